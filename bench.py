@@ -1,0 +1,454 @@
+#!/usr/bin/env python
+"""bench.py -- headline benchmark of the b2cl hot path on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl b2cl|reference]
+    python -m torch.distributed.run --nproc-per-node N ... bench.py --gpus N ...
+
+Workload (BASELINE.json configs[1], the config the metric is quoted on):
+a 4096x4096 CL_RGBA/CL_FLOAT image, normalized coordinates, LINEAR filter.
+One STEP = read_imagef over the full 4096^2 output grid under REPEAT and
+again under MIRRORED_REPEAT (map (A): translate by (0.3, 0.7) px plus a half
+period so the wrap seam crosses the output), i.e. two launches of the
+sampling kernel, 2 x 16.8 M samples.  `value` = samples / step time in
+Gsamples/s, whole job (sum over ranks; each rank owns its own image: weak
+scaling, no collective on the data path).
+
+Secondary measurements in the same JSON line (`secondary`): config 3
+(512^3 R32F trilinear), config 4 (8 GiB pitched CopyBufferRect, FillBuffer,
+CopyImageToBuffer) and the copy-size sweep, each with its HBM fraction.
+
+Timing: CUDA events on the queue's stream around every launch, after W
+untimed steps, barrier + synchronize on both sides, max over ranks.  The
+working set (256 MiB image + 2 x 256 MiB output) exceeds the 126 MB L2, so no
+flush is needed between steps.  Clocks are sampled with nvidia-smi during
+the timed region.  `--impl reference` times the CPU oracle (oracle/) on the
+host cores on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import ctypes
+import json
+import os
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "read_imagef Gsamples/s and BufferRect copy GB/s vs HBM peak at 1/2/4/8 B200"
+N2D = 4096
+WORKLOAD = "C2: 4096x4096 CL_RGBA/CL_FLOAT, normalized, LINEAR, REPEAT + MIRRORED_REPEAT, map (A)"
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+# ------------------------------------------------------------------ clocks
+class Clocks:
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.file = None
+
+    def start(self):
+        try:
+            self.file = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=self.file, stderr=subprocess.DEVNULL)
+        except (OSError, FileNotFoundError):
+            self.proc = None
+
+    def stop(self):
+        if not self.proc:
+            return None
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        self.file.flush()
+        rows = [ln.split(",") for ln in open(self.file.name).read().strip().splitlines() if ln.strip()]
+        os.unlink(self.file.name)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            try:
+                sm.append(float(r[0]))
+                mx.append(float(r[1]))
+            except (ValueError, IndexError):
+                continue
+            for n, v in zip(names, r[2:6]):
+                if v.strip() == "Active":
+                    reasons.add(n)
+        if not sm:
+            return None
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": max(mx), "samples": len(sm),
+                "reasons": sorted(reasons)}
+
+
+# ------------------------------------------------------------------ oracle (CPU) timing
+def oracle_rate(codes, n_rows_target_s: float, threads: int):
+    """Time the oracle on REPEAT + MIRRORED rows of the C2 workload.  Returns
+    (Gsamples/s, rows, seconds)."""
+    import oracle as orc
+    from paper_conf_sc_kimdjjl15_b200 import synth
+    img = orc.Image(codes, N2D, N2D, 1, dims=2, order=orc.RGBA, type=orc.FLOAT)
+    A = synth.affine_translate_2d(N2D, N2D)
+    run = lambda r0, r1: [orc.read_grid(img, True, a, orc.FILTER_LINEAR, orc.RT_F, A,
+                                        (N2D, N2D, 1), 4, yrange=(r0, r1), nthreads=threads)
+                          for a in (orc.ADDRESS_REPEAT, orc.ADDRESS_MIRRORED_REPEAT)]
+    t0 = time.perf_counter()
+    run(0, 4)
+    dt = time.perf_counter() - t0
+    rows = int(max(4, min(N2D, 4 * n_rows_target_s / max(dt, 1e-6))))
+    t0 = time.perf_counter()
+    run(0, rows)
+    dt = time.perf_counter() - t0
+    return 2 * rows * N2D / dt / 1e9, rows, dt
+
+
+def c2_codes():
+    from paper_conf_sc_kimdjjl15_b200 import cl, synth
+    g = synth.rng(2)  # the same seed the parity test of config 2 uses
+    return synth.image_codes(g, cl.CL_RGBA, cl.CL_FLOAT, N2D, N2D, 1)
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    threads = os.cpu_count() or 1
+    codes = c2_codes()
+    total_budget = 90.0
+    per_step = total_budget / max(1, args.steps + args.warmup)
+    rate, rows, _ = oracle_rate(codes, per_step, threads)  # calibrates rows per step
+    import oracle as orc
+    from paper_conf_sc_kimdjjl15_b200 import synth
+    img = orc.Image(codes, N2D, N2D, 1, dims=2, order=orc.RGBA, type=orc.FLOAT)
+    A = synth.affine_translate_2d(N2D, N2D)
+
+    def step(i):
+        y0 = (i * rows) % (N2D - rows + 1)
+        for a in (orc.ADDRESS_REPEAT, orc.ADDRESS_MIRRORED_REPEAT):
+            orc.read_grid(img, True, a, orc.FILTER_LINEAR, orc.RT_F, A, (N2D, N2D, 1), 4,
+                          yrange=(y0, y0 + rows), nthreads=threads)
+    for i in range(args.warmup):
+        step(i)
+    t0 = time.perf_counter()
+    for i in range(args.steps):
+        step(args.warmup + i)
+    dt = (time.perf_counter() - t0) / args.steps
+    value = 2 * rows * N2D / dt / 1e9
+    sample = f"{rows} rows x {N2D} columns of each pass (REPEAT, MIRRORED) per step"
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "Gsamples/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": dt * 1e3, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic (seed 20151115)",
+            "config": {"workload": WORKLOAD, "sample": sample},
+            "cpu_baseline": {"value": value, "unit": "Gsamples/s", "cores": threads,
+                             "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": "Gsamples/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ GPU arm
+class Timer:
+    """CUDA events on a torch stream (the queue's stream)."""
+
+    def __init__(self, torch, stream):
+        self.torch, self.stream = torch, stream
+
+    def event(self):
+        e = self.torch.cuda.Event(enable_timing=True)
+        e.record(self.stream)
+        return e
+
+
+def run_gpu(args):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_kimdjjl15_b200 import build, cl, synth
+    build.build()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.Stream(device=dev)
+    S = cl.Session(local, stream=stream.cuda_stream)
+    L = cl.lib()
+    T = Timer(torch, stream)
+    hbm_peak, peak_src = peaks()
+
+    # ---- inputs resident in HBM before timing ----
+    codes = c2_codes()
+    img = S.image(cl.CL_RGBA, cl.CL_FLOAT, N2D, N2D, host=codes)
+    nout = N2D * N2D * 16
+    outs = [S.buffer(nout), S.buffer(nout)]
+    smps = [S.sampler(True, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR),
+            S.sampler(True, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR)]
+    A = (ctypes.c_float * 12)(*synth.affine_translate_2d(N2D, N2D).tolist())
+    dims = cl.sz3((N2D, N2D, 1))
+
+    def launch(k):
+        cl.check(L.b2clEnqueueReadImageGrid(S.queue, img, smps[k], cl.B2CL_RTYPE_FLOAT, A, dims, 4,
+                                            outs[k], 0, 0, None, None), "read grid")
+
+    # ---- parity spot check of this exact launch configuration (bench as test) ----
+    launch(0)
+    launch(1)
+    S.finish()
+    parity = "skipped (oracle missing)"
+    try:
+        import oracle as orc
+        oimg = orc.Image(codes, N2D, N2D, 1, dims=2, order=orc.RGBA, type=orc.FLOAT)
+        Af = synth.affine_translate_2d(N2D, N2D)
+        worst = 0.0
+        for k, a in enumerate((orc.ADDRESS_REPEAT, orc.ADDRESS_MIRRORED_REPEAT)):
+            got = S.read(outs[k], nout, np.float32).reshape(N2D, N2D, 4)
+            for y in (0, N2D // 2 - 1, N2D // 2, N2D - 1, 1234):
+                exp = orc.read_grid(oimg, True, a, orc.FILTER_LINEAR, orc.RT_F, Af, (N2D, N2D, 1), 4,
+                                    yrange=(y, y + 1))[0, 0]
+                err = np.abs(got[y].astype(np.float64) - exp) / np.maximum(
+                    np.spacing(np.abs(exp)).astype(np.float64), 1e-30)
+                ok = np.all((err <= 4) | (np.abs(got[y] - exp) <= 1e-6))
+                worst = max(worst, float(np.max(np.minimum(err, 1e9))))
+                if not ok:
+                    raise SystemExit(f"bench parity check failed (pass {k}, row {y})")
+        parity = f"ok (10 rows vs oracle, worst {worst:.2f} ulp)"
+    except ImportError:
+        pass
+
+    # ---- warmup + timed steps ----
+    for _ in range(args.warmup):
+        launch(0)
+        launch(1)
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    clocks = Clocks(local)
+    clocks.start()
+    n_launch0 = cl.launch_count()
+    evs = []
+    t_start = T.event()
+    for _ in range(args.steps):
+        e0 = T.event()
+        launch(0)
+        e1 = T.event()
+        launch(1)
+        e2 = T.event()
+        evs.append((e0, e1, e2))
+    t_end = T.event()
+    torch.cuda.synchronize(dev)
+    gpu_launches = cl.launch_count() - n_launch0
+    clk = clocks.stop()
+    total_ms = t_start.elapsed_time(t_end)
+    kern_ms = [a.elapsed_time(b) for e in evs for a, b in ((e[0], e[1]), (e[1], e[2]))]
+    ms_step = total_ms / args.steps
+    if world > 1:
+        t = torch.tensor([ms_step], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_step = float(t.item())
+    samples_step = 2 * N2D * N2D
+    value = world * samples_step / (ms_step * 1e-3) / 1e9
+    k_ms = float(np.mean(kern_ms))
+    alg_bytes = N2D * N2D * 16 * 2  # every texel once (unit-scale translate covers the torus) + output
+    achieved = alg_bytes / (k_ms * 1e-3) / 1e9
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "ncu_c2_traffic.json")
+    if os.path.exists(prof):
+        traffic = json.load(open(prof)).get("dram_bytes_per_launch")
+
+    # ---- e2e: host buffers through the C-ABI, copies inside the timed region ----
+    e2e = None
+    if not args.no_e2e:
+        host_in = torch.from_numpy(codes.reshape(-1).view(np.uint8)).pin_memory()
+        host_out = [torch.empty(nout, dtype=torch.uint8).pin_memory() for _ in range(2)]
+        origin, region = cl.sz3((0, 0, 0)), cl.sz3((N2D, N2D, 1))
+
+        def e2e_step():
+            cl.check(L.clEnqueueWriteImage(S.queue, img, 0, origin, region, 0, 0,
+                                           ctypes.c_void_p(host_in.data_ptr()), 0, None, None))
+            for k in range(2):
+                launch(k)
+                cl.check(L.clEnqueueReadBuffer(S.queue, outs[k], 0, 0, nout,
+                                               ctypes.c_void_p(host_out[k].data_ptr()), 0, None, None))
+            S.finish()
+        for _ in range(2):
+            e2e_step()
+        if world > 1:
+            dist.barrier()
+        steps_e2e = max(3, args.steps // 4)
+        a = T.event()
+        for _ in range(steps_e2e):
+            e2e_step()
+        b = T.event()
+        torch.cuda.synchronize(dev)
+        e2e_ms = a.elapsed_time(b) / steps_e2e
+        if world > 1:
+            t = torch.tensor([e2e_ms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e2e_ms = float(t.item())
+        e2e = {"value": world * samples_step / (e2e_ms * 1e-3) / 1e9, "unit": "Gsamples/s",
+               "ms_per_step": e2e_ms, "h2d_bytes_per_step": int(host_in.numel()),
+               "d2h_bytes_per_step": 2 * nout}
+
+    secondary = None
+    if not args.no_secondary:
+        secondary = run_secondary(S, L, T, torch, dev, hbm_peak, args)
+
+    cpu = None
+    if rank == 0 and not args.no_cpu:
+        try:
+            threads = os.cpu_count() or 1
+            rate, rows, dt = oracle_rate(codes, args.cpu_seconds, threads)
+            cpu = {"value": rate, "unit": "Gsamples/s", "cores": threads, "kind": "oracle",
+                   "sample": f"{rows} rows x {N2D} columns of each pass (REPEAT, MIRRORED), "
+                             f"{dt:.1f} s on {threads} threads"}
+        except ImportError:
+            cpu = None
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "Gsamples/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic (numpy default_rng seed 20151115; U[0,1) RGBA32F texels)",
+            "config": {"workload": WORKLOAD, "image": "4096x4096 RGBA32F (256 MiB)",
+                       "samples_per_step": samples_step, "launches_per_step": 2,
+                       "parallelism": f"replicas x{world} (one image per GPU)",
+                       "l2": "no flush: 768 MiB working set > 126 MB L2", "parity": parity},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
+                         "frac": achieved / hbm_peak, "traffic": traffic,
+                         "kernel": "k_sample_grid<2D RGBA32F LINEAR>", "kernel_ms": k_ms,
+                         "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src},
+            "cpu_baseline": cpu, "e2e": e2e, "clocks": clk, "gpu_launches": gpu_launches,
+            "secondary": secondary,
+        }
+        print(json.dumps(line), flush=True)
+    S.release(img, *outs)
+    for s in smps:
+        L.clReleaseSampler(s)
+    S.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def _time_launches(T, torch, dev, fn, iters):
+    fn()
+    torch.cuda.synchronize(dev)
+    a = T.event()
+    for _ in range(iters):
+        fn()
+    b = T.event()
+    torch.cuda.synchronize(dev)
+    return a.elapsed_time(b) / iters
+
+
+def run_secondary(S, L, T, torch, dev, hbm_peak, args):
+    from paper_conf_sc_kimdjjl15_b200 import cl, synth
+    res = {}
+    # config 3: 512^3 R32F trilinear, stencil map, CLAMP_TO_EDGE
+    n3 = 512
+    g = synth.rng(3)
+    vol = S.image(cl.CL_R, cl.CL_FLOAT, n3, n3, n3,
+                  host=synth.image_codes(g, cl.CL_R, cl.CL_FLOAT, n3, n3, n3))
+    out3 = S.buffer(n3 ** 3 * 4)
+    smp3 = S.sampler(True, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR)
+    A3 = (ctypes.c_float * 12)(*synth.affine_stencil_3d(n3).tolist())
+    d3 = cl.sz3((n3, n3, n3))
+    ms = _time_launches(T, torch, dev, lambda: cl.check(L.b2clEnqueueReadImageGrid(
+        S.queue, vol, smp3, 0, A3, d3, 1, out3, 0, 0, None, None)), 10)
+    byt = 2 * n3 ** 3 * 4
+    res["c3_trilinear_512"] = {"Gsamples/s": n3 ** 3 / ms / 1e6, "ms": ms, "GB/s": byt / ms / 1e6,
+                               "hbm_frac": byt / ms / 1e6 / hbm_peak}
+    S.release(vol, out3)
+    L.clReleaseSampler(smp3)
+    # config 4: 8 GiB pitched CopyBufferRect (src padded, dst tight) and a misaligned variant
+    region = (16384, 2048, 256)
+    srp, ssp = 16512, 2056 * 16512
+    S_bytes = region[0] * region[1] * region[2]
+    src = S.buffer(ssp * region[2])
+    dst = S.buffer(S_bytes)
+    zero = cl.sz3((0, 0, 0))
+    ms = _time_launches(T, torch, dev, lambda: cl.check(L.clEnqueueCopyBufferRect(
+        S.queue, src, dst, zero, zero, cl.sz3(region), srp, ssp, 0, 0, 0, None, None)), 5)
+    res["c4_copy_rect_8GiB"] = {"GB/s_copied": S_bytes / ms / 1e6, "ms": ms,
+                                "hbm_frac": 2 * S_bytes / ms / 1e6 / hbm_peak}
+    reg2 = (16384, 2048, 255)
+    ms = _time_launches(T, torch, dev, lambda: cl.check(L.clEnqueueCopyBufferRect(
+        S.queue, src, dst, cl.sz3((3, 0, 0)), zero, cl.sz3(reg2), 16387, 16387 * 2056, 0, 0, 0, None,
+        None)), 5)
+    b2 = reg2[0] * reg2[1] * reg2[2]
+    res["c4_copy_rect_misaligned"] = {"GB/s_copied": b2 / ms / 1e6, "ms": ms,
+                                      "hbm_frac": 2 * b2 / ms / 1e6 / hbm_peak}
+    pat = np.arange(16, dtype=np.uint8)
+    ms = _time_launches(T, torch, dev, lambda: cl.check(L.clEnqueueFillBuffer(
+        S.queue, dst, pat.ctypes.data, 16, 0, S_bytes, 0, None, None)), 5)
+    res["c4_fill_8GiB"] = {"GB/s": S_bytes / ms / 1e6, "ms": ms, "hbm_frac": S_bytes / ms / 1e6 / hbm_peak}
+    S.release(src)
+    # CopyImageToBuffer sweep 4 KiB .. 8 GiB (RGBA32F 2D images shaped to the size)
+    sweep = []
+    for lg in range(12, 34, 3 if not args.full_sweep else 1):
+        nbytes = 1 << lg
+        w = min(32768, max(1, nbytes // 16))
+        h = max(1, nbytes // 16 // w)
+        im = S.image(cl.CL_RGBA, cl.CL_FLOAT, w, h)
+        it = 20 if nbytes < (1 << 28) else 5
+        ms = _time_launches(T, torch, dev, lambda: cl.check(L.clEnqueueCopyImageToBuffer(
+            S.queue, im, dst, zero, cl.sz3((w, h, 1)), 0, 0, None, None)), it)
+        sweep.append({"bytes": w * h * 16, "ms": ms, "GB/s_copied": w * h * 16 / ms / 1e6,
+                      "hbm_frac": 2 * w * h * 16 / ms / 1e6 / hbm_peak})
+        S.release(im)
+    res["c4_copy_image_to_buffer_sweep"] = sweep
+    S.release(dst)
+    return res
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="b2cl", choices=["b2cl", "reference"])
+    ap.add_argument("--no-secondary", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--full-sweep", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    args = ap.parse_args()
+    args.warmup = max(3, args.warmup)
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_gpu(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

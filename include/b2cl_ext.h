@@ -1,0 +1,160 @@
+/*
+ * b2cl_ext.h -- b2cl extensions to the OpenCL subset of b2cl_cl.h.
+ *
+ * The paper runs read_imageX / write_imageX as device wrappers over the
+ * CLImage pointer; there is no clBuildProgram in scope here
+ * (the translator is out of scope), so the extensions below
+ * expose those built-ins to the host as enqueue calls: one kernel launch
+ * evaluates the built-in for every sample of a coordinate list or of an
+ * affine output grid.  The per-sample arithmetic is [CL1.2 §8.1-8.3]
+ * exactly as stated in b2cl_cl.h's header, with the readings of DESIGN.md
+ * §3.  The remaining calls are runtime plumbing (torch streams and the torch
+ * allocator, raw device pointers, CUDA IPC for the one-process-per-GPU
+ * multi-device mode) and pure host validators that need no GPU.
+ */
+#ifndef B2CL_EXT_H
+#define B2CL_EXT_H
+
+#include "b2cl_cl.h"
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* return class of the read / write built-in */
+typedef cl_uint b2cl_rtype;
+#define B2CL_RTYPE_FLOAT 0 /* read_imagef / write_imagef  (float4) */
+#define B2CL_RTYPE_INT 1   /* read_imagei / write_imagei  (int4)   */
+#define B2CL_RTYPE_UINT 2  /* read_imageui / write_imageui (uint4) */
+
+/* coordinate element type of b2clEnqueueReadImageSamples */
+typedef cl_uint b2cl_ctype;
+#define B2CL_COORD_FLOAT 0
+#define B2CL_COORD_INT 1
+
+/* custom cl_mem_flags bit: allocate with cudaMalloc so that
+ * b2clGetMemIpcHandle can export the object to another process. */
+#define B2CL_MEM_IPC_EXPORTABLE ((cl_mem_flags)1 << 40)
+
+/* read_image{f,i,ui}(image, sampler, coord) for n coordinates
+ * ([CL1.2 §6.12.14.2, §8.1-8.3]; steps a3-a7).
+ *  coords:  buffer holding n coordinates starting at coords_offset, packed
+ *           per sample as 1 (1D), 2 (2D) or 4 (3D; w ignored, reading A20)
+ *           elements of 4 bytes: float (B2CL_COORD_FLOAT) or int32
+ *           (B2CL_COORD_INT: requires an unnormalized, NEAREST sampler with a
+ *           non-wrapping mode, reading A30).  coords_offset must be a
+ *           multiple of the per-sample size.
+ *  out:     n x 16 bytes (float4 / int4 / uint4) at out_offset (multiple of 16).
+ * Errors: CL_INVALID_OPERATION if rtype does not match the channel type
+ * (A7) or LINEAR is used with INT/UINT (A6); CL_INVALID_VALUE for a bad
+ * offset / size; CL_INVALID_MEM_OBJECT / CL_INVALID_SAMPLER for bad handles.
+ * n == 0 is a valid no-op. */
+cl_int b2clEnqueueReadImageSamples(cl_command_queue command_queue, cl_mem image,
+                                   cl_sampler sampler, b2cl_rtype rtype, b2cl_ctype ctype,
+                                   cl_mem coords, size_t coords_offset, size_t num_samples,
+                                   cl_mem out, size_t out_offset,
+                                   cl_uint num_events_in_wait_list,
+                                   const cl_event* event_wait_list, cl_event* event);
+
+/* read_image{f,i,ui} over an output grid of out_dims[0] x out_dims[1] x
+ * out_dims[2] samples, whose coordinates are an affine function of the
+ * output index:  for k < image dims,
+ *   coord[k] = ((affine[4k]*x + affine[4k+1]*y) + affine[4k+2]*z) + affine[4k+3]
+ * with x,y,z converted to float and EVERY operation one fp32
+ * round-to-nearest op in that order (no contraction, reading A2), so the
+ * oracle reproduces the coordinates bit for bit.  The output is tightly
+ * packed as [z][y][x][c], c < out_channels (1..4), 4 bytes per channel: the
+ * first out_channels components of the result (e.g. 1 for CL_R images).
+ * out_offset must be a multiple of 16. */
+cl_int b2clEnqueueReadImageGrid(cl_command_queue command_queue, cl_mem image,
+                                cl_sampler sampler, b2cl_rtype rtype, const float* affine,
+                                const size_t* out_dims, cl_uint out_channels, cl_mem out,
+                                size_t out_offset, cl_uint num_events_in_wait_list,
+                                const cl_event* event_wait_list, cl_event* event);
+
+/* write_image{f,i,ui}(image, int coord, color) for n samples
+ * ([CL1.2 §6.12.14.4, §8.3]; step a8).  int_coords: n x {1,2,4} int32 at
+ * coords_offset; colors: n x 16 bytes at colors_offset (multiple of 16).
+ * Out-of-range coordinates are no-ops (reading A15); if two samples hit the
+ * same texel the surviving value is one of them (unspecified which). */
+cl_int b2clEnqueueWriteImageSamples(cl_command_queue command_queue, cl_mem image,
+                                    b2cl_rtype rtype, cl_mem int_coords, size_t coords_offset,
+                                    size_t num_samples, cl_mem colors, size_t colors_offset,
+                                    cl_uint num_events_in_wait_list,
+                                    const cl_event* event_wait_list, cl_event* event);
+
+/* ---- runtime plumbing ---- */
+
+/* A queue on an existing CUDA stream (e.g. torch.cuda.Stream.cuda_stream);
+ * the stream is borrowed, not destroyed on release. */
+cl_command_queue b2clCreateCommandQueueWithStream(cl_context context, cl_device_id device,
+                                                  void* cuda_stream,
+                                                  cl_command_queue_properties properties,
+                                                  cl_int* errcode_ret);
+/* The CUDA stream (cudaStream_t) a queue launches on. */
+cl_int b2clGetCommandQueueStream(cl_command_queue command_queue, void** cuda_stream);
+/* The CUDA device ordinal behind a cl_device_id. */
+cl_int b2clGetDeviceOrdinal(cl_device_id device, cl_int* ordinal);
+
+/* Device memory provider (e.g. torch.cuda.caching_allocator_alloc/delete).
+ * alloc(size, device_ordinal, stream) returns a device pointer or NULL;
+ * free(ptr, device_ordinal, stream).  Passing NULLs restores cudaMalloc /
+ * cudaFree.  Affects objects created afterwards. */
+typedef void* (*b2cl_alloc_fn)(size_t size, int device, void* stream);
+typedef void (*b2cl_free_fn)(void* ptr, int device, void* stream);
+cl_int b2clSetAllocator(b2cl_alloc_fn alloc_fn, b2cl_free_fn free_fn);
+
+/* Wrap existing device memory (not owned, not freed) as a buffer resident
+ * on `device` of `context`. */
+cl_mem b2clCreateBufferFromDevicePointer(cl_context context, cl_device_id device,
+                                         cl_mem_flags flags, void* device_ptr, size_t size,
+                                         cl_int* errcode_ret);
+/* Device pointer of a memory object on `device` (allocated on demand; no
+ * migration).  For images this is the CLImage ptr (Fig. 6). */
+cl_int b2clGetMemDevicePointer(cl_mem memobj, cl_device_id device, void** device_ptr);
+
+/* CUDA IPC: export a B2CL_MEM_IPC_EXPORTABLE buffer (64-byte handle) and
+ * import it in another process as a buffer whose storage is the peer GPU's
+ * memory mapped over NVLink; enqueues on a queue of this process then read
+ * or write it by P2P. */
+cl_int b2clGetMemIpcHandle(cl_mem memobj, void* handle64);
+cl_mem b2clCreateBufferFromIpcHandle(cl_context context, cl_device_id device,
+                                     const void* handle64, size_t size, cl_int* errcode_ret);
+
+/* Number of b2cl kernels launched by this process so far (bench evidence). */
+cl_ulong b2clGetKernelLaunchCount(void);
+
+/* ---- pure host validators (no GPU needed; the enqueue calls use them) ---- */
+
+/* Errors of clEnqueueCopyBufferRect for buffers of src_size / dst_size
+ * bytes (same_buffer != 0 when both are one object): CL_INVALID_VALUE,
+ * CL_MEM_COPY_OVERLAP or CL_SUCCESS ([CL1.2 §5.2.2], reading A18). */
+cl_int b2clValidateCopyBufferRect(size_t src_size, size_t dst_size, cl_int same_buffer,
+                                  const size_t* src_origin, const size_t* dst_origin,
+                                  const size_t* region, size_t src_row_pitch,
+                                  size_t src_slice_pitch, size_t dst_row_pitch,
+                                  size_t dst_slice_pitch);
+/* Exact overlap test of two boxes with equal pitches in one buffer:
+ * 1 if some byte is in both, else 0. */
+cl_int b2clRectOverlap(const size_t* src_origin, const size_t* dst_origin, const size_t* region,
+                       size_t row_pitch, size_t slice_pitch);
+/* Errors of clEnqueueFillBuffer ([CL1.2 §5.2.3], reading A22). */
+cl_int b2clValidateFillBuffer(size_t buffer_size, size_t pattern_size, size_t offset,
+                              size_t size);
+/* Errors of clCreateSampler (reading A5). */
+cl_int b2clValidateSampler(cl_bool normalized_coords, cl_addressing_mode addressing_mode,
+                           cl_filter_mode filter_mode);
+/* Validates an image format / descriptor pair like clCreateImage (without
+ * a host pointer) and returns the internal layout. */
+cl_int b2clImageLayout(const cl_image_format* image_format, const cl_image_desc* image_desc,
+                       size_t* elem_size, size_t* row_pitch, size_t* slice_pitch,
+                       size_t* total_bytes);
+/* Errors of an origin / region pixel box on an image of the given type and
+ * size ([CL1.2 §5.3.3]). */
+cl_int b2clValidateImageBox(cl_mem_object_type image_type, size_t width, size_t height,
+                            size_t depth, const size_t* origin, const size_t* region);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* B2CL_EXT_H */

@@ -1,0 +1,337 @@
+"""Thin ctypes binding of libb2cl.so: the same names as include/b2cl_cl.h and
+include/b2cl_ext.h, argument marshalling only.  Every step of the hot path
+runs in the library's CUDA kernels; there is no Python or CPU fallback:
+if the library is missing, the first call raises.
+
+`Session` is a small convenience layer (one context + one queue on a device,
+numpy in / numpy out) used by the tests, smoke() and bench.py.  It calls
+only the C-ABI functions below.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from ctypes import POINTER, byref, c_float, c_int32, c_size_t, c_uint32, c_uint64, c_void_p
+
+import numpy as np
+
+LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libb2cl.so")
+
+# ---- Khronos / b2cl constants (restated from include/*.h) ----
+CL_SUCCESS = 0
+CL_DEVICE_TYPE_GPU = 1 << 2
+CL_DEVICE_TYPE_ALL = 0xFFFFFFFF
+CL_QUEUE_PROFILING_ENABLE = 1 << 1
+CL_MEM_READ_WRITE, CL_MEM_WRITE_ONLY, CL_MEM_READ_ONLY = 1, 2, 4
+CL_MEM_USE_HOST_PTR, CL_MEM_ALLOC_HOST_PTR, CL_MEM_COPY_HOST_PTR = 8, 16, 32
+B2CL_MEM_IPC_EXPORTABLE = 1 << 40
+CL_MEM_OBJECT_BUFFER, CL_MEM_OBJECT_IMAGE2D, CL_MEM_OBJECT_IMAGE3D = 0x10F0, 0x10F1, 0x10F2
+CL_MEM_OBJECT_IMAGE1D = 0x10F4
+CL_R, CL_A, CL_RG, CL_RA, CL_RGB, CL_RGBA, CL_BGRA, CL_ARGB, CL_INTENSITY, CL_LUMINANCE = range(0x10B0, 0x10BA)
+CL_SNORM_INT8, CL_SNORM_INT16, CL_UNORM_INT8, CL_UNORM_INT16 = 0x10D0, 0x10D1, 0x10D2, 0x10D3
+CL_SIGNED_INT8, CL_SIGNED_INT16, CL_SIGNED_INT32 = 0x10D7, 0x10D8, 0x10D9
+CL_UNSIGNED_INT8, CL_UNSIGNED_INT16, CL_UNSIGNED_INT32 = 0x10DA, 0x10DB, 0x10DC
+CL_HALF_FLOAT, CL_FLOAT = 0x10DD, 0x10DE
+CL_ADDRESS_NONE, CL_ADDRESS_CLAMP_TO_EDGE, CL_ADDRESS_CLAMP, CL_ADDRESS_REPEAT, \
+    CL_ADDRESS_MIRRORED_REPEAT = range(0x1130, 0x1135)
+CL_FILTER_NEAREST, CL_FILTER_LINEAR = 0x1140, 0x1141
+CL_MIGRATE_MEM_OBJECT_HOST, CL_MIGRATE_MEM_OBJECT_CONTENT_UNDEFINED = 1, 2
+CL_IMAGE_FORMAT, CL_IMAGE_ELEMENT_SIZE, CL_IMAGE_ROW_PITCH, CL_IMAGE_SLICE_PITCH = 0x1110, 0x1111, 0x1112, 0x1113
+CL_IMAGE_WIDTH, CL_IMAGE_HEIGHT, CL_IMAGE_DEPTH = 0x1114, 0x1115, 0x1116
+CL_PROFILING_COMMAND_START, CL_PROFILING_COMMAND_END = 0x1282, 0x1283
+B2CL_RTYPE_FLOAT, B2CL_RTYPE_INT, B2CL_RTYPE_UINT = 0, 1, 2
+B2CL_COORD_FLOAT, B2CL_COORD_INT = 0, 1
+
+_H = c_void_p
+_P = c_void_p
+_S = c_size_t
+_I = c_int32
+_U = c_uint32
+_L = c_uint64
+_SZ3 = POINTER(c_size_t)
+_PI = POINTER(c_int32)
+
+# name -> (restype, argtypes); covers every entry point of include/*.h
+PROTOTYPES = {
+    "clGetPlatformIDs": (_I, [_U, POINTER(_H), POINTER(_U)]),
+    "clGetPlatformInfo": (_I, [_H, _U, _S, _P, POINTER(_S)]),
+    "clGetDeviceIDs": (_I, [_H, _L, _U, POINTER(_H), POINTER(_U)]),
+    "clGetDeviceInfo": (_I, [_H, _U, _S, _P, POINTER(_S)]),
+    "clCreateContext": (_H, [_P, _U, POINTER(_H), _P, _P, _PI]),
+    "clRetainContext": (_I, [_H]),
+    "clReleaseContext": (_I, [_H]),
+    "clGetContextInfo": (_I, [_H, _U, _S, _P, POINTER(_S)]),
+    "clCreateCommandQueue": (_H, [_H, _H, _L, _PI]),
+    "clRetainCommandQueue": (_I, [_H]),
+    "clReleaseCommandQueue": (_I, [_H]),
+    "clGetCommandQueueInfo": (_I, [_H, _U, _S, _P, POINTER(_S)]),
+    "clFlush": (_I, [_H]),
+    "clFinish": (_I, [_H]),
+    "clCreateBuffer": (_H, [_H, _L, _S, _P, _PI]),
+    "clCreateImage": (_H, [_H, _L, _P, _P, _P, _PI]),
+    "clGetSupportedImageFormats": (_I, [_H, _L, _U, _U, _P, POINTER(_U)]),
+    "clRetainMemObject": (_I, [_H]),
+    "clReleaseMemObject": (_I, [_H]),
+    "clGetMemObjectInfo": (_I, [_H, _U, _S, _P, POINTER(_S)]),
+    "clGetImageInfo": (_I, [_H, _U, _S, _P, POINTER(_S)]),
+    "clCreateSampler": (_H, [_H, _U, _U, _U, _PI]),
+    "clRetainSampler": (_I, [_H]),
+    "clReleaseSampler": (_I, [_H]),
+    "clGetSamplerInfo": (_I, [_H, _U, _S, _P, POINTER(_S)]),
+    "clWaitForEvents": (_I, [_U, POINTER(_H)]),
+    "clRetainEvent": (_I, [_H]),
+    "clReleaseEvent": (_I, [_H]),
+    "clGetEventInfo": (_I, [_H, _U, _S, _P, POINTER(_S)]),
+    "clGetEventProfilingInfo": (_I, [_H, _U, _S, _P, POINTER(_S)]),
+    "clEnqueueMarkerWithWaitList": (_I, [_H, _U, POINTER(_H), POINTER(_H)]),
+    "clEnqueueBarrierWithWaitList": (_I, [_H, _U, POINTER(_H), POINTER(_H)]),
+    "clEnqueueReadBuffer": (_I, [_H, _H, _U, _S, _S, _P, _U, POINTER(_H), POINTER(_H)]),
+    "clEnqueueWriteBuffer": (_I, [_H, _H, _U, _S, _S, _P, _U, POINTER(_H), POINTER(_H)]),
+    "clEnqueueReadBufferRect": (_I, [_H, _H, _U, _SZ3, _SZ3, _SZ3, _S, _S, _S, _S, _P, _U,
+                                     POINTER(_H), POINTER(_H)]),
+    "clEnqueueWriteBufferRect": (_I, [_H, _H, _U, _SZ3, _SZ3, _SZ3, _S, _S, _S, _S, _P, _U,
+                                      POINTER(_H), POINTER(_H)]),
+    "clEnqueueCopyBuffer": (_I, [_H, _H, _H, _S, _S, _S, _U, POINTER(_H), POINTER(_H)]),
+    "clEnqueueCopyBufferRect": (_I, [_H, _H, _H, _SZ3, _SZ3, _SZ3, _S, _S, _S, _S, _U,
+                                     POINTER(_H), POINTER(_H)]),
+    "clEnqueueFillBuffer": (_I, [_H, _H, _P, _S, _S, _S, _U, POINTER(_H), POINTER(_H)]),
+    "clEnqueueReadImage": (_I, [_H, _H, _U, _SZ3, _SZ3, _S, _S, _P, _U, POINTER(_H), POINTER(_H)]),
+    "clEnqueueWriteImage": (_I, [_H, _H, _U, _SZ3, _SZ3, _S, _S, _P, _U, POINTER(_H), POINTER(_H)]),
+    "clEnqueueCopyImage": (_I, [_H, _H, _H, _SZ3, _SZ3, _SZ3, _U, POINTER(_H), POINTER(_H)]),
+    "clEnqueueFillImage": (_I, [_H, _H, _P, _SZ3, _SZ3, _U, POINTER(_H), POINTER(_H)]),
+    "clEnqueueCopyImageToBuffer": (_I, [_H, _H, _H, _SZ3, _SZ3, _S, _U, POINTER(_H), POINTER(_H)]),
+    "clEnqueueCopyBufferToImage": (_I, [_H, _H, _H, _S, _SZ3, _SZ3, _U, POINTER(_H), POINTER(_H)]),
+    "clEnqueueMigrateMemObjects": (_I, [_H, _U, POINTER(_H), _L, _U, POINTER(_H), POINTER(_H)]),
+    "b2clEnqueueReadImageSamples": (_I, [_H, _H, _H, _U, _U, _H, _S, _S, _H, _S, _U, POINTER(_H),
+                                         POINTER(_H)]),
+    "b2clEnqueueReadImageGrid": (_I, [_H, _H, _H, _U, POINTER(c_float), _SZ3, _U, _H, _S, _U,
+                                      POINTER(_H), POINTER(_H)]),
+    "b2clEnqueueWriteImageSamples": (_I, [_H, _H, _U, _H, _S, _S, _H, _S, _U, POINTER(_H),
+                                          POINTER(_H)]),
+    "b2clCreateCommandQueueWithStream": (_H, [_H, _H, _P, _L, _PI]),
+    "b2clGetCommandQueueStream": (_I, [_H, POINTER(_P)]),
+    "b2clGetDeviceOrdinal": (_I, [_H, _PI]),
+    "b2clSetAllocator": (_I, [_P, _P]),
+    "b2clCreateBufferFromDevicePointer": (_H, [_H, _H, _L, _P, _S, _PI]),
+    "b2clGetMemDevicePointer": (_I, [_H, _H, POINTER(_P)]),
+    "b2clGetMemIpcHandle": (_I, [_H, _P]),
+    "b2clCreateBufferFromIpcHandle": (_H, [_H, _H, _P, _S, _PI]),
+    "b2clGetKernelLaunchCount": (_L, []),
+    "b2clValidateCopyBufferRect": (_I, [_S, _S, _I, _SZ3, _SZ3, _SZ3, _S, _S, _S, _S]),
+    "b2clRectOverlap": (_I, [_SZ3, _SZ3, _SZ3, _S, _S]),
+    "b2clValidateFillBuffer": (_I, [_S, _S, _S, _S]),
+    "b2clValidateSampler": (_I, [_U, _U, _U]),
+    "b2clImageLayout": (_I, [_P, _P, POINTER(_S), POINTER(_S), POINTER(_S), POINTER(_S)]),
+    "b2clValidateImageBox": (_I, [_U, _S, _S, _S, _SZ3, _SZ3]),
+}
+
+
+class ImageFormat(ctypes.Structure):
+    _fields_ = [("image_channel_order", c_uint32), ("image_channel_data_type", c_uint32)]
+
+
+class ImageDesc(ctypes.Structure):
+    _fields_ = [("image_type", c_uint32), ("image_width", c_size_t), ("image_height", c_size_t),
+                ("image_depth", c_size_t), ("image_array_size", c_size_t),
+                ("image_row_pitch", c_size_t), ("image_slice_pitch", c_size_t),
+                ("num_mip_levels", c_uint32), ("num_samples", c_uint32), ("buffer", c_void_p)]
+
+
+class CLError(RuntimeError):
+    def __init__(self, code: int, what: str = ""):
+        super().__init__(f"{what} failed with OpenCL error {code}")
+        self.code = code
+
+
+_lib = None
+
+
+def lib():
+    """Load libb2cl.so (raises if it was not built: there is no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is missing: build it with "
+                               "`python -m paper_conf_sc_kimdjjl15_b200.build` (no CPU fallback)")
+        L = ctypes.CDLL(LIB_PATH)
+        for name, (res, args) in PROTOTYPES.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def __getattr__(name):  # cl.clFinish(...) etc. resolve to the C function
+    if name in PROTOTYPES:
+        return getattr(lib(), name)
+    raise AttributeError(name)
+
+
+def check(code: int, what: str = "") -> None:
+    if code != CL_SUCCESS:
+        raise CLError(code, what)
+
+
+def sz3(v) -> ctypes.Array:
+    v = [int(x) for x in v]
+    v = v + [0] * (3 - len(v)) if len(v) < 3 else v[:3]
+    return (c_size_t * 3)(*v)
+
+
+def _ptr(a: np.ndarray) -> c_void_p:
+    return c_void_p(a.ctypes.data)
+
+
+def launch_count() -> int:
+    return int(lib().b2clGetKernelLaunchCount())
+
+
+# ---- torch allocator hook (device memory from PyTorch's caching allocator) ----
+_ALLOC_T = ctypes.CFUNCTYPE(c_void_p, c_size_t, ctypes.c_int, c_void_p)
+_FREE_T = ctypes.CFUNCTYPE(None, c_void_p, ctypes.c_int, c_void_p)
+_hooks = []
+
+
+def use_torch_allocator() -> None:
+    import torch
+
+    def _alloc(size, device, stream):
+        try:
+            return torch.cuda.caching_allocator_alloc(int(size), int(device), stream or None)
+        except Exception:  # allocation failure -> NULL -> CL_MEM_OBJECT_ALLOCATION_FAILURE
+            return None
+
+    def _free(ptr, device, stream):
+        torch.cuda.caching_allocator_delete(int(ptr))
+
+    a, f = _ALLOC_T(_alloc), _FREE_T(_free)
+    _hooks[:] = [a, f]
+    check(lib().b2clSetAllocator(ctypes.cast(a, c_void_p), ctypes.cast(f, c_void_p)),
+          "b2clSetAllocator")
+
+
+def default_allocator() -> None:
+    check(lib().b2clSetAllocator(None, None), "b2clSetAllocator")
+
+
+# =============================================================== Session
+class Session:
+    """One context + one in-order queue on CUDA device `device_index`
+    (index among the platform's devices)."""
+
+    def __init__(self, device_index: int = 0, stream: int | None = None, profiling: bool = False,
+                 devices=None):
+        L = lib()
+        plat = c_void_p()
+        check(L.clGetPlatformIDs(1, byref(plat), None), "clGetPlatformIDs")
+        n = c_uint32()
+        check(L.clGetDeviceIDs(plat, CL_DEVICE_TYPE_GPU, 0, None, byref(n)), "clGetDeviceIDs")
+        devs = (c_void_p * n.value)()
+        check(L.clGetDeviceIDs(plat, CL_DEVICE_TYPE_GPU, n.value, devs, None), "clGetDeviceIDs")
+        self.all_devices = list(devs)
+        ctx_devs = [self.all_devices[i] for i in (devices or [device_index])]
+        err = c_int32()
+        arr = (c_void_p * len(ctx_devs))(*ctx_devs)
+        self.ctx = L.clCreateContext(None, len(ctx_devs), arr, None, None, byref(err))
+        check(err.value, "clCreateContext")
+        self.device = self.all_devices[device_index]
+        props = CL_QUEUE_PROFILING_ENABLE if profiling else 0
+        if stream is None:
+            self.queue = L.clCreateCommandQueue(self.ctx, self.device, props, byref(err))
+        else:
+            self.queue = L.b2clCreateCommandQueueWithStream(self.ctx, self.device, c_void_p(stream),
+                                                            props, byref(err))
+        check(err.value, "clCreateCommandQueue")
+        self._objs = []
+
+    def queue_for(self, device_index: int, profiling: bool = False):
+        err = c_int32()
+        q = lib().clCreateCommandQueue(self.ctx, self.all_devices[device_index],
+                                       CL_QUEUE_PROFILING_ENABLE if profiling else 0, byref(err))
+        check(err.value, "clCreateCommandQueue")
+        return q
+
+    def stream(self) -> int:
+        s = c_void_p()
+        check(lib().b2clGetCommandQueueStream(self.queue, byref(s)), "b2clGetCommandQueueStream")
+        return s.value or 0
+
+    def ordinal(self) -> int:
+        o = c_int32()
+        check(lib().b2clGetDeviceOrdinal(self.device, byref(o)), "b2clGetDeviceOrdinal")
+        return o.value
+
+    # ---- objects ----
+    def buffer(self, nbytes: int, host: np.ndarray | None = None, flags: int = CL_MEM_READ_WRITE):
+        err = c_int32()
+        if host is not None:
+            host = np.ascontiguousarray(host)
+            flags |= CL_MEM_COPY_HOST_PTR
+            m = lib().clCreateBuffer(self.ctx, flags, int(nbytes), _ptr(host), byref(err))
+        else:
+            m = lib().clCreateBuffer(self.ctx, flags, int(nbytes), None, byref(err))
+        check(err.value, "clCreateBuffer")
+        return m
+
+    def image(self, order: int, type_: int, width: int, height: int = 0, depth: int = 0,
+              host: np.ndarray | None = None, host_row_pitch: int = 0, host_slice_pitch: int = 0,
+              flags: int = CL_MEM_READ_WRITE):
+        dims = 3 if depth else (2 if height else 1)
+        fmt = ImageFormat(order, type_)
+        desc = ImageDesc({1: CL_MEM_OBJECT_IMAGE1D, 2: CL_MEM_OBJECT_IMAGE2D,
+                          3: CL_MEM_OBJECT_IMAGE3D}[dims], width, height, depth, 0,
+                         host_row_pitch, host_slice_pitch, 0, 0, None)
+        err = c_int32()
+        if host is not None:
+            host = np.ascontiguousarray(host)
+            m = lib().clCreateImage(self.ctx, flags | CL_MEM_COPY_HOST_PTR, byref(fmt), byref(desc),
+                                    _ptr(host), byref(err))
+        else:
+            m = lib().clCreateImage(self.ctx, flags, byref(fmt), byref(desc), None, byref(err))
+        check(err.value, "clCreateImage")
+        return m
+
+    def sampler(self, normalized: bool, addressing: int, filt: int):
+        err = c_int32()
+        s = lib().clCreateSampler(self.ctx, int(bool(normalized)), addressing, filt, byref(err))
+        check(err.value, "clCreateSampler")
+        return s
+
+    def image_info(self, img, name: int) -> int:
+        v = c_size_t()
+        check(lib().clGetImageInfo(img, name, ctypes.sizeof(v), byref(v), None), "clGetImageInfo")
+        return v.value
+
+    # ---- transfers ----
+    def write(self, buf, host: np.ndarray, offset: int = 0, blocking: bool = True) -> None:
+        host = np.ascontiguousarray(host)
+        check(lib().clEnqueueWriteBuffer(self.queue, buf, int(blocking), offset, host.nbytes,
+                                         _ptr(host), 0, None, None), "clEnqueueWriteBuffer")
+
+    def read(self, buf, nbytes: int, dtype=np.uint8, offset: int = 0) -> np.ndarray:
+        out = np.empty(nbytes, dtype=np.uint8)
+        check(lib().clEnqueueReadBuffer(self.queue, buf, 1, offset, nbytes, _ptr(out), 0, None,
+                                        None), "clEnqueueReadBuffer")
+        return out.view(dtype)
+
+    def read_image(self, img, origin, region, row_pitch=0, slice_pitch=0, nbytes=None):
+        es = self.image_info(img, CL_IMAGE_ELEMENT_SIZE)
+        rp = row_pitch or region[0] * es
+        sp = slice_pitch or rp * region[1]
+        out = np.zeros(nbytes or sp * region[2], dtype=np.uint8)
+        check(lib().clEnqueueReadImage(self.queue, img, 1, sz3(origin), sz3(region), row_pitch,
+                                       slice_pitch, _ptr(out), 0, None, None), "clEnqueueReadImage")
+        return out
+
+    def finish(self) -> None:
+        check(lib().clFinish(self.queue), "clFinish")
+
+    def release(self, *objs) -> None:
+        for o in objs:
+            lib().clReleaseMemObject(o)
+
+    def close(self) -> None:
+        L = lib()
+        L.clReleaseCommandQueue(self.queue)
+        L.clReleaseContext(self.ctx)

@@ -1,0 +1,57 @@
+// launch.h -- host-side launchers of the b2cl kernels (internal to libb2cl.so).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../device/codes.h"
+
+namespace b2cl {
+
+enum CoordMode : int { COORD_GRID = 0, COORD_LIST_F = 1, COORD_LIST_I = 2 };
+
+struct SampleParams {
+  dev::Image im;
+  dev::Sampler smp;
+  int rclass;       // dev::RetCode
+  int dims;         // 1..3
+  float A[12];      // grid: affine coordinate map
+  int ow, oh, od;   // grid: output dims
+  int outc;         // grid: output channels 1..4
+  const char* coords;  // list: coordinates (already offset)
+  uint64_t n;          // list: number of samples
+  char* out;           // output (already offset)
+};
+
+struct RectParams {
+  const char* src;   // COPY: source at origin
+  char* dst;         // destination at origin
+  uint64_t R0;       // bytes per row
+  uint32_t R1, R2;   // rows, slices
+  uint64_t srp, ssp, drp, dsp;
+  uint32_t ptile[32];     // FILL: 128-byte tile (pattern repeated)
+  uint32_t color[4];      // FILL_IMAGE: color bits
+  int type, order, es;    // FILL_IMAGE: format
+  uint32_t chunks_per_row;
+};
+
+struct WriteParams {
+  dev::Image im;
+  int rclass, dims;
+  const int32_t* coords;  // n x {1,2,4}
+  const uint32_t* colors; // n x 4
+  uint64_t n;
+};
+
+enum RectMode : int { RECT_COPY = 0, RECT_FILL = 1, RECT_FILL_IMAGE = 2 };
+
+// Each launcher enqueues exactly one kernel (or none for empty work) on
+// `stream` and returns the launch status.
+cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t stream);
+cudaError_t launch_rect(RectParams& p, int mode, cudaStream_t stream);
+cudaError_t launch_write(const WriteParams& p, cudaStream_t stream);
+
+// count of kernels launched by this library
+uint64_t launch_count();
+void count_launch();
+
+}  // namespace b2cl

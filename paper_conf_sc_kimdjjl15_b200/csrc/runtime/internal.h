@@ -1,0 +1,44 @@
+// internal.h -- host runtime internals of libb2cl (not part of the C-ABI).
+#pragma once
+#include <stddef.h>
+#include <stdint.h>
+
+#include "../../../include/b2cl_cl.h"
+#include "../../../include/b2cl_ext.h"
+#include "../device/codes.h"
+
+namespace b2cl {
+
+constexpr size_t kMax2D = 65536;  // CL_DEVICE_IMAGE2D_MAX_WIDTH/HEIGHT (and 1D width)
+constexpr size_t kMax3D = 16384;  // CL_DEVICE_IMAGE3D_MAX_*
+
+struct FormatInfo {
+  int type, order, nch, rclass;  // dev::TypeCode, dev::OrderCode, channels, dev::RetCode
+  size_t es;                     // elem_size
+};
+
+struct ImageLayout {
+  FormatInfo fmt;
+  int dims;
+  size_t w, h, d;
+  size_t row_pitch, slice_pitch, bytes;
+};
+
+int type_code(cl_channel_type t);
+int order_code(cl_channel_order o);
+cl_int format_info(const cl_image_format* f, FormatInfo* out);
+cl_int image_layout(const cl_image_format* fmt, const cl_image_desc* desc, ImageLayout* L);
+bool rect_overlap(const size_t* so, const size_t* dso, const size_t* region, size_t rp, size_t sp);
+cl_int validate_copy_rect(size_t src_size, size_t dst_size, bool same, const size_t* so,
+                          const size_t* dso, const size_t* region, size_t& srp, size_t& ssp,
+                          size_t& drp, size_t& dsp);
+cl_int validate_host_rect(size_t buf_size, const size_t* bo, const size_t* ho,
+                          const size_t* region, size_t& brp, size_t& bsp, size_t& hrp,
+                          size_t& hsp);
+cl_int validate_fill_buffer(size_t buf_size, size_t ps, size_t offset, size_t size);
+cl_int validate_sampler(cl_bool norm, cl_addressing_mode am, cl_filter_mode fm);
+cl_int validate_image_box(int dims, size_t w, size_t h, size_t d, const size_t* o,
+                          const size_t* r);
+bool image_boxes_overlap(const size_t* a, const size_t* b, const size_t* r);
+
+}  // namespace b2cl

@@ -1,0 +1,1563 @@
+// runtime.cpp -- the OpenCL 1.2 host API subset of libb2cl, over the CUDA
+// runtime (the paper's wrapper runtime, P:97-99, P:119, P:139, P:426-428,
+// re-designed for B200: one CUDA stream per queue, pitched images in HBM,
+// memory objects per context with per-device residency, peer pulls over
+// NVLink for cross-device migration).
+//
+// Every enqueue: (1) validates all arguments (no side effect on error),
+// (2) makes the touched objects resident on the queue's device,
+// (3) waits for the wait-list events, (4) launches ONE kernel (or a copy
+// engine transfer for host memory), (5) returns an event if asked.
+#include <cuda_runtime.h>
+#include <string.h>
+
+#include <algorithm>
+#include <atomic>
+#include <mutex>
+#include <new>
+#include <set>
+#include <string>
+#include <vector>
+
+#include "../kernels/launch.h"
+#include "internal.h"
+
+using namespace b2cl;
+
+// ===================================================================== objects
+struct _cl_platform_id {
+  int magic;
+};
+
+struct _cl_device_id {
+  int ordinal;
+  cudaDeviceProp prop;
+};
+
+struct _cl_context {
+  std::atomic<int> ref{1};
+  std::vector<cl_device_id> devs;  // as given (may repeat a device)
+  std::vector<int> ordinals;       // distinct CUDA ordinals
+  bool peer[64][64] = {};          // peer access enabled (dst row, src col)
+};
+
+struct _cl_command_queue {
+  std::atomic<int> ref{1};
+  cl_context ctx;
+  cl_device_id dev;
+  cudaStream_t stream;
+  bool owns_stream;
+  cl_command_queue_properties props;
+};
+
+struct Store {
+  int ordinal = -1;
+  char* ptr = nullptr;
+  int kind = 0;  // 0 none, 1 cudaMalloc, 2 allocator hook, 3 borrowed, 4 IPC import
+};
+
+struct _cl_mem {
+  std::atomic<int> ref{1};
+  cl_context ctx;
+  cl_mem_object_type type;
+  cl_mem_flags flags;
+  size_t size = 0;        // CL_MEM_SIZE (user size; images: total bytes)
+  size_t alloc_size = 0;  // rounded to 256 B
+  ImageLayout img{};      // images only
+  cl_image_format fmt{};
+  cl_image_desc desc{};
+  std::mutex mu;
+  std::vector<Store> stores;
+  uint64_t valid = 0;                   // bit per ordinal holding valid content
+  std::set<cl_command_queue> users;     // queues that enqueued work on it
+};
+
+struct _cl_sampler {
+  std::atomic<int> ref{1};
+  cl_context ctx;
+  cl_bool norm;
+  cl_addressing_mode addr;
+  cl_filter_mode filt;
+};
+
+struct _cl_event {
+  std::atomic<int> ref{1};
+  cl_context ctx;
+  cl_command_queue queue;
+  cl_command_type type;
+  int ordinal;
+  cudaEvent_t start = nullptr, end = nullptr;
+};
+
+// ===================================================================== globals
+static _cl_platform_id g_platform{0x62326c};
+static std::vector<_cl_device_id> g_devices;
+static std::once_flag g_dev_once;
+static std::mutex g_mu;                       // guards the registries below
+static std::set<cl_command_queue> g_queues;   // live queues
+static std::set<cl_mem> g_mems;
+static std::set<cl_context> g_contexts;
+static std::set<cl_sampler> g_samplers;
+static std::set<cl_event> g_events;
+static b2cl_alloc_fn g_alloc = nullptr;
+static b2cl_free_fn g_free = nullptr;
+static cudaEvent_t g_epoch[64] = {};
+
+static void init_devices() {
+  std::call_once(g_dev_once, [] {
+    int n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess) {
+      cudaGetLastError();
+      n = 0;
+    }
+    for (int i = 0; i < n; ++i) {
+      _cl_device_id d;
+      d.ordinal = i;
+      if (cudaGetDeviceProperties(&d.prop, i) != cudaSuccess) continue;
+      if (d.prop.major != 10 || d.prop.minor != 0) continue;  // kernels are sm_100a only
+      g_devices.push_back(d);
+    }
+  });
+}
+
+template <class T>
+static bool live(const std::set<T>& reg, T h) {
+  std::lock_guard<std::mutex> g(g_mu);
+  return h && reg.count(h);
+}
+
+static cl_int cuda_err(cudaError_t e) {
+  if (e == cudaSuccess) return CL_SUCCESS;
+  cudaGetLastError();
+  return e == cudaErrorMemoryAllocation ? CL_MEM_OBJECT_ALLOCATION_FAILURE : CL_OUT_OF_RESOURCES;
+}
+
+// current-device guard: the runtime sets the queue's device for its calls and
+// restores the caller's (torch's) device afterwards.
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int ordinal) {
+    cudaGetDevice(&prev);
+    if (prev != ordinal) cudaSetDevice(ordinal);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+template <class T>
+static cl_int get_info(const T& v, size_t size, void* out, size_t* size_ret) {
+  if (size_ret) *size_ret = sizeof(T);
+  if (out) {
+    if (size < sizeof(T)) return CL_INVALID_VALUE;
+    memcpy(out, &v, sizeof(T));
+  }
+  return CL_SUCCESS;
+}
+static cl_int get_str(const char* s, size_t size, void* out, size_t* size_ret) {
+  const size_t n = strlen(s) + 1;
+  if (size_ret) *size_ret = n;
+  if (out) {
+    if (size < n) return CL_INVALID_VALUE;
+    memcpy(out, s, n);
+  }
+  return CL_SUCCESS;
+}
+
+#define SET_ERR(e)             \
+  do {                         \
+    if (errcode_ret) *errcode_ret = (e); \
+  } while (0)
+
+// ===================================================================== platform / device
+extern "C" cl_int clGetPlatformIDs(cl_uint num_entries, cl_platform_id* platforms,
+                                   cl_uint* num_platforms) {
+  if ((num_entries == 0 && platforms) || (!platforms && !num_platforms)) return CL_INVALID_VALUE;
+  if (platforms && num_entries > 0) platforms[0] = &g_platform;
+  if (num_platforms) *num_platforms = 1;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clGetPlatformInfo(cl_platform_id platform, cl_platform_info name, size_t size,
+                                    void* value, size_t* size_ret) {
+  if (platform && platform != &g_platform) return CL_INVALID_PLATFORM;
+  switch (name) {
+    case CL_PLATFORM_PROFILE: return get_str("FULL_PROFILE", size, value, size_ret);
+    case CL_PLATFORM_VERSION: return get_str("OpenCL 1.2 b2cl (B200 sm_100a)", size, value, size_ret);
+    case CL_PLATFORM_NAME: return get_str("b2cl", size, value, size_ret);
+    case CL_PLATFORM_VENDOR: return get_str("b2cl", size, value, size_ret);
+    case CL_PLATFORM_EXTENSIONS: return get_str("", size, value, size_ret);
+    default: return CL_INVALID_VALUE;
+  }
+}
+
+static bool valid_device(cl_device_id d) {
+  init_devices();
+  for (auto& x : g_devices)
+    if (&x == d) return true;
+  return false;
+}
+
+extern "C" cl_int clGetDeviceIDs(cl_platform_id platform, cl_device_type type, cl_uint num_entries,
+                                 cl_device_id* devices, cl_uint* num_devices) {
+  if (platform && platform != &g_platform) return CL_INVALID_PLATFORM;
+  if ((num_entries == 0 && devices) || (!devices && !num_devices)) return CL_INVALID_VALUE;
+  const cl_device_type known = CL_DEVICE_TYPE_DEFAULT | CL_DEVICE_TYPE_CPU | CL_DEVICE_TYPE_GPU |
+                               CL_DEVICE_TYPE_ACCELERATOR;
+  if (type != CL_DEVICE_TYPE_ALL && (type & ~known)) return CL_INVALID_DEVICE_TYPE;
+  init_devices();
+  const bool gpu = type == CL_DEVICE_TYPE_ALL || (type & (CL_DEVICE_TYPE_GPU | CL_DEVICE_TYPE_DEFAULT));
+  const cl_uint n = gpu ? (cl_uint)g_devices.size() : 0;
+  if (n == 0) return CL_DEVICE_NOT_FOUND;
+  if (devices)
+    for (cl_uint i = 0; i < std::min(n, num_entries); ++i) devices[i] = &g_devices[i];
+  if (num_devices) *num_devices = n;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clGetDeviceInfo(cl_device_id d, cl_device_info name, size_t size, void* value,
+                                  size_t* size_ret) {
+  if (!valid_device(d)) return CL_INVALID_DEVICE;
+  const cudaDeviceProp& p = d->prop;
+  switch (name) {
+    case CL_DEVICE_TYPE: return get_info<cl_device_type>(CL_DEVICE_TYPE_GPU, size, value, size_ret);
+    case CL_DEVICE_VENDOR_ID: return get_info<cl_uint>(0x10DE, size, value, size_ret);
+    case CL_DEVICE_MAX_COMPUTE_UNITS: return get_info<cl_uint>(p.multiProcessorCount, size, value, size_ret);
+    case CL_DEVICE_MAX_CLOCK_FREQUENCY: {
+      int khz = 0;
+      cudaDeviceGetAttribute(&khz, cudaDevAttrClockRate, d->ordinal);
+      return get_info<cl_uint>(khz / 1000, size, value, size_ret);
+    }
+    case CL_DEVICE_GLOBAL_MEM_SIZE: return get_info<cl_ulong>(p.totalGlobalMem, size, value, size_ret);
+    case CL_DEVICE_MAX_MEM_ALLOC_SIZE: return get_info<cl_ulong>(p.totalGlobalMem, size, value, size_ret);
+    case CL_DEVICE_IMAGE_SUPPORT: return get_info<cl_bool>(CL_TRUE, size, value, size_ret);
+    case CL_DEVICE_IMAGE2D_MAX_WIDTH:
+    case CL_DEVICE_IMAGE2D_MAX_HEIGHT: return get_info<size_t>(kMax2D, size, value, size_ret);
+    case CL_DEVICE_IMAGE3D_MAX_WIDTH:
+    case CL_DEVICE_IMAGE3D_MAX_HEIGHT:
+    case CL_DEVICE_IMAGE3D_MAX_DEPTH: return get_info<size_t>(kMax3D, size, value, size_ret);
+    case CL_DEVICE_IMAGE_MAX_BUFFER_SIZE: return get_info<size_t>(0, size, value, size_ret);
+    case CL_DEVICE_AVAILABLE: return get_info<cl_bool>(CL_TRUE, size, value, size_ret);
+    case CL_DEVICE_QUEUE_PROPERTIES:
+      return get_info<cl_command_queue_properties>(
+          CL_QUEUE_PROFILING_ENABLE | CL_QUEUE_OUT_OF_ORDER_EXEC_MODE_ENABLE, size, value, size_ret);
+    case CL_DEVICE_NAME: return get_str(p.name, size, value, size_ret);
+    case CL_DEVICE_VENDOR: return get_str("NVIDIA Corporation", size, value, size_ret);
+    case CL_DRIVER_VERSION: return get_str("b2cl 0.1", size, value, size_ret);
+    case CL_DEVICE_PROFILE: return get_str("FULL_PROFILE", size, value, size_ret);
+    case CL_DEVICE_VERSION: return get_str("OpenCL 1.2 b2cl", size, value, size_ret);
+    case CL_DEVICE_PLATFORM: return get_info<cl_platform_id>(&g_platform, size, value, size_ret);
+    default: return CL_INVALID_VALUE;
+  }
+}
+
+extern "C" cl_int b2clGetDeviceOrdinal(cl_device_id d, cl_int* ordinal) {
+  if (!valid_device(d)) return CL_INVALID_DEVICE;
+  if (!ordinal) return CL_INVALID_VALUE;
+  *ordinal = d->ordinal;
+  return CL_SUCCESS;
+}
+
+// ===================================================================== context
+extern "C" cl_context clCreateContext(const cl_context_properties* props, cl_uint num_devices,
+                                      const cl_device_id* devices,
+                                      void(CL_CALLBACK* notify)(const char*, const void*, size_t, void*),
+                                      void* user_data, cl_int* errcode_ret) {
+  (void)user_data;
+  if (num_devices == 0 || !devices) { SET_ERR(CL_INVALID_VALUE); return nullptr; }
+  if (!notify && user_data) { SET_ERR(CL_INVALID_VALUE); return nullptr; }
+  if (props) {
+    for (const cl_context_properties* p = props; *p; p += 2) {
+      if (*p != 0x1084 /* CL_CONTEXT_PLATFORM */ ||
+          reinterpret_cast<cl_platform_id>(p[1]) != &g_platform) {
+        SET_ERR(CL_INVALID_PLATFORM);
+        return nullptr;
+      }
+    }
+  }
+  for (cl_uint i = 0; i < num_devices; ++i)
+    if (!valid_device(devices[i])) { SET_ERR(CL_INVALID_DEVICE); return nullptr; }
+  auto* c = new (std::nothrow) _cl_context();
+  if (!c) { SET_ERR(CL_OUT_OF_HOST_MEMORY); return nullptr; }
+  for (cl_uint i = 0; i < num_devices; ++i) {
+    c->devs.push_back(devices[i]);
+    if (std::find(c->ordinals.begin(), c->ordinals.end(), devices[i]->ordinal) == c->ordinals.end())
+      c->ordinals.push_back(devices[i]->ordinal);
+  }
+  // all-pairs peer access over NVLink / NVSwitch
+  for (int a : c->ordinals) {
+    DeviceGuard g(a);
+    if (!g_epoch[a]) cudaEventCreate(&g_epoch[a]), cudaEventRecord(g_epoch[a], 0);
+    for (int b : c->ordinals) {
+      if (a == b) continue;
+      int can = 0;
+      cudaDeviceCanAccessPeer(&can, a, b);
+      if (can) {
+        cudaError_t e = cudaDeviceEnablePeerAccess(b, 0);
+        if (e == cudaSuccess || e == cudaErrorPeerAccessAlreadyEnabled) c->peer[a][b] = true;
+        cudaGetLastError();
+      }
+    }
+  }
+  {
+    std::lock_guard<std::mutex> g(g_mu);
+    g_contexts.insert(c);
+  }
+  SET_ERR(CL_SUCCESS);
+  return c;
+}
+
+extern "C" cl_int clRetainContext(cl_context c) {
+  if (!live(g_contexts, c)) return CL_INVALID_CONTEXT;
+  c->ref++;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clReleaseContext(cl_context c) {
+  if (!live(g_contexts, c)) return CL_INVALID_CONTEXT;
+  if (--c->ref == 0) {
+    {
+      std::lock_guard<std::mutex> g(g_mu);
+      g_contexts.erase(c);
+    }
+    delete c;
+  }
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clGetContextInfo(cl_context c, cl_context_info name, size_t size, void* value,
+                                   size_t* size_ret) {
+  if (!live(g_contexts, c)) return CL_INVALID_CONTEXT;
+  switch (name) {
+    case CL_CONTEXT_REFERENCE_COUNT: return get_info<cl_uint>(c->ref.load(), size, value, size_ret);
+    case CL_CONTEXT_NUM_DEVICES: return get_info<cl_uint>((cl_uint)c->devs.size(), size, value, size_ret);
+    case CL_CONTEXT_DEVICES: {
+      const size_t n = c->devs.size() * sizeof(cl_device_id);
+      if (size_ret) *size_ret = n;
+      if (value) {
+        if (size < n) return CL_INVALID_VALUE;
+        memcpy(value, c->devs.data(), n);
+      }
+      return CL_SUCCESS;
+    }
+    default: return CL_INVALID_VALUE;
+  }
+}
+
+static bool ctx_has_device(cl_context c, cl_device_id d) {
+  return std::find(c->devs.begin(), c->devs.end(), d) != c->devs.end();
+}
+
+// ===================================================================== queue
+static cl_command_queue make_queue(cl_context c, cl_device_id d, cl_command_queue_properties props,
+                                   void* stream, cl_int* errcode_ret) {
+  if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
+  if (!valid_device(d) || !ctx_has_device(c, d)) { SET_ERR(CL_INVALID_DEVICE); return nullptr; }
+  if (props & ~(cl_command_queue_properties)(CL_QUEUE_PROFILING_ENABLE |
+                                             CL_QUEUE_OUT_OF_ORDER_EXEC_MODE_ENABLE)) {
+    SET_ERR(CL_INVALID_VALUE);
+    return nullptr;
+  }
+  auto* q = new (std::nothrow) _cl_command_queue();
+  if (!q) { SET_ERR(CL_OUT_OF_HOST_MEMORY); return nullptr; }
+  q->ctx = c;
+  q->dev = d;
+  q->props = props;
+  if (stream) {
+    q->stream = static_cast<cudaStream_t>(stream);
+    q->owns_stream = false;
+  } else {
+    DeviceGuard g(d->ordinal);
+    cudaError_t e = cudaStreamCreateWithFlags(&q->stream, cudaStreamNonBlocking);
+    if (e != cudaSuccess) {
+      delete q;
+      SET_ERR(cuda_err(e));
+      return nullptr;
+    }
+    q->owns_stream = true;
+  }
+  c->ref++;
+  {
+    std::lock_guard<std::mutex> g(g_mu);
+    g_queues.insert(q);
+  }
+  SET_ERR(CL_SUCCESS);
+  return q;
+}
+
+extern "C" cl_command_queue clCreateCommandQueue(cl_context c, cl_device_id d,
+                                                 cl_command_queue_properties props,
+                                                 cl_int* errcode_ret) {
+  return make_queue(c, d, props, nullptr, errcode_ret);
+}
+
+extern "C" cl_command_queue b2clCreateCommandQueueWithStream(cl_context c, cl_device_id d,
+                                                             void* stream,
+                                                             cl_command_queue_properties props,
+                                                             cl_int* errcode_ret) {
+  return make_queue(c, d, props, stream, errcode_ret);
+}
+
+extern "C" cl_int b2clGetCommandQueueStream(cl_command_queue q, void** stream) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  if (!stream) return CL_INVALID_VALUE;
+  *stream = q->stream;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clRetainCommandQueue(cl_command_queue q) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  q->ref++;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clReleaseCommandQueue(cl_command_queue q) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  if (--q->ref == 0) {
+    {
+      DeviceGuard g(q->dev->ordinal);
+      cudaStreamSynchronize(q->stream);  // implicit flush + finish before teardown
+      if (q->owns_stream) cudaStreamDestroy(q->stream);
+    }
+    {
+      std::lock_guard<std::mutex> g(g_mu);
+      g_queues.erase(q);
+      for (cl_mem m : g_mems) {
+        std::lock_guard<std::mutex> gm(m->mu);
+        m->users.erase(q);
+      }
+    }
+    cl_context c = q->ctx;
+    delete q;
+    clReleaseContext(c);
+  }
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clGetCommandQueueInfo(cl_command_queue q, cl_command_queue_info name,
+                                        size_t size, void* value, size_t* size_ret) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  switch (name) {
+    case CL_QUEUE_CONTEXT: return get_info<cl_context>(q->ctx, size, value, size_ret);
+    case CL_QUEUE_DEVICE: return get_info<cl_device_id>(q->dev, size, value, size_ret);
+    case CL_QUEUE_REFERENCE_COUNT: return get_info<cl_uint>(q->ref.load(), size, value, size_ret);
+    case CL_QUEUE_PROPERTIES:
+      return get_info<cl_command_queue_properties>(q->props, size, value, size_ret);
+    default: return CL_INVALID_VALUE;
+  }
+}
+
+extern "C" cl_int clFlush(cl_command_queue q) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  return CL_SUCCESS;  // CUDA submits at launch
+}
+
+extern "C" cl_int clFinish(cl_command_queue q) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  DeviceGuard g(q->dev->ordinal);
+  return cuda_err(cudaStreamSynchronize(q->stream));
+}
+
+// ===================================================================== memory objects
+static void* raw_alloc(size_t bytes, int ordinal, cudaStream_t stream, int* kind, bool ipc) {
+  DeviceGuard g(ordinal);
+  if (g_alloc && !ipc) {
+    void* p = g_alloc(bytes, ordinal, stream);
+    if (p) {
+      *kind = 2;
+      return p;
+    }
+    return nullptr;
+  }
+  void* p = nullptr;
+  if (cudaMalloc(&p, bytes) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  *kind = 1;
+  return p;
+}
+
+static void raw_free(Store& s) {
+  DeviceGuard g(s.ordinal);
+  if (s.kind == 1) cudaFree(s.ptr);
+  else if (s.kind == 2 && g_free) g_free(s.ptr, s.ordinal, nullptr);
+  else if (s.kind == 4) cudaIpcCloseMemHandle(s.ptr);
+  s.ptr = nullptr;
+  s.kind = 0;
+}
+
+static Store* find_store(cl_mem m, int ordinal) {
+  for (auto& s : m->stores)
+    if (s.ordinal == ordinal) return &s;
+  return nullptr;
+}
+
+static cl_mem new_mem(cl_context c, cl_mem_object_type type, cl_mem_flags flags, size_t size) {
+  auto* m = new (std::nothrow) _cl_mem();
+  if (!m) return nullptr;
+  m->ctx = c;
+  m->type = type;
+  m->flags = flags;
+  m->size = size;
+  m->alloc_size = (size + 255) / 256 * 256;
+  m->stores.reserve(64);  // Store pointers stay valid
+  return m;
+}
+
+static void register_mem(cl_mem m) {
+  m->ctx->ref++;
+  std::lock_guard<std::mutex> g(g_mu);
+  g_mems.insert(m);
+}
+
+static cl_int check_mem_flags(cl_mem_flags flags, void* host_ptr) {
+  const cl_mem_flags access = flags & (CL_MEM_READ_WRITE | CL_MEM_WRITE_ONLY | CL_MEM_READ_ONLY);
+  if (access && (access & (access - 1))) return CL_INVALID_VALUE;
+  const cl_mem_flags known = CL_MEM_READ_WRITE | CL_MEM_WRITE_ONLY | CL_MEM_READ_ONLY |
+                             CL_MEM_USE_HOST_PTR | CL_MEM_ALLOC_HOST_PTR | CL_MEM_COPY_HOST_PTR |
+                             CL_MEM_HOST_WRITE_ONLY | CL_MEM_HOST_READ_ONLY |
+                             CL_MEM_HOST_NO_ACCESS | B2CL_MEM_IPC_EXPORTABLE;
+  if (flags & ~known) return CL_INVALID_VALUE;
+  if (flags & CL_MEM_USE_HOST_PTR) return CL_INVALID_VALUE;  // reading A33
+  const bool copy = flags & CL_MEM_COPY_HOST_PTR;
+  if (copy != (host_ptr != nullptr)) return CL_INVALID_HOST_PTR;
+  return CL_SUCCESS;
+}
+
+// Allocate the object's storage on `ordinal` if missing (content not valid).
+static cl_int ensure_store(cl_mem m, int ordinal, cudaStream_t stream, Store** out) {
+  Store* s = find_store(m, ordinal);
+  if (!s) {
+    int kind = 0;
+    void* p = raw_alloc(m->alloc_size, ordinal, stream, &kind,
+                        (m->flags & B2CL_MEM_IPC_EXPORTABLE) != 0);
+    if (!p) return CL_MEM_OBJECT_ALLOCATION_FAILURE;
+    Store st;
+    st.ordinal = ordinal;
+    st.ptr = static_cast<char*>(p);
+    st.kind = kind;
+    m->stores.push_back(st);
+    s = &m->stores.back();
+  }
+  *out = s;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_mem clCreateBuffer(cl_context c, cl_mem_flags flags, size_t size, void* host_ptr,
+                                 cl_int* errcode_ret) {
+  if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
+  cl_int st = check_mem_flags(flags, host_ptr);
+  if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
+  if (size == 0) { SET_ERR(CL_INVALID_BUFFER_SIZE); return nullptr; }
+  cl_mem m = new_mem(c, CL_MEM_OBJECT_BUFFER, flags, size);
+  if (!m) { SET_ERR(CL_OUT_OF_HOST_MEMORY); return nullptr; }
+  const int ord = c->devs[0]->ordinal;
+  Store* s = nullptr;
+  st = ensure_store(m, ord, nullptr, &s);
+  if (st != CL_SUCCESS) { delete m; SET_ERR(st); return nullptr; }
+  if (host_ptr) {
+    DeviceGuard g(ord);
+    cudaError_t e = cudaMemcpy(s->ptr, host_ptr, size, cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) { raw_free(*s); delete m; SET_ERR(cuda_err(e)); return nullptr; }
+  }
+  m->valid = 1ull << ord;
+  register_mem(m);
+  SET_ERR(CL_SUCCESS);
+  return m;
+}
+
+extern "C" cl_mem b2clCreateBufferFromDevicePointer(cl_context c, cl_device_id d, cl_mem_flags flags,
+                                                    void* ptr, size_t size, cl_int* errcode_ret) {
+  if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
+  if (!valid_device(d) || !ctx_has_device(c, d)) { SET_ERR(CL_INVALID_DEVICE); return nullptr; }
+  if (!ptr || size == 0 || (flags & (CL_MEM_USE_HOST_PTR | CL_MEM_COPY_HOST_PTR))) {
+    SET_ERR(CL_INVALID_VALUE);
+    return nullptr;
+  }
+  cl_mem m = new_mem(c, CL_MEM_OBJECT_BUFFER, flags, size);
+  if (!m) { SET_ERR(CL_OUT_OF_HOST_MEMORY); return nullptr; }
+  Store s;
+  s.ordinal = d->ordinal;
+  s.ptr = static_cast<char*>(ptr);
+  s.kind = 3;
+  m->stores.push_back(s);
+  m->valid = 1ull << d->ordinal;
+  register_mem(m);
+  SET_ERR(CL_SUCCESS);
+  return m;
+}
+
+extern "C" cl_mem clCreateImage(cl_context c, cl_mem_flags flags, const cl_image_format* fmt,
+                                const cl_image_desc* desc, void* host_ptr, cl_int* errcode_ret) {
+  if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
+  cl_int st = check_mem_flags(flags & ~B2CL_MEM_IPC_EXPORTABLE, host_ptr);
+  if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
+  ImageLayout L;
+  st = image_layout(fmt, desc, &L);
+  if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
+  // host pitches ([CL1.2 §5.3.1]): nonzero only with a host pointer, >= tight,
+  // multiple of the element size; slice pitch only for 3D
+  size_t hrp = desc->image_row_pitch, hsp = desc->image_slice_pitch;
+  if ((hrp || hsp) && !host_ptr) { SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR); return nullptr; }
+  if (hrp == 0) hrp = L.w * L.fmt.es;
+  else if (hrp < L.w * L.fmt.es || hrp % L.fmt.es) { SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR); return nullptr; }
+  if (L.dims == 3) {
+    if (hsp == 0) hsp = hrp * L.h;
+    else if (hsp < hrp * L.h || hsp % hrp) { SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR); return nullptr; }
+  } else if (hsp != 0) {
+    SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR);
+    return nullptr;
+  }
+  cl_mem m = new_mem(c, desc->image_type, flags, L.bytes);
+  if (!m) { SET_ERR(CL_OUT_OF_HOST_MEMORY); return nullptr; }
+  m->img = L;
+  m->fmt = *fmt;
+  m->desc = *desc;
+  const int ord = c->devs[0]->ordinal;
+  Store* s = nullptr;
+  st = ensure_store(m, ord, nullptr, &s);
+  if (st != CL_SUCCESS) { delete m; SET_ERR(st); return nullptr; }
+  if (host_ptr) {  // clCreateImage uploads the contents
+    DeviceGuard g(ord);
+    for (size_t k = 0; k < L.d; ++k) {
+      cudaError_t e = cudaMemcpy2D(s->ptr + k * L.slice_pitch, L.row_pitch,
+                                   static_cast<const char*>(host_ptr) + k * hsp, hrp,
+                                   L.w * L.fmt.es, L.h, cudaMemcpyHostToDevice);
+      if (e != cudaSuccess) { raw_free(*s); delete m; SET_ERR(cuda_err(e)); return nullptr; }
+    }
+  }
+  m->valid = 1ull << ord;
+  register_mem(m);
+  SET_ERR(CL_SUCCESS);
+  return m;
+}
+
+extern "C" cl_int clGetSupportedImageFormats(cl_context c, cl_mem_flags flags,
+                                             cl_mem_object_type type, cl_uint num_entries,
+                                             cl_image_format* formats, cl_uint* num_formats) {
+  (void)flags;
+  if (!live(g_contexts, c)) return CL_INVALID_CONTEXT;
+  if (type != CL_MEM_OBJECT_IMAGE1D && type != CL_MEM_OBJECT_IMAGE2D &&
+      type != CL_MEM_OBJECT_IMAGE3D)
+    return CL_INVALID_VALUE;
+  if (num_entries == 0 && formats) return CL_INVALID_VALUE;
+  std::vector<cl_image_format> all;
+  for (cl_channel_order o = CL_R; o <= CL_LUMINANCE; ++o)
+    for (cl_channel_type t = CL_SNORM_INT8; t <= CL_FLOAT; ++t) {
+      cl_image_format f{o, t};
+      FormatInfo fi;
+      if (format_info(&f, &fi) == CL_SUCCESS) all.push_back(f);
+    }
+  if (formats)
+    for (cl_uint i = 0; i < std::min<cl_uint>(num_entries, (cl_uint)all.size()); ++i) formats[i] = all[i];
+  if (num_formats) *num_formats = (cl_uint)all.size();
+  return CL_SUCCESS;
+}
+
+static bool is_image(cl_mem m) {
+  return m->type == CL_MEM_OBJECT_IMAGE1D || m->type == CL_MEM_OBJECT_IMAGE2D ||
+         m->type == CL_MEM_OBJECT_IMAGE3D;
+}
+
+extern "C" cl_int clRetainMemObject(cl_mem m) {
+  if (!live(g_mems, m)) return CL_INVALID_MEM_OBJECT;
+  m->ref++;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clReleaseMemObject(cl_mem m) {
+  if (!live(g_mems, m)) return CL_INVALID_MEM_OBJECT;
+  if (--m->ref == 0) {
+    std::vector<cl_command_queue> users;
+    {
+      std::lock_guard<std::mutex> g(g_mu);
+      g_mems.erase(m);
+      for (cl_command_queue q : m->users)
+        if (g_queues.count(q)) users.push_back(q);
+    }
+    // stream-ordered free: drain the queues that used the object first
+    for (cl_command_queue q : users) {
+      DeviceGuard g(q->dev->ordinal);
+      cudaStreamSynchronize(q->stream);
+    }
+    for (auto& s : m->stores) raw_free(s);
+    cl_context c = m->ctx;
+    delete m;
+    clReleaseContext(c);
+  }
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clGetMemObjectInfo(cl_mem m, cl_mem_info name, size_t size, void* value,
+                                     size_t* size_ret) {
+  if (!live(g_mems, m)) return CL_INVALID_MEM_OBJECT;
+  switch (name) {
+    case CL_MEM_TYPE: return get_info<cl_mem_object_type>(m->type, size, value, size_ret);
+    case CL_MEM_FLAGS: return get_info<cl_mem_flags>(m->flags, size, value, size_ret);
+    case CL_MEM_SIZE: return get_info<size_t>(m->size, size, value, size_ret);
+    case CL_MEM_HOST_PTR: return get_info<void*>(nullptr, size, value, size_ret);
+    case CL_MEM_MAP_COUNT: return get_info<cl_uint>(0, size, value, size_ret);
+    case CL_MEM_REFERENCE_COUNT: return get_info<cl_uint>(m->ref.load(), size, value, size_ret);
+    case CL_MEM_CONTEXT: return get_info<cl_context>(m->ctx, size, value, size_ret);
+    default: return CL_INVALID_VALUE;
+  }
+}
+
+extern "C" cl_int clGetImageInfo(cl_mem m, cl_image_info name, size_t size, void* value,
+                                 size_t* size_ret) {
+  if (!live(g_mems, m) || !is_image(m)) return CL_INVALID_MEM_OBJECT;
+  const ImageLayout& L = m->img;
+  switch (name) {
+    case CL_IMAGE_FORMAT: return get_info<cl_image_format>(m->fmt, size, value, size_ret);
+    case CL_IMAGE_ELEMENT_SIZE: return get_info<size_t>(L.fmt.es, size, value, size_ret);
+    case CL_IMAGE_ROW_PITCH: return get_info<size_t>(L.row_pitch, size, value, size_ret);
+    case CL_IMAGE_SLICE_PITCH:
+      return get_info<size_t>(L.dims == 3 ? L.slice_pitch : 0, size, value, size_ret);
+    case CL_IMAGE_WIDTH: return get_info<size_t>(L.w, size, value, size_ret);
+    case CL_IMAGE_HEIGHT: return get_info<size_t>(L.dims > 1 ? L.h : 0, size, value, size_ret);
+    case CL_IMAGE_DEPTH: return get_info<size_t>(L.dims > 2 ? L.d : 0, size, value, size_ret);
+    case CL_IMAGE_ARRAY_SIZE: return get_info<size_t>(0, size, value, size_ret);
+    case CL_IMAGE_BUFFER: return get_info<cl_mem>(nullptr, size, value, size_ret);
+    case CL_IMAGE_NUM_MIP_LEVELS:
+    case CL_IMAGE_NUM_SAMPLES: return get_info<cl_uint>(0, size, value, size_ret);
+    default: return CL_INVALID_VALUE;
+  }
+}
+
+extern "C" cl_int b2clSetAllocator(b2cl_alloc_fn a, b2cl_free_fn f) {
+  if ((a == nullptr) != (f == nullptr)) return CL_INVALID_VALUE;
+  g_alloc = a;
+  g_free = f;
+  return CL_SUCCESS;
+}
+
+// ===================================================================== sampler
+extern "C" cl_sampler clCreateSampler(cl_context c, cl_bool norm, cl_addressing_mode am,
+                                      cl_filter_mode fm, cl_int* errcode_ret) {
+  if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
+  cl_int st = validate_sampler(norm, am, fm);
+  if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
+  auto* s = new (std::nothrow) _cl_sampler();
+  if (!s) { SET_ERR(CL_OUT_OF_HOST_MEMORY); return nullptr; }
+  s->ctx = c;
+  s->norm = norm;
+  s->addr = am;
+  s->filt = fm;
+  c->ref++;
+  {
+    std::lock_guard<std::mutex> g(g_mu);
+    g_samplers.insert(s);
+  }
+  SET_ERR(CL_SUCCESS);
+  return s;
+}
+
+extern "C" cl_int clRetainSampler(cl_sampler s) {
+  if (!live(g_samplers, s)) return CL_INVALID_SAMPLER;
+  s->ref++;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clReleaseSampler(cl_sampler s) {
+  if (!live(g_samplers, s)) return CL_INVALID_SAMPLER;
+  if (--s->ref == 0) {
+    {
+      std::lock_guard<std::mutex> g(g_mu);
+      g_samplers.erase(s);
+    }
+    cl_context c = s->ctx;
+    delete s;
+    clReleaseContext(c);
+  }
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clGetSamplerInfo(cl_sampler s, cl_sampler_info name, size_t size, void* value,
+                                   size_t* size_ret) {
+  if (!live(g_samplers, s)) return CL_INVALID_SAMPLER;
+  switch (name) {
+    case CL_SAMPLER_REFERENCE_COUNT: return get_info<cl_uint>(s->ref.load(), size, value, size_ret);
+    case CL_SAMPLER_CONTEXT: return get_info<cl_context>(s->ctx, size, value, size_ret);
+    case CL_SAMPLER_NORMALIZED_COORDS: return get_info<cl_bool>(s->norm, size, value, size_ret);
+    case CL_SAMPLER_ADDRESSING_MODE: return get_info<cl_addressing_mode>(s->addr, size, value, size_ret);
+    case CL_SAMPLER_FILTER_MODE: return get_info<cl_filter_mode>(s->filt, size, value, size_ret);
+    default: return CL_INVALID_VALUE;
+  }
+}
+
+// ===================================================================== events
+extern "C" cl_int clWaitForEvents(cl_uint n, const cl_event* list) {
+  if (n == 0 || !list) return CL_INVALID_VALUE;
+  for (cl_uint i = 0; i < n; ++i)
+    if (!live(g_events, list[i])) return CL_INVALID_EVENT;
+  for (cl_uint i = 0; i < n; ++i) {
+    cudaError_t e = cudaEventSynchronize(list[i]->end);
+    if (e != cudaSuccess) return cuda_err(e);
+  }
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clRetainEvent(cl_event e) {
+  if (!live(g_events, e)) return CL_INVALID_EVENT;
+  e->ref++;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clReleaseEvent(cl_event e) {
+  if (!live(g_events, e)) return CL_INVALID_EVENT;
+  if (--e->ref == 0) {
+    {
+      std::lock_guard<std::mutex> g(g_mu);
+      g_events.erase(e);
+    }
+    DeviceGuard g(e->ordinal);
+    if (e->start) cudaEventDestroy(e->start);
+    if (e->end) cudaEventDestroy(e->end);
+    cl_context c = e->ctx;
+    delete e;
+    clReleaseContext(c);
+  }
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clGetEventInfo(cl_event e, cl_event_info name, size_t size, void* value,
+                                 size_t* size_ret) {
+  if (!live(g_events, e)) return CL_INVALID_EVENT;
+  switch (name) {
+    case CL_EVENT_COMMAND_QUEUE: return get_info<cl_command_queue>(e->queue, size, value, size_ret);
+    case CL_EVENT_CONTEXT: return get_info<cl_context>(e->ctx, size, value, size_ret);
+    case CL_EVENT_COMMAND_TYPE: return get_info<cl_command_type>(e->type, size, value, size_ret);
+    case CL_EVENT_REFERENCE_COUNT: return get_info<cl_uint>(e->ref.load(), size, value, size_ret);
+    case CL_EVENT_COMMAND_EXECUTION_STATUS: {
+      cudaError_t q = cudaEventQuery(e->end);
+      cl_int status = q == cudaSuccess ? CL_COMPLETE : CL_SUBMITTED;
+      if (q != cudaSuccess && q != cudaErrorNotReady) status = CL_OUT_OF_RESOURCES;
+      cudaGetLastError();
+      return get_info<cl_int>(status, size, value, size_ret);
+    }
+    default: return CL_INVALID_VALUE;
+  }
+}
+
+extern "C" cl_int clGetEventProfilingInfo(cl_event e, cl_profiling_info name, size_t size,
+                                          void* value, size_t* size_ret) {
+  if (!live(g_events, e)) return CL_INVALID_EVENT;
+  if (!e->start) return CL_PROFILING_INFO_NOT_AVAILABLE;
+  if (cudaEventQuery(e->end) != cudaSuccess) {
+    cudaGetLastError();
+    return CL_PROFILING_INFO_NOT_AVAILABLE;
+  }
+  float ms = 0.f;
+  cudaEvent_t which = name == CL_PROFILING_COMMAND_END ? e->end : e->start;
+  if (name < CL_PROFILING_COMMAND_QUEUED || name > CL_PROFILING_COMMAND_END) return CL_INVALID_VALUE;
+  DeviceGuard g(e->ordinal);
+  if (cudaEventElapsedTime(&ms, g_epoch[e->ordinal], which) != cudaSuccess) {
+    cudaGetLastError();
+    return CL_PROFILING_INFO_NOT_AVAILABLE;
+  }
+  return get_info<cl_ulong>((cl_ulong)((double)ms * 1e6), size, value, size_ret);
+}
+
+// ===================================================================== enqueue plumbing
+struct Enq {
+  cl_command_queue q = nullptr;
+  cl_event* evout = nullptr;
+  cl_command_type type = 0;
+  cudaEvent_t start = nullptr;
+};
+
+static cl_int check_wait_list(cl_command_queue q, cl_uint n, const cl_event* list) {
+  if ((n == 0) != (list == nullptr)) return CL_INVALID_EVENT_WAIT_LIST;
+  for (cl_uint i = 0; i < n; ++i)
+    if (!live(g_events, list[i]) || list[i]->ctx != q->ctx) return CL_INVALID_EVENT_WAIT_LIST;
+  return CL_SUCCESS;
+}
+
+// after validation: make the stream wait for the wait list; start event
+static cl_int enq_begin(Enq& E, cl_uint n, const cl_event* list) {
+  for (cl_uint i = 0; i < n; ++i) cudaStreamWaitEvent(E.q->stream, list[i]->end, 0);
+  if (E.evout && (E.q->props & CL_QUEUE_PROFILING_ENABLE)) {
+    if (cudaEventCreate(&E.start) != cudaSuccess) return CL_OUT_OF_RESOURCES;
+    cudaEventRecord(E.start, E.q->stream);
+  }
+  return CL_SUCCESS;
+}
+
+static cl_int enq_end(Enq& E, cudaError_t err) {
+  if (err != cudaSuccess) {
+    if (E.start) cudaEventDestroy(E.start);
+    return cuda_err(err);
+  }
+  if (E.evout) {
+    auto* ev = new (std::nothrow) _cl_event();
+    if (!ev) return CL_OUT_OF_HOST_MEMORY;
+    ev->ctx = E.q->ctx;
+    ev->queue = E.q;
+    ev->type = E.type;
+    ev->ordinal = E.q->dev->ordinal;
+    ev->start = E.start;
+    const unsigned flags = E.start ? cudaEventDefault : cudaEventDisableTiming;
+    if (cudaEventCreateWithFlags(&ev->end, flags) != cudaSuccess) {
+      delete ev;
+      return CL_OUT_OF_RESOURCES;
+    }
+    cudaEventRecord(ev->end, E.q->stream);
+    E.q->ctx->ref++;
+    {
+      std::lock_guard<std::mutex> g(g_mu);
+      g_events.insert(ev);
+    }
+    *E.evout = ev;
+  }
+  return CL_SUCCESS;
+}
+
+// Make the object's content valid on the queue's device and return its
+// pointer there.  If another device holds the only valid copy, pull it over
+// NVLink (SM copy kernel on the peer pointer) on the queue's stream; the
+// caller's wait list orders it after the producer (OpenCL cross-queue rule).
+static cl_int resident(cl_mem m, cl_command_queue q, bool need_content, char** out) {
+  std::lock_guard<std::mutex> g(m->mu);
+  const int ord = q->dev->ordinal;
+  Store* s = nullptr;
+  cl_int st = ensure_store(m, ord, q->stream, &s);
+  if (st != CL_SUCCESS) return st;
+  const uint64_t bit = 1ull << ord;
+  if (need_content && !(m->valid & bit) && m->valid) {
+    int src = -1;
+    for (auto& o : m->stores)
+      if ((m->valid >> o.ordinal) & 1ull) { src = o.ordinal; break; }
+    Store* ss = find_store(m, src);
+    cudaError_t e;
+    if (q->ctx->peer[ord][src]) {
+      RectParams p{};
+      p.src = ss->ptr;
+      p.dst = s->ptr;
+      p.R0 = m->alloc_size;
+      p.R1 = p.R2 = 1;
+      p.srp = p.drp = m->alloc_size;
+      p.ssp = p.dsp = m->alloc_size;
+      e = launch_rect(p, RECT_COPY, q->stream);
+    } else {
+      e = cudaMemcpyPeerAsync(s->ptr, ord, ss->ptr, src, m->alloc_size, q->stream);
+    }
+    if (e != cudaSuccess) return cuda_err(e);
+    m->valid |= bit;
+  }
+  m->users.insert(q);
+  *out = s->ptr;
+  return CL_SUCCESS;
+}
+
+static void written(cl_mem m, cl_command_queue q) {
+  std::lock_guard<std::mutex> g(m->mu);
+  m->valid = 1ull << q->dev->ordinal;
+}
+
+static cl_int check_queue_mem(cl_command_queue q, cl_mem m) {
+  if (!live(g_mems, m) || m->ctx != q->ctx) return CL_INVALID_MEM_OBJECT;
+  return CL_SUCCESS;
+}
+
+#define CHECK(x)                        \
+  do {                                  \
+    cl_int _s = (x);                    \
+    if (_s != CL_SUCCESS) return _s;    \
+  } while (0)
+
+static dev::Image dev_image(cl_mem m, char* ptr) {
+  dev::Image im{};
+  const ImageLayout& L = m->img;
+  im.ptr = ptr;
+  im.w = (int)L.w;
+  im.h = (int)L.h;
+  im.d = (int)L.d;
+  im.type = L.fmt.type;
+  im.order = L.fmt.order;
+  im.es = (int)L.fmt.es;
+  im.nch = L.fmt.nch;
+  im.rp = L.row_pitch;
+  im.sp = L.slice_pitch;
+  return im;
+}
+
+// ===================================================================== host <-> device transfers
+static cl_int host_rect_copy(Enq& E, char* dev, size_t drp, size_t dsp, char* host, size_t hrp,
+                             size_t hsp, const size_t* region, bool to_device, cl_bool blocking) {
+  DeviceGuard g(E.q->dev->ordinal);
+  cudaError_t e = cudaSuccess;
+  for (size_t k = 0; k < region[2] && e == cudaSuccess; ++k) {
+    if (to_device)
+      e = cudaMemcpy2DAsync(dev + k * dsp, drp, host + k * hsp, hrp, region[0], region[1],
+                            cudaMemcpyHostToDevice, E.q->stream);
+    else
+      e = cudaMemcpy2DAsync(host + k * hsp, hrp, dev + k * dsp, drp, region[0], region[1],
+                            cudaMemcpyDeviceToHost, E.q->stream);
+  }
+  cl_int st = enq_end(E, e);
+  if (st != CL_SUCCESS) return st;
+  if (blocking) return cuda_err(cudaStreamSynchronize(E.q->stream));
+  return CL_SUCCESS;
+}
+
+static cl_int buffer_host_rect(cl_command_queue q, cl_mem buf, cl_bool blocking, const size_t* bo,
+                               const size_t* ho, const size_t* region, size_t brp, size_t bsp,
+                               size_t hrp, size_t hsp, char* ptr, bool write, cl_uint nw,
+                               const cl_event* wl, cl_event* ev, cl_command_type type) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_queue_mem(q, buf));
+  if (buf->type != CL_MEM_OBJECT_BUFFER) return CL_INVALID_MEM_OBJECT;
+  if (!ptr) return CL_INVALID_VALUE;
+  CHECK(validate_host_rect(buf->size, bo, ho, region, brp, bsp, hrp, hsp));
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = type;
+  DeviceGuard g(q->dev->ordinal);
+  char* d = nullptr;
+  CHECK(resident(buf, q, true, &d));
+  CHECK(enq_begin(E, nw, wl));
+  char* dbase = d + bo[2] * bsp + bo[1] * brp + bo[0];
+  char* hbase = ptr + ho[2] * hsp + ho[1] * hrp + ho[0];
+  cl_int st = host_rect_copy(E, dbase, brp, bsp, hbase, hrp, hsp, region, write, blocking);
+  if (st == CL_SUCCESS && write) written(buf, q);
+  return st;
+}
+
+extern "C" cl_int clEnqueueReadBuffer(cl_command_queue q, cl_mem buf, cl_bool blocking,
+                                      size_t offset, size_t size, void* ptr, cl_uint nw,
+                                      const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_queue_mem(q, buf));
+  if (size == 0 || offset > buf->size || size > buf->size - offset) return CL_INVALID_VALUE;
+  const size_t bo[3] = {offset, 0, 0}, ho[3] = {0, 0, 0}, region[3] = {size, 1, 1};
+  return buffer_host_rect(q, buf, blocking, bo, ho, region, 0, 0, 0, 0, static_cast<char*>(ptr),
+                          false, nw, wl, ev, CL_COMMAND_READ_BUFFER);
+}
+
+extern "C" cl_int clEnqueueWriteBuffer(cl_command_queue q, cl_mem buf, cl_bool blocking,
+                                       size_t offset, size_t size, const void* ptr, cl_uint nw,
+                                       const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_queue_mem(q, buf));
+  if (size == 0 || offset > buf->size || size > buf->size - offset) return CL_INVALID_VALUE;
+  const size_t bo[3] = {offset, 0, 0}, ho[3] = {0, 0, 0}, region[3] = {size, 1, 1};
+  return buffer_host_rect(q, buf, blocking, bo, ho, region, 0, 0, 0, 0,
+                          const_cast<char*>(static_cast<const char*>(ptr)), true, nw, wl, ev,
+                          CL_COMMAND_WRITE_BUFFER);
+}
+
+extern "C" cl_int clEnqueueReadBufferRect(cl_command_queue q, cl_mem buf, cl_bool blocking,
+                                          const size_t* bo, const size_t* ho, const size_t* region,
+                                          size_t brp, size_t bsp, size_t hrp, size_t hsp, void* ptr,
+                                          cl_uint nw, const cl_event* wl, cl_event* ev) {
+  return buffer_host_rect(q, buf, blocking, bo, ho, region, brp, bsp, hrp, hsp,
+                          static_cast<char*>(ptr), false, nw, wl, ev, CL_COMMAND_READ_BUFFER_RECT);
+}
+
+extern "C" cl_int clEnqueueWriteBufferRect(cl_command_queue q, cl_mem buf, cl_bool blocking,
+                                           const size_t* bo, const size_t* ho, const size_t* region,
+                                           size_t brp, size_t bsp, size_t hrp, size_t hsp,
+                                           const void* ptr, cl_uint nw, const cl_event* wl,
+                                           cl_event* ev) {
+  return buffer_host_rect(q, buf, blocking, bo, ho, region, brp, bsp, hrp, hsp,
+                          const_cast<char*>(static_cast<const char*>(ptr)), true, nw, wl, ev,
+                          CL_COMMAND_WRITE_BUFFER_RECT);
+}
+
+static cl_int image_host(cl_command_queue q, cl_mem img, cl_bool blocking, const size_t* origin,
+                         const size_t* region, size_t rp, size_t sp, char* ptr, bool write,
+                         cl_uint nw, const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_queue_mem(q, img));
+  if (!is_image(img)) return CL_INVALID_MEM_OBJECT;
+  const ImageLayout& L = img->img;
+  if (!ptr) return CL_INVALID_VALUE;
+  CHECK(validate_image_box(L.dims, L.w, L.h, L.d, origin, region));
+  const size_t es = L.fmt.es;
+  if (rp == 0) rp = region[0] * es;
+  else if (rp < region[0] * es) return CL_INVALID_VALUE;
+  if (L.dims < 3 && sp != 0) return CL_INVALID_VALUE;
+  if (sp == 0) sp = rp * region[1];
+  else if (sp < rp * region[1]) return CL_INVALID_VALUE;
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = write ? CL_COMMAND_WRITE_IMAGE : CL_COMMAND_READ_IMAGE;
+  DeviceGuard g(q->dev->ordinal);
+  char* d = nullptr;
+  CHECK(resident(img, q, true, &d));
+  CHECK(enq_begin(E, nw, wl));
+  char* dbase = d + origin[2] * L.slice_pitch + origin[1] * L.row_pitch + origin[0] * es;
+  const size_t bytes_region[3] = {region[0] * es, region[1], region[2]};
+  cl_int st = host_rect_copy(E, dbase, L.row_pitch, L.slice_pitch, ptr, rp, sp, bytes_region, write,
+                             blocking);
+  if (st == CL_SUCCESS && write) written(img, q);
+  return st;
+}
+
+extern "C" cl_int clEnqueueReadImage(cl_command_queue q, cl_mem img, cl_bool blocking,
+                                     const size_t* origin, const size_t* region, size_t rp,
+                                     size_t sp, void* ptr, cl_uint nw, const cl_event* wl,
+                                     cl_event* ev) {
+  return image_host(q, img, blocking, origin, region, rp, sp, static_cast<char*>(ptr), false, nw,
+                    wl, ev);
+}
+
+extern "C" cl_int clEnqueueWriteImage(cl_command_queue q, cl_mem img, cl_bool blocking,
+                                      const size_t* origin, const size_t* region, size_t rp,
+                                      size_t sp, const void* ptr, cl_uint nw, const cl_event* wl,
+                                      cl_event* ev) {
+  return image_host(q, img, blocking, origin, region, rp, sp,
+                    const_cast<char*>(static_cast<const char*>(ptr)), true, nw, wl, ev);
+}
+
+// ===================================================================== device rect copies / fills
+// One rect-copy kernel launch between two objects (already validated).
+static cl_int rect_copy(cl_command_queue q, cl_mem src, cl_mem dst, size_t soff, size_t doff,
+                        const size_t* region_bytes, size_t srp, size_t ssp, size_t drp, size_t dsp,
+                        cl_uint nw, const cl_event* wl, cl_event* ev, cl_command_type type) {
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = type;
+  DeviceGuard g(q->dev->ordinal);
+  char *s = nullptr, *d = nullptr;
+  CHECK(resident(src, q, true, &s));
+  CHECK(resident(dst, q, true, &d));
+  CHECK(enq_begin(E, nw, wl));
+  RectParams p{};
+  p.src = s + soff;
+  p.dst = d + doff;
+  p.R0 = region_bytes[0];
+  p.R1 = (uint32_t)region_bytes[1];
+  p.R2 = (uint32_t)region_bytes[2];
+  p.srp = srp;
+  p.ssp = ssp;
+  p.drp = drp;
+  p.dsp = dsp;
+  cl_int st = enq_end(E, launch_rect(p, RECT_COPY, q->stream));
+  if (st == CL_SUCCESS) written(dst, q);
+  return st;
+}
+
+extern "C" cl_int clEnqueueCopyBufferRect(cl_command_queue q, cl_mem src, cl_mem dst,
+                                          const size_t* so, const size_t* dso, const size_t* region,
+                                          size_t srp, size_t ssp, size_t drp, size_t dsp, cl_uint nw,
+                                          const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_queue_mem(q, src));
+  CHECK(check_queue_mem(q, dst));
+  if (src->type != CL_MEM_OBJECT_BUFFER || dst->type != CL_MEM_OBJECT_BUFFER)
+    return CL_INVALID_MEM_OBJECT;
+  CHECK(validate_copy_rect(src->size, dst->size, src == dst, so, dso, region, srp, ssp, drp, dsp));
+  if (region[1] > 0xffffffffull || region[2] > 0xffffffffull) return CL_INVALID_VALUE;
+  const size_t soff = so[2] * ssp + so[1] * srp + so[0];
+  const size_t doff = dso[2] * dsp + dso[1] * drp + dso[0];
+  return rect_copy(q, src, dst, soff, doff, region, srp, ssp, drp, dsp, nw, wl, ev,
+                   CL_COMMAND_COPY_BUFFER_RECT);
+}
+
+extern "C" cl_int clEnqueueCopyBuffer(cl_command_queue q, cl_mem src, cl_mem dst, size_t so,
+                                      size_t dso, size_t size, cl_uint nw, const cl_event* wl,
+                                      cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_queue_mem(q, src));
+  CHECK(check_queue_mem(q, dst));
+  if (src->type != CL_MEM_OBJECT_BUFFER || dst->type != CL_MEM_OBJECT_BUFFER)
+    return CL_INVALID_MEM_OBJECT;
+  if (size == 0 || so > src->size || size > src->size - so || dso > dst->size ||
+      size > dst->size - dso)
+    return CL_INVALID_VALUE;
+  if (src == dst && so < dso + size && dso < so + size) return CL_MEM_COPY_OVERLAP;
+  const size_t region[3] = {size, 1, 1};
+  return rect_copy(q, src, dst, so, dso, region, size, size, size, size, nw, wl, ev,
+                   CL_COMMAND_COPY_BUFFER);
+}
+
+extern "C" cl_int clEnqueueFillBuffer(cl_command_queue q, cl_mem buf, const void* pattern,
+                                      size_t ps, size_t offset, size_t size, cl_uint nw,
+                                      const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_queue_mem(q, buf));
+  if (buf->type != CL_MEM_OBJECT_BUFFER) return CL_INVALID_MEM_OBJECT;
+  if (!pattern) return CL_INVALID_VALUE;
+  CHECK(validate_fill_buffer(buf->size, ps, offset, size));
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = CL_COMMAND_FILL_BUFFER;
+  DeviceGuard g(q->dev->ordinal);
+  char* d = nullptr;
+  CHECK(resident(buf, q, true, &d));
+  CHECK(enq_begin(E, nw, wl));
+  RectParams p{};
+  p.dst = d + offset;
+  p.R0 = size;
+  p.R1 = p.R2 = 1;
+  p.drp = p.dsp = size;
+  // 128-byte tile indexed by absolute address: tile[X mod 128] = pattern[(X - start) mod ps]
+  const uintptr_t start = reinterpret_cast<uintptr_t>(p.dst);
+  unsigned char* tb = reinterpret_cast<unsigned char*>(p.ptile);
+  const unsigned char* pat = static_cast<const unsigned char*>(pattern);
+  for (uintptr_t k = 0; k < 128; ++k) tb[k] = pat[(k + 128 * ps - (start % ps)) % ps];
+  cl_int st = enq_end(E, launch_rect(p, RECT_FILL, q->stream));
+  if (st == CL_SUCCESS) written(buf, q);
+  return st;
+}
+
+static cl_int image_info_checked(cl_command_queue q, cl_mem m) {
+  CHECK(check_queue_mem(q, m));
+  if (!is_image(m)) return CL_INVALID_MEM_OBJECT;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clEnqueueCopyImage(cl_command_queue q, cl_mem src, cl_mem dst, const size_t* so,
+                                     const size_t* dso, const size_t* region, cl_uint nw,
+                                     const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(image_info_checked(q, src));
+  CHECK(image_info_checked(q, dst));
+  const ImageLayout &A = src->img, &B = dst->img;
+  if (A.fmt.type != B.fmt.type || A.fmt.order != B.fmt.order) return CL_IMAGE_FORMAT_MISMATCH;
+  CHECK(validate_image_box(A.dims, A.w, A.h, A.d, so, region));
+  CHECK(validate_image_box(B.dims, B.w, B.h, B.d, dso, region));
+  if (src == dst && image_boxes_overlap(so, dso, region)) return CL_MEM_COPY_OVERLAP;
+  const size_t es = A.fmt.es;
+  const size_t soff = so[2] * A.slice_pitch + so[1] * A.row_pitch + so[0] * es;
+  const size_t doff = dso[2] * B.slice_pitch + dso[1] * B.row_pitch + dso[0] * es;
+  const size_t rb[3] = {region[0] * es, region[1], region[2]};
+  return rect_copy(q, src, dst, soff, doff, rb, A.row_pitch, A.slice_pitch, B.row_pitch,
+                   B.slice_pitch, nw, wl, ev, CL_COMMAND_COPY_IMAGE);
+}
+
+extern "C" cl_int clEnqueueCopyImageToBuffer(cl_command_queue q, cl_mem src, cl_mem dst,
+                                             const size_t* so, const size_t* region, size_t doff,
+                                             cl_uint nw, const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(image_info_checked(q, src));
+  CHECK(check_queue_mem(q, dst));
+  if (dst->type != CL_MEM_OBJECT_BUFFER) return CL_INVALID_MEM_OBJECT;
+  const ImageLayout& A = src->img;
+  CHECK(validate_image_box(A.dims, A.w, A.h, A.d, so, region));
+  const size_t es = A.fmt.es, row = region[0] * es;
+  const size_t bytes = row * region[1] * region[2];
+  if (doff > dst->size || bytes > dst->size - doff) return CL_INVALID_VALUE;
+  const size_t soff = so[2] * A.slice_pitch + so[1] * A.row_pitch + so[0] * es;
+  const size_t rb[3] = {row, region[1], region[2]};
+  return rect_copy(q, src, dst, soff, doff, rb, A.row_pitch, A.slice_pitch, row, row * region[1],
+                   nw, wl, ev, CL_COMMAND_COPY_IMAGE_TO_BUFFER);
+}
+
+extern "C" cl_int clEnqueueCopyBufferToImage(cl_command_queue q, cl_mem src, cl_mem dst,
+                                             size_t soff, const size_t* dso, const size_t* region,
+                                             cl_uint nw, const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_queue_mem(q, src));
+  CHECK(image_info_checked(q, dst));
+  if (src->type != CL_MEM_OBJECT_BUFFER) return CL_INVALID_MEM_OBJECT;
+  const ImageLayout& B = dst->img;
+  CHECK(validate_image_box(B.dims, B.w, B.h, B.d, dso, region));
+  const size_t es = B.fmt.es, row = region[0] * es;
+  const size_t bytes = row * region[1] * region[2];
+  if (soff > src->size || bytes > src->size - soff) return CL_INVALID_VALUE;
+  const size_t doff = dso[2] * B.slice_pitch + dso[1] * B.row_pitch + dso[0] * es;
+  const size_t rb[3] = {row, region[1], region[2]};
+  return rect_copy(q, src, dst, soff, doff, rb, row, row * region[1], B.row_pitch, B.slice_pitch,
+                   nw, wl, ev, CL_COMMAND_COPY_BUFFER_TO_IMAGE);
+}
+
+extern "C" cl_int clEnqueueFillImage(cl_command_queue q, cl_mem img, const void* color,
+                                     const size_t* origin, const size_t* region, cl_uint nw,
+                                     const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(image_info_checked(q, img));
+  if (!color) return CL_INVALID_VALUE;
+  const ImageLayout& L = img->img;
+  CHECK(validate_image_box(L.dims, L.w, L.h, L.d, origin, region));
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = CL_COMMAND_FILL_IMAGE;
+  DeviceGuard g(q->dev->ordinal);
+  char* d = nullptr;
+  CHECK(resident(img, q, true, &d));
+  CHECK(enq_begin(E, nw, wl));
+  const size_t es = L.fmt.es;
+  RectParams p{};
+  p.dst = d + origin[2] * L.slice_pitch + origin[1] * L.row_pitch + origin[0] * es;
+  p.R0 = region[0] * es;
+  p.R1 = (uint32_t)region[1];
+  p.R2 = (uint32_t)region[2];
+  p.drp = L.row_pitch;
+  p.dsp = L.slice_pitch;
+  memcpy(p.color, color, 16);
+  p.type = L.fmt.type;
+  p.order = L.fmt.order;
+  p.es = (int)es;
+  cl_int st = enq_end(E, launch_rect(p, RECT_FILL_IMAGE, q->stream));
+  if (st == CL_SUCCESS) written(img, q);
+  return st;
+}
+
+extern "C" cl_int clEnqueueMigrateMemObjects(cl_command_queue q, cl_uint n, const cl_mem* mems,
+                                             cl_mem_migration_flags flags, cl_uint nw,
+                                             const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  if (n == 0 || !mems) return CL_INVALID_VALUE;
+  if (flags & ~(cl_mem_migration_flags)(CL_MIGRATE_MEM_OBJECT_HOST |
+                                        CL_MIGRATE_MEM_OBJECT_CONTENT_UNDEFINED))
+    return CL_INVALID_VALUE;
+  for (cl_uint i = 0; i < n; ++i) CHECK(check_queue_mem(q, mems[i]));
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = CL_COMMAND_MIGRATE_MEM_OBJECTS;
+  DeviceGuard g(q->dev->ordinal);
+  CHECK(enq_begin(E, nw, wl));
+  if (!(flags & CL_MIGRATE_MEM_OBJECT_HOST)) {  // HOST: device memory is the only storage (A24)
+    const bool undefined = flags & CL_MIGRATE_MEM_OBJECT_CONTENT_UNDEFINED;
+    for (cl_uint i = 0; i < n; ++i) {
+      char* d = nullptr;
+      CHECK(resident(mems[i], q, !undefined, &d));
+      if (undefined) written(mems[i], q);  // ownership moves without a copy
+    }
+  }
+  return enq_end(E, cudaSuccess);
+}
+
+extern "C" cl_int clEnqueueMarkerWithWaitList(cl_command_queue q, cl_uint nw, const cl_event* wl,
+                                              cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = CL_COMMAND_MARKER;
+  DeviceGuard g(q->dev->ordinal);
+  CHECK(enq_begin(E, nw, wl));
+  return enq_end(E, cudaSuccess);
+}
+
+extern "C" cl_int clEnqueueBarrierWithWaitList(cl_command_queue q, cl_uint nw, const cl_event* wl,
+                                               cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = CL_COMMAND_BARRIER;
+  DeviceGuard g(q->dev->ordinal);
+  CHECK(enq_begin(E, nw, wl));
+  return enq_end(E, cudaSuccess);
+}
+
+// ===================================================================== built-in extensions
+static cl_int check_read_combo(cl_mem img, cl_sampler smp, b2cl_rtype rtype) {
+  if (rtype > B2CL_RTYPE_UINT) return CL_INVALID_VALUE;
+  if ((int)rtype != img->img.fmt.rclass) return CL_INVALID_OPERATION;           // A7
+  if (rtype != B2CL_RTYPE_FLOAT && smp->filt == CL_FILTER_LINEAR) return CL_INVALID_OPERATION;  // A6
+  return CL_SUCCESS;
+}
+
+static void fill_sampler(SampleParams& p, cl_sampler smp) {
+  p.smp.norm = smp->norm ? 1 : 0;
+  p.smp.addr = (int)(smp->addr - CL_ADDRESS_NONE);
+  p.smp.filt = smp->filt == CL_FILTER_LINEAR ? dev::F_LINEAR : dev::F_NEAREST;
+}
+
+extern "C" cl_int b2clEnqueueReadImageSamples(cl_command_queue q, cl_mem img, cl_sampler smp,
+                                              b2cl_rtype rtype, b2cl_ctype ctype, cl_mem coords,
+                                              size_t coffset, size_t n, cl_mem out, size_t ooffset,
+                                              cl_uint nw, const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(image_info_checked(q, img));
+  if (!live(g_samplers, smp) || smp->ctx != q->ctx) return CL_INVALID_SAMPLER;
+  CHECK(check_queue_mem(q, coords));
+  CHECK(check_queue_mem(q, out));
+  if (coords->type != CL_MEM_OBJECT_BUFFER || out->type != CL_MEM_OBJECT_BUFFER)
+    return CL_INVALID_MEM_OBJECT;
+  CHECK(check_read_combo(img, smp, rtype));
+  if (ctype > B2CL_COORD_INT) return CL_INVALID_VALUE;
+  if (ctype == B2CL_COORD_INT &&
+      (smp->norm || smp->filt != CL_FILTER_NEAREST || smp->addr == CL_ADDRESS_REPEAT ||
+       smp->addr == CL_ADDRESS_MIRRORED_REPEAT))
+    return CL_INVALID_OPERATION;  // A30
+  const int dims = img->img.dims;
+  const size_t per = 4 * (dims == 1 ? 1 : (dims == 2 ? 2 : 4));
+  if (coffset % per != 0 || ooffset % 16 != 0) return CL_INVALID_VALUE;
+  if (n > 0 && (coffset > coords->size || n > (coords->size - coffset) / per ||
+                ooffset > out->size || n > (out->size - ooffset) / 16))
+    return CL_INVALID_VALUE;
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = 0x11F0;  // NDRANGE_KERNEL
+  DeviceGuard g(q->dev->ordinal);
+  char *pi = nullptr, *pc = nullptr, *po = nullptr;
+  CHECK(resident(img, q, true, &pi));
+  CHECK(resident(coords, q, true, &pc));
+  CHECK(resident(out, q, true, &po));
+  CHECK(enq_begin(E, nw, wl));
+  SampleParams p{};
+  p.im = dev_image(img, pi);
+  fill_sampler(p, smp);
+  p.rclass = (int)rtype;
+  p.dims = dims;
+  p.coords = pc + coffset;
+  p.n = n;
+  p.out = po + ooffset;
+  cl_int st = enq_end(E, launch_sample(p, ctype == B2CL_COORD_INT ? COORD_LIST_I : COORD_LIST_F,
+                                       q->stream));
+  if (st == CL_SUCCESS) written(out, q);
+  return st;
+}
+
+extern "C" cl_int b2clEnqueueReadImageGrid(cl_command_queue q, cl_mem img, cl_sampler smp,
+                                           b2cl_rtype rtype, const float* affine,
+                                           const size_t* out_dims, cl_uint outc, cl_mem out,
+                                           size_t ooffset, cl_uint nw, const cl_event* wl,
+                                           cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(image_info_checked(q, img));
+  if (!live(g_samplers, smp) || smp->ctx != q->ctx) return CL_INVALID_SAMPLER;
+  CHECK(check_queue_mem(q, out));
+  if (out->type != CL_MEM_OBJECT_BUFFER) return CL_INVALID_MEM_OBJECT;
+  CHECK(check_read_combo(img, smp, rtype));
+  if (!affine || !out_dims || outc < 1 || outc > 4 || ooffset % 16 != 0) return CL_INVALID_VALUE;
+  if (out_dims[0] > 0x7fffffff || out_dims[1] > 0x7fffffff || out_dims[2] > 65535)
+    return CL_INVALID_VALUE;
+  const unsigned __int128 bytes =
+      (unsigned __int128)out_dims[0] * out_dims[1] * out_dims[2] * outc * 4;
+  if (ooffset > out->size || bytes > out->size - ooffset) return CL_INVALID_VALUE;
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = 0x11F0;
+  DeviceGuard g(q->dev->ordinal);
+  char *pi = nullptr, *po = nullptr;
+  CHECK(resident(img, q, true, &pi));
+  CHECK(resident(out, q, true, &po));
+  CHECK(enq_begin(E, nw, wl));
+  SampleParams p{};
+  p.im = dev_image(img, pi);
+  fill_sampler(p, smp);
+  p.rclass = (int)rtype;
+  p.dims = img->img.dims;
+  memcpy(p.A, affine, sizeof(p.A));
+  p.ow = (int)out_dims[0];
+  p.oh = (int)out_dims[1];
+  p.od = (int)out_dims[2];
+  p.outc = (int)outc;
+  p.out = po + ooffset;
+  cl_int st = enq_end(E, launch_sample(p, COORD_GRID, q->stream));
+  if (st == CL_SUCCESS) written(out, q);
+  return st;
+}
+
+extern "C" cl_int b2clEnqueueWriteImageSamples(cl_command_queue q, cl_mem img, b2cl_rtype rtype,
+                                               cl_mem coords, size_t coffset, size_t n,
+                                               cl_mem colors, size_t koffset, cl_uint nw,
+                                               const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(image_info_checked(q, img));
+  CHECK(check_queue_mem(q, coords));
+  CHECK(check_queue_mem(q, colors));
+  if (coords->type != CL_MEM_OBJECT_BUFFER || colors->type != CL_MEM_OBJECT_BUFFER)
+    return CL_INVALID_MEM_OBJECT;
+  if (rtype > B2CL_RTYPE_UINT) return CL_INVALID_VALUE;
+  if ((int)rtype != img->img.fmt.rclass) return CL_INVALID_OPERATION;  // A7
+  const int dims = img->img.dims;
+  const size_t per = 4 * (dims == 1 ? 1 : (dims == 2 ? 2 : 4));
+  if (coffset % per != 0 || koffset % 16 != 0) return CL_INVALID_VALUE;
+  if (n > 0 && (coffset > coords->size || n > (coords->size - coffset) / per ||
+                koffset > colors->size || n > (colors->size - koffset) / 16))
+    return CL_INVALID_VALUE;
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = 0x11F0;
+  DeviceGuard g(q->dev->ordinal);
+  char *pi = nullptr, *pc = nullptr, *pk = nullptr;
+  CHECK(resident(img, q, true, &pi));
+  CHECK(resident(coords, q, true, &pc));
+  CHECK(resident(colors, q, true, &pk));
+  CHECK(enq_begin(E, nw, wl));
+  WriteParams p{};
+  p.im = dev_image(img, pi);
+  p.rclass = (int)rtype;
+  p.dims = dims;
+  p.coords = reinterpret_cast<const int32_t*>(pc + coffset);
+  p.colors = reinterpret_cast<const uint32_t*>(pk + koffset);
+  p.n = n;
+  cl_int st = enq_end(E, launch_write(p, q->stream));
+  if (st == CL_SUCCESS) written(img, q);
+  return st;
+}
+
+// ===================================================================== interop
+extern "C" cl_int b2clGetMemDevicePointer(cl_mem m, cl_device_id d, void** ptr) {
+  if (!live(g_mems, m)) return CL_INVALID_MEM_OBJECT;
+  if (!valid_device(d) || !ctx_has_device(m->ctx, d)) return CL_INVALID_DEVICE;
+  if (!ptr) return CL_INVALID_VALUE;
+  std::lock_guard<std::mutex> g(m->mu);
+  Store* s = nullptr;
+  CHECK(ensure_store(m, d->ordinal, nullptr, &s));
+  *ptr = s->ptr;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int b2clGetMemIpcHandle(cl_mem m, void* handle64) {
+  if (!live(g_mems, m)) return CL_INVALID_MEM_OBJECT;
+  if (!handle64) return CL_INVALID_VALUE;
+  std::lock_guard<std::mutex> g(m->mu);
+  if (!(m->flags & B2CL_MEM_IPC_EXPORTABLE) || m->stores.empty() || m->stores[0].kind != 1)
+    return CL_INVALID_OPERATION;
+  DeviceGuard dg(m->stores[0].ordinal);
+  cudaIpcMemHandle_t h;
+  cudaError_t e = cudaIpcGetMemHandle(&h, m->stores[0].ptr);
+  if (e != cudaSuccess) return cuda_err(e);
+  static_assert(sizeof(h) == 64, "IPC handle size");
+  memcpy(handle64, &h, 64);
+  return CL_SUCCESS;
+}
+
+extern "C" cl_mem b2clCreateBufferFromIpcHandle(cl_context c, cl_device_id d, const void* handle64,
+                                                size_t size, cl_int* errcode_ret) {
+  if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
+  if (!valid_device(d) || !ctx_has_device(c, d)) { SET_ERR(CL_INVALID_DEVICE); return nullptr; }
+  if (!handle64 || size == 0) { SET_ERR(CL_INVALID_VALUE); return nullptr; }
+  cudaIpcMemHandle_t h;
+  memcpy(&h, handle64, 64);
+  void* p = nullptr;
+  {
+    DeviceGuard g(d->ordinal);
+    cudaError_t e = cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) { SET_ERR(cuda_err(e)); return nullptr; }
+  }
+  cl_mem m = new_mem(c, CL_MEM_OBJECT_BUFFER, CL_MEM_READ_WRITE, size);
+  if (!m) { SET_ERR(CL_OUT_OF_HOST_MEMORY); return nullptr; }
+  Store s;
+  s.ordinal = d->ordinal;
+  s.ptr = static_cast<char*>(p);
+  s.kind = 4;
+  m->stores.push_back(s);
+  m->valid = 1ull << d->ordinal;
+  register_mem(m);
+  SET_ERR(CL_SUCCESS);
+  return m;
+}
+
+extern "C" cl_ulong b2clGetKernelLaunchCount(void) { return launch_count(); }

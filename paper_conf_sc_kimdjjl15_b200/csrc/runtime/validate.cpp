@@ -1,0 +1,269 @@
+// validate.cpp -- pure host-side argument validation (no CUDA calls).
+//
+// Every enqueue of the runtime validates through these functions before it
+// issues anything ("all validation happens before anything is enqueued").
+// They are also exported (b2cl_ext.h) so the error behaviour is testable on
+// a machine without a GPU.  Rules: [CL1.2 §5.2.2, §5.2.3, §5.3.1, §5.3.3,
+// §5.5.1] with readings A5, A18, A21, A22 of DESIGN.md §3.
+#include <stdint.h>
+
+#include "internal.h"
+
+namespace b2cl {
+
+// Khronos channel type / order -> internal codes (dev::TypeCode / OrderCode)
+int type_code(cl_channel_type t) {
+  switch (t) {
+    case CL_SNORM_INT8: return dev::T_SNORM8;
+    case CL_SNORM_INT16: return dev::T_SNORM16;
+    case CL_UNORM_INT8: return dev::T_UNORM8;
+    case CL_UNORM_INT16: return dev::T_UNORM16;
+    case CL_SIGNED_INT8: return dev::T_SINT8;
+    case CL_SIGNED_INT16: return dev::T_SINT16;
+    case CL_SIGNED_INT32: return dev::T_SINT32;
+    case CL_UNSIGNED_INT8: return dev::T_UINT8;
+    case CL_UNSIGNED_INT16: return dev::T_UINT16;
+    case CL_UNSIGNED_INT32: return dev::T_UINT32;
+    case CL_HALF_FLOAT: return dev::T_HALF;
+    case CL_FLOAT: return dev::T_FLOAT;
+    default: return -1;
+  }
+}
+
+int order_code(cl_channel_order o) {
+  switch (o) {
+    case CL_R: return dev::O_R;
+    case CL_A: return dev::O_A;
+    case CL_RG: return dev::O_RG;
+    case CL_RA: return dev::O_RA;
+    case CL_RGBA: return dev::O_RGBA;
+    case CL_BGRA: return dev::O_BGRA;
+    case CL_ARGB: return dev::O_ARGB;
+    case CL_INTENSITY: return dev::O_INTENSITY;
+    case CL_LUMINANCE: return dev::O_LUMINANCE;
+    default: return -1;
+  }
+}
+
+static bool known_type(cl_channel_type t) { return t >= 0x10D0 && t <= 0x10DE; }
+static bool known_order(cl_channel_order o) { return o >= 0x10B0 && o <= 0x10B9; }
+
+cl_int format_info(const cl_image_format* f, FormatInfo* out) {
+  if (!f || !known_type(f->image_channel_data_type) || !known_order(f->image_channel_order))
+    return CL_INVALID_IMAGE_FORMAT_DESCRIPTOR;
+  const int t = type_code(f->image_channel_data_type);
+  const int o = order_code(f->image_channel_order);
+  if (t < 0 || o < 0) return CL_IMAGE_FORMAT_NOT_SUPPORTED;  // packed types, CL_RGB
+  // [CL1.2 §5.3.1.1]: BGRA/ARGB only with 8-bit channels; INTENSITY and
+  // LUMINANCE only with UNORM/SNORM 8/16, HALF and FLOAT.
+  if (o == dev::O_BGRA || o == dev::O_ARGB) {
+    if (!(t == dev::T_UNORM8 || t == dev::T_SNORM8 || t == dev::T_SINT8 || t == dev::T_UINT8))
+      return CL_IMAGE_FORMAT_NOT_SUPPORTED;
+  }
+  if (o == dev::O_INTENSITY || o == dev::O_LUMINANCE) {
+    if (!(t == dev::T_UNORM8 || t == dev::T_UNORM16 || t == dev::T_SNORM8 ||
+          t == dev::T_SNORM16 || t == dev::T_HALF || t == dev::T_FLOAT))
+      return CL_IMAGE_FORMAT_NOT_SUPPORTED;
+  }
+  out->type = t;
+  out->order = o;
+  out->nch = dev::order_channels(o);
+  out->es = (size_t)out->nch * dev::type_bytes(t);
+  out->rclass = dev::ret_class(t);
+  return CL_SUCCESS;
+}
+
+static int image_dims(cl_mem_object_type t) {
+  switch (t) {
+    case CL_MEM_OBJECT_IMAGE1D: return 1;
+    case CL_MEM_OBJECT_IMAGE2D: return 2;
+    case CL_MEM_OBJECT_IMAGE3D: return 3;
+    default: return 0;
+  }
+}
+
+cl_int image_layout(const cl_image_format* fmt, const cl_image_desc* desc, ImageLayout* L) {
+  FormatInfo fi;
+  cl_int st = format_info(fmt, &fi);
+  if (st != CL_SUCCESS) return st;
+  if (!desc) return CL_INVALID_IMAGE_DESCRIPTOR;
+  const int dims = image_dims(desc->image_type);
+  if (dims == 0) return CL_INVALID_IMAGE_DESCRIPTOR;  // arrays / 1D buffers: NEXT(2)
+  if (desc->num_mip_levels != 0 || desc->num_samples != 0 || desc->buffer != nullptr)
+    return CL_INVALID_IMAGE_DESCRIPTOR;
+  size_t w = desc->image_width, h = dims > 1 ? desc->image_height : 1,
+         d = dims > 2 ? desc->image_depth : 1;
+  if (w == 0 || h == 0 || d == 0) return CL_INVALID_IMAGE_DESCRIPTOR;
+  const size_t maxw = dims == 3 ? kMax3D : kMax2D;
+  if (w > maxw || h > maxw || d > kMax3D) return CL_INVALID_IMAGE_SIZE;
+  L->fmt = fi;
+  L->dims = dims;
+  L->w = w; L->h = h; L->d = d;
+  // internal pitch (reading A21): rows 128-byte aligned -> every texel is
+  // naturally aligned for its vector load, and TMA boxes are legal.
+  L->row_pitch = (w * fi.es + 127) / 128 * 128;
+  L->slice_pitch = L->row_pitch * h;
+  L->bytes = L->slice_pitch * d;
+  return CL_SUCCESS;
+}
+
+// ---- rect copies ----
+static bool rect_pitches(const size_t* region, size_t& rp, size_t& sp) {
+  // pitch 0 -> defaults; a given pitch must be >= the default and the slice
+  // pitch a multiple of the row pitch ([CL1.2 §5.2.2])
+  if (rp == 0) rp = region[0];
+  else if (rp < region[0]) return false;
+  const unsigned __int128 min_sp = (unsigned __int128)region[1] * rp;
+  if (min_sp >> 64) return false;
+  if (sp == 0) sp = (size_t)min_sp;
+  else if (sp < min_sp || sp % rp != 0) return false;
+  return true;
+}
+
+// byte just past the box, or 0 on overflow
+static unsigned __int128 box_end(const size_t* o, const size_t* region, size_t rp, size_t sp) {
+  return (unsigned __int128)o[2] * sp + (unsigned __int128)o[1] * rp + o[0] +
+         (unsigned __int128)(region[2] - 1) * sp + (unsigned __int128)(region[1] - 1) * rp +
+         region[0];
+}
+
+static __int128 floor_div(__int128 a, __int128 b) {  // b > 0
+  __int128 q = a / b;
+  if ((a % b != 0) && (a < 0)) --q;
+  return q;
+}
+static __int128 ceil_div(__int128 a, __int128 b) { return -floor_div(-a, b); }
+
+// Exact test: rows are byte intervals [S + dz_s*sp + dy_s*rp, +R0); two rows
+// meet iff |delta + dz*sp + dy*rp| < R0 with |dz| < R2, |dy| < R1.  For each
+// dz the admissible dy form an interval, so the test is O(R2).
+bool rect_overlap(const size_t* so, const size_t* dso, const size_t* region, size_t rp,
+                  size_t sp) {
+  const __int128 S = (__int128)so[2] * sp + (__int128)so[1] * rp + so[0];
+  const __int128 D = (__int128)dso[2] * sp + (__int128)dso[1] * rp + dso[0];
+  const __int128 R0 = region[0], R1 = region[1], R2 = region[2];
+  const __int128 delta = S - D;
+  for (__int128 dz = -(R2 - 1); dz <= R2 - 1; ++dz) {
+    const __int128 x = delta + dz * (__int128)sp;
+    __int128 lo = floor_div(-R0 - x, (__int128)rp) + 1;
+    __int128 hi = ceil_div(R0 - x, (__int128)rp) - 1;
+    if (lo < -(R1 - 1)) lo = -(R1 - 1);
+    if (hi > R1 - 1) hi = R1 - 1;
+    if (lo <= hi) return true;
+  }
+  return false;
+}
+
+cl_int validate_copy_rect(size_t src_size, size_t dst_size, bool same, const size_t* so,
+                          const size_t* dso, const size_t* region, size_t& srp, size_t& ssp,
+                          size_t& drp, size_t& dsp) {
+  if (!so || !dso || !region) return CL_INVALID_VALUE;
+  if (region[0] == 0 || region[1] == 0 || region[2] == 0) return CL_INVALID_VALUE;
+  if (!rect_pitches(region, srp, ssp) || !rect_pitches(region, drp, dsp)) return CL_INVALID_VALUE;
+  if (box_end(so, region, srp, ssp) > src_size) return CL_INVALID_VALUE;
+  if (box_end(dso, region, drp, dsp) > dst_size) return CL_INVALID_VALUE;
+  if (same) {
+    if (srp != drp || ssp != dsp) return CL_INVALID_VALUE;  // reading A18: either differs
+    if (rect_overlap(so, dso, region, srp, ssp)) return CL_MEM_COPY_OVERLAP;
+  }
+  return CL_SUCCESS;
+}
+
+cl_int validate_host_rect(size_t buf_size, const size_t* bo, const size_t* ho,
+                          const size_t* region, size_t& brp, size_t& bsp, size_t& hrp,
+                          size_t& hsp) {
+  if (!bo || !ho || !region) return CL_INVALID_VALUE;
+  if (region[0] == 0 || region[1] == 0 || region[2] == 0) return CL_INVALID_VALUE;
+  if (!rect_pitches(region, brp, bsp) || !rect_pitches(region, hrp, hsp)) return CL_INVALID_VALUE;
+  if (box_end(bo, region, brp, bsp) > buf_size) return CL_INVALID_VALUE;
+  return CL_SUCCESS;
+}
+
+cl_int validate_fill_buffer(size_t buf_size, size_t ps, size_t offset, size_t size) {
+  if (ps == 0 || ps > 128 || (ps & (ps - 1)) != 0) return CL_INVALID_VALUE;
+  if (offset % ps != 0 || size % ps != 0) return CL_INVALID_VALUE;
+  if (offset > buf_size || size > buf_size - offset) return CL_INVALID_VALUE;
+  return CL_SUCCESS;
+}
+
+cl_int validate_sampler(cl_bool norm, cl_addressing_mode am, cl_filter_mode fm) {
+  if (norm != CL_TRUE && norm != CL_FALSE) return CL_INVALID_VALUE;
+  if (am < CL_ADDRESS_NONE || am > CL_ADDRESS_MIRRORED_REPEAT) return CL_INVALID_VALUE;
+  if (fm != CL_FILTER_NEAREST && fm != CL_FILTER_LINEAR) return CL_INVALID_VALUE;
+  if (!norm && (am == CL_ADDRESS_REPEAT || am == CL_ADDRESS_MIRRORED_REPEAT))
+    return CL_INVALID_VALUE;  // reading A5
+  return CL_SUCCESS;
+}
+
+cl_int validate_image_box(int dims, size_t w, size_t h, size_t d, const size_t* o,
+                          const size_t* r) {
+  if (!o || !r) return CL_INVALID_VALUE;
+  if (r[0] == 0 || r[1] == 0 || r[2] == 0) return CL_INVALID_VALUE;
+  if (dims < 3 && (o[2] != 0 || r[2] != 1)) return CL_INVALID_VALUE;
+  if (dims < 2 && (o[1] != 0 || r[1] != 1)) return CL_INVALID_VALUE;
+  if (o[0] > w || r[0] > w - o[0]) return CL_INVALID_VALUE;
+  if (o[1] > h || r[1] > h - o[1]) return CL_INVALID_VALUE;
+  if (o[2] > d || r[2] > d - o[2]) return CL_INVALID_VALUE;
+  return CL_SUCCESS;
+}
+
+bool image_boxes_overlap(const size_t* a, const size_t* b, const size_t* r) {
+  for (int k = 0; k < 3; ++k)
+    if (!(a[k] < b[k] + r[k] && b[k] < a[k] + r[k])) return false;
+  return true;
+}
+
+}  // namespace b2cl
+
+// ---------------------------------------------------------------- exports
+using namespace b2cl;
+
+extern "C" cl_int b2clValidateCopyBufferRect(size_t src_size, size_t dst_size, cl_int same_buffer,
+                                             const size_t* so, const size_t* dso,
+                                             const size_t* region, size_t srp, size_t ssp,
+                                             size_t drp, size_t dsp) {
+  return validate_copy_rect(src_size, dst_size, same_buffer != 0, so, dso, region, srp, ssp, drp,
+                            dsp);
+}
+
+extern "C" cl_int b2clRectOverlap(const size_t* so, const size_t* dso, const size_t* region,
+                                  size_t rp, size_t sp) {
+  if (!so || !dso || !region || region[0] == 0 || region[1] == 0 || region[2] == 0) return 0;
+  size_t r = rp, s = sp;
+  if (!rect_pitches(region, r, s)) return 0;
+  return rect_overlap(so, dso, region, r, s) ? 1 : 0;
+}
+
+extern "C" cl_int b2clValidateFillBuffer(size_t buffer_size, size_t pattern_size, size_t offset,
+                                         size_t size) {
+  return validate_fill_buffer(buffer_size, pattern_size, offset, size);
+}
+
+extern "C" cl_int b2clValidateSampler(cl_bool normalized_coords, cl_addressing_mode am,
+                                      cl_filter_mode fm) {
+  return validate_sampler(normalized_coords, am, fm);
+}
+
+extern "C" cl_int b2clImageLayout(const cl_image_format* fmt, const cl_image_desc* desc,
+                                  size_t* elem_size, size_t* row_pitch, size_t* slice_pitch,
+                                  size_t* total_bytes) {
+  ImageLayout L;
+  cl_int st = image_layout(fmt, desc, &L);
+  if (st != CL_SUCCESS) return st;
+  if (elem_size) *elem_size = L.fmt.es;
+  if (row_pitch) *row_pitch = L.row_pitch;
+  if (slice_pitch) *slice_pitch = L.slice_pitch;
+  if (total_bytes) *total_bytes = L.bytes;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int b2clValidateImageBox(cl_mem_object_type image_type, size_t width, size_t height,
+                                       size_t depth, const size_t* origin, const size_t* region) {
+  const int dims = image_type == CL_MEM_OBJECT_IMAGE1D   ? 1
+                   : image_type == CL_MEM_OBJECT_IMAGE2D ? 2
+                   : image_type == CL_MEM_OBJECT_IMAGE3D ? 3
+                                                         : 0;
+  if (!dims) return CL_INVALID_MEM_OBJECT;
+  return validate_image_box(dims, width, dims > 1 ? height : 1, dims > 2 ? depth : 1, origin,
+                            region);
+}

@@ -17,3 +17,16 @@ def orc():
     import oracle
     oracle.build()
     return oracle
+
+
+@pytest.fixture(scope="session")
+def sess():
+    """One context + queue on cuda:0 through the C-ABI (GPU tests only)."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    from paper_conf_sc_kimdjjl15_b200 import build, cl
+    build.build()
+    S = cl.Session(0)
+    yield S
+    S.close()

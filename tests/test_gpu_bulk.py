@@ -1,0 +1,287 @@
+"""GPU parity of the bulk runtime operations (steps a9-a16) through the C-ABI
+against the CPU oracle: bit-exact on every byte, including bytes the
+operation must NOT touch."""
+import ctypes
+
+import numpy as np
+import pytest
+
+from paper_conf_sc_kimdjjl15_b200 import cl, synth
+
+pytestmark = pytest.mark.gpu
+
+
+def _rand_bytes(g, n):
+    return g.integers(0, 256, n, dtype=np.uint8)
+
+
+def _copy_rect_gpu(S, src_host, dst_host, so, do, region, srp, ssp, drp, dsp, same=False):
+    sb = S.buffer(src_host.nbytes, src_host)
+    db = sb if same else S.buffer(dst_host.nbytes, dst_host)
+    st = cl.lib().clEnqueueCopyBufferRect(S.queue, sb, db, cl.sz3(so), cl.sz3(do), cl.sz3(region),
+                                          srp, ssp, drp, dsp, 0, None, None)
+    cl.check(st, "clEnqueueCopyBufferRect")
+    out = S.read(db, dst_host.nbytes if not same else src_host.nbytes)
+    S.release(sb)
+    if not same:
+        S.release(db)
+    return out
+
+
+def test_copy_buffer_rect_random_boxes(sess, orc):
+    g = synth.rng(30)
+    for it in range(150):
+        so, do, region, srp, ssp, drp, dsp = synth.random_rect(
+            g, max_region=(int(g.choice([7, 64, 300, 5000])), 9, 3), max_pad=(33, 3, 2))
+        src = _rand_bytes(g, ssp * (so[2] + region[2]) + 17)
+        dst = _rand_bytes(g, dsp * (do[2] + region[2]) + 29)
+        got = _copy_rect_gpu(sess, src, dst, so, do, region, srp, ssp, drp, dsp)
+        exp = dst.copy()
+        orc.copy_rect(src, exp, so, do, region, srp, ssp, drp, dsp)
+        assert np.array_equal(got, exp), (it, so, do, region, srp, ssp, drp, dsp)
+
+
+def test_config1_buffer_rect_all_x_origins(sess, orc):
+    """BASELINE config 1 (reading A19): region {64 B, 16, 4} out of a 64x64x4 RGBA8
+    volume (row pitch 256, slice pitch 16384), every x origin 0..192, also {16 B,16,4}."""
+    g = synth.rng(31)
+    vol = _rand_bytes(g, 256 * 64 * 4)
+    for r0 in (64, 16):
+        for x in range(0, 193):
+            so = (x, int(g.integers(0, 48)), int(g.integers(0, 1)))
+            region = (r0, 16, 4)
+            dst = np.zeros(r0 * 16 * 4 + 64, np.uint8)
+            do = (x % 7, 0, 0)
+            got = _copy_rect_gpu(sess, vol, dst, so, do, region, 256, 16384, r0 + 7, (r0 + 7) * 16)
+            exp = dst.copy()
+            orc.copy_rect(vol, exp, so, do, region, 256, 16384, r0 + 7, (r0 + 7) * 16)
+            assert np.array_equal(got, exp), (r0, x)
+
+
+def test_copy_buffer_rect_same_buffer_disjoint(sess, orc):
+    g = synth.rng(32)
+    buf = _rand_bytes(g, 64 * 8 * 3)
+    so, do, region = (0, 0, 0), (32, 0, 0), (32, 8, 3)
+    got = _copy_rect_gpu(sess, buf, buf, so, do, region, 64, 512, 64, 512, same=True)
+    exp = buf.copy()
+    orc.copy_rect(buf.copy(), exp, so, do, region, 64, 512, 64, 512)
+    assert np.array_equal(got, exp)
+    # overlap is rejected before anything is enqueued
+    sb = sess.buffer(buf.nbytes, buf)
+    st = cl.lib().clEnqueueCopyBufferRect(sess.queue, sb, sb, cl.sz3((0, 0, 0)), cl.sz3((16, 0, 0)),
+                                          cl.sz3(region), 64, 512, 64, 512, 0, None, None)
+    assert st == -8
+    assert np.array_equal(sess.read(sb, buf.nbytes), buf)
+    sess.release(sb)
+
+
+def test_copy_buffer_large_misaligned(sess):
+    g = synth.rng(33)
+    n = (1 << 22) + 13
+    src = _rand_bytes(g, n)
+    sb = sess.buffer(n, src)
+    db = sess.buffer(n + 64, np.zeros(n + 64, np.uint8))
+    for so, do, size in ((0, 0, n), (3, 5, n - 100), (17, 0, n - 17), (1, 33, 1000), (0, 1, 15)):
+        cl.check(cl.lib().clEnqueueCopyBuffer(sess.queue, sb, db, so, do, size, 0, None, None))
+        got = sess.read(db, n + 64)
+        assert np.array_equal(got[do:do + size], src[so:so + size]), (so, do, size)
+    sess.release(sb, db)
+
+
+@pytest.mark.parametrize("p", [1, 2, 4, 8, 16, 32, 64, 128])
+def test_fill_buffer(sess, orc, p):
+    g = synth.rng(34 + p)
+    n = 1 << 16
+    init = _rand_bytes(g, n)
+    pat = _rand_bytes(g, p)
+    b = sess.buffer(n, init)
+    for off, size in ((0, n), (p, 37 * p), (128 * p, 3 * p), (n - 5 * p, 5 * p), (11 * p, 1000 * p)):
+        if off + size > n:
+            continue
+        cl.check(cl.lib().clEnqueueFillBuffer(sess.queue, b, pat.ctypes.data_as(ctypes.c_void_p), p,
+                                              off, size, 0, None, None))
+        orc.fill_buffer(init, pat.tobytes(), off, size)
+        assert np.array_equal(sess.read(b, n), init), (p, off, size)
+    sess.release(b)
+
+
+def test_fill_buffer_on_unaligned_device_pointer(sess, orc):
+    """Pattern phase follows the fill start even when the buffer wraps device memory at
+    an odd address (b2clCreateBufferFromDevicePointer)."""
+    g = synth.rng(35)
+    base = sess.buffer(4096, np.zeros(4096, np.uint8))
+    ptr = ctypes.c_void_p()
+    cl.check(cl.lib().b2clGetMemDevicePointer(base, sess.device, ctypes.byref(ptr)))
+    err = ctypes.c_int32()
+    sub = cl.lib().b2clCreateBufferFromDevicePointer(sess.ctx, sess.device, 1, ptr.value + 8, 2048,
+                                                     ctypes.byref(err))
+    cl.check(err.value)
+    pat = _rand_bytes(g, 64)
+    cl.check(cl.lib().clEnqueueFillBuffer(sess.queue, sub, pat.ctypes.data_as(ctypes.c_void_p), 64,
+                                          64, 1024, 0, None, None))
+    exp = np.zeros(4096, np.uint8)
+    orc.fill_buffer(exp, pat.tobytes(), 8 + 64, 1024)
+    assert np.array_equal(sess.read(base, 4096), exp)
+    sess.release(sub, base)
+
+
+IMG_FORMATS = [(cl.CL_RGBA, cl.CL_UNORM_INT8), (cl.CL_RGBA, cl.CL_FLOAT), (cl.CL_R, cl.CL_HALF_FLOAT),
+               (cl.CL_RG, cl.CL_SIGNED_INT16), (cl.CL_BGRA, cl.CL_UNORM_INT8), (cl.CL_R, cl.CL_UNSIGNED_INT8),
+               (cl.CL_RGBA, cl.CL_UNSIGNED_INT32)]
+
+
+def _img_pair(S, orc, order, type_, W, H, D, dims, seed):
+    g = synth.rng(seed)
+    codes = synth.image_codes(g, order, type_, W, H, D)
+    img = S.image(order, type_, W, H if dims > 1 else 0, D if dims > 2 else 0, host=codes)
+    return img, orc.Image(codes.copy(), W, H, D, dims=dims, order=order, type=type_), codes
+
+
+@pytest.mark.parametrize("order,type_", IMG_FORMATS)
+def test_image_copies_and_fill(sess, orc, order, type_):
+    W, H, D = 37, 11, 5
+    a, oa, _ = _img_pair(sess, orc, order, type_, W, H, D, 3, 40)
+    b, ob, _ = _img_pair(sess, orc, order, type_, W, H, D, 3, 41)
+    c2, oc2, _ = _img_pair(sess, orc, order, type_, 29, 13, 1, 2, 42)
+    es = orc.elem_size(order, type_)
+    L = cl.lib()
+    # CopyImage 3D -> 3D, and 3D -> 2D (region[2] = 1)
+    cl.check(L.clEnqueueCopyImage(sess.queue, a, b, cl.sz3((3, 2, 1)), cl.sz3((5, 0, 2)),
+                                  cl.sz3((20, 9, 3)), 0, None, None))
+    orc.copy_image(oa, ob, (3, 2, 1), (5, 0, 2), (20, 9, 3))
+    cl.check(L.clEnqueueCopyImage(sess.queue, a, c2, cl.sz3((1, 1, 4)), cl.sz3((2, 3, 0)),
+                                  cl.sz3((25, 10, 1)), 0, None, None))
+    orc.copy_image(oa, oc2, (1, 1, 4), (2, 3, 0), (25, 10, 1))
+    # CopyImageToBuffer / CopyBufferToImage with odd offsets
+    nb = 7 + 17 * 6 * 2 * es
+    buf = sess.buffer(nb + 16, np.full(nb + 16, 0xAB, np.uint8))
+    cl.check(L.clEnqueueCopyImageToBuffer(sess.queue, b, buf, cl.sz3((4, 3, 2)), cl.sz3((17, 6, 2)),
+                                          7, 0, None, None))
+    hb = np.full(nb + 16, 0xAB, np.uint8)
+    orc.copy_image_to_buffer(ob, hb, (4, 3, 2), (17, 6, 2), 7)
+    assert np.array_equal(sess.read(buf, nb + 16), hb)
+    cl.check(L.clEnqueueCopyBufferToImage(sess.queue, buf, a, 7, cl.sz3((0, 4, 0)),
+                                          cl.sz3((17, 6, 2)), 0, None, None))
+    orc.copy_buffer_to_image(hb, oa, 7, (0, 4, 0), (17, 6, 2))
+    # FillImage with float4 / int4 / uint4 colour
+    if type_ in (cl.CL_UNSIGNED_INT8, cl.CL_UNSIGNED_INT32):
+        col, rt = np.array([7, 300, 70000, 1], np.uint32), orc.RT_UI
+    elif type_ == cl.CL_SIGNED_INT16:
+        col, rt = np.array([-7, 40000, -40000, 1], np.int32), orc.RT_I
+    else:
+        col, rt = np.array([0.25, 1.5, -0.5, 0.7071], np.float32), orc.RT_F
+    cl.check(L.clEnqueueFillImage(sess.queue, c2, col.ctypes.data_as(ctypes.c_void_p),
+                                  cl.sz3((3, 2, 0)), cl.sz3((20, 7, 1)), 0, None, None))
+    orc.fill_image(oc2, rt, col, (3, 2, 0), (20, 7, 1))
+    for img, oimg, (w, h, d) in ((a, oa, (W, H, D)), (b, ob, (W, H, D)), (c2, oc2, (29, 13, 1))):
+        got = sess.read_image(img, (0, 0, 0), (w, h, d))
+        assert np.array_equal(got, oimg.data[:got.size]), (hex(order), hex(type_))
+    sess.release(a, b, c2, buf)
+
+
+def test_read_write_image_host_pitches(sess, orc):
+    g = synth.rng(43)
+    W, H, D = 19, 7, 4
+    img, oimg, _ = _img_pair(sess, orc, cl.CL_RGBA, cl.CL_UNORM_INT16, W, H, D, 3, 43)
+    rp, sp = 8 * 12 + 5, (8 * 12 + 5) * 5 + 3
+    host = _rand_bytes(g, sp * 3)
+    L = cl.lib()
+    cl.check(L.clEnqueueWriteImage(sess.queue, img, 1, cl.sz3((4, 1, 1)), cl.sz3((12, 5, 3)), rp, sp,
+                                   host.ctypes.data_as(ctypes.c_void_p), 0, None, None))
+    orc.write_image_rect(oimg, (4, 1, 1), (12, 5, 3), rp, sp, host)
+    rp2, sp2 = 15 * 8 + 9, (15 * 8 + 9) * 6 + 11
+    out = np.zeros(sp2 * 3, np.uint8)
+    exp = np.zeros(sp2 * 3, np.uint8)
+    cl.check(L.clEnqueueReadImage(sess.queue, img, 1, cl.sz3((2, 0, 0)), cl.sz3((15, 6, 3)), rp2,
+                                  sp2, out.ctypes.data_as(ctypes.c_void_p), 0, None, None))
+    orc.read_image_rect(oimg, (2, 0, 0), (15, 6, 3), rp2, sp2, exp)
+    assert np.array_equal(out, exp)
+    sess.release(img)
+
+
+def test_read_write_buffer_rect(sess, orc):
+    g = synth.rng(44)
+    n = 64 * 10 * 4
+    dev_init = _rand_bytes(g, n)
+    b = sess.buffer(n, dev_init)
+    host = _rand_bytes(g, 50 * 12 * 3)
+    L = cl.lib()
+    cl.check(L.clEnqueueWriteBufferRect(sess.queue, b, 1, cl.sz3((3, 1, 1)), cl.sz3((5, 2, 0)),
+                                        cl.sz3((31, 7, 2)), 64, 640, 50, 600,
+                                        host.ctypes.data_as(ctypes.c_void_p), 0, None, None))
+    orc.copy_rect(host, dev_init, (5, 2, 0), (3, 1, 1), (31, 7, 2), 50, 600, 64, 640)
+    out = np.zeros(n, np.uint8)
+    cl.check(L.clEnqueueReadBufferRect(sess.queue, b, 1, cl.sz3((0, 0, 0)), cl.sz3((0, 0, 0)),
+                                       cl.sz3((64, 10, 4)), 64, 640, 64, 640,
+                                       out.ctypes.data_as(ctypes.c_void_p), 0, None, None))
+    assert np.array_equal(out, dev_init)
+    sess.release(b)
+
+
+def test_migrate_same_device_listed_twice(orc):
+    """A context with cuda:0 listed twice (two queues, one GPU): migration and
+    cross-queue events keep the data equal (reading A24 / O9)."""
+    S = cl.Session(0, devices=[0, 0])
+    q2 = S.queue_for(0)
+    g = synth.rng(45)
+    data = _rand_bytes(g, 1 << 20)
+    b = S.buffer(data.nbytes, data)
+    ev = ctypes.c_void_p()
+    L = cl.lib()
+    mems = (ctypes.c_void_p * 1)(b)
+    cl.check(L.clEnqueueMigrateMemObjects(q2, 1, mems, 0, 0, None, ctypes.byref(ev)))
+    out = np.zeros_like(data)
+    evs = (ctypes.c_void_p * 1)(ev)
+    cl.check(L.clEnqueueReadBuffer(S.queue, b, 1, 0, data.nbytes, out.ctypes.data_as(ctypes.c_void_p),
+                                   1, evs, None))
+    assert np.array_equal(out, data)
+    L.clReleaseEvent(ev)
+    L.clReleaseCommandQueue(q2)
+    S.release(b)
+    S.close()
+
+
+def test_events_profiling_and_launch_count(orc):
+    S = cl.Session(0, profiling=True)
+    b = S.buffer(1 << 24)
+    pat = np.array([1, 2, 3, 4], np.uint8)
+    ev = ctypes.c_void_p()
+    L = cl.lib()
+    before = cl.launch_count()
+    cl.check(L.clEnqueueFillBuffer(S.queue, b, pat.ctypes.data_as(ctypes.c_void_p), 4, 0, 1 << 24, 0,
+                                   None, ctypes.byref(ev)))
+    evs = (ctypes.c_void_p * 1)(ev)
+    cl.check(L.clWaitForEvents(1, evs))
+    assert cl.launch_count() == before + 1
+    t0, t1 = ctypes.c_uint64(), ctypes.c_uint64()
+    cl.check(L.clGetEventProfilingInfo(ev, cl.CL_PROFILING_COMMAND_START, 8, ctypes.byref(t0), None))
+    cl.check(L.clGetEventProfilingInfo(ev, cl.CL_PROFILING_COMMAND_END, 8, ctypes.byref(t1), None))
+    assert t1.value >= t0.value
+    st = ctypes.c_int32()
+    cl.check(L.clGetEventInfo(ev, 0x11D3, 4, ctypes.byref(st), None))
+    assert st.value == 0
+    L.clReleaseEvent(ev)
+    S.release(b)
+    S.close()
+
+
+def test_validation_has_no_side_effects(sess):
+    g = synth.rng(46)
+    data = _rand_bytes(g, 4096)
+    b = sess.buffer(4096, data)
+    L = cl.lib()
+    pat = np.zeros(3, np.uint8)
+    assert L.clEnqueueFillBuffer(sess.queue, b, pat.ctypes.data_as(ctypes.c_void_p), 3, 0, 9, 0, None,
+                                 None) == -30
+    assert L.clEnqueueCopyBufferRect(sess.queue, b, b, cl.sz3((0, 0, 0)), cl.sz3((0, 0, 0)),
+                                     cl.sz3((4096, 2, 1)), 0, 0, 0, 0, 0, None, None) == -30
+    img = sess.image(cl.CL_RGBA, cl.CL_FLOAT, 8, 8)
+    smp = sess.sampler(False, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_LINEAR)
+    assert L.b2clEnqueueReadImageSamples(sess.queue, img, smp, cl.B2CL_RTYPE_UINT, 0, b, 0, 1, b, 0,
+                                         0, None, None) == -59                     # A7
+    uimg = sess.image(cl.CL_RGBA, cl.CL_UNSIGNED_INT8, 8, 8)
+    assert L.b2clEnqueueReadImageSamples(sess.queue, uimg, smp, cl.B2CL_RTYPE_UINT, 0, b, 0, 1, b, 0,
+                                         0, None, None) == -59                     # A6
+    assert np.array_equal(sess.read(b, 4096), data)
+    sess.release(b, img, uimg)
+    cl.lib().clReleaseSampler(smp)

@@ -1,0 +1,279 @@
+"""GPU parity of the read_image / write_image path (steps a1-a8) through the C-ABI
+against the CPU oracle, on the same seeded inputs.
+
+Bar (BASELINE.json north_star): NEAREST, integer formats and writes bit-exact;
+LINEAR within 4 fp32 ulp or 1e-6 absolute, NaN iff NaN.
+"""
+import numpy as np
+import pytest
+
+from paper_conf_sc_kimdjjl15_b200 import cl, synth
+from tests.gpu_helpers import (VALID_SAMPLERS, assert_parity, coord_stride, gpu_read_grid,
+                               gpu_read_samples, make_images, rtype_of)
+
+pytestmark = pytest.mark.gpu
+
+R, RG, RA, A_, RGBA, BGRA, ARGB, INT_, LUM = (cl.CL_R, cl.CL_RG, cl.CL_RA, cl.CL_A, cl.CL_RGBA,
+                                              cl.CL_BGRA, cl.CL_ARGB, cl.CL_INTENSITY,
+                                              cl.CL_LUMINANCE)
+F32, F16, U8N, U16N, S8N, S16N = (cl.CL_FLOAT, cl.CL_HALF_FLOAT, cl.CL_UNORM_INT8,
+                                  cl.CL_UNORM_INT16, cl.CL_SNORM_INT8, cl.CL_SNORM_INT16)
+
+FLOAT_FORMATS = [(RGBA, F32), (R, F32), (RGBA, U8N), (BGRA, U8N), (RG, F16), (RGBA, U16N),
+                 (R, S8N), (RA, S16N), (A_, U8N), (INT_, U8N), (LUM, F32), (ARGB, U8N),
+                 (RGBA, F16), (RG, U8N)]
+INT_FORMATS = [(RGBA, cl.CL_UNSIGNED_INT8), (R, cl.CL_SIGNED_INT16), (RG, cl.CL_UNSIGNED_INT32),
+               (RGBA, cl.CL_SIGNED_INT32), (BGRA, cl.CL_SIGNED_INT8), (RA, cl.CL_UNSIGNED_INT16)]
+SHAPES = [(1, (37, 1, 1)), (2, (1, 1, 1)), (2, (3, 5, 1)), (2, (65, 33, 1)), (3, (7, 3, 2)),
+          (3, (9, 6, 5))]
+
+
+def _coords(g, dims, size, norm, n_rand=3000):
+    W, H, D = size
+    ns = np.array([W, H, D][:dims], np.float32)
+    sp = synth.special_floats()
+    lat = synth.coord_lattice(-2, 3, 1 / 32) if norm else synth.coord_lattice(-2, max(W, H, D) + 2, 1 / 16)
+    lo, hi = (-1.5, 2.5) if norm else (-2.0, 1.0)
+    if norm:
+        rnd = g.uniform(lo, hi, (n_rand, dims)).astype(np.float32)
+    else:
+        rnd = (g.uniform(-0.2, 1.2, (n_rand, dims)) * ns).astype(np.float32)
+    pts = [rnd]
+    for d in range(dims):
+        for vals in (lat, sp):
+            c = rnd[:vals.size].copy() if vals.size <= n_rand else np.resize(rnd, (vals.size, dims))
+            c[:, d] = vals
+            pts.append(c)
+    c = np.concatenate(pts).astype(np.float32)
+    if dims == 3:
+        c = np.concatenate([c, np.zeros((c.shape[0], 1), np.float32)], 1)
+    return np.ascontiguousarray(c)
+
+
+@pytest.mark.parametrize("order,type_", FLOAT_FORMATS)
+@pytest.mark.parametrize("dims,size", SHAPES)
+def test_read_imagef_all_samplers(sess, orc, order, type_, dims, size):
+    W, H, D = size
+    signed = type_ in (F32, F16)
+    img, oimg, _ = make_images(sess, orc, order, type_, W, H, D, dims, seed=W * 7 + H + D,
+                               signed=signed)
+    g = synth.rng(77 + W + H + D)
+    try:
+        for norm, addr, filt in VALID_SAMPLERS:
+            smp = sess.sampler(norm, addr, filt)
+            co = _coords(g, dims, size, norm)
+            got = gpu_read_samples(sess, img, smp, cl.B2CL_RTYPE_FLOAT, co)
+            exp = orc.read_samples(oimg, norm, addr, filt, orc.RT_F, co)
+            assert_parity(got, exp, filt == cl.CL_FILTER_LINEAR,
+                          f"fmt {hex(order)}/{hex(type_)} dims {dims} smp {norm},{hex(addr)},{hex(filt)}")
+            cl.lib().clReleaseSampler(smp)
+    finally:
+        sess.release(img)
+
+
+@pytest.mark.parametrize("order,type_", INT_FORMATS)
+@pytest.mark.parametrize("dims,size", [(1, (19, 1, 1)), (2, (13, 7, 1)), (3, (5, 4, 3))])
+def test_read_imagei_ui_nearest(sess, orc, order, type_, dims, size):
+    W, H, D = size
+    img, oimg, _ = make_images(sess, orc, order, type_, W, H, D, dims, seed=3 * W + H)
+    g = synth.rng(99)
+    rt = rtype_of(type_)
+    try:
+        for norm, addr, filt in VALID_SAMPLERS:
+            if filt != cl.CL_FILTER_NEAREST:
+                continue
+            smp = sess.sampler(norm, addr, filt)
+            co = _coords(g, dims, size, norm, 1500)
+            got = gpu_read_samples(sess, img, smp, rt, co)
+            exp = orc.read_samples(oimg, norm, addr, filt, rt, co)
+            assert_parity(got, exp, False, f"int fmt {hex(order)}/{hex(type_)} {norm},{hex(addr)}")
+            cl.lib().clReleaseSampler(smp)
+    finally:
+        sess.release(img)
+
+
+@pytest.mark.parametrize("dims", [1, 2, 3])
+def test_integer_coordinates(sess, orc, dims):
+    size = (11, 6, 4)
+    W, H, D = size
+    img, oimg, _ = make_images(sess, orc, RGBA, U8N, W, H, D, dims, seed=5)
+    g = synth.rng(5)
+    ic = g.integers(-3, 14, (2000, coord_stride(dims))).astype(np.int32)
+    ic[:5, 0] = [-2 ** 31, 2 ** 31 - 1, 0, -1, W]
+    for addr in (cl.CL_ADDRESS_NONE, cl.CL_ADDRESS_CLAMP, cl.CL_ADDRESS_CLAMP_TO_EDGE):
+        smp = sess.sampler(False, addr, cl.CL_FILTER_NEAREST)
+        got = gpu_read_samples(sess, img, smp, cl.B2CL_RTYPE_FLOAT, ic, int_coords=True)
+        exp = orc.read_samples(oimg, False, addr, cl.CL_FILTER_NEAREST, orc.RT_F, ic)
+        assert_parity(got, exp, False, f"icoord {hex(addr)}")
+    sess.release(img)
+
+
+def test_unorm_codes_exhaustive(sess, orc):
+    """Every UNORM/SNORM 8/16 code through read_imagef equals IEEE c/d (A11)."""
+    for type_, n in ((U8N, 256), (S8N, 256), (U16N, 65536), (S16N, 65536)):
+        codes = np.arange(n, dtype=np.uint32).astype(np.uint8 if n == 256 else np.uint16)
+        if type_ in (S8N, S16N):
+            codes = codes.view(np.int8 if n == 256 else np.int16)
+        W = 256
+        Hh = n // W
+        img = sess.image(R, type_, W, Hh, host=codes.reshape(Hh, W, 1))
+        oimg = orc.Image(codes.reshape(1, Hh, W, 1).copy(), W, Hh, 1, dims=2, order=R, type=type_)
+        smp = sess.sampler(False, cl.CL_ADDRESS_NONE, cl.CL_FILTER_NEAREST)
+        xs, ys = np.meshgrid(np.arange(W) + 0.5, np.arange(Hh) + 0.5)
+        co = np.stack([xs.ravel(), ys.ravel()], 1).astype(np.float32)
+        got = gpu_read_samples(sess, img, smp, cl.B2CL_RTYPE_FLOAT, co)
+        exp = orc.read_samples(oimg, False, cl.CL_ADDRESS_NONE, cl.CL_FILTER_NEAREST, orc.RT_F, co)
+        assert_parity(got, exp, False, f"codes {hex(type_)}")
+        sess.release(img)
+
+
+# ---------------------------------------------------------------- grid mode
+GRID_CASES = [
+    # (dims, order, type, img size, sampler, affine-maker, out dims, outc)
+    (2, RGBA, F32, (97, 61, 1), (1, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR), "translate", (97, 61, 1), 4),
+    (2, RGBA, F32, (97, 61, 1), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "translate", (97, 61, 1), 4),
+    (2, RGBA, F32, (64, 48, 1), (1, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR), "rotate", (70, 50, 1), 4),
+    (2, RGBA, F32, (64, 48, 1), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "rotate", (70, 50, 1), 4),
+    (3, R, F32, (40, 33, 17), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "stencil", (40, 33, 17), 1),
+    (2, RGBA, U8N, (64, 64, 1), (0, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_NEAREST), "unnorm", (96, 96, 1), 4),
+    (2, BGRA, U8N, (31, 17, 1), (1, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_LINEAR), "rotate", (45, 29, 1), 3),
+    (1, RG, F16, (50, 1, 1), (1, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR), "translate", (77, 1, 1), 2),
+    (3, RGBA, U16N, (9, 8, 7), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "stencil", (12, 11, 10), 4),
+]
+
+
+def _affine(kind, size, out):
+    W, H, D = size
+    if kind == "translate":
+        return synth.affine_translate_2d(W, H)
+    if kind == "rotate":
+        return synth.affine_rotate_2d(W, H, 30.0)
+    if kind == "stencil":
+        A = synth.affine_stencil_3d(W)
+        A[5] = 1.0 / H
+        A[7] = (0.5 + 0.6) / H
+        A[10] = 1.0 / D
+        A[11] = (0.5 + 0.2) / D
+        return A
+    return synth.affine_unnorm_2d(1 / 16 * 12, -2.0)
+
+
+@pytest.mark.parametrize("case", GRID_CASES)
+def test_grid_mode(sess, orc, case):
+    dims, order, type_, size, (norm, addr, filt), kind, out, outc = case
+    W, H, D = size
+    img, oimg, _ = make_images(sess, orc, order, type_, W, H, D, dims, seed=sum(size))
+    smp = sess.sampler(norm, addr, filt)
+    A = _affine(kind, size, out)
+    got = gpu_read_grid(sess, img, smp, cl.B2CL_RTYPE_FLOAT, A, out, outc)
+    exp = orc.read_grid(oimg, norm, addr, filt, orc.RT_F, A, out, outc)
+    assert_parity(got, exp, filt == cl.CL_FILTER_LINEAR, f"grid {case}")
+    sess.release(img)
+
+
+def test_config1_full_bruteforce(sess, orc):
+    """BASELINE config 1: 64x64 RGBA8, unnormalized, CLAMP + NEAREST, every
+    coordinate of a 1/16 lattice over [-2, 66)^2 (1088^2 samples), bit-exact."""
+    img, oimg, _ = make_images(sess, orc, RGBA, U8N, 64, 64, 1, 2, seed=1)
+    smp = sess.sampler(False, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_NEAREST)
+    A = synth.affine_unnorm_2d(1 / 16, -2.0)
+    out = (1088, 1088, 1)
+    got = gpu_read_grid(sess, img, smp, cl.B2CL_RTYPE_FLOAT, A, out, 4)
+    exp = orc.read_grid(oimg, False, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_NEAREST, orc.RT_F, A, out, 4,
+                        nthreads=8)
+    assert_parity(got, exp, False, "config1")
+    # and the same through the coordinate-list entry point
+    xs = (np.arange(1088) / 16 - 2).astype(np.float32)
+    co = np.stack(np.meshgrid(xs, xs), -1).reshape(-1, 2)
+    got2 = gpu_read_samples(sess, img, smp, cl.B2CL_RTYPE_FLOAT, co)
+    assert_parity(got2, exp.reshape(-1, 4), False, "config1 list")
+    sess.release(img)
+
+
+@pytest.mark.parametrize("addr", [cl.CL_ADDRESS_REPEAT, cl.CL_ADDRESS_MIRRORED_REPEAT])
+@pytest.mark.parametrize("kind", ["translate", "rotate"])
+def test_config2_full_size_sampled_rows(sess, orc, addr, kind):
+    """BASELINE config 2 at full size (4096^2 RGBA32F, normalized, LINEAR), in the
+    launch configuration bench.py times; rows sampled: all seam / edge rows and
+    every 97th row, all columns, against the oracle."""
+    N = 4096
+    img, oimg, _ = make_images(sess, orc, RGBA, F32, N, N, 1, 2, seed=2)
+    smp = sess.sampler(True, addr, cl.CL_FILTER_LINEAR)
+    A = synth.affine_translate_2d(N, N) if kind == "translate" else synth.affine_rotate_2d(N, N, 30.0)
+    got = gpu_read_grid(sess, img, smp, cl.B2CL_RTYPE_FLOAT, A, (N, N, 1), 4)
+    rows = sorted(set([0, 1, N // 2 - 1, N // 2, N // 2 + 1, N - 2, N - 1] + list(range(5, N, 97))))
+    for y in rows:
+        exp = orc.read_grid(oimg, True, addr, cl.CL_FILTER_LINEAR, orc.RT_F, A, (N, N, 1), 4,
+                            yrange=(y, y + 1))
+        assert_parity(got[0, y:y + 1], exp[0], True, f"config2 row {y}")
+    sess.release(img)
+
+
+def test_config3_full_size_sampled_slices(sess, orc):
+    """BASELINE config 3 at full size (512^3 R32F, trilinear, stencil map, CLAMP_TO_EDGE):
+    sampled rows of first / middle / last slices against the oracle."""
+    N = 512
+    img, oimg, _ = make_images(sess, orc, R, F32, N, N, N, 3, seed=3)
+    smp = sess.sampler(True, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR)
+    A = synth.affine_stencil_3d(N)
+    got = gpu_read_grid(sess, img, smp, cl.B2CL_RTYPE_FLOAT, A, (N, N, N), 1)
+    for z in (0, 1, 255, 510, 511):
+        for y in (0, 1, 100, 256, 511):
+            exp = orc.read_grid(oimg, True, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR,
+                                orc.RT_F, A, (N, N, N), 1, zrange=(z, z + 1), yrange=(y, y + 1))
+            assert_parity(got[z:z + 1, y:y + 1], exp, True, f"config3 z{z} y{y}")
+    # property at any size: the trilinear read of a [0,1) volume stays in [0,1]
+    assert np.all((got >= 0) & (got <= 1))
+    sess.release(img)
+
+
+# ---------------------------------------------------------------- write_image
+WRITE_FORMATS = [(RGBA, U8N, cl.B2CL_RTYPE_FLOAT), (BGRA, U8N, cl.B2CL_RTYPE_FLOAT),
+                 (RGBA, S8N, cl.B2CL_RTYPE_FLOAT), (RG, U16N, cl.B2CL_RTYPE_FLOAT),
+                 (R, S16N, cl.B2CL_RTYPE_FLOAT), (RGBA, F16, cl.B2CL_RTYPE_FLOAT),
+                 (RGBA, F32, cl.B2CL_RTYPE_FLOAT), (A_, U8N, cl.B2CL_RTYPE_FLOAT),
+                 (ARGB, U8N, cl.B2CL_RTYPE_FLOAT), (RA, F16, cl.B2CL_RTYPE_FLOAT),
+                 (INT_, F32, cl.B2CL_RTYPE_FLOAT), (LUM, U8N, cl.B2CL_RTYPE_FLOAT),
+                 (RGBA, cl.CL_SIGNED_INT8, cl.B2CL_RTYPE_INT), (RG, cl.CL_SIGNED_INT16, cl.B2CL_RTYPE_INT),
+                 (R, cl.CL_SIGNED_INT32, cl.B2CL_RTYPE_INT), (RGBA, cl.CL_UNSIGNED_INT8, cl.B2CL_RTYPE_UINT),
+                 (RA, cl.CL_UNSIGNED_INT16, cl.B2CL_RTYPE_UINT), (R, cl.CL_UNSIGNED_INT32, cl.B2CL_RTYPE_UINT)]
+
+
+@pytest.mark.parametrize("order,type_,rt", WRITE_FORMATS)
+@pytest.mark.parametrize("dims", [1, 2, 3])
+def test_write_image(sess, orc, order, type_, rt, dims):
+    W, H, D = 23, (9 if dims > 1 else 1), (4 if dims > 2 else 1)
+    img, oimg, codes = make_images(sess, orc, order, type_, W, H, D, dims, seed=11)
+    g = synth.rng(12)
+    n = W * H * D
+    # unique in-range coordinates (a permutation) plus out-of-range no-ops
+    perm = g.permutation(n)
+    ic = np.zeros((n + 40, {1: 1, 2: 2, 3: 4}[dims]), np.int32)
+    ic[:n, 0] = perm % W
+    if dims > 1:
+        ic[:n, 1] = (perm // W) % H
+    if dims > 2:
+        ic[:n, 2] = perm // (W * H)
+    ic[n:, 0] = g.integers(-5, 0, 40)
+    if rt == cl.B2CL_RTYPE_FLOAT:
+        col = g.uniform(-1.5, 1.5, (n + 40, 4)).astype(np.float32)
+        col[:8] = [[np.nan, 0.5, 1 / 510, 3 / 510], [2.0, -0.3, 65520.0, 6e-8], [1.0, 0.0, -0.0, 1e-40],
+                   [np.inf, -np.inf, 0.49999997, 254.5 / 255], [0.5, 0.25, 0.125, 0.0625],
+                   [-1.0, -0.999, 1.0001, 100.0], [1.5 / 255, 2.5 / 255, 1e-5, 0.9999],
+                   [65504.0, 65519.0, -65520.0, 2 ** -24]]
+        if type_ == F16:  # half NaN payloads are unspecified (reading A13): compared separately
+            col[0, 0] = 0.5
+    else:
+        col = g.integers(-2 ** 31, 2 ** 31, (n + 40, 4), dtype=np.int64).astype(np.int32)
+        col[:4] = [[300, -300, 127, -128], [70000, -70000, 32767, -32768], [255, 256, 65535, 65536],
+                   [-1, 0, 1, 2 ** 31 - 1]]
+        if rt == cl.B2CL_RTYPE_UINT:
+            col = col.view(np.uint32)
+    cbuf = sess.buffer(ic.nbytes, ic)
+    kbuf = sess.buffer(col.nbytes, col)
+    cl.check(cl.lib().b2clEnqueueWriteImageSamples(sess.queue, img, rt, cbuf, 0, ic.shape[0], kbuf, 0,
+                                                   0, None, None))
+    orc.write_samples(oimg, rt, ic, col)
+    got = sess.read_image(img, (0, 0, 0), (W, H, D))
+    assert np.array_equal(got, oimg.data[:got.size]), f"write {hex(order)}/{hex(type_)}"
+    sess.release(img, cbuf, kbuf)
