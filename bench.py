@@ -59,52 +59,87 @@ def peaks():
 
 # ------------------------------------------------------------------ clocks
 class Clocks:
-    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
-              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-              "clocks_event_reasons.sw_power_cap")
+    """SM clock + throttle reasons sampled DURING the timed region: an NVML
+    polling thread (5 ms) when pynvml finds the driver library, else
+    `nvidia-smi -lms 100` in the background."""
+
+    REASONS = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
+               "sw_power_cap": 0x4, "hw_power_brake_slowdown": 0x80}
 
     def __init__(self, index: int):
         self.index = index
-        self.proc = None
-        self.file = None
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self.thread = self.proc = None
+        self._stop = False
 
     def start(self):
         try:
+            import threading
+
+            import pynvml
+            pynvml.nvmlInit()
+            h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+
+            def poll():
+                while not self._stop:
+                    self.samples.append(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM))
+                    r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+                    for n, bit in self.REASONS.items():
+                        if r & bit:
+                            self.reasons.add(n)
+                    time.sleep(0.005)
+            self.thread = threading.Thread(target=poll, daemon=True)
+            self.thread.start()
+            time.sleep(0.01)
+            return
+        except Exception:
+            self.thread = None
+        try:
             self.file = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
             self.proc = subprocess.Popen(
-                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,"
+                 "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
                  "--format=csv,noheader,nounits", "-lms", "100"],
                 stdout=self.file, stderr=subprocess.DEVNULL)
         except (OSError, FileNotFoundError):
             self.proc = None
 
     def stop(self):
-        if not self.proc:
-            return None
-        time.sleep(0.15)
-        self.proc.terminate()
-        try:
-            self.proc.wait(timeout=5)
-        except subprocess.TimeoutExpired:
-            self.proc.kill()
-        self.file.flush()
-        rows = [ln.split(",") for ln in open(self.file.name).read().strip().splitlines() if ln.strip()]
-        os.unlink(self.file.name)
-        sm, mx, reasons = [], [], set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for r in rows:
+        if self.thread is not None:
+            self._stop = True
+            self.thread.join(timeout=2)
+            sm = self.samples
+            src = "nvml 5 ms"
+        elif self.proc is not None:
+            time.sleep(0.15)
+            self.proc.terminate()
             try:
-                sm.append(float(r[0]))
-                mx.append(float(r[1]))
-            except (ValueError, IndexError):
-                continue
-            for n, v in zip(names, r[2:6]):
-                if v.strip() == "Active":
-                    reasons.add(n)
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+            self.file.flush()
+            rows = [ln.split(",") for ln in open(self.file.name).read().splitlines() if ln.strip()]
+            os.unlink(self.file.name)
+            sm = []
+            names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+            for r in rows:
+                try:
+                    sm.append(float(r[0]))
+                    self.max_mhz = float(r[1])
+                except (ValueError, IndexError):
+                    continue
+                for n, v in zip(names, r[2:6]):
+                    if v.strip() == "Active":
+                        self.reasons.add(n)
+            src = "nvidia-smi 100 ms"
+        else:
+            return None
         if not sm:
             return None
-        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": max(mx), "samples": len(sm),
-                "reasons": sorted(reasons)}
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": self.max_mhz, "samples": len(sm),
+                "reasons": sorted(self.reasons), "source": src}
 
 
 # ------------------------------------------------------------------ oracle (CPU) timing
@@ -119,13 +154,46 @@ def oracle_rate(codes, n_rows_target_s: float, threads: int):
                                         (N2D, N2D, 1), 4, yrange=(r0, r1), nthreads=threads)
                           for a in (orc.ADDRESS_REPEAT, orc.ADDRESS_MIRRORED_REPEAT)]
     t0 = time.perf_counter()
-    run(0, 4)
+    run(0, 16)
     dt = time.perf_counter() - t0
-    rows = int(max(4, min(N2D, 4 * n_rows_target_s / max(dt, 1e-6))))
+    rows = int(max(16, 16 * n_rows_target_s / max(dt, 1e-6)))  # may exceed one full pass
     t0 = time.perf_counter()
-    run(0, rows)
+    done = 0
+    while done < rows:
+        r = min(N2D, rows - done)
+        run(0, r)
+        done += r
     dt = time.perf_counter() - t0
     return 2 * rows * N2D / dt / 1e9, rows, dt
+
+
+def _axis_taps(coef, offset, n_out, n, mode):
+    """Set of texel indices along one axis that a LINEAR read of a separable
+    affine map touches with a non-zero weight ([CL1.2 §8.2] in numpy float32;
+    measurement bookkeeping only -- the bytes a launch must move)."""
+    f32 = np.float32
+    x = np.arange(n_out, dtype=np.float32)
+    s = (f32(coef) * x).astype(f32) + f32(offset)
+    fn = f32(n)
+    if mode == "repeat":
+        u = ((s - np.floor(s)).astype(f32) * fn).astype(f32)
+    else:
+        sp = (f32(2.0) * np.rint((f32(0.5) * s).astype(f32))).astype(f32)
+        u = (np.abs((s - sp).astype(f32)) * fn).astype(f32)
+    t = (u - f32(0.5)).astype(f32)
+    b = np.floor(t).astype(np.int64)
+    a = (t - np.floor(t)).astype(f32)
+    if mode == "repeat":
+        i0, i1 = np.where(b < 0, b + n, b), np.where(b + 1 > n - 1, b + 1 - n, b + 1)
+    else:
+        i0, i1 = np.maximum(b, 0), np.minimum(b + 1, n - 1)
+    return np.unique(np.concatenate([i0[a != 1], i1[a != 0]]))
+
+
+def distinct_texels_separable(A, w_out, h_out, mode):
+    assert A[1] == 0 and A[4] == 0, "separable map expected"
+    return (_axis_taps(A[0], A[3], w_out, N2D, mode).size *
+            _axis_taps(A[5], A[7], h_out, N2D, mode).size)
 
 
 def c2_codes():
@@ -140,7 +208,7 @@ def run_reference(args):
         return 0
     threads = os.cpu_count() or 1
     codes = c2_codes()
-    total_budget = 90.0
+    total_budget = 60.0
     per_step = total_budget / max(1, args.steps + args.warmup)
     rate, rows, _ = oracle_rate(codes, per_step, threads)  # calibrates rows per step
     import oracle as orc
@@ -149,10 +217,14 @@ def run_reference(args):
     A = synth.affine_translate_2d(N2D, N2D)
 
     def step(i):
-        y0 = (i * rows) % (N2D - rows + 1)
-        for a in (orc.ADDRESS_REPEAT, orc.ADDRESS_MIRRORED_REPEAT):
-            orc.read_grid(img, True, a, orc.FILTER_LINEAR, orc.RT_F, A, (N2D, N2D, 1), 4,
-                          yrange=(y0, y0 + rows), nthreads=threads)
+        done = 0
+        while done < rows:
+            r = min(N2D, rows - done)
+            y0 = (i * 977 + done) % (N2D - r + 1)
+            for a in (orc.ADDRESS_REPEAT, orc.ADDRESS_MIRRORED_REPEAT):
+                orc.read_grid(img, True, a, orc.FILTER_LINEAR, orc.RT_F, A, (N2D, N2D, 1), 4,
+                              yrange=(y0, y0 + r), nthreads=threads)
+            done += r
     for i in range(args.warmup):
         step(i)
     t0 = time.perf_counter()
@@ -269,7 +341,8 @@ def run_gpu(args):
     gpu_launches = cl.launch_count() - n_launch0
     clk = clocks.stop()
     total_ms = t_start.elapsed_time(t_end)
-    kern_ms = [a.elapsed_time(b) for e in evs for a, b in ((e[0], e[1]), (e[1], e[2]))]
+    pass_ms = [float(np.mean([e[0].elapsed_time(e[1]) for e in evs])),
+               float(np.mean([e[1].elapsed_time(e[2]) for e in evs]))]
     ms_step = total_ms / args.steps
     if world > 1:
         t = torch.tensor([ms_step], device=dev)
@@ -277,13 +350,18 @@ def run_gpu(args):
         ms_step = float(t.item())
     samples_step = 2 * N2D * N2D
     value = world * samples_step / (ms_step * 1e-3) / 1e9
-    k_ms = float(np.mean(kern_ms))
-    alg_bytes = N2D * N2D * 16 * 2  # every texel once (unit-scale translate covers the torus) + output
-    achieved = alg_bytes / (k_ms * 1e-3) / 1e9
+    # algorithmic bytes per launch = distinct texels with a non-zero tap weight x 16 B
+    # + 16 B output per sample; counted exactly per map on the host
+    Af = synth.affine_translate_2d(N2D, N2D)
+    alg = [distinct_texels_separable(Af, N2D, N2D, m) * 16 + N2D * N2D * 16
+           for m in ("repeat", "mirrored")]
+    achieved = [alg[k] / (pass_ms[k] * 1e-3) / 1e9 for k in range(2)]
+    dom = 0 if pass_ms[0] * 1.0 >= pass_ms[1] else 1  # the kernel with the larger share of the step
     traffic = None
-    prof = os.path.join(ROOT, "profiles", "ncu_c2_traffic.json")
-    if os.path.exists(prof):
-        traffic = json.load(open(prof)).get("dram_bytes_per_launch")
+    import glob
+    profs = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*", "ncu_c2_traffic.json")))
+    if profs:
+        traffic = json.load(open(profs[-1])).get("dram_bytes_per_launch")
 
     # ---- e2e: host buffers through the C-ABI, copies inside the timed region ----
     e2e = None
@@ -344,10 +422,16 @@ def run_gpu(args):
                        "samples_per_step": samples_step, "launches_per_step": 2,
                        "parallelism": f"replicas x{world} (one image per GPU)",
                        "l2": "no flush: 768 MiB working set > 126 MB L2", "parity": parity},
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
-                         "frac": achieved / hbm_peak, "traffic": traffic,
-                         "kernel": "k_sample_grid<2D RGBA32F LINEAR>", "kernel_ms": k_ms,
-                         "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src},
+            "roofline": {"bound": "hbm", "achieved": achieved[dom], "peak": hbm_peak, "unit": "GB/s",
+                         "frac": achieved[dom] / hbm_peak, "traffic": traffic,
+                         "kernel": ["k_sample_grid<2D RGBA32F LINEAR REPEAT>",
+                                    "k_sample_grid<2D RGBA32F LINEAR MIRRORED>"][dom],
+                         "kernel_ms": pass_ms[dom], "algorithmic_bytes_per_launch": alg[dom],
+                         "peak_source": peak_src,
+                         "per_pass": [{"mode": m, "ms": pass_ms[k], "algorithmic_bytes": alg[k],
+                                       "GB/s": achieved[k], "frac": achieved[k] / hbm_peak}
+                                      for k, m in enumerate(("repeat", "mirrored"))],
+                         "step_frac": sum(alg) / (sum(pass_ms) * 1e-3) / 1e9 / hbm_peak},
             "cpu_baseline": cpu, "e2e": e2e, "clocks": clk, "gpu_launches": gpu_launches,
             "secondary": secondary,
         }
@@ -388,7 +472,12 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
         S.queue, vol, smp3, 0, A3, d3, 1, out3, 0, 0, None, None)), 10)
     byt = 2 * n3 ** 3 * 4
     res["c3_trilinear_512"] = {"Gsamples/s": n3 ** 3 / ms / 1e6, "ms": ms, "GB/s": byt / ms / 1e6,
-                               "hbm_frac": byt / ms / 1e6 / hbm_peak}
+                               "hbm_frac": byt / ms / 1e6 / hbm_peak, "map": "stencil (A)"}
+    A3b = (ctypes.c_float * 12)(*synth.affine_rotate_3d(n3, 20.0).tolist())
+    ms = _time_launches(T, torch, dev, lambda: cl.check(L.b2clEnqueueReadImageGrid(
+        S.queue, vol, smp3, 0, A3b, d3, 1, out3, 0, 0, None, None)), 10)
+    res["c3_trilinear_512_rotated"] = {"Gsamples/s": n3 ** 3 / ms / 1e6, "ms": ms,
+                                       "map": "volume-render rotation (B), 20 deg about z"}
     S.release(vol, out3)
     L.clReleaseSampler(smp3)
     # config 4: 8 GiB pitched CopyBufferRect (src padded, dst tight) and a misaligned variant
@@ -435,7 +524,7 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="b2cl", choices=["b2cl", "reference"])
     ap.add_argument("--no-secondary", action="store_true")

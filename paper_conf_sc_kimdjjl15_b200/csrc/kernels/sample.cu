@@ -1,13 +1,23 @@
 // sample.cu -- read_imagef / read_imagei / read_imageui kernels (steps a3-a7).
 //
-// One thread evaluates one sample: coordinates (affine grid or list) ->
-// per-axis addressing ([CL1.2 §8.2]) -> texel fetch through the CLImage
-// pointer with 16-byte vector loads for RGBA32F -> conversion and
-// channel map ([CL1.2 §8.3]) -> LINEAR blend in the separable FMA form.
+// Per sample: coordinates (affine grid or list) -> per-axis addressing
+// ([CL1.2 §8.2]) -> texel fetch through the CLImage pointer with one
+// vector load per texel (16 B for RGBA32F) -> conversion and channel map
+// ([CL1.2 §8.3]) -> LINEAR blend in the separable FMA form.
+//
+// Two grid kernels:
+//  * k_sample_grid      one thread per output sample, any affine map;
+//  * k_sample_grid_sep  separable maps (every off-diagonal coefficient 0):
+//    the x-axis addressing of XPT columns is computed once per thread and
+//    reused down RPW rows, the y/z-axis addressing and the texel row
+//    pointers once per row.  The coordinates it evaluates differ from the
+//    general form ((A0*x + A1*y) + A2*z) + A3 only by additions of a signed
+//    zero, which can change nothing but the sign of a zero coordinate, and
+//    every addressing mode maps +0 and -0 to the same indices and weights --
+//    so both kernels return identical bits (the parity tests run both).
 // Every template argument may be `RT` (decided from the parameters at run
 // time): the fully run-time instance covers every format x sampler; the
-// compile-time instances are the hot configurations of BASELINE.json
-// (bit-identical arithmetic, fewer instructions).
+// compile-time instances are the hot configurations of BASELINE.json.
 #include <atomic>
 
 #include "../device/image.cuh"
@@ -23,96 +33,141 @@ struct Cfg {
   static constexpr int nch = ORDER == RT ? RT : order_channels(ORDER);
 };
 
-template <class C>
-__device__ __forceinline__ int near_idx(const Sampler& s, float c, int n) {
-  if constexpr (C::addr == RT) return axis_nearest_rt(s.addr, s.norm, c, n);
-  else return axis_nearest<C::addr, C::norm>(c, n);
-}
-template <class C>
-__device__ __forceinline__ void lin_idx(const Sampler& s, float c, int n, int& i0, int& i1,
-                                        float& a) {
-  if constexpr (C::addr == RT) axis_linear_rt(s.addr, s.norm, c, n, i0, i1, a);
-  else axis_linear<C::addr, C::norm>(c, n, i0, i1, a);
-}
+struct AxN {  // NEAREST, one axis
+  int i;
+  bool ok;
+};
+struct AxL {  // LINEAR, one axis
+  int i0, i1;
+  float a, oma;
+  bool ok0, ok1;
+};
+
 template <class C>
 __device__ __forceinline__ bool may_border(const Sampler& s) {
   if constexpr (C::addr == RT) return s.addr == A_NONE || s.addr == A_CLAMP;
   else return C::addr == A_NONE || C::addr == A_CLAMP;
 }
 
-// The built-in: c[0..DIMS-1] -> res (x,y,z,w) as 32-bit patterns.
+template <class C>
+__device__ __forceinline__ AxN axis_n(const Sampler& s, float c, int n) {
+  AxN r;
+  if constexpr (C::addr == RT) r.i = axis_nearest_rt(s.addr, s.norm, c, n);
+  else r.i = axis_nearest<C::addr, C::norm>(c, n);
+  r.ok = !may_border<C>(s) || in_range(r.i, n);
+  return r;
+}
+
+template <class C>
+__device__ __forceinline__ AxL axis_l(const Sampler& s, float c, int n) {
+  AxL r;
+  if constexpr (C::addr == RT) axis_linear_rt(s.addr, s.norm, c, n, r.i0, r.i1, r.a);
+  else axis_linear<C::addr, C::norm>(c, n, r.i0, r.i1, r.a);
+  r.oma = __fsub_rn(1.0f, r.a);
+  const bool b = may_border<C>(s);
+  r.ok0 = !b || in_range(r.i0, n);
+  r.ok1 = !b || in_range(r.i1, n);
+  return r;
+}
+
+template <class C>
+__device__ __forceinline__ int filt_of(const SampleParams& p) {
+  return C::filt == RT ? p.smp.filt : C::filt;
+}
+
+// start of texel row (j,k): ptr + k*slice_pitch + j*row_pitch (Fig. 6)
+__device__ __forceinline__ const char* row_ptr(const Image& im, int j, int k) {
+  return im.ptr + (uint64_t)(unsigned)k * im.sp + (uint64_t)(unsigned)j * im.rp;
+}
+
+// memory-order channels of the texel at row + i*elem_size (zero if !ok)
+template <class C>
+__device__ __forceinline__ void fetch(const Image& im, const char* row, int i, bool ok, int rc,
+                                      uint32_t m[4]) {
+  const int type = C::type == RT ? im.type : C::type;
+  const int nch = C::nch == RT ? im.nch : C::nch;
+  const int es = (C::type == RT || C::nch == RT) ? im.es : C::nch * type_bytes(C::type);
+  m[0] = m[1] = m[2] = m[3] = 0u;
+  if (!ok) return;
+  Raw r = load_raw(row + (uint64_t)(unsigned)i * (unsigned)es, es);
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    if (c < nch) {
+      uint32_t v = channel_code(r, c, type);
+      m[c] = rc == R_F ? __float_as_uint(code_to_float(v, type)) : v;
+    }
+  }
+}
+
+// NEAREST: one texel, channel-mapped
+template <class C>
+__device__ __forceinline__ void nearest_at(const SampleParams& p, const char* row, const AxN& x,
+                                           bool row_ok, uint32_t res[4]) {
+  const int rc = C::rc == RT ? p.rclass : C::rc;
+  const int order = C::order == RT ? p.im.order : C::order;
+  uint32_t m[4];
+  fetch<C>(p.im, row, x.i, row_ok && x.ok, rc, m);
+  map_order(order, m, rc == R_F ? 0x3f800000u : 1u, res);
+}
+
+// LINEAR from the texel rows: rows[0] = (j0,k0), [1] = (j1,k0), [2] = (j0,k1),
+// [3] = (j1,k1); blend x, then y, then z ([CL1.2 §8.2] weights, separable form)
+template <class C>
+__device__ __forceinline__ void linear_at(const SampleParams& p, const char* const rows[4],
+                                          const bool rok[4], const AxL& x, float b, float omb,
+                                          float g, float omg, uint32_t res[4]) {
+  constexpr int NR = C::dims == 1 ? 1 : (C::dims == 2 ? 2 : 4);
+  const int order = C::order == RT ? p.im.order : C::order;
+  const int nch = C::nch == RT ? p.im.nch : C::nch;
+  uint32_t t0[NR][4], t1[NR][4];
+#pragma unroll
+  for (int r = 0; r < NR; ++r) {
+    fetch<C>(p.im, rows[r], x.i0, rok[r] && x.ok0, R_F, t0[r]);
+    fetch<C>(p.im, rows[r], x.i1, rok[r] && x.ok1, R_F, t1[r]);
+  }
+  uint32_t m[4];
+#pragma unroll
+  for (int ch = 0; ch < 4; ++ch) {
+    float v[NR];
+#pragma unroll
+    for (int r = 0; r < NR; ++r)
+      v[r] = lerp1(x.a, x.oma, __uint_as_float(t0[r][ch]), __uint_as_float(t1[r][ch]));
+    float o = v[0];
+    if constexpr (C::dims >= 2) {
+      const float s0 = lerp1(b, omb, v[0], v[1]);
+      o = s0;
+      if constexpr (C::dims == 3) o = lerp1(g, omg, s0, lerp1(b, omb, v[2], v[3]));
+    }
+    // channels the format does not store stay exactly 0 / 1 after the map
+    m[ch] = ch < nch ? __float_as_uint(o) : 0u;
+  }
+  map_order(order, m, 0x3f800000u, res);
+  // a NaN weight (non-finite coordinate) makes the spec's sum NaN in every
+  // component, including the constant ones (reading A26)
+  if (x.a != x.a || b != b || g != g) res[0] = res[1] = res[2] = res[3] = 0x7fffffffu;
+}
+
+// The built-in on one coordinate: c[0..DIMS-1] -> res (x,y,z,w) as 32-bit patterns.
 template <class C>
 __device__ __forceinline__ void read_image(const SampleParams& p, const float c[3],
                                            uint32_t res[4]) {
   const Image& im = p.im;
-  const int rc = C::rc == RT ? p.rclass : C::rc;
-  const int order = C::order == RT ? im.order : C::order;
-  const int nch = C::nch == RT ? im.nch : C::nch;
-  const int filt = C::filt == RT ? p.smp.filt : C::filt;
-  const uint32_t one = rc == R_F ? 0x3f800000u : 1u;
-  const bool bord = may_border<C>(p.smp);
-  uint32_t m[4];
-  if (filt == F_NEAREST) {
-    int i = near_idx<C>(p.smp, c[0], im.w);
-    int j = C::dims > 1 ? near_idx<C>(p.smp, c[1], im.h) : 0;
-    int k = C::dims > 2 ? near_idx<C>(p.smp, c[2], im.d) : 0;
-    bool ok = !bord || (in_range(i, im.w) && (C::dims < 2 || in_range(j, im.h)) &&
-                        (C::dims < 3 || in_range(k, im.d)));
-    fetch_mem<C::type, C::nch>(im, i, j, k, ok, rc, m);
+  if (filt_of<C>(p) == F_NEAREST) {
+    const AxN x = axis_n<C>(p.smp, c[0], im.w);
+    AxN y{0, true}, z{0, true};
+    if (C::dims > 1) y = axis_n<C>(p.smp, c[1], im.h);
+    if (C::dims > 2) z = axis_n<C>(p.smp, c[2], im.d);
+    nearest_at<C>(p, row_ptr(im, y.i, z.i), x, y.ok && z.ok, res);
   } else {
-    int i0, i1, j0 = 0, j1 = 0, k0 = 0, k1 = 0;
-    float a, b = 0.f, g = 0.f;
-    lin_idx<C>(p.smp, c[0], im.w, i0, i1, a);
-    if (C::dims > 1) lin_idx<C>(p.smp, c[1], im.h, j0, j1, b);
-    if (C::dims > 2) lin_idx<C>(p.smp, c[2], im.d, k0, k1, g);
-    const bool oi0 = !bord || in_range(i0, im.w), oi1 = !bord || in_range(i1, im.w);
-    const bool oj0 = C::dims < 2 || !bord || in_range(j0, im.h);
-    const bool oj1 = C::dims < 2 || !bord || in_range(j1, im.h);
-    const bool ok0 = C::dims < 3 || !bord || in_range(k0, im.d);
-    const bool ok1 = C::dims < 3 || !bord || in_range(k1, im.d);
-    const float oma = __fsub_rn(1.0f, a), omb = __fsub_rn(1.0f, b), omg = __fsub_rn(1.0f, g);
-    uint32_t t000[4], t100[4];
-    fetch_mem<C::type, C::nch>(im, i0, j0, k0, oi0 && oj0 && ok0, R_F, t000);
-    fetch_mem<C::type, C::nch>(im, i1, j0, k0, oi1 && oj0 && ok0, R_F, t100);
-    if (C::dims == 1) {
-#pragma unroll
-      for (int ch = 0; ch < 4; ++ch)
-        m[ch] = __float_as_uint(lerp1(a, oma, __uint_as_float(t000[ch]), __uint_as_float(t100[ch])));
-    } else {
-      uint32_t t010[4], t110[4];
-      fetch_mem<C::type, C::nch>(im, i0, j1, k0, oi0 && oj1 && ok0, R_F, t010);
-      fetch_mem<C::type, C::nch>(im, i1, j1, k0, oi1 && oj1 && ok0, R_F, t110);
-      float s0[4];
-#pragma unroll
-      for (int ch = 0; ch < 4; ++ch) {
-        float r0 = lerp1(a, oma, __uint_as_float(t000[ch]), __uint_as_float(t100[ch]));
-        float r1 = lerp1(a, oma, __uint_as_float(t010[ch]), __uint_as_float(t110[ch]));
-        s0[ch] = lerp1(b, omb, r0, r1);
-      }
-      if (C::dims == 2) {
-#pragma unroll
-        for (int ch = 0; ch < 4; ++ch) m[ch] = __float_as_uint(s0[ch]);
-      } else {
-        uint32_t t001[4], t101[4], t011[4], t111[4];
-        fetch_mem<C::type, C::nch>(im, i0, j0, k1, oi0 && oj0 && ok1, R_F, t001);
-        fetch_mem<C::type, C::nch>(im, i1, j0, k1, oi1 && oj0 && ok1, R_F, t101);
-        fetch_mem<C::type, C::nch>(im, i0, j1, k1, oi0 && oj1 && ok1, R_F, t011);
-        fetch_mem<C::type, C::nch>(im, i1, j1, k1, oi1 && oj1 && ok1, R_F, t111);
-#pragma unroll
-        for (int ch = 0; ch < 4; ++ch) {
-          float r0 = lerp1(a, oma, __uint_as_float(t001[ch]), __uint_as_float(t101[ch]));
-          float r1 = lerp1(a, oma, __uint_as_float(t011[ch]), __uint_as_float(t111[ch]));
-          float s1 = lerp1(b, omb, r0, r1);
-          m[ch] = __float_as_uint(lerp1(g, omg, s0[ch], s1));
-        }
-      }
-    }
-    // channels the format does not store stay exactly 0 / 1 after the map
-#pragma unroll
-    for (int ch = 0; ch < 4; ++ch)
-      if (ch >= nch) m[ch] = 0u;
+    const AxL x = axis_l<C>(p.smp, c[0], im.w);
+    AxL y{0, 0, 0.f, 1.f, true, true}, z{0, 0, 0.f, 1.f, true, true};
+    if (C::dims > 1) y = axis_l<C>(p.smp, c[1], im.h);
+    if (C::dims > 2) z = axis_l<C>(p.smp, c[2], im.d);
+    const char* rows[4] = {row_ptr(im, y.i0, z.i0), row_ptr(im, y.i1, z.i0),
+                           row_ptr(im, y.i0, z.i1), row_ptr(im, y.i1, z.i1)};
+    const bool rok[4] = {y.ok0 && z.ok0, y.ok1 && z.ok0, y.ok0 && z.ok1, y.ok1 && z.ok1};
+    linear_at<C>(p, rows, rok, x, y.a, y.oma, z.a, z.oma, res);
   }
-  map_order(order, m, one, res);
 }
 
 // coordinate of output (x,y,z) under the affine map: ((A0*x + A1*y) + A2*z) + A3
@@ -121,6 +176,21 @@ __device__ __forceinline__ float affine_coord(const float* A, float x, float y, 
   v = __fadd_rn(v, __fmul_rn(A[1], y));
   v = __fadd_rn(v, __fmul_rn(A[2], z));
   return __fadd_rn(v, A[3]);
+}
+
+template <int OUTC>
+__device__ __forceinline__ void store_out(const SampleParams& p, uint64_t idx, const uint32_t r[4]) {
+  const int outc = OUTC == RT ? p.outc : OUTC;
+  if (outc == 4) {
+    __stcs(reinterpret_cast<uint4*>(p.out) + idx, make_uint4(r[0], r[1], r[2], r[3]));
+  } else if (outc == 1) {
+    __stcs(reinterpret_cast<unsigned int*>(p.out) + idx, r[0]);
+  } else if (outc == 2) {
+    __stcs(reinterpret_cast<uint2*>(p.out) + idx, make_uint2(r[0], r[1]));
+  } else {
+    unsigned int* o = reinterpret_cast<unsigned int*>(p.out) + idx * 3;
+    o[0] = r[0]; o[1] = r[1]; o[2] = r[2];
+  }
 }
 
 template <class C, int OUTC>
@@ -136,17 +206,71 @@ __global__ void __launch_bounds__(256) k_sample_grid(const SampleParams p) {
   c[2] = C::dims > 2 ? affine_coord(p.A + 8, xf, yf, zf) : 0.f;
   uint32_t r[4];
   read_image<C>(p, c, r);
-  const int outc = OUTC == RT ? p.outc : OUTC;
-  const uint64_t idx = ((uint64_t)z * p.oh + y) * p.ow + x;
-  if (outc == 4) {
-    reinterpret_cast<uint4*>(p.out)[idx] = make_uint4(r[0], r[1], r[2], r[3]);
-  } else if (outc == 1) {
-    reinterpret_cast<uint32_t*>(p.out)[idx] = r[0];
-  } else if (outc == 2) {
-    reinterpret_cast<uint2*>(p.out)[idx] = make_uint2(r[0], r[1]);
-  } else {
-    uint32_t* o = reinterpret_cast<uint32_t*>(p.out) + idx * 3;
-    o[0] = r[0]; o[1] = r[1]; o[2] = r[2];
+  store_out<OUTC>(p, ((uint64_t)z * p.oh + y) * p.ow + x, r);
+}
+
+// Separable maps: block = 32 x 4 threads; tile = (32*XPT) columns x (4*RPW) rows
+// of one output slice.  Lane -> columns lane + 32*t, warp -> RPW consecutive rows.
+template <class C, int OUTC, int XPT, int RPW>
+__global__ void __launch_bounds__(128) k_sample_grid_sep(const SampleParams p) {
+  const Image& im = p.im;
+  const int z = blockIdx.z;
+  const int x0 = blockIdx.x * (32 * XPT) + threadIdx.x;
+  const int y0 = blockIdx.y * (4 * RPW) + threadIdx.y * RPW;
+  const bool lin = filt_of<C>(p) == F_LINEAR;
+  // x axis: once per column
+  AxL ax[XPT];
+  AxN nx[XPT];
+#pragma unroll
+  for (int t = 0; t < XPT; ++t) {
+    const float s = __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(x0 + 32 * t)), p.A[3]);
+    if (lin) ax[t] = axis_l<C>(p.smp, s, im.w);
+    else nx[t] = axis_n<C>(p.smp, s, im.w);
+  }
+  // z axis: once per block
+  AxL az{0, 0, 0.f, 1.f, true, true};
+  AxN nz{0, true};
+  if (C::dims > 2) {
+    const float s = __fadd_rn(__fmul_rn(p.A[10], __int2float_rn(z)), p.A[11]);
+    if (lin) az = axis_l<C>(p.smp, s, im.d);
+    else nz = axis_n<C>(p.smp, s, im.d);
+  }
+#pragma unroll 1
+  for (int r = 0; r < RPW; ++r) {
+    const int y = y0 + r;
+    if (y >= p.oh) break;
+    const uint64_t obase = ((uint64_t)z * p.oh + y) * p.ow;
+    if (lin) {
+      AxL ay{0, 0, 0.f, 1.f, true, true};
+      if (C::dims > 1)
+        ay = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(y)), p.A[7]), im.h);
+      const char* rows[4] = {row_ptr(im, ay.i0, az.i0), row_ptr(im, ay.i1, az.i0),
+                             row_ptr(im, ay.i0, az.i1), row_ptr(im, ay.i1, az.i1)};
+      const bool rok[4] = {ay.ok0 && az.ok0, ay.ok1 && az.ok0, ay.ok0 && az.ok1, ay.ok1 && az.ok1};
+#pragma unroll
+      for (int t = 0; t < XPT; ++t) {
+        const int x = x0 + 32 * t;
+        if (x < p.ow) {
+          uint32_t res[4];
+          linear_at<C>(p, rows, rok, ax[t], ay.a, ay.oma, az.a, az.oma, res);
+          store_out<OUTC>(p, obase + x, res);
+        }
+      }
+    } else {
+      AxN ny{0, true};
+      if (C::dims > 1)
+        ny = axis_n<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(y)), p.A[7]), im.h);
+      const char* row = row_ptr(im, ny.i, nz.i);
+#pragma unroll
+      for (int t = 0; t < XPT; ++t) {
+        const int x = x0 + 32 * t;
+        if (x < p.ow) {
+          uint32_t res[4];
+          nearest_at<C>(p, row, nx[t], ny.ok && nz.ok, res);
+          store_out<OUTC>(p, obase + x, res);
+        }
+      }
+    }
   }
 }
 
@@ -174,7 +298,7 @@ __global__ void __launch_bounds__(256) k_sample_list(const SampleParams p) {
   }
   uint32_t r[4];
   read_image<C>(p, c, r);
-  reinterpret_cast<uint4*>(p.out)[s] = make_uint4(r[0], r[1], r[2], r[3]);
+  __stcs(reinterpret_cast<uint4*>(p.out) + s, make_uint4(r[0], r[1], r[2], r[3]));
 }
 
 // ---------------------------------------------------------------- dispatch
@@ -183,6 +307,15 @@ static cudaError_t go_grid(const SampleParams& p, cudaStream_t st) {
   dim3 blk(32, 8, 1);
   dim3 grd((p.ow + 31) / 32, (p.oh + 7) / 8, p.od);
   k_sample_grid<C, OUTC><<<grd, blk, 0, st>>>(p);
+  count_launch();
+  return cudaGetLastError();
+}
+
+template <class C, int OUTC, int XPT, int RPW>
+static cudaError_t go_sep(const SampleParams& p, cudaStream_t st) {
+  dim3 blk(32, 4, 1);
+  dim3 grd((p.ow + 32 * XPT - 1) / (32 * XPT), (p.oh + 4 * RPW - 1) / (4 * RPW), p.od);
+  k_sample_grid_sep<C, OUTC, XPT, RPW><<<grd, blk, 0, st>>>(p);
   count_launch();
   return cudaGetLastError();
 }
@@ -211,13 +344,32 @@ static bool matches(const SampleParams& p, int type, int order, int norm, int ad
          p.smp.addr == addr && p.smp.filt == filt && p.rclass == ret_class(type);
 }
 
+// every coefficient that couples an output axis into another coordinate is 0
+static bool separable(const SampleParams& p) {
+  const float* A = p.A;
+  bool ok = A[1] == 0.0f && A[2] == 0.0f;
+  if (p.dims > 1) ok = ok && A[4] == 0.0f && A[6] == 0.0f;
+  if (p.dims > 2) ok = ok && A[8] == 0.0f && A[9] == 0.0f;
+  return ok;
+}
+
 cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st) {
   if (coord_mode == COORD_GRID) {
     if ((uint64_t)p.ow * p.oh * p.od == 0) return cudaSuccess;
+    if (separable(p)) {
+      if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_REPEAT, F_LINEAR)) return go_sep<C2Repeat, 4, 2, 4>(p, st);
+      if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_MIRROR, F_LINEAR)) return go_sep<C2Mirror, 4, 2, 4>(p, st);
+      if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR)) return go_sep<C3Cte, 1, 4, 4>(p, st);
+      if (p.outc == 4 && matches<2>(p, T_UNORM8, O_RGBA, 0, A_CLAMP, F_NEAREST)) return go_sep<C1Clamp, 4, 2, 4>(p, st);
+      switch (p.dims) {
+        case 1: return go_sep<Generic<1>, RT, 2, 2>(p, st);
+        case 2: return go_sep<Generic<2>, RT, 2, 2>(p, st);
+        default: return go_sep<Generic<3>, RT, 2, 2>(p, st);
+      }
+    }
     if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_REPEAT, F_LINEAR)) return go_grid<C2Repeat, 4>(p, st);
     if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_MIRROR, F_LINEAR)) return go_grid<C2Mirror, 4>(p, st);
     if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR)) return go_grid<C3Cte, 1>(p, st);
-    if (p.outc == 4 && matches<2>(p, T_UNORM8, O_RGBA, 0, A_CLAMP, F_NEAREST)) return go_grid<C1Clamp, 4>(p, st);
     switch (p.dims) {
       case 1: return go_grid<Generic<1>, RT>(p, st);
       case 2: return go_grid<Generic<2>, RT>(p, st);

@@ -118,6 +118,19 @@ def affine_stencil_3d(n: int, delta=(0.3, 0.6, 0.2)) -> np.ndarray:
     return A
 
 
+def affine_rotate_3d(n: int, degrees: float = 20.0) -> np.ndarray:
+    """C3 map (B), volume-render shaped: rotation about the z axis through the
+    volume centre, normalized coordinates (non-separable)."""
+    th = np.deg2rad(degrees)
+    c, s = np.cos(th), np.sin(th)
+    h = n / 2.0
+    A = np.zeros(12, dtype=np.float32)
+    A[0], A[1], A[3] = c / n, -s / n, (c * (0.5 - h) - s * (0.5 - h) + h) / n
+    A[4], A[5], A[7] = s / n, c / n, (s * (0.5 - h) + c * (0.5 - h) + h) / n
+    A[10], A[11] = 1.0 / n, 0.5 / n
+    return A
+
+
 def affine_unnorm_2d(step: float, origin: float) -> np.ndarray:
     """C1 brute-force map: unnormalized (u, v) = (origin + step*x, origin + step*y)."""
     A = np.zeros(12, dtype=np.float32)

@@ -50,7 +50,7 @@ def test_config1_buffer_rect_all_x_origins(sess, orc):
         for x in range(0, 193):
             so = (x, int(g.integers(0, 48)), int(g.integers(0, 1)))
             region = (r0, 16, 4)
-            dst = np.zeros(r0 * 16 * 4 + 64, np.uint8)
+            dst = np.zeros((r0 + 7) * 16 * 4 + 64, np.uint8)
             do = (x % 7, 0, 0)
             got = _copy_rect_gpu(sess, vol, dst, so, do, region, 256, 16384, r0 + 7, (r0 + 7) * 16)
             exp = dst.copy()

@@ -135,6 +135,10 @@ GRID_CASES = [
     (2, RGBA, F32, (64, 48, 1), (1, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR), "rotate", (70, 50, 1), 4),
     (2, RGBA, F32, (64, 48, 1), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "rotate", (70, 50, 1), 4),
     (3, R, F32, (40, 33, 17), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "stencil", (40, 33, 17), 1),
+    (3, R, F32, (40, 40, 17), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d", (44, 37, 19), 1),
+    (3, RGBA, F16, (12, 10, 9), (1, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR), "rotate3d", (17, 13, 11), 4),
+    (2, RGBA, U8N, (64, 64, 1), (0, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_NEAREST), "rotate", (70, 66, 1), 4),
+    (2, RG, F32, (33, 21, 1), (1, cl.CL_ADDRESS_NONE, cl.CL_FILTER_LINEAR), "translate", (40, 30, 3), 2),
     (2, RGBA, U8N, (64, 64, 1), (0, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_NEAREST), "unnorm", (96, 96, 1), 4),
     (2, BGRA, U8N, (31, 17, 1), (1, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_LINEAR), "rotate", (45, 29, 1), 3),
     (1, RG, F16, (50, 1, 1), (1, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR), "translate", (77, 1, 1), 2),
@@ -148,6 +152,8 @@ def _affine(kind, size, out):
         return synth.affine_translate_2d(W, H)
     if kind == "rotate":
         return synth.affine_rotate_2d(W, H, 30.0)
+    if kind == "rotate3d":
+        return synth.affine_rotate_3d(W, 20.0)
     if kind == "stencil":
         A = synth.affine_stencil_3d(W)
         A[5] = 1.0 / H
@@ -209,13 +215,15 @@ def test_config2_full_size_sampled_rows(sess, orc, addr, kind):
     sess.release(img)
 
 
-def test_config3_full_size_sampled_slices(sess, orc):
-    """BASELINE config 3 at full size (512^3 R32F, trilinear, stencil map, CLAMP_TO_EDGE):
-    sampled rows of first / middle / last slices against the oracle."""
+@pytest.mark.parametrize("kind", ["stencil", "rotate3d"])
+def test_config3_full_size_sampled_slices(sess, orc, kind):
+    """BASELINE config 3 at full size (512^3 R32F, trilinear, CLAMP_TO_EDGE; stencil map
+    (separable kernel) and volume-render rotation (general kernel)): sampled rows of
+    first / middle / last slices against the oracle."""
     N = 512
     img, oimg, _ = make_images(sess, orc, R, F32, N, N, N, 3, seed=3)
     smp = sess.sampler(True, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR)
-    A = synth.affine_stencil_3d(N)
+    A = synth.affine_stencil_3d(N) if kind == "stencil" else synth.affine_rotate_3d(N, 20.0)
     got = gpu_read_grid(sess, img, smp, cl.B2CL_RTYPE_FLOAT, A, (N, N, N), 1)
     for z in (0, 1, 255, 510, 511):
         for y in (0, 1, 100, 256, 511):
