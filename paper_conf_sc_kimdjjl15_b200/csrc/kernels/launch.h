@@ -31,7 +31,10 @@ struct RectParams {
   uint32_t ptile[32];     // FILL: 128-byte tile (pattern repeated)
   uint32_t color[4];      // FILL_IMAGE: color bits
   int type, order, es;    // FILL_IMAGE: format
-  uint32_t chunks_per_row;
+  // set by launch_rect: rows = R1*R2, row_step = rows walked per loop
+  // iteration of a thread, step_dz / step_dy = row_step as (slices, rows)
+  uint64_t rows, row_step;
+  uint32_t step_dz, step_dy;
 };
 
 struct WriteParams {

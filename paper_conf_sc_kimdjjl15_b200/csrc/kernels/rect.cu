@@ -72,46 +72,54 @@ __global__ void __launch_bounds__(256) k_rect(const RectParams p) {
     }
     __syncthreads();
   }
-  const uint32_t rg = blockIdx.x / p.chunks_per_row;
-  const uint32_t chunk = blockIdx.x - rg * p.chunks_per_row;
-  const uint64_t row = (uint64_t)rg * blockDim.y + threadIdx.y;
-  if (row >= (uint64_t)p.R1 * p.R2) return;
-  const uint32_t z = (uint32_t)(row / p.R1), y = (uint32_t)(row - (uint64_t)z * p.R1);
-  char* drow = p.dst + z * p.dsp + y * p.drp;
-  const char* srow = MODE == RECT_COPY ? p.src + z * p.ssp + y * p.srp : nullptr;
-  const uintptr_t dlo = reinterpret_cast<uintptr_t>(drow), dhi = dlo + p.R0;
-  const uintptr_t abase = dlo & ~uintptr_t(15);
-  const uint64_t nvec = ((dhi + 15) >> 4) - (abase >> 4);
-  const int sh = MODE == RECT_COPY ? (int)((reinterpret_cast<uintptr_t>(srow) - dlo) & 15) : 0;
-  const uint64_t v0 = (uint64_t)chunk * blockDim.x * U + threadIdx.x;
-
-  uint4 val[U];
-  bool full[U];
+  // Grid: x = chunk of a row (TX*U vectors), y = group of TY rows; each thread
+  // then walks rows with stride gridDim.y*TY (persistent in y), stepping its
+  // (z, y) row coordinates incrementally (no divisions in the loop).
+  const uint64_t v0 = (uint64_t)blockIdx.x * blockDim.x * U + threadIdx.x;
+  uint64_t row = (uint64_t)blockIdx.y * blockDim.y + threadIdx.y;
+  if (row >= p.rows) return;
+  uint32_t z = (uint32_t)(row / p.R1), y = (uint32_t)(row - (uint64_t)z * p.R1);
+  for (; row < p.rows; row += p.row_step) {
+    char* drow = p.dst + z * p.dsp + y * p.drp;
+    const char* srow = MODE == RECT_COPY ? p.src + z * p.ssp + y * p.srp : nullptr;
+    const uintptr_t dlo = reinterpret_cast<uintptr_t>(drow), dhi = dlo + p.R0;
+    const uintptr_t abase = dlo & ~uintptr_t(15);
+    const uint64_t nvec = ((dhi + 15) >> 4) - (abase >> 4);
+    // full 16-byte destination vectors are v in [vf0, vf1)
+    const uint64_t vf0 = (dlo & 15) ? 1 : 0;
+    const uint64_t vf1 = (dhi >> 4) - (abase >> 4);
+    const int sh = MODE == RECT_COPY ? (int)((reinterpret_cast<uintptr_t>(srow) - dlo) & 15) : 0;
+    uint4 val[U];
 #pragma unroll
-  for (int u = 0; u < U; ++u) {
-    const uint64_t v = v0 + (uint64_t)u * blockDim.x;
-    const uintptr_t D = abase + 16 * v;
-    full[u] = v < nvec && D >= dlo && D + 16 <= dhi;
-    if (full[u]) {
-      if (MODE == RECT_COPY) val[u] = load_shifted(srow + (D - dlo), sh);
-      else val[u] = tile[(D >> 4) & 7];
-    }
-  }
-#pragma unroll
-  for (int u = 0; u < U; ++u) {
-    const uint64_t v = v0 + (uint64_t)u * blockDim.x;
-    if (v >= nvec) continue;
-    const uintptr_t D = abase + 16 * v;
-    if (full[u]) {
-      *reinterpret_cast<uint4*>(D) = val[u];
-    } else {  // ragged head / tail of the row
-      const uintptr_t lo = D > dlo ? D : dlo, hi = D + 16 < dhi ? D + 16 : dhi;
-      for (uintptr_t X = lo; X < hi; ++X) {
-        unsigned char b;
-        if (MODE == RECT_COPY) b = static_cast<unsigned char>(srow[X - dlo]);
-        else b = reinterpret_cast<const unsigned char*>(tile)[X & 127];
-        *reinterpret_cast<unsigned char*>(X) = b;
+    for (int u = 0; u < U; ++u) {
+      const uint64_t v = v0 + (uint64_t)u * blockDim.x;
+      if (v >= vf0 && v < vf1) {
+        const uintptr_t D = abase + 16 * v;
+        if (MODE == RECT_COPY) val[u] = load_shifted(srow + (D - dlo), sh);
+        else val[u] = tile[(D >> 4) & 7];
       }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint64_t v = v0 + (uint64_t)u * blockDim.x;
+      const uintptr_t D = abase + 16 * v;
+      if (v >= vf0 && v < vf1) {
+        *reinterpret_cast<uint4*>(D) = val[u];
+      } else if (v < nvec) {  // ragged head / tail of the row
+        const uintptr_t lo = D > dlo ? D : dlo, hi = D + 16 < dhi ? D + 16 : dhi;
+        for (uintptr_t X = lo; X < hi; ++X) {
+          unsigned char b;
+          if (MODE == RECT_COPY) b = static_cast<unsigned char>(srow[X - dlo]);
+          else b = reinterpret_cast<const unsigned char*>(tile)[X & 127];
+          *reinterpret_cast<unsigned char*>(X) = b;
+        }
+      }
+    }
+    y += p.step_dy;
+    z += p.step_dz;
+    if (y >= p.R1) {
+      y -= p.R1;
+      ++z;
     }
   }
 }
@@ -120,19 +128,34 @@ cudaError_t launch_rect(RectParams& p, int mode, cudaStream_t st) {
   const uint64_t rows = (uint64_t)p.R1 * p.R2;
   if (p.R0 == 0 || rows == 0) return cudaSuccess;
   constexpr int U = 4;
+  static int nsm = 0;
+  if (nsm == 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (nsm <= 0) nsm = 148;
+  }
   const uint64_t nvec_max = (p.R0 + 15) / 16 + 1;
   unsigned tx = 32;
   while (tx < 256 && (uint64_t)tx * U < nvec_max) tx *= 2;
   const unsigned ty = 256 / tx;
   const uint64_t cpr = (nvec_max + (uint64_t)tx * U - 1) / ((uint64_t)tx * U);
-  const uint64_t blocks = cpr * ((rows + ty - 1) / ty);
-  if (cpr > 0xffffffffull || blocks > 0x7fffffffull) return cudaErrorInvalidValue;
-  p.chunks_per_row = (uint32_t)cpr;
-  dim3 blk(tx, ty, 1);
+  const uint64_t groups = (rows + ty - 1) / ty;
+  // enough blocks for ~4 resident waves; rows beyond that are walked in-kernel
+  const uint64_t want = (uint64_t)nsm * 32;
+  uint64_t gy = cpr >= want ? 1 : (want + cpr - 1) / cpr;
+  if (gy > groups) gy = groups;
+  if (gy > 65535) gy = 65535;
+  if (cpr > 0x7fffffffull) return cudaErrorInvalidValue;
+  p.rows = rows;
+  p.row_step = gy * ty;
+  p.step_dz = (uint32_t)(p.row_step / p.R1);
+  p.step_dy = (uint32_t)(p.row_step % p.R1);
+  dim3 blk(tx, ty, 1), grd((unsigned)cpr, (unsigned)gy, 1);
   switch (mode) {
-    case RECT_COPY: k_rect<RECT_COPY, U><<<(unsigned)blocks, blk, 0, st>>>(p); break;
-    case RECT_FILL: k_rect<RECT_FILL, U><<<(unsigned)blocks, blk, 0, st>>>(p); break;
-    default: k_rect<RECT_FILL_IMAGE, U><<<(unsigned)blocks, blk, 0, st>>>(p); break;
+    case RECT_COPY: k_rect<RECT_COPY, U><<<grd, blk, 0, st>>>(p); break;
+    case RECT_FILL: k_rect<RECT_FILL, U><<<grd, blk, 0, st>>>(p); break;
+    default: k_rect<RECT_FILL_IMAGE, U><<<grd, blk, 0, st>>>(p); break;
   }
   count_launch();
   return cudaGetLastError();

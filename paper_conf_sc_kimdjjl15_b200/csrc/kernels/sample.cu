@@ -77,19 +77,43 @@ __device__ __forceinline__ int filt_of(const SampleParams& p) {
 
 // start of texel row (j,k): ptr + k*slice_pitch + j*row_pitch (Fig. 6)
 __device__ __forceinline__ const char* row_ptr(const Image& im, int j, int k) {
-  return im.ptr + (uint64_t)(unsigned)k * im.sp + (uint64_t)(unsigned)j * im.rp;
+  const char* r = im.ptr + (uint64_t)(unsigned)k * im.sp + (uint64_t)(unsigned)j * im.rp;
+  // keep the absolute row pointer in registers: without this the compiler
+  // re-associates ptr + (row + i*es) and pays two extra 64-bit adds per tap
+  asm("" : "+l"(r));
+  return r;
 }
 
-// memory-order channels of the texel at row + i*elem_size (zero if !ok)
+// does any output component come from a constant of the channel map (0 or 1)?
+// Only those need the explicit NaN of reading A26; stored channels carry the
+// NaN weight through the blend by themselves.
+__device__ __forceinline__ bool const_in_output(int order, int outc) {
+  switch (order) {
+    case O_RGBA: case O_BGRA: case O_ARGB: case O_INTENSITY: return false;
+    case O_R: return outc > 1;
+    case O_RG: case O_RA: return outc > 1 + (order == O_RG);
+    case O_LUMINANCE: return outc > 3;
+    default: return true;  // O_A
+  }
+}
+
 template <class C>
+__device__ __forceinline__ int elem_size(const Image& im) {
+  return (C::type == RT || C::nch == RT) ? im.es : C::nch * type_bytes(C::type);
+}
+
+// memory-order channels of the texel at row + i*elem_size (zero if !ok);
+// SMEM: `row` points into a staged footprint in shared memory
+template <class C, bool SMEM = false>
 __device__ __forceinline__ void fetch(const Image& im, const char* row, int i, bool ok, int rc,
                                       uint32_t m[4]) {
   const int type = C::type == RT ? im.type : C::type;
   const int nch = C::nch == RT ? im.nch : C::nch;
-  const int es = (C::type == RT || C::nch == RT) ? im.es : C::nch * type_bytes(C::type);
+  const int es = elem_size<C>(im);
   m[0] = m[1] = m[2] = m[3] = 0u;
   if (!ok) return;
-  Raw r = load_raw(row + (uint64_t)(unsigned)i * (unsigned)es, es);
+  Raw r = SMEM ? load_raw_smem(row + i * es, es)
+               : load_raw(row + (uint64_t)(unsigned)i * (unsigned)es, es);
 #pragma unroll
   for (int c = 0; c < 4; ++c) {
     if (c < nch) {
@@ -112,18 +136,18 @@ __device__ __forceinline__ void nearest_at(const SampleParams& p, const char* ro
 
 // LINEAR from the texel rows: rows[0] = (j0,k0), [1] = (j1,k0), [2] = (j0,k1),
 // [3] = (j1,k1); blend x, then y, then z ([CL1.2 §8.2] weights, separable form)
-template <class C>
+template <class C, bool SMEM = false>
 __device__ __forceinline__ void linear_at(const SampleParams& p, const char* const rows[4],
                                           const bool rok[4], const AxL& x, float b, float omb,
-                                          float g, float omg, uint32_t res[4]) {
+                                          float g, float omg, uint32_t res[4], int outc = 4) {
   constexpr int NR = C::dims == 1 ? 1 : (C::dims == 2 ? 2 : 4);
   const int order = C::order == RT ? p.im.order : C::order;
   const int nch = C::nch == RT ? p.im.nch : C::nch;
   uint32_t t0[NR][4], t1[NR][4];
 #pragma unroll
   for (int r = 0; r < NR; ++r) {
-    fetch<C>(p.im, rows[r], x.i0, rok[r] && x.ok0, R_F, t0[r]);
-    fetch<C>(p.im, rows[r], x.i1, rok[r] && x.ok1, R_F, t1[r]);
+    fetch<C, SMEM>(p.im, rows[r], x.i0, rok[r] && x.ok0, R_F, t0[r]);
+    fetch<C, SMEM>(p.im, rows[r], x.i1, rok[r] && x.ok1, R_F, t1[r]);
   }
   uint32_t m[4];
 #pragma unroll
@@ -144,13 +168,14 @@ __device__ __forceinline__ void linear_at(const SampleParams& p, const char* con
   map_order(order, m, 0x3f800000u, res);
   // a NaN weight (non-finite coordinate) makes the spec's sum NaN in every
   // component, including the constant ones (reading A26)
-  if (x.a != x.a || b != b || g != g) res[0] = res[1] = res[2] = res[3] = 0x7fffffffu;
+  if (const_in_output(order, outc) && (x.a != x.a || b != b || g != g))
+    res[0] = res[1] = res[2] = res[3] = 0x7fffffffu;
 }
 
 // The built-in on one coordinate: c[0..DIMS-1] -> res (x,y,z,w) as 32-bit patterns.
 template <class C>
 __device__ __forceinline__ void read_image(const SampleParams& p, const float c[3],
-                                           uint32_t res[4]) {
+                                           uint32_t res[4], int outc = 4) {
   const Image& im = p.im;
   if (filt_of<C>(p) == F_NEAREST) {
     const AxN x = axis_n<C>(p.smp, c[0], im.w);
@@ -166,7 +191,7 @@ __device__ __forceinline__ void read_image(const SampleParams& p, const float c[
     const char* rows[4] = {row_ptr(im, y.i0, z.i0), row_ptr(im, y.i1, z.i0),
                            row_ptr(im, y.i0, z.i1), row_ptr(im, y.i1, z.i1)};
     const bool rok[4] = {y.ok0 && z.ok0, y.ok1 && z.ok0, y.ok0 && z.ok1, y.ok1 && z.ok1};
-    linear_at<C>(p, rows, rok, x, y.a, y.oma, z.a, z.oma, res);
+    linear_at<C>(p, rows, rok, x, y.a, y.oma, z.a, z.oma, res, outc);
   }
 }
 
@@ -205,7 +230,7 @@ __global__ void __launch_bounds__(256) k_sample_grid(const SampleParams p) {
   c[1] = C::dims > 1 ? affine_coord(p.A + 4, xf, yf, zf) : 0.f;
   c[2] = C::dims > 2 ? affine_coord(p.A + 8, xf, yf, zf) : 0.f;
   uint32_t r[4];
-  read_image<C>(p, c, r);
+  read_image<C>(p, c, r, OUTC == RT ? p.outc : OUTC);
   store_out<OUTC>(p, ((uint64_t)z * p.oh + y) * p.ow + x, r);
 }
 
@@ -252,7 +277,8 @@ __global__ void __launch_bounds__(128) k_sample_grid_sep(const SampleParams p) {
         const int x = x0 + 32 * t;
         if (x < p.ow) {
           uint32_t res[4];
-          linear_at<C>(p, rows, rok, ax[t], ay.a, ay.oma, az.a, az.oma, res);
+          linear_at<C>(p, rows, rok, ax[t], ay.a, ay.oma, az.a, az.oma, res,
+                       OUTC == RT ? p.outc : OUTC);
           store_out<OUTC>(p, obase + x, res);
         }
       }
@@ -271,6 +297,145 @@ __global__ void __launch_bounds__(128) k_sample_grid_sep(const SampleParams p) {
         }
       }
     }
+  }
+}
+
+// Separable map, LINEAR, compile-time format: register reuse along a walk.
+// Each warp walks consecutive outputs along the outermost image axis (y for
+// 2D, z for 3D) with lanes across x.  A step needs the texel rows at the
+// walk-axis indices (lo, hi) = (i0, i1); when step w+1's lo equals step w's
+// hi (a warp-uniform test) those rows are reused from registers, so a sample
+// costs half the taps (2 of 4 in 2D, 4 of 8 in 3D) in global loads.  The
+// loads of step w+1 are issued before step w is blended (software
+// pipelining), so a warp keeps two steps of loads in flight.  The values are
+// the same texels blended in the same order as linear_at, so the results are
+// bit-identical to the other kernels.
+//   2D: block = 32 x 4 threads, tile = (32*XPT) columns x (4*WALK) rows;
+//       warp w walks rows [y0 + w*WALK, +WALK).
+//   3D: tile = (32*XPT) columns x 4 rows x WALK slices; warp w owns one row
+//       and walks slices [z0, z0 + WALK).
+template <class C, int NJ, int XPT>
+struct WalkRows {  // converted texel values of the rows at one walk index
+  float v[NJ][XPT][C::nch][2];  // [row][column][channel][i0 / i1]
+};
+
+template <class C, int NJ, int XPT>
+__device__ __forceinline__ void walk_load(const Image& im, const AxL (&ax)[XPT], const AxL& afix,
+                                          int widx, bool wok, WalkRows<C, NJ, XPT>& out) {
+  constexpr bool D3 = C::dims == 3;
+#pragma unroll
+  for (int js = 0; js < NJ; ++js) {
+    const int j = D3 ? (js ? afix.i1 : afix.i0) : widx;
+    const int k = D3 ? widx : 0;
+    const bool rok = wok && (!D3 || (js ? afix.ok1 : afix.ok0));
+    const char* row = row_ptr(im, j, k);
+    uint32_t m0[XPT][4], m1[XPT][4];
+#pragma unroll
+    for (int t = 0; t < XPT; ++t) {
+      fetch<C>(im, row, ax[t].i0, rok && ax[t].ok0, R_F, m0[t]);
+      fetch<C>(im, row, ax[t].i1, rok && ax[t].ok1, R_F, m1[t]);
+    }
+#pragma unroll
+    for (int t = 0; t < XPT; ++t)
+#pragma unroll
+      for (int ch = 0; ch < C::nch; ++ch) {
+        out.v[js][t][ch][0] = __uint_as_float(m0[t][ch]);
+        out.v[js][t][ch][1] = __uint_as_float(m1[t][ch]);
+      }
+  }
+}
+
+template <class C, int OUTC, int XPT, int WALK>
+__global__ void __launch_bounds__(128) k_sample_grid_walk(const SampleParams p) {
+  static_assert(C::nch != RT && C::type != RT && C::order != RT, "compile-time format");
+  static_assert(C::dims >= 2, "walk needs a second axis");
+  constexpr int NCH = C::nch;
+  constexpr bool D3 = C::dims == 3;
+  constexpr int NJ = D3 ? 2 : 1;  // texel rows per walk index
+  using Rows = WalkRows<C, NJ, XPT>;
+  const Image& im = p.im;
+  // 3D: the 4 warps of a block split x (one texel row per block, wide DRAM bursts)
+  const int x0 = D3 ? blockIdx.x * (128 * XPT) + threadIdx.y * (32 * XPT) + threadIdx.x
+                    : blockIdx.x * (32 * XPT) + threadIdx.x;
+  AxL ax[XPT];
+#pragma unroll
+  for (int t = 0; t < XPT; ++t)
+    ax[t] = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(x0 + 32 * t)), p.A[3]),
+                      im.w);
+  // the fixed axis (3D: y) and the walk range
+  int yfix = 0, zfix = 0, w0;
+  AxL afix{0, 0, 0.f, 1.f, true, true};
+  if (D3) {
+    yfix = blockIdx.y;
+    if (yfix >= p.oh) return;  // warp-uniform
+    w0 = blockIdx.z * WALK;
+    afix = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(yfix)), p.A[7]), im.h);
+  } else {
+    zfix = blockIdx.z;
+    w0 = blockIdx.y * (4 * WALK) + threadIdx.y * WALK;
+  }
+  const int wlen = D3 ? p.od : p.oh;
+  if (w0 >= wlen) return;
+  const float awc = D3 ? p.A[10] : p.A[5], awo = D3 ? p.A[11] : p.A[7];
+  const int nw = D3 ? im.d : im.h;
+  auto walk_axis = [&](int wv) {
+    return axis_l<C>(p.smp, __fadd_rn(__fmul_rn(awc, __int2float_rn(wv)), awo), nw);
+  };
+  AxL aw = walk_axis(w0);
+  Rows lo, hi;
+  walk_load<C, NJ, XPT>(im, ax, afix, aw.i0, aw.ok0, lo);
+  walk_load<C, NJ, XPT>(im, ax, afix, aw.i1, aw.ok1, hi);
+#pragma unroll 1
+  for (int w = 0; w < WALK; ++w) {
+    const int wv = w0 + w;
+    // issue the next step's loads first
+    const bool next = w + 1 < WALK && wv + 1 < wlen;
+    AxL an = aw;
+    Rows nlo, nhi;
+    bool reuse = false;
+    if (next) {
+      an = walk_axis(wv + 1);
+      reuse = an.i0 == aw.i1 && an.ok0 == aw.ok1;
+      walk_load<C, NJ, XPT>(im, ax, afix, an.i1, an.ok1, nhi);
+      if (!reuse) walk_load<C, NJ, XPT>(im, ax, afix, an.i0, an.ok0, nlo);
+    }
+    // blend and store this step: x, then y, then z (as linear_at)
+    const AxL& ay = D3 ? afix : aw;
+    const float ga = D3 ? aw.a : 0.f, goma = D3 ? aw.oma : 1.f;
+    const int y = D3 ? yfix : wv, z = D3 ? wv : zfix;
+    const uint64_t obase = ((uint64_t)z * p.oh + y) * p.ow;
+#pragma unroll
+    for (int t = 0; t < XPT; ++t) {
+      const int x = x0 + 32 * t;
+      uint32_t m[4] = {0u, 0u, 0u, 0u};
+#pragma unroll
+      for (int ch = 0; ch < NCH; ++ch) {
+        const float a = ax[t].a, oma = ax[t].oma;
+        float o;
+        if (D3) {
+          // rows (j0,k0)=lo[0], (j1,k0)=lo[1], (j0,k1)=hi[0], (j1,k1)=hi[1]
+          const float r00 = lerp1(a, oma, lo.v[0][t][ch][0], lo.v[0][t][ch][1]);
+          const float r10 = lerp1(a, oma, lo.v[NJ - 1][t][ch][0], lo.v[NJ - 1][t][ch][1]);
+          const float r01 = lerp1(a, oma, hi.v[0][t][ch][0], hi.v[0][t][ch][1]);
+          const float r11 = lerp1(a, oma, hi.v[NJ - 1][t][ch][0], hi.v[NJ - 1][t][ch][1]);
+          o = lerp1(ga, goma, lerp1(ay.a, ay.oma, r00, r10), lerp1(ay.a, ay.oma, r01, r11));
+        } else {
+          const float r0 = lerp1(a, oma, lo.v[0][t][ch][0], lo.v[0][t][ch][1]);
+          const float r1 = lerp1(a, oma, hi.v[0][t][ch][0], hi.v[0][t][ch][1]);
+          o = lerp1(ay.a, ay.oma, r0, r1);
+        }
+        m[ch] = __float_as_uint(o);
+      }
+      uint32_t res[4];
+      map_order(C::order, m, 0x3f800000u, res);
+      if (const_in_output(C::order, OUTC) && (ax[t].a != ax[t].a || ay.a != ay.a || ga != ga))
+        res[0] = res[1] = res[2] = res[3] = 0x7fffffffu;
+      if (x < p.ow) store_out<OUTC>(p, obase + x, res);
+    }
+    if (!next) break;
+    lo = reuse ? hi : nlo;
+    hi = nhi;
+    aw = an;
   }
 }
 
@@ -307,6 +472,19 @@ static cudaError_t go_grid(const SampleParams& p, cudaStream_t st) {
   dim3 blk(32, 8, 1);
   dim3 grd((p.ow + 31) / 32, (p.oh + 7) / 8, p.od);
   k_sample_grid<C, OUTC><<<grd, blk, 0, st>>>(p);
+  count_launch();
+  return cudaGetLastError();
+}
+
+template <class C, int OUTC, int XPT, int WALK>
+static cudaError_t go_walk(const SampleParams& p, cudaStream_t st) {
+  dim3 blk(32, 4, 1);
+  dim3 grd;
+  if (C::dims == 3)
+    grd = dim3((p.ow + 128 * XPT - 1) / (128 * XPT), p.oh, (p.od + WALK - 1) / WALK);
+  else
+    grd = dim3((p.ow + 32 * XPT - 1) / (32 * XPT), (p.oh + 4 * WALK - 1) / (4 * WALK), p.od);
+  k_sample_grid_walk<C, OUTC, XPT, WALK><<<grd, blk, 0, st>>>(p);
   count_launch();
   return cudaGetLastError();
 }
@@ -356,10 +534,17 @@ static bool separable(const SampleParams& p) {
 cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st) {
   if (coord_mode == COORD_GRID) {
     if ((uint64_t)p.ow * p.oh * p.od == 0) return cudaSuccess;
-    if (separable(p)) {
-      if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_REPEAT, F_LINEAR)) return go_sep<C2Repeat, 4, 2, 4>(p, st);
-      if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_MIRROR, F_LINEAR)) return go_sep<C2Mirror, 4, 2, 4>(p, st);
-      if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR)) return go_sep<C3Cte, 1, 4, 4>(p, st);
+    // B2CL_GRID_KERNEL=general|sep|walk forces a kernel family (A/B runs under ncu);
+    // the default picks the variant measured fastest on B200 for each hot config
+    static const char* force = getenv("B2CL_GRID_KERNEL");
+    const int fk = !force ? 0 : (force[0] == 'g' ? 1 : (force[0] == 's' ? 2 : (force[0] == 'w' ? 3 : 0)));
+    if (separable(p) && fk != 1) {
+      if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_REPEAT, F_LINEAR))
+        return fk == 3 ? go_walk<C2Repeat, 4, 2, 8>(p, st) : go_sep<C2Repeat, 4, 2, 4>(p, st);
+      if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_MIRROR, F_LINEAR))
+        return fk == 3 ? go_walk<C2Mirror, 4, 2, 8>(p, st) : go_sep<C2Mirror, 4, 2, 4>(p, st);
+      if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR))
+        return fk == 2 ? go_sep<C3Cte, 1, 4, 4>(p, st) : go_walk<C3Cte, 1, 4, 16>(p, st);
       if (p.outc == 4 && matches<2>(p, T_UNORM8, O_RGBA, 0, A_CLAMP, F_NEAREST)) return go_sep<C1Clamp, 4, 2, 4>(p, st);
       switch (p.dims) {
         case 1: return go_sep<Generic<1>, RT, 2, 2>(p, st);

@@ -139,6 +139,13 @@ GRID_CASES = [
     (3, RGBA, F16, (12, 10, 9), (1, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR), "rotate3d", (17, 13, 11), 4),
     (2, RGBA, U8N, (64, 64, 1), (0, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_NEAREST), "rotate", (70, 66, 1), 4),
     (2, RG, F32, (33, 21, 1), (1, cl.CL_ADDRESS_NONE, cl.CL_FILTER_LINEAR), "translate", (40, 30, 3), 2),
+    # staged-footprint kernel: separable, non-wrapping, LINEAR (borders, scale != 1)
+    (3, R, F32, (30, 20, 12), (1, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_LINEAR), "stencil", (30, 20, 12), 1),
+    (3, R, F32, (30, 20, 12), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "scale2", (33, 21, 9), 1),
+    (2, RGBA, F16, (50, 40, 1), (1, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_LINEAR), "scale2", (31, 27, 1), 4),
+    (2, RGBA, F32, (64, 64, 1), (0, cl.CL_ADDRESS_NONE, cl.CL_FILTER_LINEAR), "unnorm", (96, 96, 1), 4),
+    (1, RGBA, U8N, (70, 1, 1), (0, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_LINEAR), "unnorm", (100, 3, 1), 4),
+    (2, R, S16N, (97, 61, 1), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "scale2", (300, 70, 1), 1),
     (2, RGBA, U8N, (64, 64, 1), (0, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_NEAREST), "unnorm", (96, 96, 1), 4),
     (2, BGRA, U8N, (31, 17, 1), (1, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_LINEAR), "rotate", (45, 29, 1), 3),
     (1, RG, F16, (50, 1, 1), (1, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR), "translate", (77, 1, 1), 2),
@@ -152,6 +159,12 @@ def _affine(kind, size, out):
         return synth.affine_translate_2d(W, H)
     if kind == "rotate":
         return synth.affine_rotate_2d(W, H, 30.0)
+    if kind == "scale2":  # 2x minification, separable, offset so edges hit the border
+        A = np.zeros(12, np.float32)
+        A[0], A[3] = 2.0 / W, -0.3 / W
+        A[5], A[7] = 2.0 / H, 0.45 / H
+        A[10], A[11] = 2.0 / D, -0.2 / D
+        return A
     if kind == "rotate3d":
         return synth.affine_rotate_3d(W, 20.0)
     if kind == "stencil":
