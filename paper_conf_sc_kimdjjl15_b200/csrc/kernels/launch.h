@@ -45,7 +45,7 @@ struct WriteParams {
   uint64_t n;
 };
 
-enum RectMode : int { RECT_COPY = 0, RECT_FILL = 1, RECT_FILL_IMAGE = 2 };
+enum RectMode : int { RECT_COPY = 0, RECT_FILL = 1, RECT_FILL_IMAGE = 2, RECT_COPY_ALIGNED = 3 };
 
 // Each launcher enqueues exactly one kernel (or none for empty work) on
 // `stream` and returns the launch status.

@@ -10,8 +10,9 @@
 // vectors spaced TX apart (coalesced).  Destination stores are always
 // 16-byte aligned vectors; the ragged head/tail of a row is stored byte by
 // byte.  A source that is misaligned relative to the destination (odd
-// origins or pitches) is read as two aligned 16-byte words and funnel-shifted
-// (the shift is constant along a row, so the branch is warp-uniform).
+// origins or pitches) is read as aligned 16-byte words -- one load per lane,
+// the next word by warp shuffle -- and funnel-shifted (the shift is constant
+// along a row and a warp covers one row, so the branch is warp-uniform).
 #include "../device/image.cuh"
 #include "launch.h"
 
@@ -22,12 +23,9 @@ __device__ __forceinline__ uint4 ld16(const char* p) {
   return __ldg(reinterpret_cast<const uint4*>(p));
 }
 
-// 16 bytes at S, where sh = S mod 16 (both aligned words contain needed
-// bytes, so neither leaves the source row's 16-byte blocks).
-__device__ __forceinline__ uint4 load_shifted(const char* S, int sh) {
-  if (sh == 0) return ld16(S);
-  const char* base = S - sh;
-  uint4 a = ld16(base), b = ld16(base + 16);
+// The 16 bytes starting sh bytes into the 32-byte pair (a, b) of consecutive
+// aligned source words (0 < sh < 16).
+__device__ __forceinline__ uint4 funnel16(const uint4& a, const uint4& b, int sh) {
   uint32_t w[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
   const int r = (sh & 3) * 8;
   uint4 o;
@@ -51,7 +49,8 @@ __device__ __forceinline__ uint4 load_shifted(const char* S, int sh) {
 template <int MODE, int U>
 __global__ void __launch_bounds__(256) k_rect(const RectParams p) {
   __shared__ uint4 tile[8];  // FILL modes: 128-byte pattern tile
-  if (MODE != RECT_COPY) {
+  constexpr bool COPY = MODE == RECT_COPY || MODE == RECT_COPY_ALIGNED;
+  if (!COPY) {
     if (MODE == RECT_FILL_IMAGE) {
       if (threadIdx.x == 0 && threadIdx.y == 0) {
         // convert the fill colour once with the write_image rules (A23) ...
@@ -72,16 +71,16 @@ __global__ void __launch_bounds__(256) k_rect(const RectParams p) {
     }
     __syncthreads();
   }
-  // Grid: x = chunk of a row (TX*U vectors), y = group of TY rows; each thread
-  // then walks rows with stride gridDim.y*TY (persistent in y), stepping its
-  // (z, y) row coordinates incrementally (no divisions in the loop).
+  // Grid: x = chunk of a row (TX*U vectors), y = group of TY rows; when there
+  // are more groups than the grid allows, a thread walks rows with stride
+  // gridDim.y*TY, stepping its (z, y) coordinates without divisions.
   const uint64_t v0 = (uint64_t)blockIdx.x * blockDim.x * U + threadIdx.x;
   uint64_t row = (uint64_t)blockIdx.y * blockDim.y + threadIdx.y;
   if (row >= p.rows) return;
   uint32_t z = (uint32_t)(row / p.R1), y = (uint32_t)(row - (uint64_t)z * p.R1);
   for (; row < p.rows; row += p.row_step) {
     char* drow = p.dst + z * p.dsp + y * p.drp;
-    const char* srow = MODE == RECT_COPY ? p.src + z * p.ssp + y * p.srp : nullptr;
+    const char* srow = COPY ? p.src + z * p.ssp + y * p.srp : nullptr;
     const uintptr_t dlo = reinterpret_cast<uintptr_t>(drow), dhi = dlo + p.R0;
     const uintptr_t abase = dlo & ~uintptr_t(15);
     const uint64_t nvec = ((dhi + 15) >> 4) - (abase >> 4);
@@ -90,13 +89,42 @@ __global__ void __launch_bounds__(256) k_rect(const RectParams p) {
     const uint64_t vf1 = (dhi >> 4) - (abase >> 4);
     const int sh = MODE == RECT_COPY ? (int)((reinterpret_cast<uintptr_t>(srow) - dlo) & 15) : 0;
     uint4 val[U];
+    if (MODE != RECT_COPY || sh == 0) {  // fills, aligned copies
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const uint64_t v = v0 + (uint64_t)u * blockDim.x;
-      if (v >= vf0 && v < vf1) {
-        const uintptr_t D = abase + 16 * v;
-        if (MODE == RECT_COPY) val[u] = load_shifted(srow + (D - dlo), sh);
-        else val[u] = tile[(D >> 4) & 7];
+      for (int u = 0; u < U; ++u) {
+        const uint64_t v = v0 + (uint64_t)u * blockDim.x;
+        if (v >= vf0 && v < vf1) {
+          const uintptr_t D = abase + 16 * v;
+          if (COPY) val[u] = ld16(srow + (D - dlo));
+          else val[u] = tile[(D >> 4) & 7];
+        }
+      }
+    } else if (MODE == RECT_COPY) {
+      // Misaligned source (warp-uniform: a warp covers one row): every lane
+      // loads the aligned source word under its own vector once; the word
+      // above comes from lane+1 by shuffle (lane 31, or a lane whose
+      // neighbour has no vector, loads it itself).  The head vector's word
+      // may lie before the row, so it is never loaded; every other word
+      // contains a byte of the row.
+      const unsigned lane = threadIdx.x & 31u;
+      uint4 w0[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const uint64_t v = v0 + (uint64_t)u * blockDim.x;
+        if (v >= vf0 && v < nvec) w0[u] = ld16(srow + (abase + 16 * v - dlo) - sh);
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const uint64_t v = v0 + (uint64_t)u * blockDim.x;
+        uint4 w1;
+        w1.x = __shfl_down_sync(0xffffffffu, w0[u].x, 1);
+        w1.y = __shfl_down_sync(0xffffffffu, w0[u].y, 1);
+        w1.z = __shfl_down_sync(0xffffffffu, w0[u].z, 1);
+        w1.w = __shfl_down_sync(0xffffffffu, w0[u].w, 1);
+        if (v >= vf0 && v < vf1) {
+          if (lane == 31u || v + 1 >= nvec) w1 = ld16(srow + (abase + 16 * v - dlo) - sh + 16);
+          val[u] = funnel16(w0[u], w1, sh);
+        }
       }
     }
 #pragma unroll
@@ -109,7 +137,7 @@ __global__ void __launch_bounds__(256) k_rect(const RectParams p) {
         const uintptr_t lo = D > dlo ? D : dlo, hi = D + 16 < dhi ? D + 16 : dhi;
         for (uintptr_t X = lo; X < hi; ++X) {
           unsigned char b;
-          if (MODE == RECT_COPY) b = static_cast<unsigned char>(srow[X - dlo]);
+          if (COPY) b = static_cast<unsigned char>(srow[X - dlo]);
           else b = reinterpret_cast<const unsigned char*>(tile)[X & 127];
           *reinterpret_cast<unsigned char*>(X) = b;
         }
@@ -128,31 +156,29 @@ cudaError_t launch_rect(RectParams& p, int mode, cudaStream_t st) {
   const uint64_t rows = (uint64_t)p.R1 * p.R2;
   if (p.R0 == 0 || rows == 0) return cudaSuccess;
   constexpr int U = 4;
-  static int nsm = 0;
-  if (nsm == 0) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-    if (nsm <= 0) nsm = 148;
-  }
   const uint64_t nvec_max = (p.R0 + 15) / 16 + 1;
   unsigned tx = 32;
   while (tx < 256 && (uint64_t)tx * U < nvec_max) tx *= 2;
   const unsigned ty = 256 / tx;
   const uint64_t cpr = (nvec_max + (uint64_t)tx * U - 1) / ((uint64_t)tx * U);
   const uint64_t groups = (rows + ty - 1) / ty;
-  // enough blocks for ~4 resident waves; rows beyond that are walked in-kernel
-  const uint64_t want = (uint64_t)nsm * 32;
-  uint64_t gy = cpr >= want ? 1 : (want + cpr - 1) / cpr;
-  if (gy > groups) gy = groups;
-  if (gy > 65535) gy = 65535;
+  // one block per (row group, chunk) up to the grid limit; beyond it rows are
+  // walked in-kernel (measured: short-lived blocks keep HBM busier than a
+  // persistent grid for plain copies)
+  const uint64_t gy = groups < 65535 ? groups : 65535;
   if (cpr > 0x7fffffffull) return cudaErrorInvalidValue;
   p.rows = rows;
   p.row_step = gy * ty;
   p.step_dz = (uint32_t)(p.row_step / p.R1);
   p.step_dy = (uint32_t)(p.row_step % p.R1);
   dim3 blk(tx, ty, 1), grd((unsigned)cpr, (unsigned)gy, 1);
+  // a copy whose source/destination misalignment is the same on every row
+  // and zero takes the shuffle-free instance
+  const bool aligned = mode == RECT_COPY && ((uintptr_t)p.src - (uintptr_t)p.dst) % 16 == 0 &&
+                       (p.srp - p.drp) % 16 == 0 && (p.ssp - p.dsp) % 16 == 0;
+  if (aligned) mode = RECT_COPY_ALIGNED;
   switch (mode) {
+    case RECT_COPY_ALIGNED: k_rect<RECT_COPY_ALIGNED, U><<<grd, blk, 0, st>>>(p); break;
     case RECT_COPY: k_rect<RECT_COPY, U><<<grd, blk, 0, st>>>(p); break;
     case RECT_FILL: k_rect<RECT_FILL, U><<<grd, blk, 0, st>>>(p); break;
     default: k_rect<RECT_FILL_IMAGE, U><<<grd, blk, 0, st>>>(p); break;
