@@ -264,16 +264,26 @@ def run_gpu(args):
     import torch.distributed as dist
 
     from paper_conf_sc_kimdjjl15_b200 import build, cl, synth
+    from paper_conf_sc_kimdjjl15_b200 import dist as bdist
     build.build()
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
+    # one GPU per rank; more ranks than GPUs only happens in the single-GPU
+    # rehearsal of the multi-rank path (ranks share a device, control plane on gloo)
+    ndev = torch.cuda.device_count()
+    gpu = local % ndev
+    shared = world > ndev
+    torch.cuda.set_device(gpu)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", gpu))
+    dev = torch.device("cuda", gpu)
+    red_dev = None if shared else dev  # device of the max-over-ranks tensors
     stream = torch.cuda.Stream(device=dev)
-    S = cl.Session(local, stream=stream.cuda_stream)
+    S = cl.Session(gpu, stream=stream.cuda_stream)
     L = cl.lib()
     T = Timer(torch, stream)
     hbm_peak, peak_src = peaks()
@@ -324,7 +334,7 @@ def run_gpu(args):
     torch.cuda.synchronize(dev)
     if world > 1:
         dist.barrier()
-    clocks = Clocks(local)
+    clocks = Clocks(gpu)
     clocks.start()
     n_launch0 = cl.launch_count()
     evs = []
@@ -345,9 +355,7 @@ def run_gpu(args):
                float(np.mean([e[1].elapsed_time(e[2]) for e in evs]))]
     ms_step = total_ms / args.steps
     if world > 1:
-        t = torch.tensor([ms_step], device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms_step = float(t.item())
+        ms_step = bdist.max_over_ranks(ms_step, red_dev)
     samples_step = 2 * N2D * N2D
     value = world * samples_step / (ms_step * 1e-3) / 1e9
     # algorithmic bytes per launch = distinct texels with a non-zero tap weight x 16 B
@@ -390,9 +398,7 @@ def run_gpu(args):
         torch.cuda.synchronize(dev)
         e2e_ms = a.elapsed_time(b) / steps_e2e
         if world > 1:
-            t = torch.tensor([e2e_ms], device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            e2e_ms = float(t.item())
+            e2e_ms = bdist.max_over_ranks(e2e_ms, red_dev)
         e2e = {"value": world * samples_step / (e2e_ms * 1e-3) / 1e9, "unit": "Gsamples/s",
                "ms_per_step": e2e_ms, "h2d_bytes_per_step": int(host_in.numel()),
                "d2h_bytes_per_step": 2 * nout}
@@ -400,6 +406,9 @@ def run_gpu(args):
     secondary = None
     if not args.no_secondary:
         secondary = run_secondary(S, L, T, torch, dev, hbm_peak, args)
+    if world > 1 and not args.no_p2p:
+        secondary = secondary or {}
+        secondary["p2p_ring_migrate"] = run_p2p_ring(S, L, T, torch, dev, red_dev, rank, world)
 
     cpu = None
     if rank == 0 and not args.no_cpu:
@@ -443,6 +452,51 @@ def run_gpu(args):
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def run_p2p_ring(S, L, T, torch, dev, red_dev, rank, world):
+    """Config 5 migration, one process per GPU: every rank exports an
+    IPC-exportable band buffer, opens its left neighbour's band over CUDA IPC
+    and pulls it with the library's SM copy kernel (clEnqueueCopyBuffer on the
+    peer mapping -> NVLink reads), all ranks concurrently (ring shift).  Band =
+    32768^2 RGBA32F / G rows, capped at 2 GiB.  Reported: GB/s per GPU (the
+    slowest rank) and its fraction of the 770 GB/s measured peer-copy figure
+    (B200_PROFILING.md; 900 GB/s nominal)."""
+    from paper_conf_sc_kimdjjl15_b200 import cl
+    from paper_conf_sc_kimdjjl15_b200 import dist as bdist
+    band = min((32768 * 32768 * 16) // world, 2 << 30)
+    err = ctypes.c_int32()
+    mine = L.clCreateBuffer(S.ctx, cl.CL_MEM_READ_WRITE | cl.B2CL_MEM_IPC_EXPORTABLE, band, None,
+                            ctypes.byref(err))
+    cl.check(err.value, "clCreateBuffer(IPC)")
+    pat = np.array([rank & 0xFF], np.uint8)
+    cl.check(L.clEnqueueFillBuffer(S.queue, mine, pat.ctypes.data, 1, 0, band, 0, None, None))
+    S.finish()
+    h = (ctypes.c_uint8 * 64)()
+    cl.check(L.b2clGetMemIpcHandle(mine, h), "b2clGetMemIpcHandle")
+    handles = bdist.exchange_bytes(bytes(h))
+    left, _ = bdist.ring_neighbors(rank, world)
+    hl = (ctypes.c_uint8 * 64).from_buffer_copy(handles[left])
+    peer = L.b2clCreateBufferFromIpcHandle(S.ctx, S.device, hl, band, ctypes.byref(err))
+    cl.check(err.value, "b2clCreateBufferFromIpcHandle")
+    local = S.buffer(band)
+
+    def pull():
+        cl.check(L.clEnqueueCopyBuffer(S.queue, peer, local, 0, 0, band, 0, None, None))
+    pull()
+    S.finish()
+    ok = bool(np.all(S.read(local, 4096) == (left & 0xFF)))  # data equality (O9) on a sample
+    import torch.distributed as dist
+    dist.barrier()
+    ms = _time_launches(T, torch, dev, pull, 5)
+    ms = bdist.max_over_ranks(ms, red_dev)
+    gbs = band / (ms * 1e-3) / 1e9
+    S.release(local, peer, mine)
+    return {"band_bytes": band, "ms": ms, "GB/s_per_gpu": gbs, "frac_of_770": gbs / 770.0,
+            "pattern": "ring shift, all ranks pull from rank-1 concurrently",
+            "data_check": "ok" if ok else "MISMATCH",
+            "link": ("NVLink P2P (peer GPU memory over CUDA IPC)" if red_dev is not None else
+                     "same GPU (multi-rank rehearsal with ranks sharing one device: not NVLink)")}
 
 
 def _time_launches(T, torch, dev, fn, iters):
@@ -531,6 +585,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--full-sweep", action="store_true")
+    ap.add_argument("--no-p2p", action="store_true", help="skip the N>1 NVLink ring migration")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
