@@ -72,6 +72,37 @@ cl_int b2clEnqueueReadImageGrid(cl_command_queue command_queue, cl_mem image,
                                 size_t out_offset, cl_uint num_events_in_wait_list,
                                 const cl_event* event_wait_list, cl_event* event);
 
+/* The same over the output sub-box out_origin + [0, out_region): sample
+ * (x,y,z) uses output indices (out_origin[0]+x, out_origin[1]+y,
+ * out_origin[2]+z) in the affine map -- so a band of a larger output is
+ * bit-identical to the same rows of the whole grid -- and is stored at
+ * [z][y][x][c] of the region.  origin + region must stay below 2^31. */
+cl_int b2clEnqueueReadImageGridRegion(cl_command_queue command_queue, cl_mem image,
+                                      cl_sampler sampler, b2cl_rtype rtype, const float* affine,
+                                      const size_t* out_origin, const size_t* out_region,
+                                      cl_uint out_channels, cl_mem out, size_t out_offset,
+                                      cl_uint num_events_in_wait_list,
+                                      const cl_event* event_wait_list, cl_event* event);
+
+/* An image SHARD: rows [begin, begin+count) (2D) or slices (3D) of a global
+ * image described by global_desc, plus `halo` rows/slices on each side
+ * (wrapping around the global extent), stored as a plain image of
+ * count + 2*halo rows/slices: stored row s holds global row
+ * (begin - halo + s) mod extent (row-sharded images).
+ * The read built-ins (b2clEnqueueReadImage*) address the GLOBAL image --
+ * global normalization, wrap and border -- and subtract the shard's first
+ * stored row from the integer index only, so a shard reads bit-identically
+ * to the whole image wherever its band + halo covers the filter footprint (a
+ * tap outside it reads the nearest stored row; it is the caller's job to
+ * provide the halo).  Every other operation (write_image, copies, fills,
+ * Read/WriteImage, clGetImageInfo) addresses the stored rows as a plain
+ * image.  count + 2*halo <= extent; 1D images cannot be sharded.
+ * Errors as clCreateImage, and CL_INVALID_VALUE for a bad band. */
+cl_mem b2clCreateImageShard(cl_context context, cl_mem_flags flags,
+                            const cl_image_format* image_format,
+                            const cl_image_desc* global_desc, size_t begin, size_t count,
+                            size_t halo, void* host_ptr, cl_int* errcode_ret);
+
 /* write_image{f,i,ui}(image, int coord, color) for n samples
  * ([CL1.2 §6.12.14.4, §8.3]; step a8).  int_coords: n x {1,2,4} int32 at
  * coords_offset; colors: n x 16 bytes at colors_offset (multiple of 16).

@@ -15,7 +15,8 @@ from ctypes import POINTER, byref, c_float, c_int32, c_size_t, c_uint32, c_uint6
 
 import numpy as np
 
-LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libb2cl.so")
+LIB_PATH = os.environ.get("B2CL_LIB") or os.path.join(os.path.dirname(os.path.abspath(__file__)),
+                                                    "libb2cl.so")  # B2CL_LIB: A/B builds
 
 # ---- Khronos / b2cl constants (restated from include/*.h) ----
 CL_SUCCESS = 0
@@ -106,6 +107,9 @@ PROTOTYPES = {
                                          POINTER(_H)]),
     "b2clEnqueueReadImageGrid": (_I, [_H, _H, _H, _U, POINTER(c_float), _SZ3, _U, _H, _S, _U,
                                       POINTER(_H), POINTER(_H)]),
+    "b2clEnqueueReadImageGridRegion": (_I, [_H, _H, _H, _U, POINTER(c_float), _SZ3, _SZ3, _U, _H,
+                                            _S, _U, POINTER(_H), POINTER(_H)]),
+    "b2clCreateImageShard": (_H, [_H, _L, _P, _P, _S, _S, _S, _P, _PI]),
     "b2clEnqueueWriteImageSamples": (_I, [_H, _H, _U, _H, _S, _S, _H, _S, _U, POINTER(_H),
                                           POINTER(_H)]),
     "b2clCreateCommandQueueWithStream": (_H, [_H, _H, _P, _L, _PI]),
@@ -155,7 +159,9 @@ def lib():
                                "`python -m paper_conf_sc_kimdjjl15_b200.build` (no CPU fallback)")
         L = ctypes.CDLL(LIB_PATH)
         for name, (res, args) in PROTOTYPES.items():
-            f = getattr(L, name)
+            f = getattr(L, name, None)
+            if f is None:  # an older A/B build (B2CL_LIB); the ABI test checks the real one
+                continue
             f.restype = res
             f.argtypes = args
         _lib = L
@@ -290,6 +296,26 @@ class Session:
         else:
             m = lib().clCreateImage(self.ctx, flags, byref(fmt), byref(desc), None, byref(err))
         check(err.value, "clCreateImage")
+        return m
+
+    def image_shard(self, order: int, type_: int, width: int, height: int, depth: int,
+                    begin: int, count: int, halo: int = 0, host: np.ndarray | None = None,
+                    flags: int = CL_MEM_READ_WRITE):
+        """Rows [begin, begin+count) (+halo) of a global width x height (x depth) image;
+        `host` holds the stored rows/slices, tightly packed."""
+        dims = 3 if depth else 2
+        fmt = ImageFormat(order, type_)
+        desc = ImageDesc(CL_MEM_OBJECT_IMAGE3D if dims == 3 else CL_MEM_OBJECT_IMAGE2D, width,
+                         height, depth, 0, 0, 0, 0, 0, None)
+        err = c_int32()
+        if host is not None:
+            host = np.ascontiguousarray(host)
+            m = lib().b2clCreateImageShard(self.ctx, flags | CL_MEM_COPY_HOST_PTR, byref(fmt),
+                                           byref(desc), begin, count, halo, _ptr(host), byref(err))
+        else:
+            m = lib().b2clCreateImageShard(self.ctx, flags, byref(fmt), byref(desc), begin, count,
+                                           halo, None, byref(err))
+        check(err.value, "b2clCreateImageShard")
         return m
 
     def sampler(self, normalized: bool, addressing: int, filt: int):

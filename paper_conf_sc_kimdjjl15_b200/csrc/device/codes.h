@@ -27,10 +27,15 @@ constexpr int RT = -1;  // "decided at run time" template value
 
 struct Image {            // the CLImage of Fig. 6, device view
   char* ptr;
-  int w, h, d;            // unused dimensions are 1
+  int w, h, d;            // unused dimensions are 1 (global extent for a shard)
   int type, order;        // TypeCode / OrderCode
   int es, nch;            // elem_size, channels
   uint64_t rp, sp;        // row_pitch, slice_pitch (bytes)
+  // Outer axis (rows of a 2D image, slices of a 3D image) as stored: storage
+  // row s holds global index (ob + s) mod (outer extent), s < os.  A plain
+  // image has ob = 0 and os = its extent; a shard (b2clCreateImageShard)
+  // stores its band plus halo rows of a larger global image.
+  int ob, os;
 };
 
 struct Sampler {

@@ -15,7 +15,8 @@ struct SampleParams {
   int rclass;       // dev::RetCode
   int dims;         // 1..3
   float A[12];      // grid: affine coordinate map
-  int ow, oh, od;   // grid: output dims
+  int ow, oh, od;   // grid: output region dims
+  int ox, oy, oz;   // grid: output region origin (coordinates use origin + index)
   int outc;         // grid: output channels 1..4
   const char* coords;  // list: coordinates (already offset)
   uint64_t n;          // list: number of samples

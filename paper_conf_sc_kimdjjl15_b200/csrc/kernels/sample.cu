@@ -33,6 +33,12 @@ struct Cfg {
   static constexpr int nch = ORDER == RT ? RT : order_channels(ORDER);
 };
 
+// C with the image-shard row mapping compiled in (SH) or out (plain images)
+template <class C, bool SH>
+struct WithShard : C {
+  static constexpr bool shard = SH;
+};
+
 struct AxN {  // NEAREST, one axis
   int i;
   bool ok;
@@ -76,7 +82,23 @@ __device__ __forceinline__ int filt_of(const SampleParams& p) {
 }
 
 // start of texel row (j,k): ptr + k*slice_pitch + j*row_pitch (Fig. 6)
+// The outer index o (j of a 2D image, k of a 3D image) is a global index; its
+// storage row is (o - ob) mod extent, clamped into the stored rows (a tap
+// outside a shard's band + halo reads the nearest stored row: the caller
+// provides the halo; this only keeps the access in bounds).
+__device__ __forceinline__ int storage_row(const Image& im, int o, int extent) {
+  int l = o - im.ob;
+  l += l < 0 ? extent : 0;
+  l -= l >= extent ? extent : 0;
+  return min(max(l, 0), im.os - 1);
+}
+
+template <class C>
 __device__ __forceinline__ const char* row_ptr(const Image& im, int j, int k) {
+  if constexpr (C::shard) {
+    if (C::dims == 3) k = storage_row(im, k, im.d);
+    else if (C::dims == 2) j = storage_row(im, j, im.h);
+  }
   const char* r = im.ptr + (uint64_t)(unsigned)k * im.sp + (uint64_t)(unsigned)j * im.rp;
   // keep the absolute row pointer in registers: without this the compiler
   // re-associates ptr + (row + i*es) and pays two extra 64-bit adds per tap
@@ -182,14 +204,14 @@ __device__ __forceinline__ void read_image(const SampleParams& p, const float c[
     AxN y{0, true}, z{0, true};
     if (C::dims > 1) y = axis_n<C>(p.smp, c[1], im.h);
     if (C::dims > 2) z = axis_n<C>(p.smp, c[2], im.d);
-    nearest_at<C>(p, row_ptr(im, y.i, z.i), x, y.ok && z.ok, res);
+    nearest_at<C>(p, row_ptr<C>(im, y.i, z.i), x, y.ok && z.ok, res);
   } else {
     const AxL x = axis_l<C>(p.smp, c[0], im.w);
     AxL y{0, 0, 0.f, 1.f, true, true}, z{0, 0, 0.f, 1.f, true, true};
     if (C::dims > 1) y = axis_l<C>(p.smp, c[1], im.h);
     if (C::dims > 2) z = axis_l<C>(p.smp, c[2], im.d);
-    const char* rows[4] = {row_ptr(im, y.i0, z.i0), row_ptr(im, y.i1, z.i0),
-                           row_ptr(im, y.i0, z.i1), row_ptr(im, y.i1, z.i1)};
+    const char* rows[4] = {row_ptr<C>(im, y.i0, z.i0), row_ptr<C>(im, y.i1, z.i0),
+                           row_ptr<C>(im, y.i0, z.i1), row_ptr<C>(im, y.i1, z.i1)};
     const bool rok[4] = {y.ok0 && z.ok0, y.ok1 && z.ok0, y.ok0 && z.ok1, y.ok1 && z.ok1};
     linear_at<C>(p, rows, rok, x, y.a, y.oma, z.a, z.oma, res, outc);
   }
@@ -224,7 +246,8 @@ __global__ void __launch_bounds__(256) k_sample_grid(const SampleParams p) {
   const int y = blockIdx.y * blockDim.y + threadIdx.y;
   const int z = blockIdx.z;
   if (x >= p.ow || y >= p.oh) return;
-  const float xf = __int2float_rn(x), yf = __int2float_rn(y), zf = __int2float_rn(z);
+  const float xf = __int2float_rn(p.ox + x), yf = __int2float_rn(p.oy + y),
+              zf = __int2float_rn(p.oz + z);
   float c[3];
   c[0] = affine_coord(p.A, xf, yf, zf);
   c[1] = C::dims > 1 ? affine_coord(p.A + 4, xf, yf, zf) : 0.f;
@@ -237,7 +260,7 @@ __global__ void __launch_bounds__(256) k_sample_grid(const SampleParams p) {
 // Separable maps: block = 32 x 4 threads; tile = (32*XPT) columns x (4*RPW) rows
 // of one output slice.  Lane -> columns lane + 32*t, warp -> RPW consecutive rows.
 template <class C, int OUTC, int XPT, int RPW>
-__global__ void __launch_bounds__(128) k_sample_grid_sep(const SampleParams p) {
+__global__ void __launch_bounds__(128, 12) k_sample_grid_sep(const SampleParams p) {
   const Image& im = p.im;
   const int z = blockIdx.z;
   const int x0 = blockIdx.x * (32 * XPT) + threadIdx.x;
@@ -248,7 +271,7 @@ __global__ void __launch_bounds__(128) k_sample_grid_sep(const SampleParams p) {
   AxN nx[XPT];
 #pragma unroll
   for (int t = 0; t < XPT; ++t) {
-    const float s = __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(x0 + 32 * t)), p.A[3]);
+    const float s = __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(p.ox + x0 + 32 * t)), p.A[3]);
     if (lin) ax[t] = axis_l<C>(p.smp, s, im.w);
     else nx[t] = axis_n<C>(p.smp, s, im.w);
   }
@@ -256,7 +279,7 @@ __global__ void __launch_bounds__(128) k_sample_grid_sep(const SampleParams p) {
   AxL az{0, 0, 0.f, 1.f, true, true};
   AxN nz{0, true};
   if (C::dims > 2) {
-    const float s = __fadd_rn(__fmul_rn(p.A[10], __int2float_rn(z)), p.A[11]);
+    const float s = __fadd_rn(__fmul_rn(p.A[10], __int2float_rn(p.oz + z)), p.A[11]);
     if (lin) az = axis_l<C>(p.smp, s, im.d);
     else nz = axis_n<C>(p.smp, s, im.d);
   }
@@ -268,9 +291,9 @@ __global__ void __launch_bounds__(128) k_sample_grid_sep(const SampleParams p) {
     if (lin) {
       AxL ay{0, 0, 0.f, 1.f, true, true};
       if (C::dims > 1)
-        ay = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(y)), p.A[7]), im.h);
-      const char* rows[4] = {row_ptr(im, ay.i0, az.i0), row_ptr(im, ay.i1, az.i0),
-                             row_ptr(im, ay.i0, az.i1), row_ptr(im, ay.i1, az.i1)};
+        ay = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(p.oy + y)), p.A[7]), im.h);
+      const char* rows[4] = {row_ptr<C>(im, ay.i0, az.i0), row_ptr<C>(im, ay.i1, az.i0),
+                             row_ptr<C>(im, ay.i0, az.i1), row_ptr<C>(im, ay.i1, az.i1)};
       const bool rok[4] = {ay.ok0 && az.ok0, ay.ok1 && az.ok0, ay.ok0 && az.ok1, ay.ok1 && az.ok1};
 #pragma unroll
       for (int t = 0; t < XPT; ++t) {
@@ -285,8 +308,8 @@ __global__ void __launch_bounds__(128) k_sample_grid_sep(const SampleParams p) {
     } else {
       AxN ny{0, true};
       if (C::dims > 1)
-        ny = axis_n<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(y)), p.A[7]), im.h);
-      const char* row = row_ptr(im, ny.i, nz.i);
+        ny = axis_n<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(p.oy + y)), p.A[7]), im.h);
+      const char* row = row_ptr<C>(im, ny.i, nz.i);
 #pragma unroll
       for (int t = 0; t < XPT; ++t) {
         const int x = x0 + 32 * t;
@@ -328,7 +351,7 @@ __device__ __forceinline__ void walk_load(const Image& im, const AxL (&ax)[XPT],
     const int j = D3 ? (js ? afix.i1 : afix.i0) : widx;
     const int k = D3 ? widx : 0;
     const bool rok = wok && (!D3 || (js ? afix.ok1 : afix.ok0));
-    const char* row = row_ptr(im, j, k);
+    const char* row = row_ptr<C>(im, j, k);
     uint32_t m0[XPT][4], m1[XPT][4];
 #pragma unroll
     for (int t = 0; t < XPT; ++t) {
@@ -360,7 +383,7 @@ __global__ void __launch_bounds__(128) k_sample_grid_walk(const SampleParams p) 
   AxL ax[XPT];
 #pragma unroll
   for (int t = 0; t < XPT; ++t)
-    ax[t] = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(x0 + 32 * t)), p.A[3]),
+    ax[t] = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(p.ox + x0 + 32 * t)), p.A[3]),
                       im.w);
   // the fixed axis (3D: y) and the walk range
   int yfix = 0, zfix = 0, w0;
@@ -369,7 +392,7 @@ __global__ void __launch_bounds__(128) k_sample_grid_walk(const SampleParams p) 
     yfix = blockIdx.y;
     if (yfix >= p.oh) return;  // warp-uniform
     w0 = blockIdx.z * WALK;
-    afix = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(yfix)), p.A[7]), im.h);
+    afix = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(p.oy + yfix)), p.A[7]), im.h);
   } else {
     zfix = blockIdx.z;
     w0 = blockIdx.y * (4 * WALK) + threadIdx.y * WALK;
@@ -378,8 +401,9 @@ __global__ void __launch_bounds__(128) k_sample_grid_walk(const SampleParams p) 
   if (w0 >= wlen) return;
   const float awc = D3 ? p.A[10] : p.A[5], awo = D3 ? p.A[11] : p.A[7];
   const int nw = D3 ? im.d : im.h;
+  const int wor = D3 ? p.oz : p.oy;  // origin of the output region along the walk
   auto walk_axis = [&](int wv) {
-    return axis_l<C>(p.smp, __fadd_rn(__fmul_rn(awc, __int2float_rn(wv)), awo), nw);
+    return axis_l<C>(p.smp, __fadd_rn(__fmul_rn(awc, __int2float_rn(wor + wv)), awo), nw);
   };
   AxL aw = walk_axis(w0);
   Rows lo, hi;
@@ -467,11 +491,18 @@ __global__ void __launch_bounds__(256) k_sample_list(const SampleParams p) {
 }
 
 // ---------------------------------------------------------------- dispatch
+// a shard stores a window of the outer axis (b2clCreateImageShard)
+static bool is_shard(const SampleParams& p) {
+  if (p.dims < 2) return false;
+  return p.im.ob != 0 || p.im.os != (p.dims == 3 ? p.im.d : p.im.h);
+}
+
 template <class C, int OUTC>
 static cudaError_t go_grid(const SampleParams& p, cudaStream_t st) {
   dim3 blk(32, 8, 1);
   dim3 grd((p.ow + 31) / 32, (p.oh + 7) / 8, p.od);
-  k_sample_grid<C, OUTC><<<grd, blk, 0, st>>>(p);
+  if (is_shard(p)) k_sample_grid<WithShard<C, true>, OUTC><<<grd, blk, 0, st>>>(p);
+  else k_sample_grid<WithShard<C, false>, OUTC><<<grd, blk, 0, st>>>(p);
   count_launch();
   return cudaGetLastError();
 }
@@ -484,7 +515,8 @@ static cudaError_t go_walk(const SampleParams& p, cudaStream_t st) {
     grd = dim3((p.ow + 128 * XPT - 1) / (128 * XPT), p.oh, (p.od + WALK - 1) / WALK);
   else
     grd = dim3((p.ow + 32 * XPT - 1) / (32 * XPT), (p.oh + 4 * WALK - 1) / (4 * WALK), p.od);
-  k_sample_grid_walk<C, OUTC, XPT, WALK><<<grd, blk, 0, st>>>(p);
+  if (is_shard(p)) k_sample_grid_walk<WithShard<C, true>, OUTC, XPT, WALK><<<grd, blk, 0, st>>>(p);
+  else k_sample_grid_walk<WithShard<C, false>, OUTC, XPT, WALK><<<grd, blk, 0, st>>>(p);
   count_launch();
   return cudaGetLastError();
 }
@@ -493,7 +525,8 @@ template <class C, int OUTC, int XPT, int RPW>
 static cudaError_t go_sep(const SampleParams& p, cudaStream_t st) {
   dim3 blk(32, 4, 1);
   dim3 grd((p.ow + 32 * XPT - 1) / (32 * XPT), (p.oh + 4 * RPW - 1) / (4 * RPW), p.od);
-  k_sample_grid_sep<C, OUTC, XPT, RPW><<<grd, blk, 0, st>>>(p);
+  if (is_shard(p)) k_sample_grid_sep<WithShard<C, true>, OUTC, XPT, RPW><<<grd, blk, 0, st>>>(p);
+  else k_sample_grid_sep<WithShard<C, false>, OUTC, XPT, RPW><<<grd, blk, 0, st>>>(p);
   count_launch();
   return cudaGetLastError();
 }
@@ -501,8 +534,16 @@ static cudaError_t go_sep(const SampleParams& p, cudaStream_t st) {
 template <class C>
 static cudaError_t go_list(const SampleParams& p, bool int_coord, cudaStream_t st) {
   const uint64_t blocks = (p.n + 255) / 256;
-  if (int_coord) k_sample_list<C, true><<<(unsigned)blocks, 256, 0, st>>>(p);
-  else k_sample_list<C, false><<<(unsigned)blocks, 256, 0, st>>>(p);
+  using Cs = WithShard<C, true>;
+  using Cp = WithShard<C, false>;
+  const bool sh = is_shard(p);
+  if (int_coord) {
+    if (sh) k_sample_list<Cs, true><<<(unsigned)blocks, 256, 0, st>>>(p);
+    else k_sample_list<Cp, true><<<(unsigned)blocks, 256, 0, st>>>(p);
+  } else {
+    if (sh) k_sample_list<Cs, false><<<(unsigned)blocks, 256, 0, st>>>(p);
+    else k_sample_list<Cp, false><<<(unsigned)blocks, 256, 0, st>>>(p);
+  }
   count_launch();
   return cudaGetLastError();
 }

@@ -63,7 +63,13 @@ struct _cl_mem {
   cl_mem_flags flags;
   size_t size = 0;        // CL_MEM_SIZE (user size; images: total bytes)
   size_t alloc_size = 0;  // rounded to 256 B
-  ImageLayout img{};      // images only
+  ImageLayout img{};      // images only (a shard: the layout of its stored rows)
+  // image shards (b2clCreateImageShard): the outer axis (2D rows / 3D slices)
+  // of a global image of extent shard_extent; stored row s is global index
+  // (shard_ob + s) mod shard_extent
+  bool shard = false;
+  size_t shard_extent = 0;
+  long long shard_ob = 0;
   cl_image_format fmt{};
   cl_image_desc desc{};
   std::mutex mu;
@@ -635,6 +641,35 @@ extern "C" cl_mem clCreateImage(cl_context c, cl_mem_flags flags, const cl_image
   return m;
 }
 
+extern "C" cl_mem b2clCreateImageShard(cl_context c, cl_mem_flags flags, const cl_image_format* fmt,
+                                       const cl_image_desc* global_desc, size_t begin,
+                                       size_t count, size_t halo, void* host_ptr,
+                                       cl_int* errcode_ret) {
+  if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
+  if (!global_desc) { SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR); return nullptr; }
+  ImageLayout G;
+  cl_int st = image_layout(fmt, global_desc, &G);
+  if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
+  if (G.dims < 2) { SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR); return nullptr; }
+  const size_t extent = G.dims == 3 ? G.d : G.h;
+  // the band may wrap around the global extent (begin + count > extent)
+  if (count == 0 || begin >= extent || count + 2 * halo > extent ||
+      global_desc->image_row_pitch || global_desc->image_slice_pitch) {
+    SET_ERR(CL_INVALID_VALUE);
+    return nullptr;
+  }
+  // the stored rows as a plain image of count + 2*halo rows (or slices)
+  cl_image_desc sd = *global_desc;
+  if (G.dims == 3) sd.image_depth = count + 2 * halo;
+  else sd.image_height = count + 2 * halo;
+  cl_mem m = clCreateImage(c, flags, fmt, &sd, host_ptr, errcode_ret);
+  if (!m) return nullptr;
+  m->shard = true;
+  m->shard_extent = extent;
+  m->shard_ob = (long long)begin - (long long)halo;
+  return m;
+}
+
 extern "C" cl_int clGetSupportedImageFormats(cl_context c, cl_mem_flags flags,
                                              cl_mem_object_type type, cl_uint num_entries,
                                              cl_image_format* formats, cl_uint* num_formats) {
@@ -968,7 +1003,10 @@ static cl_int check_queue_mem(cl_command_queue q, cl_mem m) {
     if (_s != CL_SUCCESS) return _s;    \
   } while (0)
 
-static dev::Image dev_image(cl_mem m, char* ptr) {
+// Device view of an image.  For the read built-ins (sampling) a shard
+// presents its global extent on the outer axis with the stored window (ob,
+// os); every other operation addresses the stored rows as a plain image.
+static dev::Image dev_image(cl_mem m, char* ptr, bool sampling = false) {
   dev::Image im{};
   const ImageLayout& L = m->img;
   im.ptr = ptr;
@@ -981,6 +1019,13 @@ static dev::Image dev_image(cl_mem m, char* ptr) {
   im.nch = L.fmt.nch;
   im.rp = L.row_pitch;
   im.sp = L.slice_pitch;
+  im.ob = 0;
+  im.os = L.dims == 3 ? im.d : im.h;
+  if (sampling && m->shard) {
+    im.ob = (int)m->shard_ob;
+    if (L.dims == 3) im.d = (int)m->shard_extent;
+    else im.h = (int)m->shard_extent;
+  }
   return im;
 }
 
@@ -1410,7 +1455,7 @@ extern "C" cl_int b2clEnqueueReadImageSamples(cl_command_queue q, cl_mem img, cl
   CHECK(resident(out, q, true, &po));
   CHECK(enq_begin(E, nw, wl));
   SampleParams p{};
-  p.im = dev_image(img, pi);
+  p.im = dev_image(img, pi, true);
   fill_sampler(p, smp);
   p.rclass = (int)rtype;
   p.dims = dims;
@@ -1423,22 +1468,26 @@ extern "C" cl_int b2clEnqueueReadImageSamples(cl_command_queue q, cl_mem img, cl
   return st;
 }
 
-extern "C" cl_int b2clEnqueueReadImageGrid(cl_command_queue q, cl_mem img, cl_sampler smp,
-                                           b2cl_rtype rtype, const float* affine,
-                                           const size_t* out_dims, cl_uint outc, cl_mem out,
-                                           size_t ooffset, cl_uint nw, const cl_event* wl,
-                                           cl_event* ev) {
+extern "C" cl_int b2clEnqueueReadImageGridRegion(cl_command_queue q, cl_mem img, cl_sampler smp,
+                                                 b2cl_rtype rtype, const float* affine,
+                                                 const size_t* out_origin, const size_t* out_region,
+                                                 cl_uint outc, cl_mem out, size_t ooffset,
+                                                 cl_uint nw, const cl_event* wl, cl_event* ev) {
   if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
   CHECK(image_info_checked(q, img));
   if (!live(g_samplers, smp) || smp->ctx != q->ctx) return CL_INVALID_SAMPLER;
   CHECK(check_queue_mem(q, out));
   if (out->type != CL_MEM_OBJECT_BUFFER) return CL_INVALID_MEM_OBJECT;
   CHECK(check_read_combo(img, smp, rtype));
-  if (!affine || !out_dims || outc < 1 || outc > 4 || ooffset % 16 != 0) return CL_INVALID_VALUE;
-  if (out_dims[0] > 0x7fffffff || out_dims[1] > 0x7fffffff || out_dims[2] > 65535)
+  if (!affine || !out_origin || !out_region || outc < 1 || outc > 4 || ooffset % 16 != 0)
     return CL_INVALID_VALUE;
+  // output indices origin + [0, region) must be exact int32 -> float conversions' domain
+  for (int k = 0; k < 3; ++k)
+    if (out_origin[k] > 0x7fffffff || out_region[k] > 0x7fffffff - out_origin[k])
+      return CL_INVALID_VALUE;
+  if (out_region[2] > 65535) return CL_INVALID_VALUE;
   const unsigned __int128 bytes =
-      (unsigned __int128)out_dims[0] * out_dims[1] * out_dims[2] * outc * 4;
+      (unsigned __int128)out_region[0] * out_region[1] * out_region[2] * outc * 4;
   if (ooffset > out->size || bytes > out->size - ooffset) return CL_INVALID_VALUE;
   CHECK(check_wait_list(q, nw, wl));
   Enq E;
@@ -1451,19 +1500,32 @@ extern "C" cl_int b2clEnqueueReadImageGrid(cl_command_queue q, cl_mem img, cl_sa
   CHECK(resident(out, q, true, &po));
   CHECK(enq_begin(E, nw, wl));
   SampleParams p{};
-  p.im = dev_image(img, pi);
+  p.im = dev_image(img, pi, true);
   fill_sampler(p, smp);
   p.rclass = (int)rtype;
   p.dims = img->img.dims;
   memcpy(p.A, affine, sizeof(p.A));
-  p.ow = (int)out_dims[0];
-  p.oh = (int)out_dims[1];
-  p.od = (int)out_dims[2];
+  p.ow = (int)out_region[0];
+  p.oh = (int)out_region[1];
+  p.od = (int)out_region[2];
+  p.ox = (int)out_origin[0];
+  p.oy = (int)out_origin[1];
+  p.oz = (int)out_origin[2];
   p.outc = (int)outc;
   p.out = po + ooffset;
   cl_int st = enq_end(E, launch_sample(p, COORD_GRID, q->stream));
   if (st == CL_SUCCESS) written(out, q);
   return st;
+}
+
+extern "C" cl_int b2clEnqueueReadImageGrid(cl_command_queue q, cl_mem img, cl_sampler smp,
+                                           b2cl_rtype rtype, const float* affine,
+                                           const size_t* out_dims, cl_uint outc, cl_mem out,
+                                           size_t ooffset, cl_uint nw, const cl_event* wl,
+                                           cl_event* ev) {
+  const size_t origin[3] = {0, 0, 0};
+  return b2clEnqueueReadImageGridRegion(q, img, smp, rtype, affine, origin, out_dims, outc, out,
+                                        ooffset, nw, wl, ev);
 }
 
 extern "C" cl_int b2clEnqueueWriteImageSamples(cl_command_queue q, cl_mem img, b2cl_rtype rtype,
