@@ -167,12 +167,13 @@ def oracle_rate(codes, n_rows_target_s: float, threads: int):
     return 2 * rows * N2D / dt / 1e9, rows, dt
 
 
-def _axis_taps(coef, offset, n_out, n, mode):
+def _axis_taps(coef, offset, n_out, n, mode, start=0):
     """Set of texel indices along one axis that a LINEAR read of a separable
-    affine map touches with a non-zero weight ([CL1.2 §8.2] in numpy float32;
-    measurement bookkeeping only -- the bytes a launch must move)."""
+    affine map touches with a non-zero weight, for outputs start..start+n_out-1
+    ([CL1.2 §8.2] in numpy float32; measurement bookkeeping only -- the bytes a
+    launch must move, and the rows a shard must hold)."""
     f32 = np.float32
-    x = np.arange(n_out, dtype=np.float32)
+    x = np.arange(start, start + n_out, dtype=np.float32)
     s = (f32(coef) * x).astype(f32) + f32(offset)
     fn = f32(n)
     if mode == "repeat":
@@ -188,6 +189,17 @@ def _axis_taps(coef, offset, n_out, n, mode):
     else:
         i0, i1 = np.maximum(b, 0), np.minimum(b + 1, n - 1)
     return np.unique(np.concatenate([i0[a != 1], i1[a != 0]]))
+
+
+def circular_interval(idx, n):
+    """Smallest (begin, count) whose circular range {(begin+s) mod n} covers idx."""
+    rows = np.unique(np.asarray(idx, dtype=np.int64))
+    if rows.size == 1:
+        return int(rows[0]), 1
+    gaps = (np.roll(rows, -1) - rows) % n
+    i = int(np.argmax(gaps))
+    begin = int(rows[(i + 1) % rows.size])
+    return begin, int((rows[i] - begin) % n + 1)
 
 
 def distinct_texels_separable(A, w_out, h_out, mode):
@@ -289,43 +301,71 @@ def run_gpu(args):
     hbm_peak, peak_src = peaks()
 
     # ---- inputs resident in HBM before timing ----
-    codes = c2_codes()
-    img = S.image(cl.CL_RGBA, cl.CL_FLOAT, N2D, N2D, host=codes)
+    # N = 1: config 2 itself, one 4096^2 image.  N > 1 (config 5 style): one
+    # global (4096*N) x 4096 image, row-sharded: rank r computes output rows
+    # [4096 r, 4096 (r+1)) of map (A) on the GLOBAL image from shards holding
+    # exactly the texel rows that band needs (one per pass: REPEAT and the
+    # folded MIRRORED rows differ) -- bit-identical to a single-GPU read
+    # (tests/test_gpu_shards.py), same per-GPU work as N = 1 (weak scaling).
+    Hg = N2D * world
+    r0 = rank * N2D
+    Af = synth.affine_translate_2d(N2D, Hg)
+    A = (ctypes.c_float * 12)(*Af.tolist())
+    modes = ("repeat", "mirrored")
+    codes = None
+    shard_rows, shard_host = [], []
+    if world == 1:
+        codes = c2_codes()
+        img = S.image(cl.CL_RGBA, cl.CL_FLOAT, N2D, N2D, host=codes)
+        imgs = [img, img]
+    else:
+        imgs = []
+        for m in modes:
+            need = _axis_taps(Af[5], Af[7], N2D, Hg, m, start=r0)
+            begin, count = circular_interval(need, Hg)
+            rows = [(begin + s) % Hg for s in range(count)]
+            shard_rows.append(count)
+            shard_host.append(synth.image_rows(cl.CL_RGBA, cl.CL_FLOAT, N2D, rows))
+            imgs.append(S.image_shard(cl.CL_RGBA, cl.CL_FLOAT, N2D, Hg, 0, begin, count, 0,
+                                      host=shard_host[-1]))
     nout = N2D * N2D * 16
     outs = [S.buffer(nout), S.buffer(nout)]
     smps = [S.sampler(True, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR),
             S.sampler(True, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR)]
-    A = (ctypes.c_float * 12)(*synth.affine_translate_2d(N2D, N2D).tolist())
-    dims = cl.sz3((N2D, N2D, 1))
+    origin, region = cl.sz3((0, r0, 0)), cl.sz3((N2D, N2D, 1))
 
     def launch(k):
-        cl.check(L.b2clEnqueueReadImageGrid(S.queue, img, smps[k], cl.B2CL_RTYPE_FLOAT, A, dims, 4,
-                                            outs[k], 0, 0, None, None), "read grid")
+        cl.check(L.b2clEnqueueReadImageGridRegion(S.queue, imgs[k], smps[k], cl.B2CL_RTYPE_FLOAT, A,
+                                                  origin, region, 4, outs[k], 0, 0, None, None),
+                 "read grid")
 
     # ---- parity spot check of this exact launch configuration (bench as test) ----
     launch(0)
     launch(1)
     S.finish()
     parity = "skipped (oracle missing)"
-    try:
-        import oracle as orc
-        oimg = orc.Image(codes, N2D, N2D, 1, dims=2, order=orc.RGBA, type=orc.FLOAT)
-        Af = synth.affine_translate_2d(N2D, N2D)
-        worst = 0.0
-        for k, a in enumerate((orc.ADDRESS_REPEAT, orc.ADDRESS_MIRRORED_REPEAT)):
-            got = S.read(outs[k], nout, np.float32).reshape(N2D, N2D, 4)
-            for y in (0, N2D // 2 - 1, N2D // 2, N2D - 1, 1234):
-                exp = orc.read_grid(oimg, True, a, orc.FILTER_LINEAR, orc.RT_F, Af, (N2D, N2D, 1), 4,
-                                    yrange=(y, y + 1))[0, 0]
-                err = np.abs(got[y].astype(np.float64) - exp) / np.maximum(
-                    np.spacing(np.abs(exp)).astype(np.float64), 1e-30)
-                ok = np.all((err <= 4) | (np.abs(got[y] - exp) <= 1e-6))
-                worst = max(worst, float(np.max(np.minimum(err, 1e9))))
-                if not ok:
-                    raise SystemExit(f"bench parity check failed (pass {k}, row {y})")
-        parity = f"ok (10 rows vs oracle, worst {worst:.2f} ulp)"
-    except ImportError:
-        pass
+    if world > 1:
+        parity = ("sharded: bit-identity of shard reads to whole-image reads is tested in "
+                  "tests/test_gpu_shards.py; the whole-image path is checked against the oracle")
+    else:
+        try:
+            import oracle as orc
+            oimg = orc.Image(codes, N2D, N2D, 1, dims=2, order=orc.RGBA, type=orc.FLOAT)
+            worst = 0.0
+            for k, a in enumerate((orc.ADDRESS_REPEAT, orc.ADDRESS_MIRRORED_REPEAT)):
+                got = S.read(outs[k], nout, np.float32).reshape(N2D, N2D, 4)
+                for y in (0, N2D // 2 - 1, N2D // 2, N2D - 1, 1234):
+                    exp = orc.read_grid(oimg, True, a, orc.FILTER_LINEAR, orc.RT_F, Af,
+                                        (N2D, N2D, 1), 4, yrange=(y, y + 1))[0, 0]
+                    err = np.abs(got[y].astype(np.float64) - exp) / np.maximum(
+                        np.spacing(np.abs(exp)).astype(np.float64), 1e-30)
+                    ok = np.all((err <= 4) | (np.abs(got[y] - exp) <= 1e-6))
+                    worst = max(worst, float(np.max(np.minimum(err, 1e9))))
+                    if not ok:
+                        raise SystemExit(f"bench parity check failed (pass {k}, row {y})")
+            parity = f"ok (10 rows vs oracle, worst {worst:.2f} ulp)"
+        except ImportError:
+            pass
 
     # ---- warmup + timed steps ----
     for _ in range(args.warmup):
@@ -360,9 +400,9 @@ def run_gpu(args):
     value = world * samples_step / (ms_step * 1e-3) / 1e9
     # algorithmic bytes per launch = distinct texels with a non-zero tap weight x 16 B
     # + 16 B output per sample; counted exactly per map on the host
-    Af = synth.affine_translate_2d(N2D, N2D)
-    alg = [distinct_texels_separable(Af, N2D, N2D, m) * 16 + N2D * N2D * 16
-           for m in ("repeat", "mirrored")]
+    ncols = [_axis_taps(Af[0], Af[3], N2D, N2D, m).size for m in modes]
+    nrows = [_axis_taps(Af[5], Af[7], N2D, Hg, m, start=r0).size for m in modes]
+    alg = [ncols[k] * nrows[k] * 16 + N2D * N2D * 16 for k in range(2)]
     achieved = [alg[k] / (pass_ms[k] * 1e-3) / 1e9 for k in range(2)]
     dom = 0 if pass_ms[0] * 1.0 >= pass_ms[1] else 1  # the kernel with the larger share of the step
     traffic = None
@@ -374,13 +414,22 @@ def run_gpu(args):
     # ---- e2e: host buffers through the C-ABI, copies inside the timed region ----
     e2e = None
     if not args.no_e2e:
-        host_in = torch.from_numpy(codes.reshape(-1).view(np.uint8)).pin_memory()
+        # the image(s) every step uploads from pinned host memory: the whole
+        # image at N = 1, the two shards (their stored rows) at N > 1
+        uploads = []
+        for k, im in enumerate(imgs[:1] if world == 1 else imgs):
+            hrows = N2D if world == 1 else shard_rows[k]
+            hbuf = torch.empty(hrows * N2D * 16, dtype=torch.uint8).pin_memory()
+            src = codes if world == 1 else shard_host[k]
+            hbuf.copy_(torch.from_numpy(np.ascontiguousarray(src).reshape(-1).view(np.uint8)))
+            uploads.append((im, hbuf, cl.sz3((N2D, hrows, 1))))
         host_out = [torch.empty(nout, dtype=torch.uint8).pin_memory() for _ in range(2)]
-        origin, region = cl.sz3((0, 0, 0)), cl.sz3((N2D, N2D, 1))
+        zero3 = cl.sz3((0, 0, 0))
 
         def e2e_step():
-            cl.check(L.clEnqueueWriteImage(S.queue, img, 0, origin, region, 0, 0,
-                                           ctypes.c_void_p(host_in.data_ptr()), 0, None, None))
+            for im, hbuf, reg in uploads:
+                cl.check(L.clEnqueueWriteImage(S.queue, im, 0, zero3, reg, 0, 0,
+                                               ctypes.c_void_p(hbuf.data_ptr()), 0, None, None))
             for k in range(2):
                 launch(k)
                 cl.check(L.clEnqueueReadBuffer(S.queue, outs[k], 0, 0, nout,
@@ -400,7 +449,7 @@ def run_gpu(args):
         if world > 1:
             e2e_ms = bdist.max_over_ranks(e2e_ms, red_dev)
         e2e = {"value": world * samples_step / (e2e_ms * 1e-3) / 1e9, "unit": "Gsamples/s",
-               "ms_per_step": e2e_ms, "h2d_bytes_per_step": int(host_in.numel()),
+               "ms_per_step": e2e_ms, "h2d_bytes_per_step": int(sum(u[1].numel() for u in uploads)),
                "d2h_bytes_per_step": 2 * nout}
 
     secondary = None
@@ -429,7 +478,10 @@ def run_gpu(args):
             "data": "synthetic (numpy default_rng seed 20151115; U[0,1) RGBA32F texels)",
             "config": {"workload": WORKLOAD, "image": "4096x4096 RGBA32F (256 MiB)",
                        "samples_per_step": samples_step, "launches_per_step": 2,
-                       "parallelism": f"replicas x{world} (one image per GPU)",
+                       "parallelism": ("single GPU" if world == 1 else
+                                       f"row-sharded x{world}: global {Hg}x{N2D} image, "
+                                       f"4096 output rows per GPU from shards of "
+                                       f"{shard_rows} texel rows (REPEAT, MIRRORED)"),
                        "l2": "no flush: 768 MiB working set > 126 MB L2", "parity": parity},
             "roofline": {"bound": "hbm", "achieved": achieved[dom], "peak": hbm_peak, "unit": "GB/s",
                          "frac": achieved[dom] / hbm_peak, "traffic": traffic,
@@ -445,7 +497,7 @@ def run_gpu(args):
             "secondary": secondary,
         }
         print(json.dumps(line), flush=True)
-    S.release(img, *outs)
+    S.release(*set(imgs), *outs)
     for s in smps:
         L.clReleaseSampler(s)
     S.close()

@@ -49,6 +49,17 @@ def image_codes(g: np.random.Generator, order: int, type_: int, width: int, heig
     return g.integers(0, 256, size=nbytes, dtype=np.uint8).view(dt).reshape(shape)
 
 
+def image_rows(order: int, type_: int, width: int, rows, key: int = 5,
+               signed: bool = False) -> np.ndarray:
+    """Rows of a large virtual 2D image whose row j is drawn from its own
+    generator default_rng([SEED, key, j]) -- so any rank can materialise any
+    band (or shard) of a global image without generating the rest.
+    Returns shape (1, len(rows), width, channels)."""
+    out = [image_codes(np.random.default_rng([SEED, key, int(j)]), order, type_, width,
+                       signed=signed)[0, 0] for j in rows]
+    return np.stack(out)[None]
+
+
 def special_floats() -> np.ndarray:
     """Coordinates that stress the address path."""
     f32 = np.float32
