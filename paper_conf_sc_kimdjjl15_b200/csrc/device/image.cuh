@@ -135,20 +135,6 @@ __device__ __forceinline__ Raw load_raw(const char* p, int es) {
   return r;
 }
 
-// the same from shared memory (staged footprints)
-__device__ __forceinline__ Raw load_raw_smem(const char* p, int es) {
-  Raw r;
-  r.w[0] = r.w[1] = r.w[2] = r.w[3] = 0u;
-  switch (es) {
-    case 16: { uint4 v = *reinterpret_cast<const uint4*>(p); r.w[0] = v.x; r.w[1] = v.y; r.w[2] = v.z; r.w[3] = v.w; break; }
-    case 8: { uint2 v = *reinterpret_cast<const uint2*>(p); r.w[0] = v.x; r.w[1] = v.y; break; }
-    case 4: r.w[0] = *reinterpret_cast<const unsigned int*>(p); break;
-    case 2: r.w[0] = *reinterpret_cast<const unsigned short*>(p); break;
-    default: r.w[0] = *reinterpret_cast<const unsigned char*>(p); break;
-  }
-  return r;
-}
-
 // stored code of channel c (memory order), zero/sign extended to 32 bits
 __device__ __forceinline__ uint32_t channel_code(const Raw& r, int c, int type) {
   const int tb = type_bytes(type);

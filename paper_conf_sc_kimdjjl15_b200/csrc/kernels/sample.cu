@@ -5,8 +5,10 @@
 // vector load per texel (16 B for RGBA32F) -> conversion and channel map
 // ([CL1.2 §8.3]) -> LINEAR blend in the separable FMA form.
 //
-// Two grid kernels:
+// Grid kernels:
 //  * k_sample_grid      one thread per output sample, any affine map;
+//  * k_sample_grid_walk separable maps, compile-time format: register reuse
+//    of texel rows along the outermost axis (see its comment);
 //  * k_sample_grid_sep  separable maps (every off-diagonal coefficient 0):
 //    the x-axis addressing of XPT columns is computed once per thread and
 //    reused down RPW rows, the y/z-axis addressing and the texel row
@@ -124,9 +126,8 @@ __device__ __forceinline__ int elem_size(const Image& im) {
   return (C::type == RT || C::nch == RT) ? im.es : C::nch * type_bytes(C::type);
 }
 
-// memory-order channels of the texel at row + i*elem_size (zero if !ok);
-// SMEM: `row` points into a staged footprint in shared memory
-template <class C, bool SMEM = false>
+// memory-order channels of the texel at row + i*elem_size (zero if !ok)
+template <class C>
 __device__ __forceinline__ void fetch(const Image& im, const char* row, int i, bool ok, int rc,
                                       uint32_t m[4]) {
   const int type = C::type == RT ? im.type : C::type;
@@ -134,8 +135,7 @@ __device__ __forceinline__ void fetch(const Image& im, const char* row, int i, b
   const int es = elem_size<C>(im);
   m[0] = m[1] = m[2] = m[3] = 0u;
   if (!ok) return;
-  Raw r = SMEM ? load_raw_smem(row + i * es, es)
-               : load_raw(row + (uint64_t)(unsigned)i * (unsigned)es, es);
+  Raw r = load_raw(row + (uint64_t)(unsigned)i * (unsigned)es, es);
 #pragma unroll
   for (int c = 0; c < 4; ++c) {
     if (c < nch) {
@@ -158,7 +158,7 @@ __device__ __forceinline__ void nearest_at(const SampleParams& p, const char* ro
 
 // LINEAR from the texel rows: rows[0] = (j0,k0), [1] = (j1,k0), [2] = (j0,k1),
 // [3] = (j1,k1); blend x, then y, then z ([CL1.2 §8.2] weights, separable form)
-template <class C, bool SMEM = false>
+template <class C>
 __device__ __forceinline__ void linear_at(const SampleParams& p, const char* const rows[4],
                                           const bool rok[4], const AxL& x, float b, float omb,
                                           float g, float omg, uint32_t res[4], int outc = 4) {
@@ -168,8 +168,8 @@ __device__ __forceinline__ void linear_at(const SampleParams& p, const char* con
   uint32_t t0[NR][4], t1[NR][4];
 #pragma unroll
   for (int r = 0; r < NR; ++r) {
-    fetch<C, SMEM>(p.im, rows[r], x.i0, rok[r] && x.ok0, R_F, t0[r]);
-    fetch<C, SMEM>(p.im, rows[r], x.i1, rok[r] && x.ok1, R_F, t1[r]);
+    fetch<C>(p.im, rows[r], x.i0, rok[r] && x.ok0, R_F, t0[r]);
+    fetch<C>(p.im, rows[r], x.i1, rok[r] && x.ok1, R_F, t1[r]);
   }
   uint32_t m[4];
 #pragma unroll
