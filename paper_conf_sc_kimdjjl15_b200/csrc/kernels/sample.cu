@@ -264,7 +264,12 @@ __global__ void __launch_bounds__(128, 12) k_sample_grid_sep(const SampleParams 
   const Image& im = p.im;
   const int z = blockIdx.z;
   const int x0 = blockIdx.x * (32 * XPT) + threadIdx.x;
-  const int y0 = blockIdx.y * (4 * RPW) + threadIdx.y * RPW;
+  // MIRRORED_REPEAT folds output rows onto shared texel rows symmetrically
+  // about the mirror axis; taking row tiles alternately from both ends keeps
+  // those texel rows in L2 between their two uses (a traversal order only)
+  int ty = blockIdx.y;
+  if (C::addr == A_MIRROR) ty = (ty & 1) ? gridDim.y - 1 - (ty >> 1) : (ty >> 1);
+  const int y0 = ty * (4 * RPW) + threadIdx.y * RPW;
   const bool lin = filt_of<C>(p) == F_LINEAR;
   // x axis: once per column
   AxL ax[XPT];
