@@ -79,6 +79,10 @@ typedef struct _cl_command_queue* cl_command_queue;
 typedef struct _cl_mem* cl_mem;
 typedef struct _cl_sampler* cl_sampler;
 typedef struct _cl_event* cl_event;
+typedef struct _cl_program* cl_program;
+typedef struct _cl_kernel* cl_kernel;
+typedef cl_uint cl_program_build_info;
+typedef cl_uint cl_kernel_info;
 
 typedef struct _cl_image_format {
   cl_channel_order image_channel_order;
@@ -126,6 +130,30 @@ typedef struct _cl_image_desc {
 #define CL_INVALID_OPERATION -59
 #define CL_INVALID_BUFFER_SIZE -61
 #define CL_INVALID_IMAGE_DESCRIPTOR -65
+#define CL_BUILD_PROGRAM_FAILURE -11
+#define CL_INVALID_BINARY -42
+#define CL_INVALID_BUILD_OPTIONS -43
+#define CL_INVALID_PROGRAM -44
+#define CL_INVALID_PROGRAM_EXECUTABLE -45
+#define CL_INVALID_KERNEL_NAME -46
+#define CL_INVALID_KERNEL -48
+#define CL_INVALID_ARG_INDEX -49
+#define CL_INVALID_ARG_VALUE -50
+#define CL_INVALID_ARG_SIZE -51
+#define CL_INVALID_KERNEL_ARGS -52
+#define CL_INVALID_WORK_DIMENSION -53
+#define CL_INVALID_WORK_GROUP_SIZE -54
+#define CL_INVALID_WORK_ITEM_SIZE -55
+#define CL_INVALID_GLOBAL_OFFSET -56
+#define CL_PROGRAM_BUILD_STATUS 0x1181
+#define CL_PROGRAM_BUILD_LOG 0x1183
+#define CL_BUILD_SUCCESS 0
+#define CL_BUILD_NONE -1
+#define CL_BUILD_ERROR -2
+#define CL_KERNEL_FUNCTION_NAME 0x1190
+#define CL_KERNEL_NUM_ARGS 0x1191
+#define CL_KERNEL_REFERENCE_COUNT 0x1192
+#define CL_COMMAND_NDRANGE_KERNEL 0x11F0
 
 #define CL_FALSE 0
 #define CL_TRUE 1
@@ -529,6 +557,65 @@ cl_int CL_API_CALL clEnqueueMigrateMemObjects(cl_command_queue command_queue,
                                               cl_mem_migration_flags flags,
                                               cl_uint num_events_in_wait_list,
                                               const cl_event* event_wait_list, cl_event* event);
+
+/* ================= programs and kernels (launch glue) ================= */
+
+/* The paper builds an OpenCL program by translating it to CUDA C, compiling
+ * it with nvcc and loading the module with cuModuleLoad.  Here the
+ * translated kernel (written against include/b2cl_device.cuh) is compiled
+ * with nvcc ahead of time, and its cubin / fatbin / PTX image is the program
+ * binary.  binaries[i] (lengths[i] bytes) is the module for devices[i];
+ * binary_status[i] receives CL_SUCCESS or CL_INVALID_BINARY. */
+cl_program CL_API_CALL clCreateProgramWithBinary(cl_context context, cl_uint num_devices,
+                                                 const cl_device_id* device_list,
+                                                 const size_t* lengths,
+                                                 const unsigned char** binaries,
+                                                 cl_int* binary_status, cl_int* errcode_ret);
+/* Loads the module on every device of the program (cudaLibraryLoadData);
+ * options are ignored; CL_BUILD_PROGRAM_FAILURE if a device rejects it. */
+cl_int CL_API_CALL clBuildProgram(cl_program program, cl_uint num_devices,
+                                  const cl_device_id* device_list, const char* options,
+                                  void(CL_CALLBACK* pfn_notify)(cl_program, void*),
+                                  void* user_data);
+cl_int CL_API_CALL clGetProgramBuildInfo(cl_program program, cl_device_id device,
+                                         cl_program_build_info param_name,
+                                         size_t param_value_size, void* param_value,
+                                         size_t* param_value_size_ret);
+cl_int CL_API_CALL clRetainProgram(cl_program program);
+cl_int CL_API_CALL clReleaseProgram(cl_program program);
+
+/* A __global__ function of the built program (extern "C" name). */
+cl_kernel CL_API_CALL clCreateKernel(cl_program program, const char* kernel_name,
+                                     cl_int* errcode_ret);
+cl_int CL_API_CALL clRetainKernel(cl_kernel kernel);
+cl_int CL_API_CALL clReleaseKernel(cl_kernel kernel);
+cl_int CL_API_CALL clGetKernelInfo(cl_kernel kernel, cl_kernel_info param_name,
+                                   size_t param_value_size, void* param_value,
+                                   size_t* param_value_size_ret);
+
+/* Records argument arg_index, as the paper's wrapper does ("the parameters
+ * of cuLaunchKernel() ... are collected when clSetKernelArg() is called",
+ * P:139).  arg_value == NULL: a __local argument of arg_size bytes -- the
+ * kernel receives the size (size_t) and the launch reserves the sum of all
+ * __local sizes as dynamic shared memory (Fig. 5(b)).  arg_value
+ * pointing to a cl_mem: a buffer passes its device pointer, an image its
+ * descriptor by value (b2cl_device.cuh image*_t).  To a cl_sampler: its
+ * 32-bit CLK_* bits.  Anything else: the arg_size bytes. */
+cl_int CL_API_CALL clSetKernelArg(cl_kernel kernel, cl_uint arg_index, size_t arg_size,
+                                  const void* arg_value);
+
+/* [CL1.2 §5.8]: work_dim 1..3, global_work_size[d] > 0, local_work_size
+ * (or a chosen one when NULL) must divide it (CL_INVALID_WORK_GROUP_SIZE)
+ * with at most 1024 work-items per group; global_work_offset is passed to
+ * get_global_id through the module's __b2cl_global_offset.  One
+ * cudaLaunchKernel: grid = global / local, block = local.  Buffers and
+ * images passed to the kernel count as written by it (residency). */
+cl_int CL_API_CALL clEnqueueNDRangeKernel(cl_command_queue command_queue, cl_kernel kernel,
+                                          cl_uint work_dim, const size_t* global_work_offset,
+                                          const size_t* global_work_size,
+                                          const size_t* local_work_size,
+                                          cl_uint num_events_in_wait_list,
+                                          const cl_event* event_wait_list, cl_event* event);
 
 #ifdef __cplusplus
 }

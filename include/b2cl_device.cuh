@@ -1,0 +1,209 @@
+// b2cl_device.cuh -- OpenCL C built-ins for translated kernels (CUDA C, sm_100a).
+//
+// The paper translates an OpenCL kernel to CUDA C and implements the OpenCL
+// built-ins it calls as CUDA device wrappers (read_imageX /
+// write_imageX "handle the CLImage object to read or to write image data
+// through pointer ptr"; §3.5 kernel launch; Fig. 5 dynamic __local carving).
+// A kernel written against this header is compiled by nvcc to a cubin and
+// run through clCreateProgramWithBinary / clBuildProgram / clCreateKernel /
+// clSetKernelArg / clEnqueueNDRangeKernel of libb2cl.
+//
+// Argument conventions (what clSetKernelArg passes for each OpenCL argument):
+//   __global / __constant buffer (cl_mem)  -> a device pointer
+//   image1d_t / image2d_t / image3d_t      -> the image descriptor by value
+//                                             (the paper's CLImage, Fig. 6;
+//                                             reading A27)
+//   sampler_t (cl_sampler)                 -> 32-bit CLK_* bits below
+//   __local pointer (arg_value == NULL)    -> size_t size of that local
+//                                             object; the kernel carves
+//                                             __OC2CU_shared_mem by the
+//                                             running sum of the sizes, in
+//                                             argument order (Fig. 5(b))
+//   anything else                          -> the bytes given
+// The read / write built-ins are the library's own (csrc/device/read.cuh):
+// same arithmetic, same readings as the enqueue extensions.
+#pragma once
+#include <stddef.h>
+
+#include "../paper_conf_sc_kimdjjl15_b200/csrc/device/read.cuh"
+
+// ---- image and sampler types ----
+struct image1d_t { b2cl::dev::Image im; };
+struct image2d_t { b2cl::dev::Image im; };
+struct image3d_t { b2cl::dev::Image im; };
+typedef unsigned int sampler_t;
+
+// sampler bits (clang's CLK_* encoding)
+#define CLK_NORMALIZED_COORDS_FALSE 0x0u
+#define CLK_NORMALIZED_COORDS_TRUE 0x1u
+#define CLK_ADDRESS_NONE 0x0u
+#define CLK_ADDRESS_CLAMP_TO_EDGE 0x2u
+#define CLK_ADDRESS_CLAMP 0x4u
+#define CLK_ADDRESS_REPEAT 0x6u
+#define CLK_ADDRESS_MIRRORED_REPEAT 0x8u
+#define CLK_FILTER_NEAREST 0x10u
+#define CLK_FILTER_LINEAR 0x20u
+
+#define CLK_LOCAL_MEM_FENCE 0x1u
+#define CLK_GLOBAL_MEM_FENCE 0x2u
+
+// one dynamic shared array for every __local argument (Fig. 5(b))
+extern __shared__ __align__(16) char __OC2CU_shared_mem[];
+
+// global work offset of clEnqueueNDRangeKernel, written by the runtime before
+// each launch when the module defines it (this header does)
+__device__ size_t __b2cl_global_offset[3];
+
+// ---- work-item functions ----
+__device__ __forceinline__ size_t get_local_id(unsigned d) {
+  return d == 0 ? threadIdx.x : (d == 1 ? threadIdx.y : (d == 2 ? threadIdx.z : 0));
+}
+__device__ __forceinline__ size_t get_local_size(unsigned d) {
+  return d == 0 ? blockDim.x : (d == 1 ? blockDim.y : (d == 2 ? blockDim.z : 1));
+}
+__device__ __forceinline__ size_t get_group_id(unsigned d) {
+  return d == 0 ? blockIdx.x : (d == 1 ? blockIdx.y : (d == 2 ? blockIdx.z : 0));
+}
+__device__ __forceinline__ size_t get_num_groups(unsigned d) {
+  return d == 0 ? gridDim.x : (d == 1 ? gridDim.y : (d == 2 ? gridDim.z : 1));
+}
+__device__ __forceinline__ size_t get_global_offset(unsigned d) {
+  return d < 3 ? __b2cl_global_offset[d] : 0;
+}
+__device__ __forceinline__ size_t get_global_id(unsigned d) {
+  return get_group_id(d) * get_local_size(d) + get_local_id(d) + get_global_offset(d);
+}
+__device__ __forceinline__ size_t get_global_size(unsigned d) {
+  return get_num_groups(d) * get_local_size(d);
+}
+__device__ __forceinline__ void barrier(unsigned) { __syncthreads(); }
+
+// ---- read built-ins ([CL1.2 §6.12.14.2]) ----
+namespace b2cl {
+namespace cl_builtin {
+
+struct ReadParams {  // the P of read.cuh
+  dev::Image im;
+  dev::Sampler smp;
+  int rclass;
+};
+
+__device__ __forceinline__ dev::Sampler decode(sampler_t s) {
+  dev::Sampler r;
+  r.norm = (int)(s & 1u);
+  r.addr = (int)((s & 0xEu) >> 1);  // NONE, CTE, CLAMP, REPEAT, MIRRORED -> 0..4
+  r.filt = (s & CLK_FILTER_LINEAR) ? dev::F_LINEAR : dev::F_NEAREST;
+  return r;
+}
+
+template <int DIMS>
+__device__ __forceinline__ uint4 read(const dev::Image& im, sampler_t s, int rclass, float c0,
+                                      float c1, float c2) {
+  using C = WithShard<Cfg<DIMS, RT, RT, RT, RT, RT, RT>, true>;
+  ReadParams p{im, decode(s), rclass};
+  // LINEAR with read_imagei/ui is undefined; NEAREST is used (reading A6)
+  if (rclass != dev::R_F) p.smp.filt = dev::F_NEAREST;
+  const float c[3] = {c0, c1, c2};
+  uint32_t r[4];
+  read_image<C>(p, c, r, 4);
+  return make_uint4(r[0], r[1], r[2], r[3]);
+}
+
+__device__ __forceinline__ float4 as_f4(uint4 v) {
+  return make_float4(__uint_as_float(v.x), __uint_as_float(v.y), __uint_as_float(v.z),
+                     __uint_as_float(v.w));
+}
+__device__ __forceinline__ int4 as_i4(uint4 v) {
+  return make_int4((int)v.x, (int)v.y, (int)v.z, (int)v.w);
+}
+
+// integer coordinates: u = (float)i (reading A30); samplerless reads use
+// NEAREST, unnormalized, CLK_ADDRESS_NONE (reading A31)
+constexpr sampler_t kSamplerless = CLK_NORMALIZED_COORDS_FALSE | CLK_ADDRESS_NONE | CLK_FILTER_NEAREST;
+
+template <int DIMS>
+__device__ __forceinline__ void write(const dev::Image& im, int i, int j, int k, uint4 col) {
+  if (!dev::in_range(i, im.w) || !dev::in_range(j, im.h) || !dev::in_range(k, im.d)) return;  // A15
+  // global outer index -> stored row of a shard; rows the shard does not hold: no-op
+  int& o = DIMS == 3 ? k : j;
+  const int extent = DIMS == 3 ? im.d : im.h;
+  if (DIMS > 1) {
+    int l = o - im.ob;
+    l += l < 0 ? extent : 0;
+    l -= l >= extent ? extent : 0;
+    if (l >= im.os) return;
+    o = l;
+  }
+  const uint32_t cc[4] = {col.x, col.y, col.z, col.w};
+  dev::Raw t = dev::encode_texel(cc, im.type, im.order);
+  dev::store_raw(const_cast<char*>(dev::texel_ptr(im, i, j, k)), im.es, t);
+}
+
+}  // namespace cl_builtin
+}  // namespace b2cl
+
+#define B2CL_READ_OVERLOADS(RET, NAME, RC, CONV)                                                 \
+  __device__ __forceinline__ RET NAME(image1d_t im, sampler_t s, float c) {                      \
+    return CONV(b2cl::cl_builtin::read<1>(im.im, s, RC, c, 0.f, 0.f));                           \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image1d_t im, sampler_t s, int c) {                        \
+    return CONV(b2cl::cl_builtin::read<1>(im.im, s, RC, __int2float_rn(c), 0.f, 0.f));           \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image2d_t im, sampler_t s, float2 c) {                     \
+    return CONV(b2cl::cl_builtin::read<2>(im.im, s, RC, c.x, c.y, 0.f));                         \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image2d_t im, sampler_t s, int2 c) {                       \
+    return CONV(b2cl::cl_builtin::read<2>(im.im, s, RC, __int2float_rn(c.x), __int2float_rn(c.y), \
+                                          0.f));                                                 \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image3d_t im, sampler_t s, float4 c) {                     \
+    return CONV(b2cl::cl_builtin::read<3>(im.im, s, RC, c.x, c.y, c.z));                         \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image3d_t im, sampler_t s, int4 c) {                       \
+    return CONV(b2cl::cl_builtin::read<3>(im.im, s, RC, __int2float_rn(c.x), __int2float_rn(c.y), \
+                                          __int2float_rn(c.z)));                                 \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image2d_t im, int2 c) {                                    \
+    return NAME(im, b2cl::cl_builtin::kSamplerless, c);                                          \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image3d_t im, int4 c) {                                    \
+    return NAME(im, b2cl::cl_builtin::kSamplerless, c);                                          \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image1d_t im, int c) {                                     \
+    return NAME(im, b2cl::cl_builtin::kSamplerless, c);                                          \
+  }
+
+#define B2CL_ID(v) (v)
+B2CL_READ_OVERLOADS(float4, read_imagef, b2cl::dev::R_F, b2cl::cl_builtin::as_f4)
+B2CL_READ_OVERLOADS(int4, read_imagei, b2cl::dev::R_I, b2cl::cl_builtin::as_i4)
+B2CL_READ_OVERLOADS(uint4, read_imageui, b2cl::dev::R_UI, B2CL_ID)
+
+// ---- write built-ins ([CL1.2 §6.12.14.4]); 3D writes as cl_khr_3d_image_writes ----
+__device__ __forceinline__ void write_imagef(image1d_t im, int c, float4 v) {
+  b2cl::cl_builtin::write<1>(im.im, c, 0, 0, make_uint4(__float_as_uint(v.x), __float_as_uint(v.y),
+                                                       __float_as_uint(v.z), __float_as_uint(v.w)));
+}
+__device__ __forceinline__ void write_imagef(image2d_t im, int2 c, float4 v) {
+  b2cl::cl_builtin::write<2>(im.im, c.x, c.y, 0,
+                             make_uint4(__float_as_uint(v.x), __float_as_uint(v.y),
+                                        __float_as_uint(v.z), __float_as_uint(v.w)));
+}
+__device__ __forceinline__ void write_imagef(image3d_t im, int4 c, float4 v) {
+  b2cl::cl_builtin::write<3>(im.im, c.x, c.y, c.z,
+                             make_uint4(__float_as_uint(v.x), __float_as_uint(v.y),
+                                        __float_as_uint(v.z), __float_as_uint(v.w)));
+}
+__device__ __forceinline__ void write_imagei(image2d_t im, int2 c, int4 v) {
+  b2cl::cl_builtin::write<2>(im.im, c.x, c.y, 0, make_uint4(v.x, v.y, v.z, v.w));
+}
+__device__ __forceinline__ void write_imageui(image2d_t im, int2 c, uint4 v) {
+  b2cl::cl_builtin::write<2>(im.im, c.x, c.y, 0, v);
+}
+
+// ---- image queries ([CL1.2 §6.12.14.5]) ----
+__device__ __forceinline__ int get_image_width(image1d_t im) { return im.im.w; }
+__device__ __forceinline__ int get_image_width(image2d_t im) { return im.im.w; }
+__device__ __forceinline__ int get_image_width(image3d_t im) { return im.im.w; }
+__device__ __forceinline__ int get_image_height(image2d_t im) { return im.im.h; }
+__device__ __forceinline__ int get_image_height(image3d_t im) { return im.im.h; }
+__device__ __forceinline__ int get_image_depth(image3d_t im) { return im.im.d; }

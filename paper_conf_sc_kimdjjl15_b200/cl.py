@@ -103,6 +103,17 @@ PROTOTYPES = {
     "clEnqueueCopyImageToBuffer": (_I, [_H, _H, _H, _SZ3, _SZ3, _S, _U, POINTER(_H), POINTER(_H)]),
     "clEnqueueCopyBufferToImage": (_I, [_H, _H, _H, _S, _SZ3, _SZ3, _U, POINTER(_H), POINTER(_H)]),
     "clEnqueueMigrateMemObjects": (_I, [_H, _U, POINTER(_H), _L, _U, POINTER(_H), POINTER(_H)]),
+    "clCreateProgramWithBinary": (_H, [_H, _U, POINTER(_H), POINTER(_S), _P, _PI, _PI]),
+    "clBuildProgram": (_I, [_H, _U, POINTER(_H), ctypes.c_char_p, _P, _P]),
+    "clGetProgramBuildInfo": (_I, [_H, _H, _U, _S, _P, POINTER(_S)]),
+    "clRetainProgram": (_I, [_H]),
+    "clReleaseProgram": (_I, [_H]),
+    "clCreateKernel": (_H, [_H, ctypes.c_char_p, _PI]),
+    "clRetainKernel": (_I, [_H]),
+    "clReleaseKernel": (_I, [_H]),
+    "clGetKernelInfo": (_I, [_H, _U, _S, _P, POINTER(_S)]),
+    "clSetKernelArg": (_I, [_H, _U, _S, _P]),
+    "clEnqueueNDRangeKernel": (_I, [_H, _H, _U, _SZ3, _SZ3, _SZ3, _U, POINTER(_H), POINTER(_H)]),
     "b2clEnqueueReadImageSamples": (_I, [_H, _H, _H, _U, _U, _H, _S, _S, _H, _S, _U, POINTER(_H),
                                          POINTER(_H)]),
     "b2clEnqueueReadImageGrid": (_I, [_H, _H, _H, _U, POINTER(c_float), _SZ3, _U, _H, _S, _U,
@@ -349,6 +360,47 @@ class Session:
         check(lib().clEnqueueReadImage(self.queue, img, 1, sz3(origin), sz3(region), row_pitch,
                                        slice_pitch, _ptr(out), 0, None, None), "clEnqueueReadImage")
         return out
+
+    # ---- programs and kernels (translated kernels, include/b2cl_device.cuh) ----
+    def program(self, binary: bytes):
+        err = c_int32()
+        buf = ctypes.create_string_buffer(binary, len(binary))
+        bins = (c_void_p * 1)(ctypes.cast(buf, c_void_p))
+        lens = (c_size_t * 1)(len(binary))
+        devs = (c_void_p * 1)(self.device)
+        prog = lib().clCreateProgramWithBinary(self.ctx, 1, devs, lens, bins, None, byref(err))
+        check(err.value, "clCreateProgramWithBinary")
+        st = lib().clBuildProgram(prog, 0, None, None, None, None)
+        if st != CL_SUCCESS:
+            log = ctypes.create_string_buffer(4096)
+            lib().clGetProgramBuildInfo(prog, self.device, 0x1183, 4096, log, None)
+            raise CLError(st, f"clBuildProgram ({log.value.decode(errors='replace')})")
+        return prog
+
+    def kernel(self, prog, name: str):
+        err = c_int32()
+        k = lib().clCreateKernel(prog, name.encode(), byref(err))
+        check(err.value, "clCreateKernel")
+        return k
+
+    def set_args(self, k, *args) -> None:
+        """Each arg: a handle (c_void_p: cl_mem / cl_sampler), ("local", nbytes), or a
+        ctypes scalar (c_int32(3), c_float(2.0), ...)."""
+        for i, a in enumerate(args):
+            if isinstance(a, tuple) and a[0] == "local":
+                st = lib().clSetKernelArg(k, i, int(a[1]), None)
+            elif isinstance(a, (int, c_void_p)) and not isinstance(a, bool):
+                h = c_void_p(a.value if isinstance(a, c_void_p) else a)
+                st = lib().clSetKernelArg(k, i, ctypes.sizeof(h), byref(h))
+            else:
+                st = lib().clSetKernelArg(k, i, ctypes.sizeof(a), byref(a))
+            check(st, f"clSetKernelArg({i})")
+
+    def ndrange(self, k, gws, lws=None, offset=None) -> None:
+        dim = len(gws)
+        check(lib().clEnqueueNDRangeKernel(self.queue, k, dim, sz3(offset) if offset else None,
+                                           sz3(gws), sz3(lws) if lws else None, 0, None, None),
+              "clEnqueueNDRangeKernel")
 
     def finish(self) -> None:
         check(lib().clFinish(self.queue), "clFinish")

@@ -1,0 +1,204 @@
+// read.cuh -- the read built-in (read_imagef / read_imagei / read_imageui)
+// for one coordinate, shared by the library's kernels (csrc/kernels/sample.cu)
+// and by user kernels through include/b2cl_device.cuh.
+//
+// Everything is templated on a configuration C (Cfg: dims, format, sampler,
+// each possibly decided at run time) and on a parameter block P providing
+// `im` (dev::Image), `smp` (dev::Sampler) and `rclass` (dev::RetCode).
+// Rules: [CL1.2 §8.1-8.3] as implemented in image.cuh.
+#pragma once
+#include "image.cuh"
+
+namespace b2cl {
+using namespace dev;
+
+template <int DIMS, int TYPE, int ORDER, int NORM, int ADDR, int FILT, int RC>
+struct Cfg {
+  static constexpr int dims = DIMS, type = TYPE, order = ORDER, norm = NORM, addr = ADDR,
+                       filt = FILT, rc = RC;
+  static constexpr int nch = ORDER == RT ? RT : order_channels(ORDER);
+};
+
+// C with the image-shard row mapping compiled in (SH) or out (plain images)
+template <class C, bool SH>
+struct WithShard : C {
+  static constexpr bool shard = SH;
+};
+
+struct AxN {  // NEAREST, one axis
+  int i;
+  bool ok;
+};
+struct AxL {  // LINEAR, one axis
+  int i0, i1;
+  float a, oma;
+  bool ok0, ok1;
+};
+
+template <class C>
+__device__ __forceinline__ bool may_border(const Sampler& s) {
+  if constexpr (C::addr == RT) return s.addr == A_NONE || s.addr == A_CLAMP;
+  else return C::addr == A_NONE || C::addr == A_CLAMP;
+}
+
+template <class C>
+__device__ __forceinline__ AxN axis_n(const Sampler& s, float c, int n) {
+  AxN r;
+  if constexpr (C::addr == RT) r.i = axis_nearest_rt(s.addr, s.norm, c, n);
+  else r.i = axis_nearest<C::addr, C::norm>(c, n);
+  r.ok = !may_border<C>(s) || in_range(r.i, n);
+  return r;
+}
+
+template <class C>
+__device__ __forceinline__ AxL axis_l(const Sampler& s, float c, int n) {
+  AxL r;
+  if constexpr (C::addr == RT) axis_linear_rt(s.addr, s.norm, c, n, r.i0, r.i1, r.a);
+  else axis_linear<C::addr, C::norm>(c, n, r.i0, r.i1, r.a);
+  r.oma = __fsub_rn(1.0f, r.a);
+  const bool b = may_border<C>(s);
+  r.ok0 = !b || in_range(r.i0, n);
+  r.ok1 = !b || in_range(r.i1, n);
+  return r;
+}
+
+template <class C, class P>
+__device__ __forceinline__ int filt_of(const P& p) {
+  return C::filt == RT ? p.smp.filt : C::filt;
+}
+
+// start of texel row (j,k): ptr + k*slice_pitch + j*row_pitch (Fig. 6)
+// The outer index o (j of a 2D image, k of a 3D image) is a global index; its
+// storage row is (o - ob) mod extent, clamped into the stored rows (a tap
+// outside a shard's band + halo reads the nearest stored row: the caller
+// provides the halo; this only keeps the access in bounds).
+__device__ __forceinline__ int storage_row(const Image& im, int o, int extent) {
+  int l = o - im.ob;
+  l += l < 0 ? extent : 0;
+  l -= l >= extent ? extent : 0;
+  return min(max(l, 0), im.os - 1);
+}
+
+template <class C>
+__device__ __forceinline__ const char* row_ptr(const Image& im, int j, int k) {
+  if constexpr (C::shard) {
+    if (C::dims == 3) k = storage_row(im, k, im.d);
+    else if (C::dims == 2) j = storage_row(im, j, im.h);
+  }
+  const char* r = im.ptr + (uint64_t)(unsigned)k * im.sp + (uint64_t)(unsigned)j * im.rp;
+  // keep the absolute row pointer in registers: without this the compiler
+  // re-associates ptr + (row + i*es) and pays two extra 64-bit adds per tap
+  asm("" : "+l"(r));
+  return r;
+}
+
+// does any output component come from a constant of the channel map (0 or 1)?
+// Only those need the explicit NaN of reading A26; stored channels carry the
+// NaN weight through the blend by themselves.
+__device__ __forceinline__ bool const_in_output(int order, int outc) {
+  switch (order) {
+    case O_RGBA: case O_BGRA: case O_ARGB: case O_INTENSITY: return false;
+    case O_R: return outc > 1;
+    case O_RG: case O_RA: return outc > 1 + (order == O_RG);
+    case O_LUMINANCE: return outc > 3;
+    default: return true;  // O_A
+  }
+}
+
+template <class C>
+__device__ __forceinline__ int elem_size(const Image& im) {
+  return (C::type == RT || C::nch == RT) ? im.es : C::nch * type_bytes(C::type);
+}
+
+// memory-order channels of the texel at row + i*elem_size (zero if !ok)
+template <class C>
+__device__ __forceinline__ void fetch(const Image& im, const char* row, int i, bool ok, int rc,
+                                      uint32_t m[4]) {
+  const int type = C::type == RT ? im.type : C::type;
+  const int nch = C::nch == RT ? im.nch : C::nch;
+  const int es = elem_size<C>(im);
+  m[0] = m[1] = m[2] = m[3] = 0u;
+  if (!ok) return;
+  Raw r = load_raw(row + (uint64_t)(unsigned)i * (unsigned)es, es);
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    if (c < nch) {
+      uint32_t v = channel_code(r, c, type);
+      m[c] = rc == R_F ? __float_as_uint(code_to_float(v, type)) : v;
+    }
+  }
+}
+
+// NEAREST: one texel, channel-mapped
+template <class C, class P>
+__device__ __forceinline__ void nearest_at(const P& p, const char* row, const AxN& x,
+                                           bool row_ok, uint32_t res[4]) {
+  const int rc = C::rc == RT ? p.rclass : C::rc;
+  const int order = C::order == RT ? p.im.order : C::order;
+  uint32_t m[4];
+  fetch<C>(p.im, row, x.i, row_ok && x.ok, rc, m);
+  map_order(order, m, rc == R_F ? 0x3f800000u : 1u, res);
+}
+
+// LINEAR from the texel rows: rows[0] = (j0,k0), [1] = (j1,k0), [2] = (j0,k1),
+// [3] = (j1,k1); blend x, then y, then z ([CL1.2 §8.2] weights, separable form)
+template <class C, class P>
+__device__ __forceinline__ void linear_at(const P& p, const char* const rows[4],
+                                          const bool rok[4], const AxL& x, float b, float omb,
+                                          float g, float omg, uint32_t res[4], int outc = 4) {
+  constexpr int NR = C::dims == 1 ? 1 : (C::dims == 2 ? 2 : 4);
+  const int order = C::order == RT ? p.im.order : C::order;
+  const int nch = C::nch == RT ? p.im.nch : C::nch;
+  uint32_t t0[NR][4], t1[NR][4];
+#pragma unroll
+  for (int r = 0; r < NR; ++r) {
+    fetch<C>(p.im, rows[r], x.i0, rok[r] && x.ok0, R_F, t0[r]);
+    fetch<C>(p.im, rows[r], x.i1, rok[r] && x.ok1, R_F, t1[r]);
+  }
+  uint32_t m[4];
+#pragma unroll
+  for (int ch = 0; ch < 4; ++ch) {
+    float v[NR];
+#pragma unroll
+    for (int r = 0; r < NR; ++r)
+      v[r] = lerp1(x.a, x.oma, __uint_as_float(t0[r][ch]), __uint_as_float(t1[r][ch]));
+    float o = v[0];
+    if constexpr (C::dims >= 2) {
+      const float s0 = lerp1(b, omb, v[0], v[1]);
+      o = s0;
+      if constexpr (C::dims == 3) o = lerp1(g, omg, s0, lerp1(b, omb, v[2], v[3]));
+    }
+    // channels the format does not store stay exactly 0 / 1 after the map
+    m[ch] = ch < nch ? __float_as_uint(o) : 0u;
+  }
+  map_order(order, m, 0x3f800000u, res);
+  // a NaN weight (non-finite coordinate) makes the spec's sum NaN in every
+  // component, including the constant ones (reading A26)
+  if (const_in_output(order, outc) && (x.a != x.a || b != b || g != g))
+    res[0] = res[1] = res[2] = res[3] = 0x7fffffffu;
+}
+
+// The built-in on one coordinate: c[0..DIMS-1] -> res (x,y,z,w) as 32-bit patterns.
+template <class C, class P>
+__device__ __forceinline__ void read_image(const P& p, const float c[3],
+                                           uint32_t res[4], int outc = 4) {
+  const Image& im = p.im;
+  if (filt_of<C>(p) == F_NEAREST) {
+    const AxN x = axis_n<C>(p.smp, c[0], im.w);
+    AxN y{0, true}, z{0, true};
+    if (C::dims > 1) y = axis_n<C>(p.smp, c[1], im.h);
+    if (C::dims > 2) z = axis_n<C>(p.smp, c[2], im.d);
+    nearest_at<C>(p, row_ptr<C>(im, y.i, z.i), x, y.ok && z.ok, res);
+  } else {
+    const AxL x = axis_l<C>(p.smp, c[0], im.w);
+    AxL y{0, 0, 0.f, 1.f, true, true}, z{0, 0, 0.f, 1.f, true, true};
+    if (C::dims > 1) y = axis_l<C>(p.smp, c[1], im.h);
+    if (C::dims > 2) z = axis_l<C>(p.smp, c[2], im.d);
+    const char* rows[4] = {row_ptr<C>(im, y.i0, z.i0), row_ptr<C>(im, y.i1, z.i0),
+                           row_ptr<C>(im, y.i0, z.i1), row_ptr<C>(im, y.i1, z.i1)};
+    const bool rok[4] = {y.ok0 && z.ok0, y.ok1 && z.ok0, y.ok0 && z.ok1, y.ok1 && z.ok1};
+    linear_at<C>(p, rows, rok, x, y.a, y.oma, z.a, z.oma, res, outc);
+  }
+}
+
+}  // namespace b2cl

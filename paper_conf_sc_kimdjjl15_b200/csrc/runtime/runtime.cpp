@@ -1622,4 +1622,363 @@ extern "C" cl_mem b2clCreateBufferFromIpcHandle(cl_context c, cl_device_id d, co
   return m;
 }
 
+// ===================================================================== programs and kernels
+// The paper's OpenCL-to-CUDA launch path: clBuildProgram -> module load
+// (P:119-121), clSetKernelArg collects the arguments, clEnqueueNDRangeKernel
+// -> one launch with grid = global / local, __local arguments as
+// sizes carving one dynamic shared array (Fig. 5(b)).
+struct KArg {
+  int kind = 0;  // 0 unset, 1 bytes, 2 memory object, 3 sampler, 4 __local
+  std::vector<unsigned char> bytes;
+  cl_mem mem = nullptr;
+  cl_sampler smp = nullptr;
+  size_t local = 0;
+};
+
+struct _cl_program {
+  std::atomic<int> ref{1};
+  cl_context ctx;
+  std::vector<int> ordinals;                        // one module per device
+  std::vector<std::vector<unsigned char>> images;   // NUL-terminated (PTX text is allowed)
+  std::vector<cudaLibrary_t> libs;
+  std::vector<void*> offset_sym;                    // __b2cl_global_offset per module (or null)
+  cl_int status = CL_BUILD_NONE;
+  std::string log;
+};
+
+struct _cl_kernel {
+  std::atomic<int> ref{1};
+  cl_program prog;
+  std::string name;
+  std::vector<cudaKernel_t> kerns;  // per program module
+  std::vector<size_t> psize;        // parameter sizes
+  std::vector<KArg> args;
+};
+
+static std::set<cl_program> g_programs;
+static std::set<cl_kernel> g_kernels;
+
+extern "C" cl_program clCreateProgramWithBinary(cl_context c, cl_uint n, const cl_device_id* devs,
+                                                const size_t* lengths, const unsigned char** bins,
+                                                cl_int* binary_status, cl_int* errcode_ret) {
+  if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
+  if (n == 0 || !devs || !lengths || !bins) { SET_ERR(CL_INVALID_VALUE); return nullptr; }
+  auto* p = new (std::nothrow) _cl_program();
+  if (!p) { SET_ERR(CL_OUT_OF_HOST_MEMORY); return nullptr; }
+  p->ctx = c;
+  for (cl_uint i = 0; i < n; ++i) {
+    if (!valid_device(devs[i]) || !ctx_has_device(c, devs[i])) {
+      delete p;
+      SET_ERR(CL_INVALID_DEVICE);
+      return nullptr;
+    }
+    if (lengths[i] == 0 || !bins[i]) {
+      if (binary_status) binary_status[i] = CL_INVALID_VALUE;
+      delete p;
+      SET_ERR(CL_INVALID_VALUE);
+      return nullptr;
+    }
+    if (binary_status) binary_status[i] = CL_SUCCESS;
+    if (std::find(p->ordinals.begin(), p->ordinals.end(), devs[i]->ordinal) != p->ordinals.end())
+      continue;
+    p->ordinals.push_back(devs[i]->ordinal);
+    std::vector<unsigned char> img(bins[i], bins[i] + lengths[i]);
+    img.push_back(0);
+    p->images.push_back(std::move(img));
+  }
+  c->ref++;
+  {
+    std::lock_guard<std::mutex> g(g_mu);
+    g_programs.insert(p);
+  }
+  SET_ERR(CL_SUCCESS);
+  return p;
+}
+
+extern "C" cl_int clBuildProgram(cl_program p, cl_uint n, const cl_device_id* devs,
+                                 const char* options, void(CL_CALLBACK* notify)(cl_program, void*),
+                                 void* user_data) {
+  (void)options;
+  if (!live(g_programs, p)) return CL_INVALID_PROGRAM;
+  if ((n == 0) != (devs == nullptr) || (!notify && user_data)) return CL_INVALID_VALUE;
+  if (!p->libs.empty()) return CL_INVALID_OPERATION;  // already built (kernels may exist)
+  p->log.clear();
+  for (size_t i = 0; i < p->ordinals.size(); ++i) {
+    DeviceGuard g(p->ordinals[i]);
+    cudaLibrary_t lib = nullptr;
+    cudaError_t e = cudaLibraryLoadData(&lib, p->images[i].data(), nullptr, nullptr, 0, nullptr,
+                                        nullptr, 0);
+    // module loading may be lazy: an image with no kernel is a failed build
+    unsigned nk = 0;
+    if (e == cudaSuccess && (cudaLibraryGetKernelCount(&nk, lib) != cudaSuccess || nk == 0)) {
+      cudaLibraryUnload(lib);
+      e = cudaErrorInvalidKernelImage;
+    }
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      p->log = std::string("module load failed on device ") + std::to_string(p->ordinals[i]) +
+               ": " + cudaGetErrorString(e);
+      for (auto l : p->libs) cudaLibraryUnload(l);
+      p->libs.clear();
+      p->offset_sym.clear();
+      p->status = CL_BUILD_ERROR;
+      if (notify) notify(p, user_data);
+      return CL_BUILD_PROGRAM_FAILURE;
+    }
+    void* sym = nullptr;
+    size_t bytes = 0;
+    if (cudaLibraryGetGlobal(&sym, &bytes, lib, "__b2cl_global_offset") != cudaSuccess ||
+        bytes < 3 * sizeof(size_t)) {
+      cudaGetLastError();
+      sym = nullptr;
+    }
+    p->libs.push_back(lib);
+    p->offset_sym.push_back(sym);
+  }
+  p->status = CL_BUILD_SUCCESS;
+  if (notify) notify(p, user_data);
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clGetProgramBuildInfo(cl_program p, cl_device_id d, cl_program_build_info name,
+                                        size_t size, void* value, size_t* size_ret) {
+  if (!live(g_programs, p)) return CL_INVALID_PROGRAM;
+  if (!valid_device(d)) return CL_INVALID_DEVICE;
+  switch (name) {
+    case CL_PROGRAM_BUILD_STATUS: return get_info<cl_int>(p->status, size, value, size_ret);
+    case CL_PROGRAM_BUILD_LOG: return get_str(p->log.c_str(), size, value, size_ret);
+    default: return CL_INVALID_VALUE;
+  }
+}
+
+extern "C" cl_int clRetainProgram(cl_program p) {
+  if (!live(g_programs, p)) return CL_INVALID_PROGRAM;
+  p->ref++;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clReleaseProgram(cl_program p) {
+  if (!live(g_programs, p)) return CL_INVALID_PROGRAM;
+  if (--p->ref == 0) {
+    {
+      std::lock_guard<std::mutex> g(g_mu);
+      g_programs.erase(p);
+    }
+    for (size_t i = 0; i < p->libs.size(); ++i) {
+      DeviceGuard g(p->ordinals[i]);
+      cudaDeviceSynchronize();  // no launch of the module may still be running
+      cudaLibraryUnload(p->libs[i]);
+    }
+    cl_context c = p->ctx;
+    delete p;
+    clReleaseContext(c);
+  }
+  return CL_SUCCESS;
+}
+
+extern "C" cl_kernel clCreateKernel(cl_program p, const char* name, cl_int* errcode_ret) {
+  if (!live(g_programs, p)) { SET_ERR(CL_INVALID_PROGRAM); return nullptr; }
+  if (!name) { SET_ERR(CL_INVALID_VALUE); return nullptr; }
+  if (p->status != CL_BUILD_SUCCESS) { SET_ERR(CL_INVALID_PROGRAM_EXECUTABLE); return nullptr; }
+  auto* k = new (std::nothrow) _cl_kernel();
+  if (!k) { SET_ERR(CL_OUT_OF_HOST_MEMORY); return nullptr; }
+  k->prog = p;
+  k->name = name;
+  for (size_t i = 0; i < p->libs.size(); ++i) {
+    DeviceGuard g(p->ordinals[i]);
+    cudaKernel_t kern = nullptr;
+    if (cudaLibraryGetKernel(&kern, p->libs[i], name) != cudaSuccess) {
+      cudaGetLastError();
+      delete k;
+      SET_ERR(CL_INVALID_KERNEL_NAME);
+      return nullptr;
+    }
+    k->kerns.push_back(kern);
+  }
+  // parameter sizes from the module's metadata
+  {
+    DeviceGuard g(p->ordinals[0]);
+    for (size_t idx = 0;; ++idx) {
+      size_t off = 0, sz = 0;
+      if (cudaFuncGetParamInfo(reinterpret_cast<const void*>(k->kerns[0]), idx, &off, &sz) !=
+          cudaSuccess) {
+        cudaGetLastError();
+        break;
+      }
+      k->psize.push_back(sz);
+    }
+  }
+  k->args.resize(k->psize.size());
+  p->ref++;
+  {
+    std::lock_guard<std::mutex> g(g_mu);
+    g_kernels.insert(k);
+  }
+  SET_ERR(CL_SUCCESS);
+  return k;
+}
+
+extern "C" cl_int clRetainKernel(cl_kernel k) {
+  if (!live(g_kernels, k)) return CL_INVALID_KERNEL;
+  k->ref++;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clReleaseKernel(cl_kernel k) {
+  if (!live(g_kernels, k)) return CL_INVALID_KERNEL;
+  if (--k->ref == 0) {
+    {
+      std::lock_guard<std::mutex> g(g_mu);
+      g_kernels.erase(k);
+    }
+    cl_program p = k->prog;
+    delete k;
+    clReleaseProgram(p);
+  }
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int clGetKernelInfo(cl_kernel k, cl_kernel_info name, size_t size, void* value,
+                                  size_t* size_ret) {
+  if (!live(g_kernels, k)) return CL_INVALID_KERNEL;
+  switch (name) {
+    case CL_KERNEL_FUNCTION_NAME: return get_str(k->name.c_str(), size, value, size_ret);
+    case CL_KERNEL_NUM_ARGS: return get_info<cl_uint>((cl_uint)k->psize.size(), size, value, size_ret);
+    case CL_KERNEL_REFERENCE_COUNT: return get_info<cl_uint>(k->ref.load(), size, value, size_ret);
+    default: return CL_INVALID_VALUE;
+  }
+}
+
+extern "C" cl_int clSetKernelArg(cl_kernel k, cl_uint index, size_t size, const void* value) {
+  if (!live(g_kernels, k)) return CL_INVALID_KERNEL;
+  if (index >= k->psize.size()) return CL_INVALID_ARG_INDEX;
+  const size_t want = k->psize[index];
+  KArg a;
+  if (!value) {  // __local: the kernel parameter is the size (Fig. 5(b))
+    if (size == 0) return CL_INVALID_ARG_SIZE;
+    if (want != sizeof(size_t)) return CL_INVALID_ARG_VALUE;
+    a.kind = 4;
+    a.local = size;
+  } else {
+    void* h = nullptr;
+    if (size == sizeof(void*)) memcpy(&h, value, sizeof(void*));
+    if (h && live(g_mems, static_cast<cl_mem>(h))) {
+      cl_mem m = static_cast<cl_mem>(h);
+      if (m->ctx != k->prog->ctx) return CL_INVALID_MEM_OBJECT;
+      if (want != (is_image(m) ? sizeof(dev::Image) : sizeof(void*))) return CL_INVALID_ARG_SIZE;
+      a.kind = 2;
+      a.mem = m;
+    } else if (h && live(g_samplers, static_cast<cl_sampler>(h))) {
+      if (want != sizeof(uint32_t)) return CL_INVALID_ARG_SIZE;
+      a.kind = 3;
+      a.smp = static_cast<cl_sampler>(h);
+    } else {
+      if (size != want) return CL_INVALID_ARG_SIZE;
+      a.kind = 1;
+      a.bytes.assign(static_cast<const unsigned char*>(value),
+                     static_cast<const unsigned char*>(value) + size);
+    }
+  }
+  k->args[index] = std::move(a);
+  return CL_SUCCESS;
+}
+
+// largest divisor of g not above cap
+static size_t pick_local(size_t g, size_t cap) {
+  for (size_t l = std::min(g, cap); l > 1; --l)
+    if (g % l == 0) return l;
+  return 1;
+}
+
+extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uint work_dim,
+                                         const size_t* goff, const size_t* gws, const size_t* lws,
+                                         cl_uint nw, const cl_event* wl, cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  if (!live(g_kernels, k)) return CL_INVALID_KERNEL;
+  if (k->prog->ctx != q->ctx) return CL_INVALID_CONTEXT;
+  const auto it = std::find(k->prog->ordinals.begin(), k->prog->ordinals.end(), q->dev->ordinal);
+  if (it == k->prog->ordinals.end()) return CL_INVALID_PROGRAM_EXECUTABLE;
+  const size_t mi = it - k->prog->ordinals.begin();
+  if (work_dim < 1 || work_dim > 3) return CL_INVALID_WORK_DIMENSION;
+  if (!gws) return CL_INVALID_VALUE;
+  for (const KArg& a : k->args)
+    if (a.kind == 0) return CL_INVALID_KERNEL_ARGS;
+  size_t G[3] = {1, 1, 1}, Lw[3] = {1, 1, 1}, O[3] = {0, 0, 0};
+  for (cl_uint d = 0; d < work_dim; ++d) {
+    G[d] = gws[d];
+    if (G[d] == 0) return -63;  // CL_INVALID_GLOBAL_WORK_SIZE
+    if (goff) O[d] = goff[d];
+  }
+  if (lws) {
+    for (cl_uint d = 0; d < work_dim; ++d) {
+      Lw[d] = lws[d];
+      if (Lw[d] == 0 || G[d] % Lw[d] != 0) return CL_INVALID_WORK_GROUP_SIZE;
+    }
+    if (Lw[0] > 1024 || Lw[1] > 1024 || Lw[2] > 64) return CL_INVALID_WORK_ITEM_SIZE;
+    if (Lw[0] * Lw[1] * Lw[2] > 1024) return CL_INVALID_WORK_GROUP_SIZE;
+  } else {
+    const size_t caps[3][3] = {{256, 1, 1}, {32, 8, 1}, {32, 4, 2}};
+    for (cl_uint d = 0; d < work_dim; ++d) Lw[d] = pick_local(G[d], caps[work_dim - 1][d]);
+  }
+  const size_t grid[3] = {G[0] / Lw[0], G[1] / Lw[1], G[2] / Lw[2]};
+  if (grid[0] > 0x7fffffffull || grid[1] > 65535 || grid[2] > 65535) return -63;
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = CL_COMMAND_NDRANGE_KERNEL;
+  DeviceGuard g(q->dev->ordinal);
+  // argument values, in parameter order
+  const size_t na = k->args.size();
+  std::vector<std::vector<unsigned char>> vals(na);
+  std::vector<void*> argp(na);
+  size_t local_bytes = 0;
+  for (size_t i = 0; i < na; ++i) {
+    const KArg& a = k->args[i];
+    if (a.kind == 1) {
+      vals[i] = a.bytes;
+    } else if (a.kind == 2) {
+      char* ptr = nullptr;
+      CHECK(resident(a.mem, q, true, &ptr));
+      if (is_image(a.mem)) {
+        const dev::Image im = dev_image(a.mem, ptr, true);
+        vals[i].resize(sizeof(im));
+        memcpy(vals[i].data(), &im, sizeof(im));
+      } else {
+        vals[i].resize(sizeof(ptr));
+        memcpy(vals[i].data(), &ptr, sizeof(ptr));
+      }
+    } else if (a.kind == 3) {
+      const uint32_t bits = (a.smp->norm ? 1u : 0u) | ((a.smp->addr - CL_ADDRESS_NONE) << 1) |
+                            (a.smp->filt == CL_FILTER_LINEAR ? 0x20u : 0x10u);
+      vals[i].resize(4);
+      memcpy(vals[i].data(), &bits, 4);
+    } else {
+      vals[i].resize(sizeof(size_t));
+      memcpy(vals[i].data(), &a.local, sizeof(size_t));
+      local_bytes += a.local;
+    }
+    argp[i] = vals[i].data();
+  }
+  CHECK(enq_begin(E, nw, wl));
+  const void* fn = reinterpret_cast<const void*>(k->kerns[mi]);
+  cudaError_t e = cudaSuccess;
+  if (local_bytes > 48 * 1024)
+    e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)local_bytes);
+  void* osym = k->prog->offset_sym[mi];
+  if (e == cudaSuccess && osym)  // get_global_offset(): pageable source, staged before return
+    e = cudaMemcpyAsync(osym, O, sizeof(O), cudaMemcpyHostToDevice, q->stream);
+  if (e == cudaSuccess) {
+    e = cudaLaunchKernel(fn, dim3((unsigned)grid[0], (unsigned)grid[1], (unsigned)grid[2]),
+                         dim3((unsigned)Lw[0], (unsigned)Lw[1], (unsigned)Lw[2]), argp.data(),
+                         local_bytes, q->stream);
+    if (e == cudaSuccess) count_launch();
+  }
+  cl_int st = enq_end(E, e);
+  if (st == CL_SUCCESS)
+    for (const KArg& a : k->args)
+      if (a.kind == 2) written(a.mem, q);
+  return st;
+}
+
 extern "C" cl_ulong b2clGetKernelLaunchCount(void) { return launch_count(); }
