@@ -54,6 +54,19 @@ extern __shared__ __align__(16) char __OC2CU_shared_mem[];
 // each launch when the module defines it (this header does)
 __device__ size_t __b2cl_global_offset[3];
 
+// Dynamic __constant arguments (Fig. 5(b) line 2): one constant
+// array; each __constant argument becomes its size (size_t) and the kernel
+// carves the array by the running sum, in argument order.  The buffer stays
+// in global memory until the launch, which copies it here (the paper's
+// deferred placement).  A kernel declares which arguments are
+// __constant with B2CL_KERNEL_CONSTANT_ARGS(name, bitmask of argument indices).
+#ifndef B2CL_MAX_CONST_SIZE
+#define B2CL_MAX_CONST_SIZE 32768
+#endif
+__constant__ __align__(16) char __OC2CU_const_mem[B2CL_MAX_CONST_SIZE];
+#define B2CL_KERNEL_CONSTANT_ARGS(kernel_name, mask) \
+  extern "C" __device__ const unsigned int __b2cl_const_args_##kernel_name = (mask)
+
 // ---- work-item functions ----
 __device__ __forceinline__ size_t get_local_id(unsigned d) {
   return d == 0 ? threadIdx.x : (d == 1 ? threadIdx.y : (d == 2 ? threadIdx.z : 0));

@@ -1628,7 +1628,7 @@ extern "C" cl_mem b2clCreateBufferFromIpcHandle(cl_context c, cl_device_id d, co
 // -> one launch with grid = global / local, __local arguments as
 // sizes carving one dynamic shared array (Fig. 5(b)).
 struct KArg {
-  int kind = 0;  // 0 unset, 1 bytes, 2 memory object, 3 sampler, 4 __local
+  int kind = 0;  // 0 unset, 1 bytes, 2 memory object, 3 sampler, 4 __local, 5 __constant
   std::vector<unsigned char> bytes;
   cl_mem mem = nullptr;
   cl_sampler smp = nullptr;
@@ -1642,6 +1642,8 @@ struct _cl_program {
   std::vector<std::vector<unsigned char>> images;   // NUL-terminated (PTX text is allowed)
   std::vector<cudaLibrary_t> libs;
   std::vector<void*> offset_sym;                    // __b2cl_global_offset per module (or null)
+  std::vector<void*> const_sym;                     // __OC2CU_const_mem per module (or null)
+  size_t const_bytes = 0;
   cl_int status = CL_BUILD_NONE;
   std::string log;
 };
@@ -1653,6 +1655,7 @@ struct _cl_kernel {
   std::vector<cudaKernel_t> kerns;  // per program module
   std::vector<size_t> psize;        // parameter sizes
   std::vector<KArg> args;
+  uint32_t const_mask = 0;          // __constant arguments (B2CL_KERNEL_CONSTANT_ARGS)
 };
 
 static std::set<cl_program> g_programs;
@@ -1721,6 +1724,7 @@ extern "C" cl_int clBuildProgram(cl_program p, cl_uint n, const cl_device_id* de
       for (auto l : p->libs) cudaLibraryUnload(l);
       p->libs.clear();
       p->offset_sym.clear();
+      p->const_sym.clear();
       p->status = CL_BUILD_ERROR;
       if (notify) notify(p, user_data);
       return CL_BUILD_PROGRAM_FAILURE;
@@ -1732,8 +1736,17 @@ extern "C" cl_int clBuildProgram(cl_program p, cl_uint n, const cl_device_id* de
       cudaGetLastError();
       sym = nullptr;
     }
+    void* csym = nullptr;
+    size_t cbytes = 0;
+    if (cudaLibraryGetGlobal(&csym, &cbytes, lib, "__OC2CU_const_mem") != cudaSuccess) {
+      cudaGetLastError();
+      csym = nullptr;
+      cbytes = 0;
+    }
     p->libs.push_back(lib);
     p->offset_sym.push_back(sym);
+    p->const_sym.push_back(csym);
+    p->const_bytes = cbytes;
   }
   p->status = CL_BUILD_SUCCESS;
   if (notify) notify(p, user_data);
@@ -1809,6 +1822,16 @@ extern "C" cl_kernel clCreateKernel(cl_program p, const char* name, cl_int* errc
     }
   }
   k->args.resize(k->psize.size());
+  {  // which arguments are __constant (a module global written by the translator)
+    DeviceGuard g(p->ordinals[0]);
+    void* m = nullptr;
+    size_t mb = 0;
+    const std::string sym = "__b2cl_const_args_" + k->name;
+    if (cudaLibraryGetGlobal(&m, &mb, p->libs[0], sym.c_str()) == cudaSuccess && mb == 4) {
+      if (cudaMemcpy(&k->const_mask, m, 4, cudaMemcpyDeviceToHost) != cudaSuccess) k->const_mask = 0;
+    }
+    cudaGetLastError();
+  }
   p->ref++;
   {
     std::lock_guard<std::mutex> g(g_mu);
@@ -1854,7 +1877,17 @@ extern "C" cl_int clSetKernelArg(cl_kernel k, cl_uint index, size_t size, const 
   if (index >= k->psize.size()) return CL_INVALID_ARG_INDEX;
   const size_t want = k->psize[index];
   KArg a;
-  if (!value) {  // __local: the kernel parameter is the size (Fig. 5(b))
+  const bool is_const = index < 32 && ((k->const_mask >> index) & 1u);
+  if (is_const) {  // __constant buffer: the parameter is its size (Fig. 5(b))
+    void* h = nullptr;
+    if (value && size == sizeof(void*)) memcpy(&h, value, sizeof(void*));
+    cl_mem m = static_cast<cl_mem>(h);
+    if (!h || !live(g_mems, m) || m->type != CL_MEM_OBJECT_BUFFER) return CL_INVALID_ARG_VALUE;
+    if (m->ctx != k->prog->ctx) return CL_INVALID_MEM_OBJECT;
+    if (want != sizeof(size_t)) return CL_INVALID_ARG_SIZE;
+    a.kind = 5;
+    a.mem = m;
+  } else if (!value) {  // __local: the kernel parameter is the size (Fig. 5(b))
     if (size == 0) return CL_INVALID_ARG_SIZE;
     if (want != sizeof(size_t)) return CL_INVALID_ARG_VALUE;
     a.kind = 4;
@@ -1932,7 +1965,12 @@ extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uin
   const size_t na = k->args.size();
   std::vector<std::vector<unsigned char>> vals(na);
   std::vector<void*> argp(na);
-  size_t local_bytes = 0;
+  size_t local_bytes = 0, const_bytes = 0;
+  for (const KArg& a : k->args)
+    if (a.kind == 5) const_bytes += a.mem->size;
+  if (const_bytes && (!k->prog->const_sym[mi] || const_bytes > k->prog->const_bytes))
+    return CL_OUT_OF_RESOURCES;  // more __constant data than the module's constant array
+  std::vector<std::pair<char*, size_t>> const_src;  // (device pointer, bytes) in argument order
   for (size_t i = 0; i < na; ++i) {
     const KArg& a = k->args[i];
     if (a.kind == 1) {
@@ -1953,6 +1991,12 @@ extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uin
                             (a.smp->filt == CL_FILTER_LINEAR ? 0x20u : 0x10u);
       vals[i].resize(4);
       memcpy(vals[i].data(), &bits, 4);
+    } else if (a.kind == 5) {
+      char* ptr = nullptr;
+      CHECK(resident(a.mem, q, true, &ptr));
+      const_src.emplace_back(ptr, a.mem->size);
+      vals[i].resize(sizeof(size_t));
+      memcpy(vals[i].data(), &a.mem->size, sizeof(size_t));
     } else {
       vals[i].resize(sizeof(size_t));
       memcpy(vals[i].data(), &a.local, sizeof(size_t));
@@ -1968,6 +2012,14 @@ extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uin
   void* osym = k->prog->offset_sym[mi];
   if (e == cudaSuccess && osym)  // get_global_offset(): pageable source, staged before return
     e = cudaMemcpyAsync(osym, O, sizeof(O), cudaMemcpyHostToDevice, q->stream);
+  // deferred placement of __constant buffers: copied at launch
+  size_t coff = 0;
+  for (const auto& cs : const_src) {
+    if (e != cudaSuccess) break;
+    e = cudaMemcpyAsync(static_cast<char*>(k->prog->const_sym[mi]) + coff, cs.first, cs.second,
+                        cudaMemcpyDeviceToDevice, q->stream);
+    coff += cs.second;
+  }
   if (e == cudaSuccess) {
     e = cudaLaunchKernel(fn, dim3((unsigned)grid[0], (unsigned)grid[1], (unsigned)grid[2]),
                          dim3((unsigned)Lw[0], (unsigned)Lw[1], (unsigned)Lw[2]), argp.data(),
@@ -1977,7 +2029,7 @@ extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uin
   cl_int st = enq_end(E, e);
   if (st == CL_SUCCESS)
     for (const KArg& a : k->args)
-      if (a.kind == 2) written(a.mem, q);
+      if (a.kind == 2) written(a.mem, q);  // __constant (kind 5) buffers are only read
   return st;
 }
 

@@ -141,3 +141,28 @@ def test_launch_glue_errors(sess, prog):
     L.clReleaseKernel(k)
     sess.release(out, img)
     L.clReleaseSampler(smp)
+
+
+def test_dynamic_constant_arguments(sess, prog):
+    """__constant buffers stay in global memory until the launch copies them into
+    the module's constant array."""
+    g = synth.rng(82)
+    n1, n2, N = 37, 100, 1024
+    lut1 = g.uniform(-1, 1, n1).astype(np.float32)
+    lut2 = g.uniform(-1, 1, n2).astype(np.float32)
+    b1, b2 = sess.buffer(lut1.nbytes, lut1), sess.buffer(lut2.nbytes, lut2)
+    out = sess.buffer(N * 4)
+    k = sess.kernel(prog, "const_lut")
+    sess.set_args(k, out, b1, b2, ctypes.c_int32(n1), ctypes.c_int32(n2))
+    sess.ndrange(k, (N,), (128,))
+    i = np.arange(N)
+    assert np.array_equal(sess.read(out, N * 4, np.float32), lut1[i % n1] + lut2[i % n2])
+    # new contents are picked up by the next launch (copied at launch time)
+    sess.write(b1, -lut1)
+    sess.ndrange(k, (N,), (128,))
+    assert np.array_equal(sess.read(out, N * 4, np.float32), -lut1[i % n1] + lut2[i % n2])
+    # a non-buffer for a __constant argument is rejected
+    v = ctypes.c_int64(5)
+    assert cl.lib().clSetKernelArg(k, 1, 8, ctypes.byref(v)) == -50
+    cl.lib().clReleaseKernel(k)
+    sess.release(b1, b2, out)
