@@ -222,22 +222,21 @@ __global__ void __launch_bounds__(128) k_sample_grid_walk(const SampleParams p) 
     return axis_l<C>(p.smp, __fadd_rn(__fmul_rn(awc, __int2float_rn(wor + wv)), awo), nw);
   };
   AxL aw = walk_axis(w0);
-  Rows lo, hi;
-  walk_load<C, NJ, XPT>(im, ax, afix, aw.i0, aw.ok0, lo);
-  walk_load<C, NJ, XPT>(im, ax, afix, aw.i1, aw.ok1, hi);
-#pragma unroll 1
-  for (int w = 0; w < WALK; ++w) {
+  // Three row buffers in fixed rotating roles (lo, hi, next-hi): no register
+  // copies between steps.  A step issues the next hi rows, blends (lo, hi),
+  // and -- only when the next lo rows are not this hi (no reuse) -- reloads
+  // them into the hi buffer after the blend, which becomes the next lo.
+  Rows B0, B1, B2;
+  walk_load<C, NJ, XPT>(im, ax, afix, aw.i0, aw.ok0, B0);
+  walk_load<C, NJ, XPT>(im, ax, afix, aw.i1, aw.ok1, B1);
+  // one step with (lo, hi, nx) = rows at aw; returns false after the last step
+  auto step = [&](int w, Rows& lo, Rows& hi, Rows& nx) -> bool {
     const int wv = w0 + w;
-    // issue the next step's loads first
     const bool next = w + 1 < WALK && wv + 1 < wlen;
     AxL an = aw;
-    Rows nlo, nhi;
-    bool reuse = false;
     if (next) {
       an = walk_axis(wv + 1);
-      reuse = an.i0 == aw.i1 && an.ok0 == aw.ok1;
-      walk_load<C, NJ, XPT>(im, ax, afix, an.i1, an.ok1, nhi);
-      if (!reuse) walk_load<C, NJ, XPT>(im, ax, afix, an.i0, an.ok0, nlo);
+      walk_load<C, NJ, XPT>(im, ax, afix, an.i1, an.ok1, nx);
     }
     // blend and store this step: x, then y, then z (as linear_at)
     const AxL& ay = D3 ? afix : aw;
@@ -272,10 +271,18 @@ __global__ void __launch_bounds__(128) k_sample_grid_walk(const SampleParams p) 
         res[0] = res[1] = res[2] = res[3] = 0x7fffffffu;
       if (x < p.ow) store_out<OUTC>(p, obase + x, res);
     }
-    if (!next) break;
-    lo = reuse ? hi : nlo;
-    hi = nhi;
+    if (!next) return false;
+    // the next step's lo rows are this step's hi rows unless the walk skips
+    if (!(an.i0 == aw.i1 && an.ok0 == aw.ok1))
+      walk_load<C, NJ, XPT>(im, ax, afix, an.i0, an.ok0, hi);
     aw = an;
+    return true;
+  };
+#pragma unroll 1
+  for (int w = 0; w < WALK; w += 3) {
+    if (!step(w, B0, B1, B2)) break;
+    if (!step(w + 1, B1, B2, B0)) break;
+    if (!step(w + 2, B2, B0, B1)) break;
   }
 }
 
