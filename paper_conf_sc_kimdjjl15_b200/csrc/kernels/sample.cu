@@ -71,7 +71,7 @@ __global__ void __launch_bounds__(256) k_sample_grid(const SampleParams p) {
 // Separable maps: block = 32 x 4 threads; tile = (32*XPT) columns x (4*RPW) rows
 // of one output slice.  Lane -> columns lane + 32*t, warp -> RPW consecutive rows.
 template <class C, int OUTC, int XPT, int RPW>
-__global__ void __launch_bounds__(128, 12) k_sample_grid_sep(const SampleParams p) {
+__global__ void __launch_bounds__(128, 11) k_sample_grid_sep(const SampleParams p) {
   const Image& im = p.im;
   const int z = blockIdx.z;
   const int x0 = blockIdx.x * (32 * XPT) + threadIdx.x;
