@@ -51,7 +51,8 @@ class _Image(ctypes.Structure):
     _fields_ = [("data", ctypes.c_void_p),
                 ("width", ctypes.c_int64), ("height", ctypes.c_int64), ("depth", ctypes.c_int64),
                 ("row_pitch", ctypes.c_int64), ("slice_pitch", ctypes.c_int64),
-                ("dims", ctypes.c_int32), ("order", ctypes.c_uint32), ("type", ctypes.c_uint32)]
+                ("dims", ctypes.c_int32), ("order", ctypes.c_uint32), ("type", ctypes.c_uint32),
+                ("arrayed", ctypes.c_int32)]
 
 
 _lib = None
@@ -77,6 +78,8 @@ def lib():
         L.oracle_axis_nearest.argtypes = [ctypes.c_float, i64, i32, u32, ctypes.POINTER(i64)]
         L.oracle_axis_linear.argtypes = [ctypes.c_float, i64, i32, u32, ctypes.POINTER(i64),
                                          ctypes.POINTER(i64), ctypes.POINTER(ctypes.c_float)]
+        L.oracle_layer_index.argtypes = [ctypes.c_float, i64]
+        L.oracle_layer_index.restype = i64
         L.oracle_read_samples.argtypes = [P, i32, u32, u32, i32, i32, P, i64, i64, P]
         L.oracle_read_grid.argtypes = [P, i32, u32, u32, i32, P, i64, i64, i64, i32,
                                        i64, i64, i64, i64, P, i32]
@@ -114,11 +117,14 @@ def _ptr(a: np.ndarray) -> ctypes.c_void_p:
 
 
 class Image:
-    """A host image for the oracle: a byte array plus the Fig. 6 fields."""
+    """A host image for the oracle: a byte array plus the Fig. 6 fields.
+
+    Image arrays: ``arrayed=True`` with ``dims`` the sampled axes (1 or 2); the
+    layers are ``height`` (1D array) or ``depth`` (2D array)."""
 
     def __init__(self, data: np.ndarray, width: int, height: int = 1, depth: int = 1,
                  dims: int = 2, order: int = RGBA, type: int = FLOAT,
-                 row_pitch: int = 0, slice_pitch: int = 0):
+                 row_pitch: int = 0, slice_pitch: int = 0, arrayed: bool = False):
         es = elem_size(order, type)
         if es < 0:
             raise ValueError("format not supported")
@@ -131,10 +137,14 @@ class Image:
             raise ValueError(f"image data too small: {self.data.size} < {need}")
         self.width, self.height, self.depth, self.dims = width, height, depth, dims
         self.order, self.type = order, type
+        self.arrayed = bool(arrayed)
+        if self.arrayed and dims not in (1, 2):
+            raise ValueError("image arrays are 1D or 2D")
 
     def cstruct(self) -> _Image:
         return _Image(self.data.ctypes.data, self.width, self.height, self.depth,
-                      self.row_pitch, self.slice_pitch, self.dims, self.order, self.type)
+                      self.row_pitch, self.slice_pitch, self.dims, self.order, self.type,
+                      int(self.arrayed))
 
 
 def elem_size(order: int, type: int) -> int:
@@ -252,6 +262,11 @@ def write_image_rect(img: Image, origin, region, row_pitch, slice_pitch, host: n
 def rect_overlap(src_origin, dst_origin, region, srp=0, ssp=0, drp=0, dsp=0) -> bool:
     return bool(lib().oracle_rect_overlap(_sz3(src_origin), _sz3(dst_origin), _sz3(region),
                                           srp, ssp, drp, dsp))
+
+
+def layer_index(c: float, n: int) -> int:
+    """[CL1.2 §8.4] layer = clamp(rint(c), 0, n - 1)."""
+    return lib().oracle_layer_index(c, n)
 
 
 def axis_nearest(s: float, n: int, normalized: bool, addressing: int) -> int:

@@ -333,14 +333,27 @@ static int check_read(const oracle_image* img, int normalized, uint32_t addressi
 
 static void store16(const val32* v, void* out16) { memcpy(out16, v, 16); }
 
+/* [CL1.2 §8.4] "Selecting an Image from an Image Array": the layer is
+ * clamp(rint(w), 0, d - 1); rintf rounds half to even in the default mode. */
+int64_t oracle_layer_index(float c, int64_t n) {
+  if (isnan(c)) return 0;                                    /* A35 */
+  float r = rintf(c);
+  int64_t l = r >= 2147483648.0f ? INT32_MAX : (r < -2147483648.0f ? INT32_MIN : (int64_t)r);
+  return clamp64(l, 0, n - 1);
+}
+
 static void sample_checked(const oracle_image* img, int normalized, uint32_t addressing,
                            uint32_t filter, int rtype, const float* coord, void* out16) {
-  int dims = img->dims;
+  int dims = img->dims, nc = dims + (img->arrayed ? 1 : 0);
   int64_t n[3] = {img->width, img->height, img->depth};
-  float c[3] = {coord[0], dims > 1 ? coord[1] : 0.0f, dims > 2 ? coord[2] : 0.0f};
+  float c[3] = {coord[0], nc > 1 ? coord[1] : 0.0f, nc > 2 ? coord[2] : 0.0f};
+  /* an array's layer axis (the one after the sampled axes) is selected, not
+     addressed: the sampler's normalization, addressing and filter skip it */
+  int64_t layer = img->arrayed ? oracle_layer_index(c[dims], n[dims]) : 0;
   if (filter == OR_FILTER_NEAREST) {
     int64_t ix[3] = {0, 0, 0};
     for (int d = 0; d < dims; ++d) oracle_axis_nearest(c[d], n[d], normalized, addressing, &ix[d]);
+    if (img->arrayed) ix[dims] = layer;
     val32 t[4];
     fetch(img, ix[0], ix[1], ix[2], rtype, t);
     store16(t, out16);
@@ -352,6 +365,7 @@ static void sample_checked(const oracle_image* img, int normalized, uint32_t add
   float w[3] = {0.0f, 0.0f, 0.0f};
   for (int d = 0; d < dims; ++d)
     oracle_axis_linear(c[d], n[d], normalized, addressing, &lo[d], &hi[d], &w[d]);
+  if (img->arrayed) lo[dims] = hi[dims] = layer;   /* one layer, weight 1 */
   double acc[4] = {0.0, 0.0, 0.0, 0.0};
   int nk = dims > 2 ? 2 : 1, nj = dims > 1 ? 2 : 1;
   for (int kk = 0; kk < nk; ++kk) {
@@ -390,7 +404,7 @@ int oracle_read_image_icoord(const oracle_image* img, int normalized, uint32_t a
       addressing == OR_ADDRESS_MIRRORED_REPEAT)
     return OR_INVALID_OPERATION;
   float c[3];
-  for (int d = 0; d < 3; ++d) c[d] = d < img->dims ? (float)icoord[d] : 0.0f;
+  for (int d = 0; d < 3; ++d) c[d] = d < img->dims + img->arrayed ? (float)icoord[d] : 0.0f;
   sample_checked(img, normalized, addressing, filter, rtype, c, out16);
   return OR_SUCCESS;
 }
@@ -426,7 +440,7 @@ typedef struct {
 
 static void grid_rows(const grid_job* g) {
   int64_t ny = g->y1 - g->y0;
-  int dims = g->img->dims;
+  int dims = g->img->dims + (g->img->arrayed ? 1 : 0);   /* + the layer coordinate */
   for (int64_t r = g->row_begin; r < g->row_end; ++r) {
     int64_t z = g->z0 + r / ny, y = g->y0 + r % ny;
     uint8_t* orow = g->out + r * g->out_w * 4 * g->out_channels;
@@ -535,7 +549,8 @@ int oracle_write_samples(oracle_image* img, int rtype, const int32_t* icoords,
   if (rtype != rtype_of(img->type)) return OR_INVALID_OPERATION;
   for (int64_t s = 0; s < n; ++s) {
     const int32_t* ic = icoords + s * cstride;
-    int64_t i = ic[0], j = img->dims > 1 ? ic[1] : 0, k = img->dims > 2 ? ic[2] : 0;
+    int nc = img->dims + (img->arrayed ? 1 : 0);  /* an array's layer is coordinate dims */
+    int64_t i = ic[0], j = nc > 1 ? ic[1] : 0, k = nc > 2 ? ic[2] : 0;
     if (i < 0 || i >= img->width || j < 0 || j >= img->height || k < 0 || k >= img->depth)
       continue;                                              /* A15: no-op */
     uint8_t texel[16];
@@ -631,12 +646,27 @@ void oracle_copy_buffer_to_image(const uint8_t* src, oracle_image* dst, size_t s
 }
 
 /* clEnqueueReadImage / clEnqueueWriteImage ([CL1.2 §5.3.3]): host row_pitch
- * 0 -> region[0]*elem_size; slice_pitch 0 -> row_pitch*region[1]. */
+ * 0 -> region[0]*elem_size; slice_pitch 0 -> row_pitch*region[1].  For a 1D
+ * image array region[1] counts layers and the host layers are slice_pitch
+ * apart (0 -> row_pitch): "slice_pitch ... the size in bytes of ... each
+ * image in a 1D or 2D image array ... calculated as row_pitch for a 1D image
+ * array" -- so there the host row stride is slice_pitch. */
+static void host_pitches(const oracle_image* img, const size_t* region, int es,
+                         size_t* row_pitch, size_t* slice_pitch) {
+  if (*row_pitch == 0) *row_pitch = region[0] * (size_t)es;
+  if (img->arrayed && img->dims == 1) {
+    if (*slice_pitch == 0) *slice_pitch = *row_pitch;
+    *row_pitch = *slice_pitch;                  /* layer y at host + y*slice_pitch */
+    *slice_pitch = *row_pitch * region[1];
+    return;
+  }
+  if (*slice_pitch == 0) *slice_pitch = *row_pitch * region[1];
+}
+
 void oracle_read_image_rect(const oracle_image* img, const size_t* origin, const size_t* region,
                             size_t row_pitch, size_t slice_pitch, uint8_t* host) {
   int es = oracle_elem_size(img->order, img->type);
-  if (row_pitch == 0) row_pitch = region[0] * (size_t)es;
-  if (slice_pitch == 0) slice_pitch = row_pitch * region[1];
+  host_pitches(img, region, es, &row_pitch, &slice_pitch);
   for (size_t z = 0; z < region[2]; ++z)
     for (size_t y = 0; y < region[1]; ++y)
       for (size_t x = 0; x < region[0]; ++x)
@@ -647,8 +677,7 @@ void oracle_read_image_rect(const oracle_image* img, const size_t* origin, const
 void oracle_write_image_rect(oracle_image* img, const size_t* origin, const size_t* region,
                              size_t row_pitch, size_t slice_pitch, const uint8_t* host) {
   int es = oracle_elem_size(img->order, img->type);
-  if (row_pitch == 0) row_pitch = region[0] * (size_t)es;
-  if (slice_pitch == 0) slice_pitch = row_pitch * region[1];
+  host_pitches(img, region, es, &row_pitch, &slice_pitch);
   for (size_t z = 0; z < region[2]; ++z)
     for (size_t y = 0; y < region[1]; ++y)
       for (size_t x = 0; x < region[0]; ++x)

@@ -79,13 +79,19 @@ extern "C" {
 #define OR_IMAGE_FORMAT_NOT_SUPPORTED (-10)
 
 /* An image as the oracle sees it: texel (i,j,k) lives at
- * data + k*slice_pitch + j*row_pitch + i*elem_size   (Fig. 6 fields). */
+ * data + k*slice_pitch + j*row_pitch + i*elem_size   (Fig. 6 fields).
+ * Image arrays ([CL1.2 §5.3.1], §8.4): `arrayed` = 1 and `dims` is the number
+ * of SAMPLED axes; the layer is the next axis -- a 1D image array of L layers
+ * is width x L (j = layer, row_pitch = bytes per layer), a 2D image array is
+ * width x height x L (k = layer, slice_pitch = bytes per layer).  A 1D image
+ * buffer is a plain dims = 1 image over the buffer's bytes. */
 typedef struct {
   uint8_t* data;
   int64_t width, height, depth;   /* unused dimensions are 1 */
   int64_t row_pitch, slice_pitch; /* bytes */
-  int32_t dims;                   /* 1, 2 or 3 */
+  int32_t dims;                   /* sampled axes: 1, 2 or 3 */
   uint32_t order, type;
+  int32_t arrayed;                /* 0, or 1 for a 1D / 2D image array */
 } oracle_image;
 
 /* bytes per element, or -1 if (order,type) is not an in-scope format */
@@ -107,8 +113,14 @@ void oracle_axis_nearest(float s, int64_t n, int normalized, uint32_t addressing
 void oracle_axis_linear(float s, int64_t n, int normalized, uint32_t addressing,
                         int64_t* i0, int64_t* i1, float* a);
 
+/* ---- image-array layer selection ([CL1.2 §8.4]) ----
+ * layer = clamp(rint(c), 0, n - 1), rint = round half to even; NaN -> 0
+ * (reading A35).  The layer coordinate is never normalized or filtered. */
+int64_t oracle_layer_index(float c, int64_t n);
+
 /* ---- the read built-ins ----
- * coord: dims floats (1D: s, 2D: s,t, 3D: s,t,r).  out: 16 bytes
+ * coord: dims (+1 for an array: the layer) floats (1D: s, 2D: s,t, 3D: s,t,r;
+ * 1D array: s,layer; 2D array: s,t,layer).  out: 16 bytes
  * (float4 / int4 / uint4).  Returns OR_SUCCESS or a Khronos error for
  * combinations the readings A5/A6/A7 reject. */
 int oracle_read_image(const oracle_image* img, int normalized, uint32_t addressing,
