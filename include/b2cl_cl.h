@@ -192,6 +192,7 @@ typedef struct _cl_image_desc {
 #define CL_DEVICE_VERSION 0x102F
 #define CL_DEVICE_PLATFORM 0x1031
 #define CL_DEVICE_IMAGE_MAX_BUFFER_SIZE 0x1040
+#define CL_DEVICE_IMAGE_MAX_ARRAY_SIZE 0x1041
 
 /* ---- context / queue ---- */
 #define CL_CONTEXT_REFERENCE_COUNT 0x1080
@@ -257,6 +258,8 @@ typedef struct _cl_image_desc {
 #define CL_MEM_MAP_COUNT 0x1104
 #define CL_MEM_REFERENCE_COUNT 0x1105
 #define CL_MEM_CONTEXT 0x1106
+#define CL_MEM_ASSOCIATED_MEMOBJECT 0x1107
+#define CL_MEM_OFFSET 0x1108
 
 #define CL_IMAGE_FORMAT 0x1110
 #define CL_IMAGE_ELEMENT_SIZE 0x1111
@@ -374,7 +377,18 @@ cl_mem CL_API_CALL clCreateBuffer(cl_context context, cl_mem_flags flags, size_t
                                   void* host_ptr, cl_int* errcode_ret);
 
 /* [CL1.2 §5.3.1]; the paper's CLImage (Fig. 6).
- * image_type: CL_MEM_OBJECT_IMAGE1D / IMAGE2D / IMAGE3D.  Formats: orders
+ * image_type: CL_MEM_OBJECT_IMAGE1D / IMAGE2D / IMAGE3D / IMAGE1D_ARRAY /
+ * IMAGE2D_ARRAY / IMAGE1D_BUFFER.  An image array of L layers is stored as a
+ * width x L (1D array) or width x height x L (2D array) image: layer l at
+ * ptr + l*row_pitch (1D array) or ptr + l*slice_pitch (2D array); pixel boxes
+ * select layers through origin/region[1] (1D array) or [2] (2D array), and
+ * reads select the layer clamp(rint(coord), 0, L-1) ([CL1.2 §8.4]).  For a 1D
+ * array image_slice_pitch is the host size of each layer (>= image_row_pitch,
+ * 0 = image_row_pitch).  IMAGE1D_BUFFER: desc->buffer is a buffer of the same
+ * context holding >= width*elem_size bytes; the image aliases its bytes
+ * tightly packed (row_pitch = width*elem_size), retains it, and takes no
+ * host_ptr, host pitches or host-pointer flags (CL_INVALID_VALUE, reading
+ * A34); width <= CL_DEVICE_IMAGE_MAX_BUFFER_SIZE = 2^31-1 texels.  Formats: orders
  * R, A, RG, RA, RGBA with every non-packed channel type; BGRA and ARGB with
  * the 8-bit types; INTENSITY and LUMINANCE with UNORM/SNORM 8/16, HALF,
  * FLOAT ([CL1.2 §5.3.1.1]).  Storage is pitched linear in HBM: texel (i,j,k)

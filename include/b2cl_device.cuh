@@ -10,7 +10,9 @@
 //
 // Argument conventions (what clSetKernelArg passes for each OpenCL argument):
 //   __global / __constant buffer (cl_mem)  -> a device pointer
-//   image1d_t / image2d_t / image3d_t      -> the image descriptor by value
+//   image1d_t / image2d_t / image3d_t /    -> the image descriptor by value
+//   image1d_array_t / image2d_array_t /
+//   image1d_buffer_t
 //                                             (the paper's CLImage, Fig. 6;
 //                                             reading A27)
 //   sampler_t (cl_sampler)                 -> 32-bit CLK_* bits below
@@ -25,12 +27,19 @@
 #pragma once
 #include <stddef.h>
 
+#include <type_traits>
+
 #include "../paper_conf_sc_kimdjjl15_b200/csrc/device/read.cuh"
 
 // ---- image and sampler types ----
 struct image1d_t { b2cl::dev::Image im; };
 struct image2d_t { b2cl::dev::Image im; };
 struct image3d_t { b2cl::dev::Image im; };
+// arrays: layers on the storage axis after the sampled ones (h of a 1D array,
+// d of a 2D array); a 1D image buffer is a 1D image over a buffer's bytes
+struct image1d_array_t { b2cl::dev::Image im; };
+struct image2d_array_t { b2cl::dev::Image im; };
+struct image1d_buffer_t { b2cl::dev::Image im; };
 typedef unsigned int sampler_t;
 
 // sampler bits (clang's CLK_* encoding)
@@ -122,16 +131,44 @@ __device__ __forceinline__ uint4 read(const dev::Image& im, sampler_t s, int rcl
   return make_uint4(r[0], r[1], r[2], r[3]);
 }
 
+// image arrays ([CL1.2 §8.4]): coordinate DIMS is the layer, selected as
+// clamp(rint(c), 0, layers - 1); arrays are never shards
+template <int DIMS>
+__device__ __forceinline__ uint4 read_array(const dev::Image& im, sampler_t s, int rclass, float c0,
+                                            float c1, float c2) {
+  using C = WithShard<Layered<Cfg<DIMS, RT, RT, RT, RT, RT, RT>>, false>;
+  ReadParams p{im, decode(s), rclass};
+  if (rclass != dev::R_F) p.smp.filt = dev::F_NEAREST;
+  const float c[3] = {c0, c1, c2};
+  uint32_t r[4];
+  read_image<C>(p, c, r, 4);
+  return make_uint4(r[0], r[1], r[2], r[3]);
+}
+
+// integer coordinates (reading A30): the coordinate is the texel index,
+// exact at any width (a 1D image buffer reaches 2^31 - 1 texels)
+template <int DIMS, bool ARR>
+__device__ __forceinline__ uint4 read_int(const dev::Image& im, sampler_t s, int rclass, int c0,
+                                          int c1, int c2) {
+  using Base = Cfg<DIMS, RT, RT, RT, RT, RT, RT>;
+  using C = std::conditional_t<ARR, WithShard<Layered<Base>, false>, WithShard<Base, true>>;
+  ReadParams p{im, decode(s), rclass};
+  const int ic[3] = {c0, c1, c2};
+  uint32_t r[4];
+  read_image_int<C>(p, ic, r);
+  return make_uint4(r[0], r[1], r[2], r[3]);
+}
+
 __device__ __forceinline__ float4 as_f4(uint4 v) {
   return make_float4(__uint_as_float(v.x), __uint_as_float(v.y), __uint_as_float(v.z),
                      __uint_as_float(v.w));
 }
+__device__ __forceinline__ uint4 as_u4(uint4 v) { return v; }
 __device__ __forceinline__ int4 as_i4(uint4 v) {
   return make_int4((int)v.x, (int)v.y, (int)v.z, (int)v.w);
 }
 
-// integer coordinates: u = (float)i (reading A30); samplerless reads use
-// NEAREST, unnormalized, CLK_ADDRESS_NONE (reading A31)
+// samplerless reads use NEAREST, unnormalized, CLK_ADDRESS_NONE (reading A31)
 constexpr sampler_t kSamplerless = CLK_NORMALIZED_COORDS_FALSE | CLK_ADDRESS_NONE | CLK_FILTER_NEAREST;
 
 template <int DIMS>
@@ -160,21 +197,19 @@ __device__ __forceinline__ void write(const dev::Image& im, int i, int j, int k,
     return CONV(b2cl::cl_builtin::read<1>(im.im, s, RC, c, 0.f, 0.f));                           \
   }                                                                                              \
   __device__ __forceinline__ RET NAME(image1d_t im, sampler_t s, int c) {                        \
-    return CONV(b2cl::cl_builtin::read<1>(im.im, s, RC, __int2float_rn(c), 0.f, 0.f));           \
+    return CONV(b2cl::cl_builtin::read_int<1, false>(im.im, s, RC, c, 0, 0));           \
   }                                                                                              \
   __device__ __forceinline__ RET NAME(image2d_t im, sampler_t s, float2 c) {                     \
     return CONV(b2cl::cl_builtin::read<2>(im.im, s, RC, c.x, c.y, 0.f));                         \
   }                                                                                              \
   __device__ __forceinline__ RET NAME(image2d_t im, sampler_t s, int2 c) {                       \
-    return CONV(b2cl::cl_builtin::read<2>(im.im, s, RC, __int2float_rn(c.x), __int2float_rn(c.y), \
-                                          0.f));                                                 \
+    return CONV(b2cl::cl_builtin::read_int<2, false>(im.im, s, RC, c.x, c.y, 0));                                                 \
   }                                                                                              \
   __device__ __forceinline__ RET NAME(image3d_t im, sampler_t s, float4 c) {                     \
     return CONV(b2cl::cl_builtin::read<3>(im.im, s, RC, c.x, c.y, c.z));                         \
   }                                                                                              \
   __device__ __forceinline__ RET NAME(image3d_t im, sampler_t s, int4 c) {                       \
-    return CONV(b2cl::cl_builtin::read<3>(im.im, s, RC, __int2float_rn(c.x), __int2float_rn(c.y), \
-                                          __int2float_rn(c.z)));                                 \
+    return CONV(b2cl::cl_builtin::read_int<3, false>(im.im, s, RC, c.x, c.y, c.z));                                 \
   }                                                                                              \
   __device__ __forceinline__ RET NAME(image2d_t im, int2 c) {                                    \
     return NAME(im, b2cl::cl_builtin::kSamplerless, c);                                          \
@@ -184,34 +219,70 @@ __device__ __forceinline__ void write(const dev::Image& im, int i, int j, int k,
   }                                                                                              \
   __device__ __forceinline__ RET NAME(image1d_t im, int c) {                                     \
     return NAME(im, b2cl::cl_builtin::kSamplerless, c);                                          \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image1d_array_t im, sampler_t s, float2 c) {               \
+    return CONV(b2cl::cl_builtin::read_array<1>(im.im, s, RC, c.x, c.y, 0.f));                   \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image1d_array_t im, sampler_t s, int2 c) {                 \
+    return CONV(b2cl::cl_builtin::read_int<1, true>(im.im, s, RC, c.x, c.y, 0));                      \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image2d_array_t im, sampler_t s, float4 c) {               \
+    return CONV(b2cl::cl_builtin::read_array<2>(im.im, s, RC, c.x, c.y, c.z));                   \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image2d_array_t im, sampler_t s, int4 c) {                 \
+    return CONV(b2cl::cl_builtin::read_int<2, true>(im.im, s, RC, c.x, c.y, c.z));      \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image1d_array_t im, int2 c) {                              \
+    return NAME(im, b2cl::cl_builtin::kSamplerless, c);                                          \
+  }                                                                                              \
+  __device__ __forceinline__ RET NAME(image2d_array_t im, int4 c) {                              \
+    return NAME(im, b2cl::cl_builtin::kSamplerless, c);                                          \
+  }                                                                                              \
+  /* image1d_buffer_t: samplerless reads only ([CL1.2 §6.12.14.2]) */                            \
+  __device__ __forceinline__ RET NAME(image1d_buffer_t im, int c) {                              \
+    return CONV(b2cl::cl_builtin::read_int<1, false>(im.im, b2cl::cl_builtin::kSamplerless, RC, c, 0, 0));                         \
   }
 
-#define B2CL_ID(v) (v)
 B2CL_READ_OVERLOADS(float4, read_imagef, b2cl::dev::R_F, b2cl::cl_builtin::as_f4)
 B2CL_READ_OVERLOADS(int4, read_imagei, b2cl::dev::R_I, b2cl::cl_builtin::as_i4)
-B2CL_READ_OVERLOADS(uint4, read_imageui, b2cl::dev::R_UI, B2CL_ID)
+B2CL_READ_OVERLOADS(uint4, read_imageui, b2cl::dev::R_UI, b2cl::cl_builtin::as_u4)
 
 // ---- write built-ins ([CL1.2 §6.12.14.4]); 3D writes as cl_khr_3d_image_writes ----
-__device__ __forceinline__ void write_imagef(image1d_t im, int c, float4 v) {
-  b2cl::cl_builtin::write<1>(im.im, c, 0, 0, make_uint4(__float_as_uint(v.x), __float_as_uint(v.y),
-                                                       __float_as_uint(v.z), __float_as_uint(v.w)));
+// Arrays write as the storage image they are (layer = the last coordinate,
+// out of range -> no-op like every other out-of-range write, reading A15).
+namespace b2cl {
+namespace cl_builtin {
+__device__ __forceinline__ uint4 bits(float4 v) {
+  return make_uint4(__float_as_uint(v.x), __float_as_uint(v.y), __float_as_uint(v.z),
+                    __float_as_uint(v.w));
 }
-__device__ __forceinline__ void write_imagef(image2d_t im, int2 c, float4 v) {
-  b2cl::cl_builtin::write<2>(im.im, c.x, c.y, 0,
-                             make_uint4(__float_as_uint(v.x), __float_as_uint(v.y),
-                                        __float_as_uint(v.z), __float_as_uint(v.w)));
-}
-__device__ __forceinline__ void write_imagef(image3d_t im, int4 c, float4 v) {
-  b2cl::cl_builtin::write<3>(im.im, c.x, c.y, c.z,
-                             make_uint4(__float_as_uint(v.x), __float_as_uint(v.y),
-                                        __float_as_uint(v.z), __float_as_uint(v.w)));
-}
-__device__ __forceinline__ void write_imagei(image2d_t im, int2 c, int4 v) {
-  b2cl::cl_builtin::write<2>(im.im, c.x, c.y, 0, make_uint4(v.x, v.y, v.z, v.w));
-}
-__device__ __forceinline__ void write_imageui(image2d_t im, int2 c, uint4 v) {
-  b2cl::cl_builtin::write<2>(im.im, c.x, c.y, 0, v);
-}
+__device__ __forceinline__ uint4 bits(int4 v) { return make_uint4(v.x, v.y, v.z, v.w); }
+__device__ __forceinline__ uint4 bits(uint4 v) { return v; }
+}  // namespace cl_builtin
+}  // namespace b2cl
+
+#define B2CL_WRITE_OVERLOADS(NAME, VT)                                                           \
+  __device__ __forceinline__ void NAME(image1d_t im, int c, VT v) {                              \
+    b2cl::cl_builtin::write<1>(im.im, c, 0, 0, b2cl::cl_builtin::bits(v));                       \
+  }                                                                                              \
+  __device__ __forceinline__ void NAME(image1d_buffer_t im, int c, VT v) {                       \
+    b2cl::cl_builtin::write<1>(im.im, c, 0, 0, b2cl::cl_builtin::bits(v));                       \
+  }                                                                                              \
+  __device__ __forceinline__ void NAME(image2d_t im, int2 c, VT v) {                             \
+    b2cl::cl_builtin::write<2>(im.im, c.x, c.y, 0, b2cl::cl_builtin::bits(v));                   \
+  }                                                                                              \
+  __device__ __forceinline__ void NAME(image1d_array_t im, int2 c, VT v) {                       \
+    b2cl::cl_builtin::write<2>(im.im, c.x, c.y, 0, b2cl::cl_builtin::bits(v));                   \
+  }                                                                                              \
+  __device__ __forceinline__ void NAME(image3d_t im, int4 c, VT v) {                             \
+    b2cl::cl_builtin::write<3>(im.im, c.x, c.y, c.z, b2cl::cl_builtin::bits(v));                 \
+  }                                                                                              \
+  __device__ __forceinline__ void NAME(image2d_array_t im, int4 c, VT v) {                       \
+    b2cl::cl_builtin::write<3>(im.im, c.x, c.y, c.z, b2cl::cl_builtin::bits(v));                 \
+  }
+B2CL_WRITE_OVERLOADS(write_imagef, float4)
+B2CL_WRITE_OVERLOADS(write_imagei, int4)
+B2CL_WRITE_OVERLOADS(write_imageui, uint4)
 
 // ---- image queries ([CL1.2 §6.12.14.5]) ----
 __device__ __forceinline__ int get_image_width(image1d_t im) { return im.im.w; }
@@ -220,3 +291,9 @@ __device__ __forceinline__ int get_image_width(image3d_t im) { return im.im.w; }
 __device__ __forceinline__ int get_image_height(image2d_t im) { return im.im.h; }
 __device__ __forceinline__ int get_image_height(image3d_t im) { return im.im.h; }
 __device__ __forceinline__ int get_image_depth(image3d_t im) { return im.im.d; }
+__device__ __forceinline__ int get_image_width(image1d_buffer_t im) { return im.im.w; }
+__device__ __forceinline__ int get_image_width(image1d_array_t im) { return im.im.w; }
+__device__ __forceinline__ int get_image_width(image2d_array_t im) { return im.im.w; }
+__device__ __forceinline__ int get_image_height(image2d_array_t im) { return im.im.h; }
+__device__ __forceinline__ size_t get_image_array_size(image1d_array_t im) { return im.im.h; }
+__device__ __forceinline__ size_t get_image_array_size(image2d_array_t im) { return im.im.d; }

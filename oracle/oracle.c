@@ -395,7 +395,11 @@ int oracle_read_image(const oracle_image* img, int normalized, uint32_t addressi
 }
 
 /* Integer coordinates (reading A30): legal only with unnormalized coordinates,
- * NEAREST and a non-wrapping mode; then u = (float)i. */
+ * NEAREST and a non-wrapping mode.  The coordinate is the texel index itself,
+ * i = address_mode(coord) ([CL1.2 §8.2] with floor(u) = coord exactly), and an
+ * array's layer is clamp(coord, 0, n - 1) ([CL1.2 §8.4]: rint of an integer
+ * is itself).  For |coord| <= 2^24 this is the float path at u = (float)coord;
+ * beyond, it stays exact (1D image buffers reach 2^31 - 1 texels). */
 int oracle_read_image_icoord(const oracle_image* img, int normalized, uint32_t addressing,
                              uint32_t filter, int rtype, const int32_t* icoord, void* out16) {
   int st = check_read(img, normalized, addressing, filter, rtype);
@@ -403,9 +407,13 @@ int oracle_read_image_icoord(const oracle_image* img, int normalized, uint32_t a
   if (normalized || filter != OR_FILTER_NEAREST || addressing == OR_ADDRESS_REPEAT ||
       addressing == OR_ADDRESS_MIRRORED_REPEAT)
     return OR_INVALID_OPERATION;
-  float c[3];
-  for (int d = 0; d < 3; ++d) c[d] = d < img->dims + img->arrayed ? (float)icoord[d] : 0.0f;
-  sample_checked(img, normalized, addressing, filter, rtype, c, out16);
+  int64_t n[3] = {img->width, img->height, img->depth};
+  int64_t ix[3] = {0, 0, 0};
+  for (int d = 0; d < img->dims; ++d) ix[d] = am(addressing, icoord[d], n[d]);
+  if (img->arrayed) ix[img->dims] = clamp64(icoord[img->dims], 0, n[img->dims] - 1);
+  val32 t[4];
+  fetch(img, ix[0], ix[1], ix[2], rtype, t);
+  store16(t, out16);
   return OR_SUCCESS;
 }
 

@@ -27,7 +27,8 @@ CL_MEM_READ_WRITE, CL_MEM_WRITE_ONLY, CL_MEM_READ_ONLY = 1, 2, 4
 CL_MEM_USE_HOST_PTR, CL_MEM_ALLOC_HOST_PTR, CL_MEM_COPY_HOST_PTR = 8, 16, 32
 B2CL_MEM_IPC_EXPORTABLE = 1 << 40
 CL_MEM_OBJECT_BUFFER, CL_MEM_OBJECT_IMAGE2D, CL_MEM_OBJECT_IMAGE3D = 0x10F0, 0x10F1, 0x10F2
-CL_MEM_OBJECT_IMAGE1D = 0x10F4
+CL_MEM_OBJECT_IMAGE2D_ARRAY, CL_MEM_OBJECT_IMAGE1D = 0x10F3, 0x10F4
+CL_MEM_OBJECT_IMAGE1D_ARRAY, CL_MEM_OBJECT_IMAGE1D_BUFFER = 0x10F5, 0x10F6
 CL_R, CL_A, CL_RG, CL_RA, CL_RGB, CL_RGBA, CL_BGRA, CL_ARGB, CL_INTENSITY, CL_LUMINANCE = range(0x10B0, 0x10BA)
 CL_SNORM_INT8, CL_SNORM_INT16, CL_UNORM_INT8, CL_UNORM_INT16 = 0x10D0, 0x10D1, 0x10D2, 0x10D3
 CL_SIGNED_INT8, CL_SIGNED_INT16, CL_SIGNED_INT32 = 0x10D7, 0x10D8, 0x10D9
@@ -39,6 +40,7 @@ CL_FILTER_NEAREST, CL_FILTER_LINEAR = 0x1140, 0x1141
 CL_MIGRATE_MEM_OBJECT_HOST, CL_MIGRATE_MEM_OBJECT_CONTENT_UNDEFINED = 1, 2
 CL_IMAGE_FORMAT, CL_IMAGE_ELEMENT_SIZE, CL_IMAGE_ROW_PITCH, CL_IMAGE_SLICE_PITCH = 0x1110, 0x1111, 0x1112, 0x1113
 CL_IMAGE_WIDTH, CL_IMAGE_HEIGHT, CL_IMAGE_DEPTH = 0x1114, 0x1115, 0x1116
+CL_IMAGE_ARRAY_SIZE, CL_IMAGE_BUFFER = 0x1117, 0x1118
 CL_PROFILING_COMMAND_START, CL_PROFILING_COMMAND_END = 0x1282, 0x1283
 B2CL_RTYPE_FLOAT, B2CL_RTYPE_INT, B2CL_RTYPE_UINT = 0, 1, 2
 B2CL_COORD_FLOAT, B2CL_COORD_INT = 0, 1
@@ -307,6 +309,32 @@ class Session:
         else:
             m = lib().clCreateImage(self.ctx, flags, byref(fmt), byref(desc), None, byref(err))
         check(err.value, "clCreateImage")
+        return m
+
+    def image_array(self, order: int, type_: int, width: int, layers: int, height: int = 0,
+                    host: np.ndarray | None = None, host_row_pitch: int = 0,
+                    host_slice_pitch: int = 0, flags: int = CL_MEM_READ_WRITE):
+        """A 1D image array (height 0) or 2D image array of `layers` layers."""
+        fmt = ImageFormat(order, type_)
+        desc = ImageDesc(CL_MEM_OBJECT_IMAGE2D_ARRAY if height else CL_MEM_OBJECT_IMAGE1D_ARRAY,
+                         width, height, 0, layers, host_row_pitch, host_slice_pitch, 0, 0, None)
+        err = c_int32()
+        if host is not None:
+            host = np.ascontiguousarray(host)
+            m = lib().clCreateImage(self.ctx, flags | CL_MEM_COPY_HOST_PTR, byref(fmt), byref(desc),
+                                    _ptr(host), byref(err))
+        else:
+            m = lib().clCreateImage(self.ctx, flags, byref(fmt), byref(desc), None, byref(err))
+        check(err.value, "clCreateImage (array)")
+        return m
+
+    def image_buffer(self, order: int, type_: int, width: int, buffer, flags: int = 0):
+        """A 1D image buffer over `buffer`'s bytes (CL_MEM_OBJECT_IMAGE1D_BUFFER)."""
+        fmt = ImageFormat(order, type_)
+        desc = ImageDesc(CL_MEM_OBJECT_IMAGE1D_BUFFER, width, 0, 0, 0, 0, 0, 0, 0, buffer)
+        err = c_int32()
+        m = lib().clCreateImage(self.ctx, flags, byref(fmt), byref(desc), None, byref(err))
+        check(err.value, "clCreateImage (1D buffer)")
         return m
 
     def image_shard(self, order: int, type_: int, width: int, height: int, depth: int,

@@ -17,6 +17,8 @@ struct Cfg {
   static constexpr int dims = DIMS, type = TYPE, order = ORDER, norm = NORM, addr = ADDR,
                        filt = FILT, rc = RC;
   static constexpr int nch = ORDER == RT ? RT : order_channels(ORDER);
+  static constexpr bool arr = false;   // image array (see Layered)
+  static constexpr int cdims = DIMS;   // coordinates per sample
 };
 
 // C with the image-shard row mapping compiled in (SH) or out (plain images)
@@ -24,6 +26,20 @@ template <class C, bool SH>
 struct WithShard : C {
   static constexpr bool shard = SH;
 };
+
+// C read from an image array: coordinate dims selects the layer, stored on
+// the axis after the sampled ones (rows of a 1D array, slices of a 2D array)
+template <class C>
+struct Layered : C {
+  static constexpr bool arr = true;
+  static constexpr int cdims = C::dims + 1;
+};
+
+// [CL1.2 §8.4]: layer = clamp(rint(c), 0, n - 1).  cvt.rni rounds half to
+// even, saturates, and gives 0 for NaN (reading A35).
+__device__ __forceinline__ int layer_of(float c, int n) {
+  return min(max(__float2int_rn(c), 0), n - 1);
+}
 
 struct AxN {  // NEAREST, one axis
   int i;
@@ -183,22 +199,47 @@ template <class C, class P>
 __device__ __forceinline__ void read_image(const P& p, const float c[3],
                                            uint32_t res[4], int outc = 4) {
   const Image& im = p.im;
+  // an array's layer: the row (1D array) or slice (2D array) index, always
+  // in range, weight 1 -- the sampler never touches it
+  int layer = 0;
+  if constexpr (C::arr) layer = layer_of(c[C::dims], C::dims == 1 ? im.h : im.d);
   if (filt_of<C>(p) == F_NEAREST) {
     const AxN x = axis_n<C>(p.smp, c[0], im.w);
     AxN y{0, true}, z{0, true};
     if (C::dims > 1) y = axis_n<C>(p.smp, c[1], im.h);
     if (C::dims > 2) z = axis_n<C>(p.smp, c[2], im.d);
+    if constexpr (C::arr) (C::dims == 1 ? y : z) = AxN{layer, true};
     nearest_at<C>(p, row_ptr<C>(im, y.i, z.i), x, y.ok && z.ok, res);
   } else {
     const AxL x = axis_l<C>(p.smp, c[0], im.w);
     AxL y{0, 0, 0.f, 1.f, true, true}, z{0, 0, 0.f, 1.f, true, true};
     if (C::dims > 1) y = axis_l<C>(p.smp, c[1], im.h);
     if (C::dims > 2) z = axis_l<C>(p.smp, c[2], im.d);
+    if constexpr (C::arr) (C::dims == 1 ? y : z) = AxL{layer, layer, 0.f, 1.f, true, true};
     const char* rows[4] = {row_ptr<C>(im, y.i0, z.i0), row_ptr<C>(im, y.i1, z.i0),
                            row_ptr<C>(im, y.i0, z.i1), row_ptr<C>(im, y.i1, z.i1)};
     const bool rok[4] = {y.ok0 && z.ok0, y.ok1 && z.ok0, y.ok0 && z.ok1, y.ok1 && z.ok1};
     linear_at<C>(p, rows, rok, x, y.a, y.oma, z.a, z.oma, res, outc);
   }
+}
+
+// The built-in on integer coordinates (reading A30): NEAREST, unnormalized,
+// non-wrapping; the coordinate IS the texel index, i = address_mode(coord)
+// (CLAMP_TO_EDGE clamps into [0, n-1]; NONE and CLAMP give the border out of
+// range), exact at any width.  An array's layer is clamp(coord, 0, n-1).
+template <class C, class P>
+__device__ __forceinline__ void read_image_int(const P& p, const int ic[3], uint32_t res[4]) {
+  const Image& im = p.im;
+  const int addr = C::addr == RT ? p.smp.addr : C::addr;
+  const int n[3] = {im.w, im.h, im.d};
+  AxN a[3] = {{0, true}, {0, true}, {0, true}};
+#pragma unroll
+  for (int d = 0; d < C::dims; ++d) {
+    a[d].i = addr == A_CTE ? min(max(ic[d], 0), n[d] - 1) : ic[d];
+    a[d].ok = in_range(a[d].i, n[d]);
+  }
+  if constexpr (C::arr) a[C::dims] = AxN{min(max(ic[C::dims], 0), n[C::dims] - 1), true};
+  nearest_at<C>(p, row_ptr<C>(im, a[1].i, a[2].i), a[0], a[1].ok && a[2].ok, res);
 }
 
 }  // namespace b2cl

@@ -13,7 +13,8 @@ struct SampleParams {
   dev::Image im;
   dev::Sampler smp;
   int rclass;       // dev::RetCode
-  int dims;         // 1..3
+  int dims;         // sampled axes 1..3
+  int arr;          // 1: image array; coordinate `dims` selects the layer ([CL1.2 §8.4])
   float A[12];      // grid: affine coordinate map
   int ow, oh, od;   // grid: output region dims
   int ox, oy, oz;   // grid: output region origin (coordinates use origin + index)

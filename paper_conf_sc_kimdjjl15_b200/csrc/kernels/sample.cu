@@ -61,8 +61,8 @@ __global__ void __launch_bounds__(256) k_sample_grid(const SampleParams p) {
               zf = __int2float_rn(p.oz + z);
   float c[3];
   c[0] = affine_coord(p.A, xf, yf, zf);
-  c[1] = C::dims > 1 ? affine_coord(p.A + 4, xf, yf, zf) : 0.f;
-  c[2] = C::dims > 2 ? affine_coord(p.A + 8, xf, yf, zf) : 0.f;
+  c[1] = C::cdims > 1 ? affine_coord(p.A + 4, xf, yf, zf) : 0.f;
+  c[2] = C::cdims > 2 ? affine_coord(p.A + 8, xf, yf, zf) : 0.f;
   uint32_t r[4];
   read_image<C>(p, c, r, OUTC == RT ? p.outc : OUTC);
   store_out<OUTC>(p, ((uint64_t)z * p.oh + y) * p.ow + x, r);
@@ -290,13 +290,16 @@ template <class C, bool INT_COORD>
 __global__ void __launch_bounds__(256) k_sample_list(const SampleParams p) {
   const uint64_t s = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (s >= p.n) return;
-  float c[3] = {0.f, 0.f, 0.f};
-  constexpr int stride = C::dims == 1 ? 1 : (C::dims == 2 ? 2 : 4);
+  constexpr int stride = C::cdims == 1 ? 1 : (C::cdims == 2 ? 2 : 4);
+  uint32_t r[4];
   if (INT_COORD) {
     const int32_t* q = reinterpret_cast<const int32_t*>(p.coords) + s * stride;
+    int ic[3] = {0, 0, 0};
 #pragma unroll
-    for (int d = 0; d < C::dims; ++d) c[d] = __int2float_rn(q[d]);  // u = (float)i (A30)
+    for (int d = 0; d < C::cdims; ++d) ic[d] = q[d];
+    read_image_int<C>(p, ic, r);  // the coordinate is the texel index (A30)
   } else {
+    float c[3] = {0.f, 0.f, 0.f};
     const float* q = reinterpret_cast<const float*>(p.coords) + s * stride;
     if (stride == 4) {
       float4 v = *reinterpret_cast<const float4*>(q);
@@ -307,16 +310,15 @@ __global__ void __launch_bounds__(256) k_sample_list(const SampleParams p) {
     } else {
       c[0] = q[0];
     }
+    read_image<C>(p, c, r);
   }
-  uint32_t r[4];
-  read_image<C>(p, c, r);
   __stcs(reinterpret_cast<uint4*>(p.out) + s, make_uint4(r[0], r[1], r[2], r[3]));
 }
 
 // ---------------------------------------------------------------- dispatch
 // a shard stores a window of the outer axis (b2clCreateImageShard)
 static bool is_shard(const SampleParams& p) {
-  if (p.dims < 2) return false;
+  if (p.dims < 2 || p.arr) return false;
   return p.im.ob != 0 || p.im.os != (p.dims == 3 ? p.im.d : p.im.h);
 }
 
@@ -402,6 +404,8 @@ cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st
     // the default picks the variant measured fastest on B200 for each hot config
     static const char* force = getenv("B2CL_GRID_KERNEL");
     const int fk = !force ? 0 : (force[0] == 'g' ? 1 : (force[0] == 's' ? 2 : (force[0] == 'w' ? 3 : 0)));
+    if (p.arr)  // image arrays: the general kernel, fully run-time format and sampler
+      return p.dims == 1 ? go_grid<Layered<Generic<1>>, RT>(p, st) : go_grid<Layered<Generic<2>>, RT>(p, st);
     if (separable(p) && fk != 1) {
       if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_REPEAT, F_LINEAR))
         return fk == 3 ? go_walk<C2Repeat, 4, 2, 8>(p, st) : go_sep<C2Repeat, 4, 2, 4>(p, st);
@@ -427,6 +431,8 @@ cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st
   }
   if (p.n == 0) return cudaSuccess;
   const bool ic = coord_mode == COORD_LIST_I;
+  if (p.arr)
+    return p.dims == 1 ? go_list<Layered<Generic<1>>>(p, ic, st) : go_list<Layered<Generic<2>>>(p, ic, st);
   if (!ic && matches<2>(p, T_FLOAT, O_RGBA, 1, A_REPEAT, F_LINEAR)) return go_list<C2Repeat>(p, false, st);
   if (!ic && matches<2>(p, T_FLOAT, O_RGBA, 1, A_MIRROR, F_LINEAR)) return go_list<C2Mirror>(p, false, st);
   if (!ic && matches<2>(p, T_UNORM8, O_RGBA, 0, A_CLAMP, F_NEAREST)) return go_list<C1Clamp>(p, false, st);

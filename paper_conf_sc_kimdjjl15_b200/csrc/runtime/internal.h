@@ -11,15 +11,26 @@ namespace b2cl {
 
 constexpr size_t kMax2D = 65536;  // CL_DEVICE_IMAGE2D_MAX_WIDTH/HEIGHT (and 1D width)
 constexpr size_t kMax3D = 16384;  // CL_DEVICE_IMAGE3D_MAX_*
+constexpr size_t kMaxArray = 65536;            // CL_DEVICE_IMAGE_MAX_ARRAY_SIZE
+constexpr size_t kMaxBuffer = (1ull << 31) - 1;  // CL_DEVICE_IMAGE_MAX_BUFFER_SIZE (texels):
+                                                 // the int coordinate's range, not a texture limit
 
 struct FormatInfo {
   int type, order, nch, rclass;  // dev::TypeCode, dev::OrderCode, channels, dev::RetCode
   size_t es;                     // elem_size
 };
 
+// Storage view of every image type.  `dims` counts STORAGE axes: an image
+// array keeps its layers on the axis after the sampled ones -- a 1D image
+// array is stored as a w x layers 2D image (dims 2, arrayed), a 2D image
+// array as a w x h x layers 3D image (dims 3, arrayed) -- so every pixel-box
+// operation (copies, fills, host transfers) addresses it as that image, with
+// origin/region[1] (1D array) or [2] (2D array) selecting layers as
+// [CL1.2 §5.3.3] specifies.  Sampling uses dims - arrayed axes plus the layer.
 struct ImageLayout {
   FormatInfo fmt;
   int dims;
+  int arrayed;  // 1 for CL_MEM_OBJECT_IMAGE1D_ARRAY / IMAGE2D_ARRAY
   size_t w, h, d;
   size_t row_pitch, slice_pitch, bytes;
 };

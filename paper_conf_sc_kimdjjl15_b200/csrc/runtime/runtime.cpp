@@ -72,6 +72,9 @@ struct _cl_mem {
   long long shard_ob = 0;
   cl_image_format fmt{};
   cl_image_desc desc{};
+  // a 1D image buffer (CL_MEM_OBJECT_IMAGE1D_BUFFER) owns no storage: its
+  // texels are the bytes of this buffer, which it retains
+  cl_mem parent = nullptr;
   std::mutex mu;
   std::vector<Store> stores;
   uint64_t valid = 0;                   // bit per ordinal holding valid content
@@ -244,7 +247,8 @@ extern "C" cl_int clGetDeviceInfo(cl_device_id d, cl_device_info name, size_t si
     case CL_DEVICE_IMAGE3D_MAX_WIDTH:
     case CL_DEVICE_IMAGE3D_MAX_HEIGHT:
     case CL_DEVICE_IMAGE3D_MAX_DEPTH: return get_info<size_t>(kMax3D, size, value, size_ret);
-    case CL_DEVICE_IMAGE_MAX_BUFFER_SIZE: return get_info<size_t>(0, size, value, size_ret);
+    case CL_DEVICE_IMAGE_MAX_BUFFER_SIZE: return get_info<size_t>(kMaxBuffer, size, value, size_ret);
+    case CL_DEVICE_IMAGE_MAX_ARRAY_SIZE: return get_info<size_t>(kMaxArray, size, value, size_ret);
     case CL_DEVICE_AVAILABLE: return get_info<cl_bool>(CL_TRUE, size, value, size_ret);
     case CL_DEVICE_QUEUE_PROPERTIES:
       return get_info<cl_command_queue_properties>(
@@ -596,23 +600,58 @@ extern "C" cl_mem b2clCreateBufferFromDevicePointer(cl_context c, cl_device_id d
   return m;
 }
 
+// A 1D image buffer ([CL1.2 §5.3.1]): an image view of a buffer's bytes.
+static cl_mem image_from_buffer(cl_context c, cl_mem_flags flags, const cl_image_format* fmt,
+                                const cl_image_desc* desc, const ImageLayout& L, void* host_ptr,
+                                cl_int* errcode_ret) {
+  cl_mem b = desc->buffer;
+  if (!live(g_mems, b) || b->type != CL_MEM_OBJECT_BUFFER || b->ctx != c) {
+    SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR);
+    return nullptr;
+  }
+  // the pixels are the buffer's (no host pointer, no host pitches: reading A34)
+  if (host_ptr || (flags & (CL_MEM_COPY_HOST_PTR | CL_MEM_USE_HOST_PTR | CL_MEM_ALLOC_HOST_PTR)) ||
+      desc->image_row_pitch || desc->image_slice_pitch) {
+    SET_ERR(CL_INVALID_VALUE);
+    return nullptr;
+  }
+  if (L.bytes > b->size) { SET_ERR(CL_INVALID_IMAGE_SIZE); return nullptr; }
+  cl_mem m = new_mem(c, CL_MEM_OBJECT_IMAGE1D_BUFFER, flags ? flags : b->flags, L.bytes);
+  if (!m) { SET_ERR(CL_OUT_OF_HOST_MEMORY); return nullptr; }
+  m->img = L;
+  m->fmt = *fmt;
+  m->desc = *desc;
+  b->ref++;
+  m->parent = b;
+  register_mem(m);
+  SET_ERR(CL_SUCCESS);
+  return m;
+}
+
 extern "C" cl_mem clCreateImage(cl_context c, cl_mem_flags flags, const cl_image_format* fmt,
                                 const cl_image_desc* desc, void* host_ptr, cl_int* errcode_ret) {
   if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
-  cl_int st = check_mem_flags(flags & ~B2CL_MEM_IPC_EXPORTABLE, host_ptr);
-  if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
   ImageLayout L;
-  st = image_layout(fmt, desc, &L);
+  cl_int st = image_layout(fmt, desc, &L);
+  if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
+  if (desc->image_type == CL_MEM_OBJECT_IMAGE1D_BUFFER)
+    return image_from_buffer(c, flags, fmt, desc, L, host_ptr, errcode_ret);
+  st = check_mem_flags(flags & ~B2CL_MEM_IPC_EXPORTABLE, host_ptr);
   if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
   // host pitches ([CL1.2 §5.3.1]): nonzero only with a host pointer, >= tight,
-  // multiple of the element size; slice pitch only for 3D
+  // multiple of the element size.  Slice pitch: 3D images and 2D arrays
+  // (>= row_pitch * height), 1D arrays (the size of each layer, >= row_pitch),
+  // in both cases a multiple of row_pitch; 0 for 1D and 2D images.
   size_t hrp = desc->image_row_pitch, hsp = desc->image_slice_pitch;
   if ((hrp || hsp) && !host_ptr) { SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR); return nullptr; }
   if (hrp == 0) hrp = L.w * L.fmt.es;
   else if (hrp < L.w * L.fmt.es || hrp % L.fmt.es) { SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR); return nullptr; }
-  if (L.dims == 3) {
-    if (hsp == 0) hsp = hrp * L.h;
-    else if (hsp < hrp * L.h || hsp % hrp) { SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR); return nullptr; }
+  const bool arr1 = L.arrayed && L.dims == 2;
+  if (L.dims == 3 || arr1) {
+    const size_t min_sp = arr1 ? hrp : hrp * L.h;
+    if (hsp == 0) hsp = min_sp;
+    else if (hsp < min_sp || hsp % hrp) { SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR); return nullptr; }
+    if (arr1) hrp = hsp;  // layer l of a 1D array is host row l, hsp apart
   } else if (hsp != 0) {
     SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR);
     return nullptr;
@@ -650,7 +689,7 @@ extern "C" cl_mem b2clCreateImageShard(cl_context c, cl_mem_flags flags, const c
   ImageLayout G;
   cl_int st = image_layout(fmt, global_desc, &G);
   if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
-  if (G.dims < 2) { SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR); return nullptr; }
+  if (G.dims < 2 || G.arrayed) { SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR); return nullptr; }
   const size_t extent = G.dims == 3 ? G.d : G.h;
   // the band may wrap around the global extent (begin + count > extent)
   if (count == 0 || begin >= extent || count + 2 * halo > extent ||
@@ -675,9 +714,7 @@ extern "C" cl_int clGetSupportedImageFormats(cl_context c, cl_mem_flags flags,
                                              cl_image_format* formats, cl_uint* num_formats) {
   (void)flags;
   if (!live(g_contexts, c)) return CL_INVALID_CONTEXT;
-  if (type != CL_MEM_OBJECT_IMAGE1D && type != CL_MEM_OBJECT_IMAGE2D &&
-      type != CL_MEM_OBJECT_IMAGE3D)
-    return CL_INVALID_VALUE;
+  if (type < CL_MEM_OBJECT_IMAGE2D || type > CL_MEM_OBJECT_IMAGE1D_BUFFER) return CL_INVALID_VALUE;
   if (num_entries == 0 && formats) return CL_INVALID_VALUE;
   std::vector<cl_image_format> all;
   for (cl_channel_order o = CL_R; o <= CL_LUMINANCE; ++o)
@@ -693,8 +730,7 @@ extern "C" cl_int clGetSupportedImageFormats(cl_context c, cl_mem_flags flags,
 }
 
 static bool is_image(cl_mem m) {
-  return m->type == CL_MEM_OBJECT_IMAGE1D || m->type == CL_MEM_OBJECT_IMAGE2D ||
-         m->type == CL_MEM_OBJECT_IMAGE3D;
+  return m->type >= CL_MEM_OBJECT_IMAGE2D && m->type <= CL_MEM_OBJECT_IMAGE1D_BUFFER;
 }
 
 extern "C" cl_int clRetainMemObject(cl_mem m) {
@@ -720,7 +756,9 @@ extern "C" cl_int clReleaseMemObject(cl_mem m) {
     }
     for (auto& s : m->stores) raw_free(s);
     cl_context c = m->ctx;
+    cl_mem parent = m->parent;
     delete m;
+    if (parent) clReleaseMemObject(parent);
     clReleaseContext(c);
   }
   return CL_SUCCESS;
@@ -737,6 +775,8 @@ extern "C" cl_int clGetMemObjectInfo(cl_mem m, cl_mem_info name, size_t size, vo
     case CL_MEM_MAP_COUNT: return get_info<cl_uint>(0, size, value, size_ret);
     case CL_MEM_REFERENCE_COUNT: return get_info<cl_uint>(m->ref.load(), size, value, size_ret);
     case CL_MEM_CONTEXT: return get_info<cl_context>(m->ctx, size, value, size_ret);
+    case CL_MEM_ASSOCIATED_MEMOBJECT: return get_info<cl_mem>(m->parent, size, value, size_ret);
+    case CL_MEM_OFFSET: return get_info<size_t>(0, size, value, size_ret);
     default: return CL_INVALID_VALUE;
   }
 }
@@ -749,13 +789,19 @@ extern "C" cl_int clGetImageInfo(cl_mem m, cl_image_info name, size_t size, void
     case CL_IMAGE_FORMAT: return get_info<cl_image_format>(m->fmt, size, value, size_ret);
     case CL_IMAGE_ELEMENT_SIZE: return get_info<size_t>(L.fmt.es, size, value, size_ret);
     case CL_IMAGE_ROW_PITCH: return get_info<size_t>(L.row_pitch, size, value, size_ret);
-    case CL_IMAGE_SLICE_PITCH:
-      return get_info<size_t>(L.dims == 3 ? L.slice_pitch : 0, size, value, size_ret);
+    case CL_IMAGE_SLICE_PITCH: {
+      // 3D: bytes per slice; arrays: bytes per layer; 1D, 1D buffer and 2D: 0
+      const size_t sp = (L.dims == 3) ? L.slice_pitch : (L.arrayed ? L.row_pitch : 0);
+      return get_info<size_t>(sp, size, value, size_ret);
+    }
     case CL_IMAGE_WIDTH: return get_info<size_t>(L.w, size, value, size_ret);
-    case CL_IMAGE_HEIGHT: return get_info<size_t>(L.dims > 1 ? L.h : 0, size, value, size_ret);
-    case CL_IMAGE_DEPTH: return get_info<size_t>(L.dims > 2 ? L.d : 0, size, value, size_ret);
-    case CL_IMAGE_ARRAY_SIZE: return get_info<size_t>(0, size, value, size_ret);
-    case CL_IMAGE_BUFFER: return get_info<cl_mem>(nullptr, size, value, size_ret);
+    case CL_IMAGE_HEIGHT:
+      return get_info<size_t>(L.dims - L.arrayed > 1 ? L.h : 0, size, value, size_ret);
+    case CL_IMAGE_DEPTH:
+      return get_info<size_t>(L.dims == 3 && !L.arrayed ? L.d : 0, size, value, size_ret);
+    case CL_IMAGE_ARRAY_SIZE:
+      return get_info<size_t>(!L.arrayed ? 0 : (L.dims == 2 ? L.h : L.d), size, value, size_ret);
+    case CL_IMAGE_BUFFER: return get_info<cl_mem>(m->parent, size, value, size_ret);
     case CL_IMAGE_NUM_MIP_LEVELS:
     case CL_IMAGE_NUM_SAMPLES: return get_info<cl_uint>(0, size, value, size_ret);
     default: return CL_INVALID_VALUE;
@@ -955,6 +1001,7 @@ static cl_int enq_end(Enq& E, cudaError_t err) {
 // NVLink (SM copy kernel on the peer pointer) on the queue's stream; the
 // caller's wait list orders it after the producer (OpenCL cross-queue rule).
 static cl_int resident(cl_mem m, cl_command_queue q, bool need_content, char** out) {
+  if (m->parent) m = m->parent;  // a 1D image buffer lives in its buffer
   std::lock_guard<std::mutex> g(m->mu);
   const int ord = q->dev->ordinal;
   Store* s = nullptr;
@@ -988,6 +1035,7 @@ static cl_int resident(cl_mem m, cl_command_queue q, bool need_content, char** o
 }
 
 static void written(cl_mem m, cl_command_queue q) {
+  if (m->parent) m = m->parent;
   std::lock_guard<std::mutex> g(m->mu);
   m->valid = 1ull << q->dev->ordinal;
 }
@@ -1126,9 +1174,18 @@ static cl_int image_host(cl_command_queue q, cl_mem img, cl_bool blocking, const
   const size_t es = L.fmt.es;
   if (rp == 0) rp = region[0] * es;
   else if (rp < region[0] * es) return CL_INVALID_VALUE;
-  if (L.dims < 3 && sp != 0) return CL_INVALID_VALUE;
-  if (sp == 0) sp = rp * region[1];
-  else if (sp < rp * region[1]) return CL_INVALID_VALUE;
+  if (L.arrayed && L.dims == 2) {
+    // 1D image array: region[1] counts layers, host layers are slice_pitch
+    // apart (0 -> row_pitch) ([CL1.2 §5.3.3]); they are the host's "rows"
+    if (sp == 0) sp = rp;
+    else if (sp < rp) return CL_INVALID_VALUE;
+    rp = sp;
+    sp = rp * region[1];
+  } else {
+    if (L.dims < 3 && sp != 0) return CL_INVALID_VALUE;
+    if (sp == 0) sp = rp * region[1];
+    else if (sp < rp * region[1]) return CL_INVALID_VALUE;
+  }
   CHECK(check_wait_list(q, nw, wl));
   Enq E;
   E.q = q;
@@ -1458,7 +1515,8 @@ extern "C" cl_int b2clEnqueueReadImageSamples(cl_command_queue q, cl_mem img, cl
   p.im = dev_image(img, pi, true);
   fill_sampler(p, smp);
   p.rclass = (int)rtype;
-  p.dims = dims;
+  p.dims = dims - img->img.arrayed;  // sampled axes; an array's layer is coordinate p.dims
+  p.arr = img->img.arrayed;
   p.coords = pc + coffset;
   p.n = n;
   p.out = po + ooffset;
@@ -1503,7 +1561,8 @@ extern "C" cl_int b2clEnqueueReadImageGridRegion(cl_command_queue q, cl_mem img,
   p.im = dev_image(img, pi, true);
   fill_sampler(p, smp);
   p.rclass = (int)rtype;
-  p.dims = img->img.dims;
+  p.dims = img->img.dims - img->img.arrayed;
+  p.arr = img->img.arrayed;
   memcpy(p.A, affine, sizeof(p.A));
   p.ow = (int)out_region[0];
   p.oh = (int)out_region[1];
@@ -1574,6 +1633,7 @@ extern "C" cl_int b2clGetMemDevicePointer(cl_mem m, cl_device_id d, void** ptr) 
   if (!live(g_mems, m)) return CL_INVALID_MEM_OBJECT;
   if (!valid_device(d) || !ctx_has_device(m->ctx, d)) return CL_INVALID_DEVICE;
   if (!ptr) return CL_INVALID_VALUE;
+  if (m->parent) m = m->parent;  // a 1D image buffer's texels are its buffer's
   std::lock_guard<std::mutex> g(m->mu);
   Store* s = nullptr;
   CHECK(ensure_store(m, d->ordinal, nullptr, &s));

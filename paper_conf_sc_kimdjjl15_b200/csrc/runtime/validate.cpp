@@ -75,9 +75,12 @@ cl_int format_info(const cl_image_format* f, FormatInfo* out) {
 
 static int image_dims(cl_mem_object_type t) {
   switch (t) {
-    case CL_MEM_OBJECT_IMAGE1D: return 1;
-    case CL_MEM_OBJECT_IMAGE2D: return 2;
-    case CL_MEM_OBJECT_IMAGE3D: return 3;
+    case CL_MEM_OBJECT_IMAGE1D:
+    case CL_MEM_OBJECT_IMAGE1D_BUFFER: return 1;
+    case CL_MEM_OBJECT_IMAGE2D:
+    case CL_MEM_OBJECT_IMAGE1D_ARRAY: return 2;
+    case CL_MEM_OBJECT_IMAGE3D:
+    case CL_MEM_OBJECT_IMAGE2D_ARRAY: return 3;
     default: return 0;
   }
 }
@@ -87,21 +90,37 @@ cl_int image_layout(const cl_image_format* fmt, const cl_image_desc* desc, Image
   cl_int st = format_info(fmt, &fi);
   if (st != CL_SUCCESS) return st;
   if (!desc) return CL_INVALID_IMAGE_DESCRIPTOR;
-  const int dims = image_dims(desc->image_type);
-  if (dims == 0) return CL_INVALID_IMAGE_DESCRIPTOR;  // arrays / 1D buffers: NEXT(2)
-  if (desc->num_mip_levels != 0 || desc->num_samples != 0 || desc->buffer != nullptr)
+  const cl_mem_object_type t = desc->image_type;
+  const int dims = image_dims(t);
+  if (dims == 0) return CL_INVALID_IMAGE_DESCRIPTOR;
+  const bool arr1 = t == CL_MEM_OBJECT_IMAGE1D_ARRAY, arr2 = t == CL_MEM_OBJECT_IMAGE2D_ARRAY;
+  const bool from_buffer = t == CL_MEM_OBJECT_IMAGE1D_BUFFER;
+  if (desc->num_mip_levels != 0 || desc->num_samples != 0 ||
+      (desc->buffer != nullptr) != from_buffer)
     return CL_INVALID_IMAGE_DESCRIPTOR;
-  size_t w = desc->image_width, h = dims > 1 ? desc->image_height : 1,
-         d = dims > 2 ? desc->image_depth : 1;
+  // storage extents: the layers of an array are its last storage axis
+  size_t w = desc->image_width, h = 1, d = 1;
+  if (arr1) h = desc->image_array_size;
+  else if (dims > 1) h = desc->image_height;
+  if (arr2) d = desc->image_array_size;
+  else if (dims > 2) d = desc->image_depth;
   if (w == 0 || h == 0 || d == 0) return CL_INVALID_IMAGE_DESCRIPTOR;
-  const size_t maxw = dims == 3 ? kMax3D : kMax2D;
-  if (w > maxw || h > maxw || d > kMax3D) return CL_INVALID_IMAGE_SIZE;
+  if (from_buffer) {
+    if (w > kMaxBuffer) return CL_INVALID_IMAGE_SIZE;
+  } else if (arr1 || arr2) {
+    if (w > kMax2D || (arr1 ? h : d) > kMaxArray || (arr2 && h > kMax2D)) return CL_INVALID_IMAGE_SIZE;
+  } else {
+    const size_t maxw = dims == 3 ? kMax3D : kMax2D;
+    if (w > maxw || h > maxw || d > kMax3D) return CL_INVALID_IMAGE_SIZE;
+  }
   L->fmt = fi;
   L->dims = dims;
+  L->arrayed = (arr1 || arr2) ? 1 : 0;
   L->w = w; L->h = h; L->d = d;
   // internal pitch (reading A21): rows 128-byte aligned -> every texel is
-  // naturally aligned for its vector load, and TMA boxes are legal.
-  L->row_pitch = (w * fi.es + 127) / 128 * 128;
+  // naturally aligned for its vector load, and TMA boxes are legal.  A 1D
+  // image buffer is the buffer's bytes, tightly packed (one row).
+  L->row_pitch = from_buffer ? w * fi.es : (w * fi.es + 127) / 128 * 128;
   L->slice_pitch = L->row_pitch * h;
   L->bytes = L->slice_pitch * d;
   return CL_SUCCESS;

@@ -166,3 +166,34 @@ def test_dynamic_constant_arguments(sess, prog):
     assert cl.lib().clSetKernelArg(k, 1, 8, ctypes.byref(v)) == -50
     cl.lib().clReleaseKernel(k)
     sess.release(b1, b2, out)
+
+
+def test_arrays_and_buffer_images_in_translated_kernel(sess, orc, prog):
+    """image2d_array_t / image1d_buffer_t / image1d_array_t arguments: a weighted
+    sum over layers, each layer read with the library's read built-in."""
+    W, H, L = 40, 6, 5
+    g = synth.rng(83)
+    codes = synth.image_codes(g, cl.CL_RGBA, cl.CL_UNORM_INT8, W, H, L)
+    arr = sess.image_array(cl.CL_RGBA, cl.CL_UNORM_INT8, W, L, H, host=codes)
+    wts = g.uniform(-1, 1, 8).astype(np.float32)
+    wb = sess.buffer(wts.nbytes, wts)
+    wimg = sess.image_buffer(cl.CL_R, cl.CL_FLOAT, 8, wb)
+    dst = sess.image_array(cl.CL_RGBA, cl.CL_FLOAT, W, H)
+    smp = sess.sampler(False, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_NEAREST)
+    k = sess.kernel(prog, "layer_mix")
+    sess.set_args(k, arr, smp, wimg, dst)
+    sess.ndrange(k, (W, H), (8, 2))
+    got = sess.read_image(dst, (0, 0, 0), (W, H, 1)).view(np.float32).reshape(H, W, 4)
+    oarr = orc.Image(codes.copy(), W, H, L, dims=2, order=orc.RGBA, type=orc.UNORM_INT8,
+                     arrayed=True)
+    xs, ys = np.meshgrid(np.arange(W) + 0.5, np.arange(H) + 0.5)
+    exp = np.zeros((H * W, 4), np.float32)
+    for l in range(L):
+        co = np.stack([xs.ravel(), ys.ravel(), np.full(W * H, l), np.zeros(W * H)], 1)
+        t = orc.read_samples(oarr, False, orc.ADDRESS_CLAMP_TO_EDGE, orc.FILTER_NEAREST, orc.RT_F,
+                             co.astype(np.float32))
+        exp = (exp + (t * wts[l]).astype(np.float32)).astype(np.float32)
+    assert np.array_equal(got.reshape(-1, 4), exp)
+    cl.lib().clReleaseKernel(k)
+    cl.lib().clReleaseSampler(smp)
+    sess.release(arr, wimg, wb, dst)

@@ -161,3 +161,32 @@ def test_p8_grid_mode_on_arrays(orc):
     co = np.stack(co, 1)
     ref = orc.read_samples(img, False, ADDR["CLAMP"], FILT["LINEAR"], orc.RT_F, co)
     assert np.array_equal(got.reshape(-1, 4).view(np.uint32), ref.view(np.uint32))
+
+
+def test_p8_integer_coordinates_are_exact_indices(orc):
+    """Reading A30: an integer coordinate is the texel index itself -- equal to
+    the float path at u = (float)i while i is exactly representable (|i| <= 2^24),
+    and still the texel at i beyond (a 1D image buffer reaches 2^31 - 1)."""
+    n = (1 << 25) + 64
+    data = (np.arange(n, dtype=np.int64) * 2654435761 % 251).astype(np.uint8)
+    img = orc.Image(data, n, 1, 1, dims=1, order=orc.R, type=orc.UNSIGNED_INT8)
+    g = synth.rng(306)
+    big = np.concatenate([g.integers((1 << 24) + 1, n, 500), [n - 1, (1 << 24) + 1, (1 << 25) + 1]])
+    for addr in (ADDR["NONE"], ADDR["CLAMP_TO_EDGE"], ADDR["CLAMP"]):
+        got = orc.read_samples(img, False, addr, FILT["NEAREST"], orc.RT_UI,
+                               big.astype(np.int32)[:, None].copy())
+        assert np.array_equal(got[:, 0], data[big]), addr          # the definition: texel i
+        small = np.concatenate([g.integers(-5, 1 << 24, 500), [1 << 24, -1, n, n + 7]])
+        gi = orc.read_samples(img, False, addr, FILT["NEAREST"], orc.RT_UI,
+                              small.astype(np.int32)[:, None].copy())
+        gf = orc.read_samples(img, False, addr, FILT["NEAREST"], orc.RT_UI,
+                              small.astype(np.float32)[:, None].copy())
+        ok = np.abs(small) <= (1 << 24)
+        assert np.array_equal(gi[ok], gf[ok]), addr
+    # out of range under CLAMP_TO_EDGE: the edge texel; under NONE/CLAMP: the border (0,0,0,1)
+    got = orc.read_samples(img, False, ADDR["CLAMP_TO_EDGE"], FILT["NEAREST"], orc.RT_UI,
+                           np.array([[n + 100], [-7]], np.int32))
+    assert got[:, 0].tolist() == [data[n - 1], data[0]]
+    got = orc.read_samples(img, False, ADDR["CLAMP"], FILT["NEAREST"], orc.RT_UI,
+                           np.array([[n + 100]], np.int32))
+    assert got.tolist() == [[0, 0, 0, 1]]
