@@ -376,23 +376,28 @@ def run_gpu(args):
         dist.barrier()
     clocks = Clocks(gpu)
     clocks.start()
+    # (1) the step time: K steps back to back, events only at the two ends
+    # (an event between launches serialises the kernel boundary: +3.5 us each)
     n_launch0 = cl.launch_count()
-    evs = []
     t_start = T.event()
     for _ in range(args.steps):
-        e0 = T.event()
         launch(0)
-        e1 = T.event()
         launch(1)
-        e2 = T.event()
-        evs.append((e0, e1, e2))
     t_end = T.event()
     torch.cuda.synchronize(dev)
     gpu_launches = cl.launch_count() - n_launch0
-    clk = clocks.stop()
     total_ms = t_start.elapsed_time(t_end)
-    pass_ms = [float(np.mean([e[0].elapsed_time(e[1]) for e in evs])),
-               float(np.mean([e[1].elapsed_time(e[2]) for e in evs]))]
+    # (2) each kernel's average launch duration for the roofline: K launches of
+    # it back to back between two events on the launching stream
+    pass_ms = []
+    for k in range(2):
+        a = T.event()
+        for _ in range(args.steps):
+            launch(k)
+        b = T.event()
+        torch.cuda.synchronize(dev)
+        pass_ms.append(a.elapsed_time(b) / args.steps)
+    clk = clocks.stop()
     ms_step = total_ms / args.steps
     if world > 1:
         ms_step = bdist.max_over_ranks(ms_step, red_dev)
@@ -478,6 +483,8 @@ def run_gpu(args):
             "data": "synthetic (numpy default_rng seed 20151115; U[0,1) RGBA32F texels)",
             "config": {"workload": WORKLOAD, "image": "4096x4096 RGBA32F (256 MiB)",
                        "samples_per_step": samples_step, "launches_per_step": 2,
+                       "timing": ("step: K steps between two events; kernel_ms: K back-to-back "
+                                  "launches of that kernel between two events, right after"),
                        "parallelism": ("single GPU" if world == 1 else
                                        f"row-sharded x{world}: global {Hg}x{N2D} image, "
                                        f"4096 output rows per GPU from shards of "

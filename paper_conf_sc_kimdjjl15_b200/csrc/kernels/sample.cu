@@ -71,7 +71,7 @@ __global__ void __launch_bounds__(256) k_sample_grid(const SampleParams p) {
 // Separable maps: block = 32 x 4 threads; tile = (32*XPT) columns x (4*RPW) rows
 // of one output slice.  Lane -> columns lane + 32*t, warp -> RPW consecutive rows.
 template <class C, int OUTC, int XPT, int RPW>
-__global__ void __launch_bounds__(128, 11) k_sample_grid_sep(const SampleParams p) {
+__global__ void __launch_bounds__(128, (C::type == RT ? 1 : 11)) k_sample_grid_sep(const SampleParams p) {
   const Image& im = p.im;
   const int z = blockIdx.z;
   const int x0 = blockIdx.x * (32 * XPT) + threadIdx.x;
@@ -141,47 +141,60 @@ __global__ void __launch_bounds__(128, 11) k_sample_grid_sep(const SampleParams 
 
 // Separable map, LINEAR, compile-time format: register reuse along a walk.
 // Each warp walks consecutive outputs along the outermost image axis (y for
-// 2D, z for 3D) with lanes across x.  A step needs the texel rows at the
-// walk-axis indices (lo, hi) = (i0, i1); when step w+1's lo equals step w's
-// hi (a warp-uniform test) those rows are reused from registers, so a sample
-// costs half the taps (2 of 4 in 2D, 4 of 8 in 3D) in global loads.  The
-// loads of step w+1 are issued before step w is blended (software
-// pipelining), so a warp keeps two steps of loads in flight.  The values are
-// the same texels blended in the same order as linear_at, so the results are
-// bit-identical to the other kernels.
+// 2D, z for 3D) with lanes across x.  The blend is separable -- x, then y,
+// then z, as linear_at -- and every partial result before the walk-axis
+// blend depends only on the texel row(s) at one walk index and on the fixed
+// x (and 3D: y) weights.  So a step keeps, per column and channel, ONE value
+// for each of the two walk indices it blends (lo, hi):
+//   2D: the x-blended row            lerp(a, T[j][i0], T[j][i1])
+//   3D: the x- then y-blended slice   lerp(b, lerp(a, T[j0][k][i0..]), lerp(a, T[j1][k][i0..]))
+// and blends them along the walk axis.  When step w+1's lo index equals step
+// w's hi (warp-uniform test) that value is reused from registers, so a
+// sample costs half the taps in global loads and half the x/y blends.  The
+// next hi is loaded and pre-blended before this step is finished (software
+// pipelining).  The operations and their order are exactly linear_at's, so
+// the results are bit-identical to the other kernels.
 //   2D: block = 32 x 4 threads, tile = (32*XPT) columns x (4*WALK) rows;
 //       warp w walks rows [y0 + w*WALK, +WALK).
 //   3D: tile = (32*XPT) columns x 4 rows x WALK slices; warp w owns one row
 //       and walks slices [z0, z0 + WALK).
-template <class C, int NJ, int XPT>
-struct WalkRows {  // converted texel values of the rows at one walk index
-  float v[NJ][XPT][C::nch][2];  // [row][column][channel][i0 / i1]
+template <class C, int XPT>
+struct WalkVals {  // pre-blended values at one walk index: [column][channel]
+  float v[XPT][C::nch];
 };
 
-template <class C, int NJ, int XPT>
+template <class C, int XPT>
 __device__ __forceinline__ void walk_load(const Image& im, const AxL (&ax)[XPT], const AxL& afix,
-                                          int widx, bool wok, WalkRows<C, NJ, XPT>& out) {
+                                          int widx, bool wok, WalkVals<C, XPT>& out) {
   constexpr bool D3 = C::dims == 3;
+  constexpr int NJ = D3 ? 2 : 1;  // texel rows per walk index
+  uint32_t m0[NJ][XPT][4], m1[NJ][XPT][4];
 #pragma unroll
   for (int js = 0; js < NJ; ++js) {
     const int j = D3 ? (js ? afix.i1 : afix.i0) : widx;
     const int k = D3 ? widx : 0;
     const bool rok = wok && (!D3 || (js ? afix.ok1 : afix.ok0));
     const char* row = row_ptr<C>(im, j, k);
-    uint32_t m0[XPT][4], m1[XPT][4];
 #pragma unroll
     for (int t = 0; t < XPT; ++t) {
-      fetch<C>(im, row, ax[t].i0, rok && ax[t].ok0, R_F, m0[t]);
-      fetch<C>(im, row, ax[t].i1, rok && ax[t].ok1, R_F, m1[t]);
+      fetch<C>(im, row, ax[t].i0, rok && ax[t].ok0, R_F, m0[js][t]);
+      fetch<C>(im, row, ax[t].i1, rok && ax[t].ok1, R_F, m1[js][t]);
     }
-#pragma unroll
-    for (int t = 0; t < XPT; ++t)
-#pragma unroll
-      for (int ch = 0; ch < C::nch; ++ch) {
-        out.v[js][t][ch][0] = __uint_as_float(m0[t][ch]);
-        out.v[js][t][ch][1] = __uint_as_float(m1[t][ch]);
-      }
   }
+#pragma unroll
+  for (int t = 0; t < XPT; ++t)
+#pragma unroll
+    for (int ch = 0; ch < C::nch; ++ch) {
+      const float r0 = lerp1(ax[t].a, ax[t].oma, __uint_as_float(m0[0][t][ch]),
+                             __uint_as_float(m1[0][t][ch]));
+      if constexpr (D3) {
+        const float r1 = lerp1(ax[t].a, ax[t].oma, __uint_as_float(m0[NJ - 1][t][ch]),
+                               __uint_as_float(m1[NJ - 1][t][ch]));
+        out.v[t][ch] = lerp1(afix.a, afix.oma, r0, r1);
+      } else {
+        out.v[t][ch] = r0;
+      }
+    }
 }
 
 template <class C, int OUTC, int XPT, int WALK>
@@ -190,8 +203,7 @@ __global__ void __launch_bounds__(128) k_sample_grid_walk(const SampleParams p) 
   static_assert(C::dims >= 2, "walk needs a second axis");
   constexpr int NCH = C::nch;
   constexpr bool D3 = C::dims == 3;
-  constexpr int NJ = D3 ? 2 : 1;  // texel rows per walk index
-  using Rows = WalkRows<C, NJ, XPT>;
+  using Vals = WalkVals<C, XPT>;
   const Image& im = p.im;
   // 3D: the 4 warps of a block split x (one texel row per block, wide DRAM bursts)
   const int x0 = D3 ? blockIdx.x * (128 * XPT) + threadIdx.y * (32 * XPT) + threadIdx.x
@@ -222,25 +234,23 @@ __global__ void __launch_bounds__(128) k_sample_grid_walk(const SampleParams p) 
     return axis_l<C>(p.smp, __fadd_rn(__fmul_rn(awc, __int2float_rn(wor + wv)), awo), nw);
   };
   AxL aw = walk_axis(w0);
-  // Three row buffers in fixed rotating roles (lo, hi, next-hi): no register
-  // copies between steps.  A step issues the next hi rows, blends (lo, hi),
-  // and -- only when the next lo rows are not this hi (no reuse) -- reloads
-  // them into the hi buffer after the blend, which becomes the next lo.
-  Rows B0, B1, B2;
-  walk_load<C, NJ, XPT>(im, ax, afix, aw.i0, aw.ok0, B0);
-  walk_load<C, NJ, XPT>(im, ax, afix, aw.i1, aw.ok1, B1);
-  // one step with (lo, hi, nx) = rows at aw; returns false after the last step
-  auto step = [&](int w, Rows& lo, Rows& hi, Rows& nx) -> bool {
+  // Three value buffers in fixed rotating roles (lo, hi, next-hi): no
+  // register copies between steps.  A step loads the next hi, blends
+  // (lo, hi), and -- only when the next lo is not this hi (no reuse) --
+  // reloads it into the hi buffer after the blend, which becomes the next lo.
+  Vals B0, B1, B2;
+  walk_load<C, XPT>(im, ax, afix, aw.i0, aw.ok0, B0);
+  walk_load<C, XPT>(im, ax, afix, aw.i1, aw.ok1, B1);
+  const float fa = D3 ? afix.a : 0.f;  // 3D: the fixed y weight (NaN test of A26)
+  // one step with (lo, hi, nx) = values at aw; returns false after the last step
+  auto step = [&](int w, Vals& lo, Vals& hi, Vals& nx) -> bool {
     const int wv = w0 + w;
     const bool next = w + 1 < WALK && wv + 1 < wlen;
     AxL an = aw;
     if (next) {
       an = walk_axis(wv + 1);
-      walk_load<C, NJ, XPT>(im, ax, afix, an.i1, an.ok1, nx);
+      walk_load<C, XPT>(im, ax, afix, an.i1, an.ok1, nx);
     }
-    // blend and store this step: x, then y, then z (as linear_at)
-    const AxL& ay = D3 ? afix : aw;
-    const float ga = D3 ? aw.a : 0.f, goma = D3 ? aw.oma : 1.f;
     const int y = D3 ? yfix : wv, z = D3 ? wv : zfix;
     const uint64_t obase = ((uint64_t)z * p.oh + y) * p.ow;
 #pragma unroll
@@ -248,33 +258,17 @@ __global__ void __launch_bounds__(128) k_sample_grid_walk(const SampleParams p) 
       const int x = x0 + 32 * t;
       uint32_t m[4] = {0u, 0u, 0u, 0u};
 #pragma unroll
-      for (int ch = 0; ch < NCH; ++ch) {
-        const float a = ax[t].a, oma = ax[t].oma;
-        float o;
-        if (D3) {
-          // rows (j0,k0)=lo[0], (j1,k0)=lo[1], (j0,k1)=hi[0], (j1,k1)=hi[1]
-          const float r00 = lerp1(a, oma, lo.v[0][t][ch][0], lo.v[0][t][ch][1]);
-          const float r10 = lerp1(a, oma, lo.v[NJ - 1][t][ch][0], lo.v[NJ - 1][t][ch][1]);
-          const float r01 = lerp1(a, oma, hi.v[0][t][ch][0], hi.v[0][t][ch][1]);
-          const float r11 = lerp1(a, oma, hi.v[NJ - 1][t][ch][0], hi.v[NJ - 1][t][ch][1]);
-          o = lerp1(ga, goma, lerp1(ay.a, ay.oma, r00, r10), lerp1(ay.a, ay.oma, r01, r11));
-        } else {
-          const float r0 = lerp1(a, oma, lo.v[0][t][ch][0], lo.v[0][t][ch][1]);
-          const float r1 = lerp1(a, oma, hi.v[0][t][ch][0], hi.v[0][t][ch][1]);
-          o = lerp1(ay.a, ay.oma, r0, r1);
-        }
-        m[ch] = __float_as_uint(o);
-      }
+      for (int ch = 0; ch < NCH; ++ch)
+        m[ch] = __float_as_uint(lerp1(aw.a, aw.oma, lo.v[t][ch], hi.v[t][ch]));
       uint32_t res[4];
       map_order(C::order, m, 0x3f800000u, res);
-      if (const_in_output(C::order, OUTC) && (ax[t].a != ax[t].a || ay.a != ay.a || ga != ga))
+      if (const_in_output(C::order, OUTC) && (ax[t].a != ax[t].a || aw.a != aw.a || fa != fa))
         res[0] = res[1] = res[2] = res[3] = 0x7fffffffu;
       if (x < p.ow) store_out<OUTC>(p, obase + x, res);
     }
     if (!next) return false;
-    // the next step's lo rows are this step's hi rows unless the walk skips
-    if (!(an.i0 == aw.i1 && an.ok0 == aw.ok1))
-      walk_load<C, NJ, XPT>(im, ax, afix, an.i0, an.ok0, hi);
+    // the next step's lo is this step's hi unless the walk skips
+    if (!(an.i0 == aw.i1 && an.ok0 == aw.ok1)) walk_load<C, XPT>(im, ax, afix, an.i0, an.ok0, hi);
     aw = an;
     return true;
   };
@@ -284,6 +278,132 @@ __global__ void __launch_bounds__(128) k_sample_grid_walk(const SampleParams p) 
     if (!step(w + 1, B1, B2, B0)) break;
     if (!step(w + 2, B2, B0, B1)) break;
   }
+}
+
+// 3D walk for one-channel 32-bit float images (config 3: R32F trilinear),
+// four CONSECUTIVE columns per thread (a warp covers 128 columns).  When the
+// x axis is a unit-stride stencil over the warp -- column x+t taps
+// (i0 + t, i0 + t + 1), all in range, i0 16-byte aligned, the next lane
+// starting 4 texels further (warp-uniform vote, once per thread) -- a texel
+// row costs one 16-byte load plus one shuffle for the fifth texel, instead
+// of eight scalar loads, and the four outputs leave in one 16-byte store.
+// Otherwise (image edges, other maps) the same columns load texel by texel.
+// Blend order and operands are walk_load's and linear_at's: bit-identical.
+template <class C>
+struct Walk4 {
+  float v[4];  // x- then y-blended value of this slice for the 4 columns
+};
+
+template <class C>
+__device__ __forceinline__ void walk4_load(const Image& im, const AxL (&ax)[4], const AxL& afix,
+                                           int k, bool kok, bool vec, Walk4<C>& out) {
+  float r[2][4];
+#pragma unroll
+  for (int js = 0; js < 2; ++js) {
+    const int j = js ? afix.i1 : afix.i0;
+    const bool rok = kok && (js ? afix.ok1 : afix.ok0);
+    const char* row = row_ptr<C>(im, j, k);
+    float T0[4], T1[4];
+    if (vec) {
+      float4 q = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (rok) q = __ldg(reinterpret_cast<const float4*>(row + (uint64_t)(unsigned)ax[0].i0 * 4u));
+      float e = __shfl_down_sync(0xffffffffu, q.x, 1);
+      if ((threadIdx.x & 31) == 31)
+        e = rok ? __ldg(reinterpret_cast<const float*>(row + (uint64_t)(unsigned)ax[3].i1 * 4u)) : 0.f;
+      T0[0] = q.x; T0[1] = q.y; T0[2] = q.z; T0[3] = q.w;
+      T1[0] = q.y; T1[1] = q.z; T1[2] = q.w; T1[3] = e;
+    } else {
+#pragma unroll
+      for (int t = 0; t < 4; ++t) {
+        uint32_t m0[4], m1[4];
+        fetch<C>(im, row, ax[t].i0, rok && ax[t].ok0, R_F, m0);
+        fetch<C>(im, row, ax[t].i1, rok && ax[t].ok1, R_F, m1);
+        T0[t] = __uint_as_float(m0[0]);
+        T1[t] = __uint_as_float(m1[0]);
+      }
+    }
+#pragma unroll
+    for (int t = 0; t < 4; ++t) r[js][t] = lerp1(ax[t].a, ax[t].oma, T0[t], T1[t]);
+  }
+#pragma unroll
+  for (int t = 0; t < 4; ++t) out.v[t] = lerp1(afix.a, afix.oma, r[0][t], r[1][t]);
+}
+
+// the walk of one thread (VEC: the 16-byte row loads; else texel by texel)
+template <class C, int WALK, bool VEC>
+__device__ __forceinline__ void walk4_run(const SampleParams& p, const AxL (&ax)[4], int x0,
+                                          int yfix, int w0, bool vst) {
+  const Image& im = p.im;
+  const AxL afix =
+      axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(p.oy + yfix)), p.A[7]), im.h);
+  auto walk_axis = [&](int wv) {
+    return axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[10], __int2float_rn(p.oz + wv)), p.A[11]), im.d);
+  };
+  AxL aw = walk_axis(w0);
+  Walk4<C> B0, B1, B2;
+  walk4_load<C>(im, ax, afix, aw.i0, aw.ok0, VEC, B0);
+  walk4_load<C>(im, ax, afix, aw.i1, aw.ok1, VEC, B1);
+  float* obase = reinterpret_cast<float*>(p.out) + (uint64_t)yfix * p.ow + x0;
+  const uint64_t zstride = (uint64_t)p.oh * p.ow;
+  auto step = [&](int w, Walk4<C>& lo, Walk4<C>& hi, Walk4<C>& nx) -> bool {
+    const int wv = w0 + w;
+    const bool next = w + 1 < WALK && wv + 1 < p.od;
+    AxL an = aw;
+    if (next) {
+      an = walk_axis(wv + 1);
+      walk4_load<C>(im, ax, afix, an.i1, an.ok1, VEC, nx);
+    }
+    float o[4];
+#pragma unroll
+    for (int t = 0; t < 4; ++t) o[t] = lerp1(aw.a, aw.oma, lo.v[t], hi.v[t]);
+    float* orow = obase + (uint64_t)wv * zstride;
+    if (vst) {
+      __stcs(reinterpret_cast<float4*>(orow), make_float4(o[0], o[1], o[2], o[3]));
+    } else {
+#pragma unroll
+      for (int t = 0; t < 4; ++t)
+        if (x0 + t < p.ow) __stcs(orow + t, o[t]);
+    }
+    if (!next) return false;
+    if (!(an.i0 == aw.i1 && an.ok0 == aw.ok1)) walk4_load<C>(im, ax, afix, an.i0, an.ok0, VEC, hi);
+    aw = an;
+    return true;
+  };
+#pragma unroll 1
+  for (int w = 0; w < WALK; w += 3) {
+    if (!step(w, B0, B1, B2)) break;
+    if (!step(w + 1, B1, B2, B0)) break;
+    if (!step(w + 2, B2, B0, B1)) break;
+  }
+}
+
+#ifndef B2CL_W4_MINB
+#define B2CL_W4_MINB 12
+#endif
+template <class C, int WALK>
+__global__ void __launch_bounds__(128, B2CL_W4_MINB) k_sample_grid_walk4(const SampleParams p) {
+  static_assert(C::dims == 3 && C::nch == 1 && C::type == T_FLOAT, "R32F-type 3D images");
+  const Image& im = p.im;
+  const int lane = threadIdx.x & 31;
+  const int x0 = blockIdx.x * 512 + threadIdx.y * 128 + lane * 4;
+  AxL ax[4];
+#pragma unroll
+  for (int t = 0; t < 4; ++t)
+    ax[t] = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(p.ox + x0 + t)), p.A[3]),
+                      im.w);
+  bool ok = (ax[0].i0 & 3) == 0 && x0 + 3 < p.ow;
+#pragma unroll
+  for (int t = 0; t < 4; ++t)
+    ok = ok && ax[t].ok0 && ax[t].ok1 && ax[t].i0 == ax[0].i0 + t && ax[t].i1 == ax[t].i0 + 1;
+  const int nb = __shfl_down_sync(0xffffffffu, ax[0].i0, 1);
+  if (lane < 31) ok = ok && nb == ax[0].i0 + 4;
+  const bool vec = __all_sync(0xffffffffu, ok);
+  const bool vst = (p.ow & 3) == 0 && x0 + 3 < p.ow;  // 16-byte output stores
+  const int yfix = blockIdx.y;
+  const int w0 = blockIdx.z * WALK;
+  if (yfix >= p.oh || w0 >= p.od) return;  // block-uniform
+  if (vec) walk4_run<C, WALK, true>(p, ax, x0, yfix, w0, vst);
+  else walk4_run<C, WALK, false>(p, ax, x0, yfix, w0, vst);
 }
 
 template <class C, bool INT_COORD>
@@ -346,6 +466,16 @@ static cudaError_t go_walk(const SampleParams& p, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+template <class C, int WALK>
+static cudaError_t go_walk4(const SampleParams& p, cudaStream_t st) {
+  dim3 blk(32, 4, 1);
+  dim3 grd((p.ow + 511) / 512, p.oh, (p.od + WALK - 1) / WALK);
+  if (is_shard(p)) k_sample_grid_walk4<WithShard<C, true>, WALK><<<grd, blk, 0, st>>>(p);
+  else k_sample_grid_walk4<WithShard<C, false>, WALK><<<grd, blk, 0, st>>>(p);
+  count_launch();
+  return cudaGetLastError();
+}
+
 template <class C, int OUTC, int XPT, int RPW>
 static cudaError_t go_sep(const SampleParams& p, cudaStream_t st) {
   dim3 blk(32, 4, 1);
@@ -376,6 +506,15 @@ static cudaError_t go_list(const SampleParams& p, bool int_coord, cudaStream_t s
 template <int DIMS>
 using Generic = Cfg<DIMS, RT, RT, RT, RT, RT, RT>;
 
+// tile shapes of the hot instances (overridable at build time for A/B
+// variants, tools/build_variant.py)
+#ifndef B2CL_C3_XPT
+#define B2CL_C3_XPT 4
+#endif
+#ifndef B2CL_C3_WALK
+#define B2CL_C3_WALK 32
+#endif
+
 // hot configurations (BASELINE.json configs 1-3)
 using C2Repeat = Cfg<2, T_FLOAT, O_RGBA, 1, A_REPEAT, F_LINEAR, R_F>;
 using C2Mirror = Cfg<2, T_FLOAT, O_RGBA, 1, A_MIRROR, F_LINEAR, R_F>;
@@ -400,10 +539,10 @@ static bool separable(const SampleParams& p) {
 cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st) {
   if (coord_mode == COORD_GRID) {
     if ((uint64_t)p.ow * p.oh * p.od == 0) return cudaSuccess;
-    // B2CL_GRID_KERNEL=general|sep|walk forces a kernel family (A/B runs under ncu);
+    // B2CL_GRID_KERNEL=general|sep|walk|4 forces a kernel family (A/B runs under ncu);
     // the default picks the variant measured fastest on B200 for each hot config
     static const char* force = getenv("B2CL_GRID_KERNEL");
-    const int fk = !force ? 0 : (force[0] == 'g' ? 1 : (force[0] == 's' ? 2 : (force[0] == 'w' ? 3 : 0)));
+    const int fk = !force ? 0 : (force[0] == 'g' ? 1 : (force[0] == 's' ? 2 : (force[0] == 'w' ? 3 : (force[0] == '4' ? 4 : 0))));
     if (p.arr)  // image arrays: the general kernel, fully run-time format and sampler
       return p.dims == 1 ? go_grid<Layered<Generic<1>>, RT>(p, st) : go_grid<Layered<Generic<2>>, RT>(p, st);
     if (separable(p) && fk != 1) {
@@ -412,7 +551,9 @@ cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st
       if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_MIRROR, F_LINEAR))
         return fk == 3 ? go_walk<C2Mirror, 4, 2, 8>(p, st) : go_sep<C2Mirror, 4, 2, 4>(p, st);
       if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR))
-        return fk == 2 ? go_sep<C3Cte, 1, 4, 4>(p, st) : go_walk<C3Cte, 1, 4, 16>(p, st);
+        return fk == 2   ? go_sep<C3Cte, 1, 4, 4>(p, st)
+               : fk == 3 ? go_walk<C3Cte, 1, B2CL_C3_XPT, B2CL_C3_WALK>(p, st)
+                         : go_walk4<C3Cte, B2CL_C3_WALK>(p, st);
       if (p.outc == 4 && matches<2>(p, T_UNORM8, O_RGBA, 0, A_CLAMP, F_NEAREST)) return go_sep<C1Clamp, 4, 2, 4>(p, st);
       switch (p.dims) {
         case 1: return go_sep<Generic<1>, RT, 2, 2>(p, st);

@@ -150,6 +150,14 @@ GRID_CASES = [
     (2, BGRA, U8N, (31, 17, 1), (1, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_LINEAR), "rotate", (45, 29, 1), 3),
     (1, RG, F16, (50, 1, 1), (1, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR), "translate", (77, 1, 1), 2),
     (3, RGBA, U16N, (9, 8, 7), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "stencil", (12, 11, 10), 4),
+    # config-3 kernel (k_sample_grid_walk4): 16-byte stencil rows in the interior
+    # warps, texel-by-texel at the right edge and the ragged last warp, a ragged walk
+    (3, R, F32, (300, 7, 37), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "stencil", (300, 7, 37), 1),
+    (3, R, F32, (1030, 3, 5), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "stencil", (1030, 3, 5), 1),
+    # shifted by one texel (i0 = x + 1: not 16-byte aligned) and by five (the 5th
+    # texel of the last lane comes from the next 16 bytes), output width not /4
+    (3, R, F32, (260, 4, 19), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "stencil+1", (258, 4, 19), 1),
+    (3, R, F32, (260, 4, 19), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "stencil+4", (250, 4, 19), 1),
 ]
 
 
@@ -167,8 +175,10 @@ def _affine(kind, size, out):
         return A
     if kind == "rotate3d":
         return synth.affine_rotate_3d(W, 20.0)
-    if kind == "stencil":
+    if kind.startswith("stencil"):
         A = synth.affine_stencil_3d(W)
+        if "+" in kind:  # shift the x taps by whole texels
+            A[3] = (0.5 + 0.3 + int(kind.split("+")[1])) / W
         A[5] = 1.0 / H
         A[7] = (0.5 + 0.6) / H
         A[10] = 1.0 / D

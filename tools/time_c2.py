@@ -39,8 +39,25 @@ def main():
         e1.record(st)
         torch.cuda.synchronize()
         res.append(e0.elapsed_time(e1) / 50 * 1e3)
+    # the bench step: REPEAT then MIRRORED back to back, no events in between
+    smps = [S.sampler(True, a, cl.CL_FILTER_LINEAR)
+            for a in (cl.CL_ADDRESS_REPEAT, cl.CL_ADDRESS_MIRRORED_REPEAT)]
+    outs = [out, S.buffer(n * n * 16)]
+
+    def step():
+        for k in range(2):
+            cl.check(L.b2clEnqueueReadImageGrid(S.queue, img, smps[k], 0, A, d, 4, outs[k], 0, 0,
+                                                None, None))
+    for _ in range(5):
+        step()
+    e0.record(st)
+    for _ in range(50):
+        step()
+    e1.record(st)
+    torch.cuda.synchronize()
+    pair = e0.elapsed_time(e1) / 50 * 1e3
     print(f"{os.path.basename(os.environ.get('B2CL_LIB', 'libb2cl.so'))}: REPEAT {res[0]:.1f} us, "
-          f"MIRRORED {res[1]:.1f} us")
+          f"MIRRORED {res[1]:.1f} us, sum {res[0] + res[1]:.1f} us, step {pair:.1f} us")
 
 
 if __name__ == "__main__":
