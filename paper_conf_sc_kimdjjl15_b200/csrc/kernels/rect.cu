@@ -13,6 +13,12 @@
 // origins or pitches) is read as aligned 16-byte words -- one load per lane,
 // the next word by warp shuffle -- and funnel-shifted (the shift is constant
 // along a row and a warp covers one row, so the branch is warp-uniform).
+// Misaligned copies of rows of 2 KiB or more take k_rect_staged instead
+// (bulk-async staging through shared memory, below).  Sources are always
+// local to the launching device except for migration, whose source and
+// destination offsets are both 0 (the aligned instance).
+#include <atomic>
+
 #include "../device/image.cuh"
 #include "launch.h"
 
@@ -152,6 +158,171 @@ __global__ void __launch_bounds__(256) k_rect(const RectParams p) {
   }
 }
 
+// ------------------------------------------------- staged misaligned copy
+// A copy whose source is misaligned against its destination, with rows long
+// enough to amortize a stage: each unit (up to ST_CH destination bytes of one
+// row) has the 16-byte-aligned cover of its source bytes brought into shared
+// memory by one bulk async copy (cp.async.bulk, the TMA engine) completing on
+// an mbarrier; ST_NS stages keep ST_NS-1 units in flight per block while the
+// threads funnel-shift the current one out of shared memory into aligned
+// 16-byte global stores.  The loads need no registers and no shuffles, so the
+// bytes in flight no longer depend on occupancy.  A persistent grid of
+// ST_BPS blocks per SM strides over the units.
+#ifndef B2CL_ST_CH
+#define B2CL_ST_CH 16384
+#endif
+#ifndef B2CL_ST_NS
+#define B2CL_ST_NS 3
+#endif
+#ifndef B2CL_ST_BPS
+#define B2CL_ST_BPS 3
+#endif
+constexpr int ST_CH = B2CL_ST_CH;   // destination bytes per unit (chunk 0: up to 15 more)
+constexpr int ST_BUF = ST_CH + 48;  // aligned cover of its source bytes
+constexpr int ST_NS = B2CL_ST_NS;   // stages per block
+constexpr int ST_BPS = B2CL_ST_BPS; // blocks per SM
+#ifndef B2CL_ST_THREADS
+#define B2CL_ST_THREADS 256
+#endif
+constexpr int ST_THREADS = B2CL_ST_THREADS;
+constexpr uint64_t ST_MIN_ROW = 2048;  // shorter rows: the register/shuffle kernel
+
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+struct StUnit {
+  const char* srow;
+  uintptr_t dlo, dhi, abase;
+  uintptr_t u0, u1;  // destination bytes of the unit: [u0, u1)
+  const char* sa;    // aligned source cover: [sa, sa + bytes)
+  uint32_t bytes;
+};
+
+__device__ __forceinline__ StUnit st_unit(const RectParams& p, uint64_t u, uint64_t cpr) {
+  StUnit w;
+  const uint64_t row = u / cpr, c = u - row * cpr;
+  const uint64_t z = row / p.R1, y = row - z * p.R1;
+  w.srow = p.src + z * p.ssp + y * p.srp;
+  w.dlo = reinterpret_cast<uintptr_t>(p.dst + z * p.dsp + y * p.drp);
+  w.dhi = w.dlo + p.R0;
+  w.abase = w.dlo & ~uintptr_t(15);
+  // chunk boundaries at h + c*ST_CH, h = the first 16-byte boundary at or
+  // after the row start; chunk 0 also takes the partial head vector
+  const uintptr_t h = (w.dlo + 15) & ~uintptr_t(15);
+  const uintptr_t c1 = h + (c + 1) * ST_CH;
+  w.u0 = c == 0 ? w.dlo : h + c * ST_CH;
+  w.u1 = c1 < w.dhi ? c1 : w.dhi;
+  if (w.u1 <= w.u0) {  // a row with fewer chunks than the grid's maximum
+    w.u1 = w.u0;
+    w.sa = w.srow;
+    w.bytes = 0;
+    return w;
+  }
+  const uintptr_t s0 = reinterpret_cast<uintptr_t>(w.srow) + (w.u0 - w.dlo);
+  const uintptr_t s1 = reinterpret_cast<uintptr_t>(w.srow) + (w.u1 - w.dlo);
+  const uintptr_t a0 = s0 & ~uintptr_t(15), a1 = (s1 + 15) & ~uintptr_t(15);
+  w.sa = reinterpret_cast<const char*>(a0);
+  w.bytes = static_cast<uint32_t>(a1 - a0);
+  return w;
+}
+
+__device__ __forceinline__ void st_issue(const StUnit& w, char* buf, uint64_t* bar) {
+  const uint32_t b = smem_addr(bar);
+  // (an empty unit arrives with no transaction bytes: the phase completes at once)
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(b), "r"(w.bytes)
+               : "memory");
+  if (w.bytes == 0) return;
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_addr(buf)),
+      "l"(w.sa), "r"(w.bytes), "r"(b)
+      : "memory");
+}
+
+__device__ __forceinline__ void st_wait(uint64_t* bar, uint32_t parity) {
+  const uint32_t b = smem_addr(bar);
+  uint32_t done;
+  do {
+    asm volatile(
+        "{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2; selp.u32 %0, 1, 0, P; }"
+        : "=r"(done)
+        : "r"(b), "r"(parity)
+        : "memory");
+  } while (!done);
+}
+
+__global__ void __launch_bounds__(ST_THREADS, ST_BPS)
+    k_rect_staged(const RectParams p, const uint64_t cpr, const uint64_t units) {
+  extern __shared__ __align__(128) char sbuf[];
+  __shared__ uint64_t full[ST_NS];
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < ST_NS; ++s)
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_addr(&full[s])) : "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  __syncthreads();
+  const uint64_t u_first = blockIdx.x, u_step = gridDim.x;
+  if (threadIdx.x == 0)
+    for (int s = 0; s < ST_NS; ++s) {
+      const uint64_t u = u_first + s * u_step;
+      if (u < units) st_issue(st_unit(p, u, cpr), sbuf + s * ST_BUF, &full[s]);
+    }
+  uint64_t i = 0;
+  for (uint64_t u = u_first; u < units; u += u_step, ++i) {
+    const int s = (int)(i % ST_NS);
+    const char* buf = sbuf + s * ST_BUF;
+    const StUnit w = st_unit(p, u, cpr);
+    st_wait(&full[s], (uint32_t)((i / ST_NS) & 1));
+    // destination vectors of the unit, 16-byte aligned: [v0, v1) counted from abase
+    const uint64_t va = (w.u0 - w.abase) >> 4, vb = (w.u1 - w.abase + 15) >> 4;
+    const uintptr_t sbase = reinterpret_cast<uintptr_t>(w.sa);
+    for (uint64_t v = va + threadIdx.x; v < vb; v += ST_THREADS) {
+      const uintptr_t D = w.abase + 16 * v;
+      // source byte of D, as an offset into the staged cover
+      const uint32_t o = (uint32_t)(reinterpret_cast<uintptr_t>(w.srow) + (D - w.dlo) - sbase);
+      if (D >= w.dlo && D + 16 <= w.dhi) {
+        const uint4* q = reinterpret_cast<const uint4*>(buf + (o & ~15u));
+        const int sh = (int)(o & 15u);
+        *reinterpret_cast<uint4*>(D) = sh ? funnel16(q[0], q[1], sh) : q[0];
+      } else {  // ragged head / tail of the row
+        const uintptr_t lo = D > w.dlo ? D : w.dlo, hi = D + 16 < w.dhi ? D + 16 : w.dhi;
+        for (uintptr_t X = lo; X < hi; ++X)
+          *reinterpret_cast<char*>(X) = buf[o + (uint32_t)(X - D)];
+      }
+    }
+    __syncthreads();  // every thread is done with stage s
+    if (threadIdx.x == 0) {
+      const uint64_t un = u + ST_NS * u_step;
+      if (un < units) {
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        st_issue(st_unit(p, un, cpr), sbuf + s * ST_BUF, &full[s]);
+      }
+    }
+  }
+}
+
+static cudaError_t launch_rect_staged(const RectParams& p, cudaStream_t st) {
+  int dev = 0, sms = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (e != cudaSuccess) return e;
+  const int smem = ST_NS * ST_BUF;
+  static std::atomic<uint64_t> attr_set{0};  // per-device bit: opt-in to > 48 KiB
+  if (!((attr_set.load() >> (dev & 63)) & 1)) {
+    e = cudaFuncSetAttribute(k_rect_staged, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    attr_set.fetch_or(1ull << (dev & 63));
+  }
+  // chunks per row (a row's bytes past its first 16-byte boundary number at most R0)
+  const uint64_t cpr = (p.R0 + ST_CH - 1) / ST_CH;
+  const uint64_t units = cpr * p.R1 * p.R2;
+  const uint64_t blocks = units < (uint64_t)sms * ST_BPS ? units : (uint64_t)sms * ST_BPS;
+  k_rect_staged<<<(unsigned)blocks, ST_THREADS, smem, st>>>(p, cpr, units);
+  count_launch();
+  return cudaGetLastError();
+}
+
 cudaError_t launch_rect(RectParams& p, int mode, cudaStream_t st) {
   const uint64_t rows = (uint64_t)p.R1 * p.R2;
   if (p.R0 == 0 || rows == 0) return cudaSuccess;
@@ -177,6 +348,8 @@ cudaError_t launch_rect(RectParams& p, int mode, cudaStream_t st) {
   const bool aligned = mode == RECT_COPY && ((uintptr_t)p.src - (uintptr_t)p.dst) % 16 == 0 &&
                        (p.srp - p.drp) % 16 == 0 && (p.ssp - p.dsp) % 16 == 0;
   if (aligned) mode = RECT_COPY_ALIGNED;
+  // misaligned copies of rows long enough to fill a stage: bulk-async staged
+  if (mode == RECT_COPY && p.R0 >= ST_MIN_ROW) return launch_rect_staged(p, st);
   switch (mode) {
     case RECT_COPY_ALIGNED: k_rect<RECT_COPY_ALIGNED, U><<<grd, blk, 0, st>>>(p); break;
     case RECT_COPY: k_rect<RECT_COPY, U><<<grd, blk, 0, st>>>(p); break;

@@ -41,6 +41,29 @@ def test_copy_buffer_rect_random_boxes(sess, orc):
         assert np.array_equal(got, exp), (it, so, do, region, srp, ssp, drp, dsp)
 
 
+def test_copy_buffer_rect_staged_long_rows(sess, orc):
+    """Misaligned copies with rows >= 2 KiB take the bulk-async staged kernel (16 KiB
+    destination chunks): rows around and across chunk boundaries, destination
+    alignment constant per row or varying (odd pitches), bytes outside the box kept."""
+    g = synth.rng(36)
+    cases = [(16384, 3, 0), (16383, 5, 1), (16385, 1, 15), (32768 + 5, 7, 3), (2048, 9, 2),
+             (40000, 15, 8), (16384 - 7, 8, 0)]
+    for it, (r0, sx, dx) in enumerate(cases):
+        for odd_pitch in (False, True):
+            region = (r0, int(g.integers(1, 6)), int(g.integers(1, 4)))
+            srp = r0 + sx + int(g.integers(0, 40))
+            drp = r0 + dx + (int(g.integers(1, 30)) if odd_pitch else 16 * int(g.integers(0, 3)))
+            ssp = srp * (region[1] + int(g.integers(0, 3)))
+            dsp = drp * (region[1] + int(g.integers(0, 3)))
+            so, do = (sx, int(g.integers(0, 2)), 0), (dx, 0, int(g.integers(0, 2)))
+            src = _rand_bytes(g, ssp * (so[2] + region[2]) + srp * 2 + 64)
+            dst = _rand_bytes(g, dsp * (do[2] + region[2]) + drp * 2 + 64)
+            got = _copy_rect_gpu(sess, src, dst, so, do, region, srp, ssp, drp, dsp)
+            exp = dst.copy()
+            orc.copy_rect(src, exp, so, do, region, srp, ssp, drp, dsp)
+            assert np.array_equal(got, exp), (it, odd_pitch, so, do, region, srp, ssp, drp, dsp)
+
+
 def test_config1_buffer_rect_all_x_origins(sess, orc):
     """BASELINE config 1 (reading A19): region {64 B, 16, 4} out of a 64x64x4 RGBA8
     volume (row pitch 256, slice pitch 16384), every x origin 0..192, also {16 B,16,4}."""
