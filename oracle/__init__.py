@@ -28,6 +28,8 @@ SNORM_INT8, SNORM_INT16, UNORM_INT8, UNORM_INT16 = 0x10D0, 0x10D1, 0x10D2, 0x10D
 SIGNED_INT8, SIGNED_INT16, SIGNED_INT32 = 0x10D7, 0x10D8, 0x10D9
 UNSIGNED_INT8, UNSIGNED_INT16, UNSIGNED_INT32 = 0x10DA, 0x10DB, 0x10DC
 HALF_FLOAT, FLOAT = 0x10DD, 0x10DE
+Rx, RGx, RGBx = 0x10BA, 0x10BB, 0x10BC
+UNORM_SHORT_565, UNORM_SHORT_555, UNORM_INT_101010 = 0x10D4, 0x10D5, 0x10D6
 ADDRESS_NONE, ADDRESS_CLAMP_TO_EDGE, ADDRESS_CLAMP, ADDRESS_REPEAT, ADDRESS_MIRRORED_REPEAT = range(0x1130, 0x1135)
 FILTER_NEAREST, FILTER_LINEAR = 0x1140, 0x1141
 RT_F, RT_I, RT_UI = 0, 1, 2

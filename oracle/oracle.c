@@ -40,18 +40,43 @@ static int type_bytes(uint32_t type) {
   }
 }
 
+/* The packed channel types ([CL1.2 §5.3.1.1]): a normalized 5-6-5 RGB, or
+ * x-5-5-5 / x-10-10-10 xRGB, in one 16- or 32-bit little-endian word, legal
+ * only with the orders CL_RGB and CL_RGBx. */
+static int is_packed(uint32_t type) {
+  return type == OR_UNORM_SHORT_565 || type == OR_UNORM_SHORT_555 || type == OR_UNORM_INT_101010;
+}
+
+/* width and lowest bit of stored channel c (0 = R, 1 = G, 2 = B) of a packed word */
+static void packed_field(uint32_t type, int c, int* bits, int* shift) {
+  static const int w565[3] = {5, 6, 5}, s565[3] = {11, 5, 0};
+  static const int w555[3] = {5, 5, 5}, s555[3] = {10, 5, 0};
+  static const int w10[3] = {10, 10, 10}, s10[3] = {20, 10, 0};
+  const int *w = w10, *sh = s10;
+  if (type == OR_UNORM_SHORT_565) { w = w565; sh = s565; }
+  if (type == OR_UNORM_SHORT_555) { w = w555; sh = s555; }
+  *bits = w[c];
+  *shift = sh[c];
+}
+
 int oracle_channels(uint32_t order) {
   switch (order) {
     case OR_R: case OR_A: case OR_INTENSITY: case OR_LUMINANCE: return 1;
     case OR_RG: case OR_RA: return 2;
+    case OR_RGB: case OR_RGBx: return 3;   /* packed types only */
     case OR_RGBA: case OR_BGRA: case OR_ARGB: return 4;
-    default: return -1; /* CL_RGB is only legal with packed types: out of scope */
+    default: return -1; /* CL_Rx, CL_RGx: not supported (reading A37) */
   }
 }
 
-/* The [CL1.2 §5.3.1.1] table of legal (order, type) pairs, minus packed types. */
+/* The [CL1.2 §5.3.1.1] table of legal (order, type) pairs. */
 static int format_ok(uint32_t order, uint32_t type) {
-  if (type_bytes(type) < 0 || oracle_channels(order) < 0) return 0;
+  if (oracle_channels(order) < 0) return 0;
+  /* "CL_RGB or CL_RGBx: only if the channel data type is CL_UNORM_SHORT_565,
+     CL_UNORM_SHORT_555 or CL_UNORM_INT_101010" -- and those types need them */
+  if (order == OR_RGB || order == OR_RGBx || is_packed(type))
+    return (order == OR_RGB || order == OR_RGBx) && is_packed(type);
+  if (type_bytes(type) < 0) return 0;
   if (order == OR_BGRA || order == OR_ARGB)
     return type == OR_UNORM_INT8 || type == OR_SNORM_INT8 || type == OR_SIGNED_INT8 ||
            type == OR_UNSIGNED_INT8;
@@ -63,6 +88,7 @@ static int format_ok(uint32_t order, uint32_t type) {
 
 int oracle_elem_size(uint32_t order, uint32_t type) {
   if (!format_ok(order, type)) return -1;
+  if (is_packed(type)) return type == OR_UNORM_INT_101010 ? 4 : 2;  /* one packed word */
   return oracle_channels(order) * type_bytes(type); /* elem_size, Fig. 6 */
 }
 
@@ -187,13 +213,16 @@ static void map_to_xyzw(uint32_t order, const val32* mem, val32 zero, val32 one,
     case OR_ARGB:      out[0] = mem[1]; out[1] = mem[2]; out[2] = mem[3]; out[3] = mem[0]; break;
     case OR_INTENSITY: out[0] = mem[0]; out[1] = mem[0]; out[2] = mem[0]; out[3] = mem[0]; break;
     case OR_LUMINANCE: out[0] = mem[0]; out[1] = mem[0]; out[2] = mem[0]; out[3] = one;    break;
+    case OR_RGB:       out[0] = mem[0]; out[1] = mem[1]; out[2] = mem[2]; out[3] = one;    break;
+    case OR_RGBx:      out[0] = mem[0]; out[1] = mem[1]; out[2] = mem[2]; out[3] = one;    break;
     default:           out[0] = zero;   out[1] = zero;   out[2] = zero;   out[3] = zero;   break;
   }
 }
 
 /* Border colour of CLK_ADDRESS_CLAMP ([CL1.2 §6.12.14.1]; reading A4 extends
- * it to CLK_ADDRESS_NONE out of range): (0,0,0,0) for A, INTENSITY, RA, ARGB,
- * BGRA, RGBA; (0,0,0,1) for R, RG, RGB, LUMINANCE. */
+ * it to CLK_ADDRESS_NONE out of range): (0,0,0,0) for A, INTENSITY, Rx, RA,
+ * RGx, RGBx, ARGB, BGRA, RGBA; (0,0,0,1) for R, RG, RGB, LUMINANCE.  (So for
+ * CL_RGBx the border's alpha 0 differs from an in-range texel's alpha 1.) */
 static void border_color(uint32_t order, val32 zero, val32 one, val32* out) {
   out[0] = zero; out[1] = zero; out[2] = zero;
   out[3] = (order == OR_R || order == OR_RG || order == OR_RGB || order == OR_LUMINANCE)
@@ -212,9 +241,24 @@ static void fetch(const oracle_image* img, int64_t i, int64_t j, int64_t k, int 
   }
   int nc = oracle_channels(img->order);
   int tb = type_bytes(img->type);
+  int es = oracle_elem_size(img->order, img->type);
   const uint8_t* p = img->data + k * img->slice_pitch + j * img->row_pitch +
-                     i * (int64_t)(nc * tb);                  /* P:403-404, P:428 */
+                     i * (int64_t)es;                         /* P:403-404, P:428 */
   val32 mem[4];
+  if (is_packed(img->type)) {
+    /* the word, little endian; each field c / (2^bits - 1) ([CL1.2 §8.3.1.1],
+       correctly rounded as for the other normalized types, reading A11) */
+    uint32_t word = 0;
+    for (int b = 0; b < es; ++b) word |= (uint32_t)p[b] << (8 * b);
+    for (int c = 0; c < 3; ++c) {
+      int bits, shift;
+      packed_field(img->type, c, &bits, &shift);
+      uint32_t code = (word >> shift) & ((1u << bits) - 1u);
+      mem[c].f = (float)code / (float)((1u << bits) - 1u);
+    }
+    map_to_xyzw(img->order, mem, zero, one, out);
+    return;
+  }
   for (int c = 0; c < nc; ++c) {
     int64_t code = load_code(p + c * tb, img->type);
     switch (img->type) {
@@ -526,6 +570,20 @@ int oracle_convert_texel(uint32_t order, uint32_t type, int rtype, const void* c
     case OR_BGRA: slot[0] = 2; slot[1] = 1; slot[2] = 0; slot[3] = 3; break;
     case OR_ARGB: slot[0] = 3; slot[1] = 0; slot[2] = 1; slot[3] = 2; break;
     default: break;
+  }
+  if (is_packed(type)) {
+    /* R, G, B = convert_sat_rte(x, y, z times 2^bits - 1), the product one fp32
+       RN op (reading A12); the unused x bits are written 0 (reading A38) */
+    uint32_t word = 0;
+    for (int c = 0; c < 3; ++c) {
+      int bits, shift;
+      packed_field(type, c, &bits, &shift);
+      int32_t hi = (int32_t)((1u << bits) - 1u);
+      word |= (uint32_t)sat_rte(col[c].f * (float)hi, 0, hi) << shift;
+    }
+    int es = oracle_elem_size(order, type);
+    for (int b = 0; b < es; ++b) texel_out[b] = (uint8_t)(word >> (8 * b));
+    return OR_SUCCESS;
   }
   int nc = oracle_channels(order), tb = type_bytes(type);
   for (int c = 0; c < nc; ++c) {

@@ -45,11 +45,17 @@ extern "C" {
 #define OR_ARGB       0x10B7
 #define OR_INTENSITY  0x10B8
 #define OR_LUMINANCE  0x10B9
+#define OR_Rx         0x10BA   /* not supported (reading A37) */
+#define OR_RGx        0x10BB   /* not supported (reading A37) */
+#define OR_RGBx       0x10BC
 
 #define OR_SNORM_INT8      0x10D0
 #define OR_SNORM_INT16     0x10D1
 #define OR_UNORM_INT8      0x10D2
 #define OR_UNORM_INT16     0x10D3
+#define OR_UNORM_SHORT_565  0x10D4  /* packed: R 15:11, G 10:5, B 4:0 (CL_RGB / CL_RGBx) */
+#define OR_UNORM_SHORT_555  0x10D5  /* packed: x 15, R 14:10, G 9:5, B 4:0 */
+#define OR_UNORM_INT_101010 0x10D6  /* packed: x 31:30, R 29:20, G 19:10, B 9:0 */
 #define OR_SIGNED_INT8     0x10D7
 #define OR_SIGNED_INT16    0x10D8
 #define OR_SIGNED_INT32    0x10D9

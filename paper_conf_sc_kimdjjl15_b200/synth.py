@@ -18,11 +18,12 @@ SEED = 20151115
 
 # Khronos values (public cl.h); the product binding has its own copy.
 _CHANNELS = {0x10B0: 1, 0x10B1: 1, 0x10B2: 2, 0x10B3: 2, 0x10B5: 4, 0x10B6: 4, 0x10B7: 4,
-             0x10B8: 1, 0x10B9: 1}
+             0x10B8: 1, 0x10B9: 1, 0x10B4: 1, 0x10BC: 1}  # CL_RGB / CL_RGBx: one packed word
 _TYPE_DTYPE = {0x10D0: np.int8, 0x10D1: np.int16, 0x10D2: np.uint8, 0x10D3: np.uint16,
                0x10D7: np.int8, 0x10D8: np.int16, 0x10D9: np.int32,
                0x10DA: np.uint8, 0x10DB: np.uint16, 0x10DC: np.uint32,
-               0x10DD: np.float16, 0x10DE: np.float32}
+               0x10DD: np.float16, 0x10DE: np.float32,
+               0x10D4: np.uint16, 0x10D5: np.uint16, 0x10D6: np.uint32}  # packed words
 
 
 def rng(offset: int = 0) -> np.random.Generator:
