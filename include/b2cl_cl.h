@@ -229,11 +229,17 @@ typedef struct _cl_image_desc {
 #define CL_ARGB 0x10B7
 #define CL_INTENSITY 0x10B8
 #define CL_LUMINANCE 0x10B9
+#define CL_Rx 0x10BA
+#define CL_RGx 0x10BB
+#define CL_RGBx 0x10BC
 
 #define CL_SNORM_INT8 0x10D0
 #define CL_SNORM_INT16 0x10D1
 #define CL_UNORM_INT8 0x10D2
 #define CL_UNORM_INT16 0x10D3
+#define CL_UNORM_SHORT_565 0x10D4
+#define CL_UNORM_SHORT_555 0x10D5
+#define CL_UNORM_INT_101010 0x10D6
 #define CL_SIGNED_INT8 0x10D7
 #define CL_SIGNED_INT16 0x10D8
 #define CL_SIGNED_INT32 0x10D9

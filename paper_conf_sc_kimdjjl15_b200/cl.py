@@ -34,6 +34,8 @@ CL_SNORM_INT8, CL_SNORM_INT16, CL_UNORM_INT8, CL_UNORM_INT16 = 0x10D0, 0x10D1, 0
 CL_SIGNED_INT8, CL_SIGNED_INT16, CL_SIGNED_INT32 = 0x10D7, 0x10D8, 0x10D9
 CL_UNSIGNED_INT8, CL_UNSIGNED_INT16, CL_UNSIGNED_INT32 = 0x10DA, 0x10DB, 0x10DC
 CL_HALF_FLOAT, CL_FLOAT = 0x10DD, 0x10DE
+CL_Rx, CL_RGx, CL_RGBx = 0x10BA, 0x10BB, 0x10BC
+CL_UNORM_SHORT_565, CL_UNORM_SHORT_555, CL_UNORM_INT_101010 = 0x10D4, 0x10D5, 0x10D6
 CL_ADDRESS_NONE, CL_ADDRESS_CLAMP_TO_EDGE, CL_ADDRESS_CLAMP, CL_ADDRESS_REPEAT, \
     CL_ADDRESS_MIRRORED_REPEAT = range(0x1130, 0x1135)
 CL_FILTER_NEAREST, CL_FILTER_LINEAR = 0x1140, 0x1141

@@ -15,10 +15,13 @@ namespace dev {
 // ---- internal format codes (host maps the Khronos enums onto these) ----
 enum TypeCode : int {
   T_SNORM8 = 0, T_SNORM16, T_UNORM8, T_UNORM16, T_SINT8, T_SINT16, T_SINT32,
-  T_UINT8, T_UINT16, T_UINT32, T_HALF, T_FLOAT, T_COUNT
+  T_UINT8, T_UINT16, T_UINT32, T_HALF, T_FLOAT,
+  // packed normalized RGB words ([CL1.2 §5.3.1.1]), orders O_RGB / O_RGBX only
+  T_U565, T_U555, T_U101010, T_COUNT
 };
 enum OrderCode : int {
-  O_R = 0, O_A, O_RG, O_RA, O_RGBA, O_BGRA, O_ARGB, O_INTENSITY, O_LUMINANCE, O_COUNT
+  O_R = 0, O_A, O_RG, O_RA, O_RGBA, O_BGRA, O_ARGB, O_INTENSITY, O_LUMINANCE, O_RGB, O_RGBX,
+  O_COUNT
 };
 enum AddrCode : int { A_NONE = 0, A_CTE, A_CLAMP, A_REPEAT, A_MIRROR };
 enum FiltCode : int { F_NEAREST = 0, F_LINEAR = 1 };
@@ -42,15 +45,22 @@ struct Sampler {
   int norm, addr, filt;
 };
 
+B2CL_HD constexpr bool is_packed(int t) { return t == T_U565 || t == T_U555 || t == T_U101010; }
+// bytes of one channel (a packed type: of the whole word)
 B2CL_HD constexpr int type_bytes(int t) {
-  return (t == T_SNORM8 || t == T_UNORM8 || t == T_SINT8 || t == T_UINT8) ? 1
-         : (t == T_SINT32 || t == T_UINT32 || t == T_FLOAT)               ? 4
-                                                                          : 2;
+  return (t == T_SNORM8 || t == T_UNORM8 || t == T_SINT8 || t == T_UINT8)   ? 1
+         : (t == T_SINT32 || t == T_UINT32 || t == T_FLOAT || t == T_U101010) ? 4
+                                                                              : 2;
 }
 B2CL_HD constexpr int order_channels(int o) {
   return (o == O_R || o == O_A || o == O_INTENSITY || o == O_LUMINANCE) ? 1
          : (o == O_RG || o == O_RA)                                   ? 2
+         : (o == O_RGB || o == O_RGBX)                                ? 3
                                                                       : 4;
+}
+// element size (CLImage.elem_size, Fig. 6): channels x channel bytes, or the packed word
+B2CL_HD constexpr int texel_bytes(int t, int o) {
+  return is_packed(t) ? type_bytes(t) : order_channels(o) * type_bytes(t);
 }
 B2CL_HD constexpr int ret_class(int t) {
   return (t == T_SINT8 || t == T_SINT16 || t == T_SINT32)    ? R_I

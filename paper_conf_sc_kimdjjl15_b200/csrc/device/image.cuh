@@ -163,7 +163,28 @@ __device__ __forceinline__ float code_to_float(uint32_t v, int type) {
   }
 }
 
+// Packed word ([CL1.2 §5.3.1.1]: 565 = R 15:11, G 10:5, B 4:0; 555 = x 15,
+// R 14:10, G 9:5, B 4:0; 101010 = x 31:30, R 29:20, G 19:10, B 9:0) ->
+// R, G, B as floats c / (2^bits - 1), correctly rounded (reading A11)
+__device__ __forceinline__ void unpack_rgb(uint32_t w, int type, uint32_t m[3]) {
+  uint32_t c[3];
+  float d[3];
+  if (type == T_U565) {
+    c[0] = (w >> 11) & 31u; c[1] = (w >> 5) & 63u; c[2] = w & 31u;
+    d[0] = 31.0f; d[1] = 63.0f; d[2] = 31.0f;
+  } else if (type == T_U555) {
+    c[0] = (w >> 10) & 31u; c[1] = (w >> 5) & 31u; c[2] = w & 31u;
+    d[0] = d[1] = d[2] = 31.0f;
+  } else {
+    c[0] = (w >> 20) & 1023u; c[1] = (w >> 10) & 1023u; c[2] = w & 1023u;
+    d[0] = d[1] = d[2] = 1023.0f;
+  }
+#pragma unroll
+  for (int k = 0; k < 3; ++k) m[k] = __float_as_uint(__fdiv_rn(__uint2float_rn(c[k]), d[k]));
+}
+
 // memory-order channel slots -> (x,y,z,w); one = 1.0f bits or integer 1
+// (CL_RGBx: the fetch supplies slot 3 -- 1 in range, 0 for the border)
 __device__ __forceinline__ void map_order(int order, const uint32_t m[4], uint32_t one,
                                           uint32_t out[4]) {
   switch (order) {
@@ -175,6 +196,7 @@ __device__ __forceinline__ void map_order(int order, const uint32_t m[4], uint32
     case O_ARGB: out[0] = m[1]; out[1] = m[2]; out[2] = m[3]; out[3] = m[0]; break;
     case O_INTENSITY: out[0] = m[0]; out[1] = m[0]; out[2] = m[0]; out[3] = m[0]; break;
     case O_LUMINANCE: out[0] = m[0]; out[1] = m[0]; out[2] = m[0]; out[3] = one; break;
+    case O_RGB: out[0] = m[0]; out[1] = m[1]; out[2] = m[2]; out[3] = one; break;
     default: out[0] = m[0]; out[1] = m[1]; out[2] = m[2]; out[3] = m[3]; break;
   }
 }
@@ -183,26 +205,6 @@ __device__ __forceinline__ void map_order(int order, const uint32_t m[4], uint32
 __device__ __forceinline__ const char* texel_ptr(const Image& im, int i, int j, int k) {
   return im.ptr + (uint64_t)(unsigned)k * im.sp + (uint64_t)(unsigned)j * im.rp +
          (uint64_t)(unsigned)i * (unsigned)im.es;
-}
-
-// Memory-order channel values of texel (i,j,k) for return class F (converted
-// floats as bits) or I/UI (extended codes); all zero when out of range.
-template <int TYPE, int NCH>
-__device__ __forceinline__ void fetch_mem(const Image& im, int i, int j, int k, bool ok,
-                                          int rclass, uint32_t m[4]) {
-  const int type = TYPE == RT ? im.type : TYPE;
-  const int nch = NCH == RT ? im.nch : NCH;
-  const int es = (TYPE == RT || NCH == RT) ? im.es : NCH * type_bytes(TYPE);
-  m[0] = m[1] = m[2] = m[3] = 0u;
-  if (!ok) return;
-  Raw r = load_raw(texel_ptr(im, i, j, k), es);
-#pragma unroll
-  for (int c = 0; c < 4; ++c) {
-    if (c < nch) {
-      uint32_t v = channel_code(r, c, type);
-      m[c] = rclass == R_F ? __float_as_uint(code_to_float(v, type)) : v;
-    }
-  }
 }
 
 // ------------------------------------------------------------------------
@@ -228,8 +230,26 @@ __device__ __forceinline__ uint32_t int_to_code(uint32_t v, int type) {
   }
 }
 
+// (x,y,z,w) color -> packed word: convert_sat_rte(component * (2^bits - 1))
+// (reading A12); the unused x bits are written 0 (reading A38)
+__device__ __forceinline__ uint32_t pack_rgb(const uint32_t col[4], int type) {
+  const float f[3] = {__uint_as_float(col[0]), __uint_as_float(col[1]), __uint_as_float(col[2])};
+  auto q = [](float v, int hi) {
+    return (uint32_t)min(max(__float2int_rn(__fmul_rn(v, (float)hi)), 0), hi);
+  };
+  if (type == T_U565) return (q(f[0], 31) << 11) | (q(f[1], 63) << 5) | q(f[2], 31);
+  if (type == T_U555) return (q(f[0], 31) << 10) | (q(f[1], 31) << 5) | q(f[2], 31);
+  return (q(f[0], 1023) << 20) | (q(f[1], 1023) << 10) | q(f[2], 1023);
+}
+
 // (x,y,z,w) color -> stored texel bytes in 4 words (little endian)
 __device__ __forceinline__ Raw encode_texel(const uint32_t col[4], int type, int order) {
+  if (is_packed(type)) {
+    Raw r;
+    r.w[0] = pack_rgb(col, type);
+    r.w[1] = r.w[2] = r.w[3] = 0u;
+    return r;
+  }
   int slot[4] = {0, 1, 2, 3};
   if (order == O_A) slot[0] = 3;
   else if (order == O_RA) slot[1] = 3;

@@ -113,7 +113,8 @@ __device__ __forceinline__ const char* row_ptr(const Image& im, int j, int k) {
 // NaN weight through the blend by themselves.
 __device__ __forceinline__ bool const_in_output(int order, int outc) {
   switch (order) {
-    case O_RGBA: case O_BGRA: case O_ARGB: case O_INTENSITY: return false;
+    case O_RGBA: case O_BGRA: case O_ARGB: case O_INTENSITY: case O_RGBX: return false;
+    case O_RGB: return outc > 3;
     case O_R: return outc > 1;
     case O_RG: case O_RA: return outc > 1 + (order == O_RG);
     case O_LUMINANCE: return outc > 3;
@@ -123,7 +124,7 @@ __device__ __forceinline__ bool const_in_output(int order, int outc) {
 
 template <class C>
 __device__ __forceinline__ int elem_size(const Image& im) {
-  return (C::type == RT || C::nch == RT) ? im.es : C::nch * type_bytes(C::type);
+  return (C::type == RT || C::nch == RT) ? im.es : texel_bytes(C::type, C::order);
 }
 
 // memory-order channels of the texel at row + i*elem_size (zero if !ok)
@@ -136,6 +137,13 @@ __device__ __forceinline__ void fetch(const Image& im, const char* row, int i, b
   m[0] = m[1] = m[2] = m[3] = 0u;
   if (!ok) return;
   Raw r = load_raw(row + (uint64_t)(unsigned)i * (unsigned)es, es);
+  if (is_packed(type)) {  // normalized only (read_imagef)
+    unpack_rgb(r.w[0], type, m);
+    // CL_RGBx: the in-range alpha 1 is carried as a channel, so that a border
+    // tap (alpha 0, [CL1.2 §6.12.14.1]) blends into it
+    if ((C::order == RT ? im.order : C::order) == O_RGBX) m[3] = 0x3f800000u;
+    return;
+  }
 #pragma unroll
   for (int c = 0; c < 4; ++c) {
     if (c < nch) {
@@ -164,7 +172,8 @@ __device__ __forceinline__ void linear_at(const P& p, const char* const rows[4],
                                           float g, float omg, uint32_t res[4], int outc = 4) {
   constexpr int NR = C::dims == 1 ? 1 : (C::dims == 2 ? 2 : 4);
   const int order = C::order == RT ? p.im.order : C::order;
-  const int nch = C::nch == RT ? p.im.nch : C::nch;
+  // channels blended: the stored ones (CL_RGBx: also its alpha, see fetch)
+  const int nch = order == O_RGBX ? 4 : (C::nch == RT ? p.im.nch : C::nch);
   uint32_t t0[NR][4], t1[NR][4];
 #pragma unroll
   for (int r = 0; r < NR; ++r) {

@@ -717,7 +717,7 @@ extern "C" cl_int clGetSupportedImageFormats(cl_context c, cl_mem_flags flags,
   if (type < CL_MEM_OBJECT_IMAGE2D || type > CL_MEM_OBJECT_IMAGE1D_BUFFER) return CL_INVALID_VALUE;
   if (num_entries == 0 && formats) return CL_INVALID_VALUE;
   std::vector<cl_image_format> all;
-  for (cl_channel_order o = CL_R; o <= CL_LUMINANCE; ++o)
+  for (cl_channel_order o = CL_R; o <= CL_RGBx; ++o)
     for (cl_channel_type t = CL_SNORM_INT8; t <= CL_FLOAT; ++t) {
       cl_image_format f{o, t};
       FormatInfo fi;

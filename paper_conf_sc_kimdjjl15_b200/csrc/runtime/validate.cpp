@@ -26,6 +26,9 @@ int type_code(cl_channel_type t) {
     case CL_UNSIGNED_INT32: return dev::T_UINT32;
     case CL_HALF_FLOAT: return dev::T_HALF;
     case CL_FLOAT: return dev::T_FLOAT;
+    case CL_UNORM_SHORT_565: return dev::T_U565;
+    case CL_UNORM_SHORT_555: return dev::T_U555;
+    case CL_UNORM_INT_101010: return dev::T_U101010;
     default: return -1;
   }
 }
@@ -41,19 +44,25 @@ int order_code(cl_channel_order o) {
     case CL_ARGB: return dev::O_ARGB;
     case CL_INTENSITY: return dev::O_INTENSITY;
     case CL_LUMINANCE: return dev::O_LUMINANCE;
-    default: return -1;
+    case CL_RGB: return dev::O_RGB;
+    case CL_RGBx: return dev::O_RGBX;
+    default: return -1;  // CL_Rx, CL_RGx: not supported (reading A37)
   }
 }
 
 static bool known_type(cl_channel_type t) { return t >= 0x10D0 && t <= 0x10DE; }
-static bool known_order(cl_channel_order o) { return o >= 0x10B0 && o <= 0x10B9; }
+static bool known_order(cl_channel_order o) { return o >= 0x10B0 && o <= 0x10BC; }
 
 cl_int format_info(const cl_image_format* f, FormatInfo* out) {
   if (!f || !known_type(f->image_channel_data_type) || !known_order(f->image_channel_order))
     return CL_INVALID_IMAGE_FORMAT_DESCRIPTOR;
   const int t = type_code(f->image_channel_data_type);
   const int o = order_code(f->image_channel_order);
-  if (t < 0 || o < 0) return CL_IMAGE_FORMAT_NOT_SUPPORTED;  // packed types, CL_RGB
+  if (t < 0 || o < 0) return CL_IMAGE_FORMAT_NOT_SUPPORTED;  // CL_Rx, CL_RGx (A37)
+  // "CL_RGB or CL_RGBx: only if the channel data type is CL_UNORM_SHORT_565,
+  // CL_UNORM_SHORT_555 or CL_UNORM_INT_101010" -- and those types need them
+  const bool rgb = o == dev::O_RGB || o == dev::O_RGBX;
+  if (rgb != dev::is_packed(t)) return CL_IMAGE_FORMAT_NOT_SUPPORTED;
   // [CL1.2 §5.3.1.1]: BGRA/ARGB only with 8-bit channels; INTENSITY and
   // LUMINANCE only with UNORM/SNORM 8/16, HALF and FLOAT.
   if (o == dev::O_BGRA || o == dev::O_ARGB) {
@@ -68,7 +77,7 @@ cl_int format_info(const cl_image_format* f, FormatInfo* out) {
   out->type = t;
   out->order = o;
   out->nch = dev::order_channels(o);
-  out->es = (size_t)out->nch * dev::type_bytes(t);
+  out->es = (size_t)dev::texel_bytes(t, o);
   out->rclass = dev::ret_class(t);
   return CL_SUCCESS;
 }

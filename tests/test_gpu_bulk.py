@@ -150,7 +150,8 @@ def test_fill_buffer_on_unaligned_device_pointer(sess, orc):
 
 IMG_FORMATS = [(cl.CL_RGBA, cl.CL_UNORM_INT8), (cl.CL_RGBA, cl.CL_FLOAT), (cl.CL_R, cl.CL_HALF_FLOAT),
                (cl.CL_RG, cl.CL_SIGNED_INT16), (cl.CL_BGRA, cl.CL_UNORM_INT8), (cl.CL_R, cl.CL_UNSIGNED_INT8),
-               (cl.CL_RGBA, cl.CL_UNSIGNED_INT32)]
+               (cl.CL_RGBA, cl.CL_UNSIGNED_INT32), (cl.CL_RGB, cl.CL_UNORM_SHORT_565),
+               (cl.CL_RGBx, cl.CL_UNORM_INT_101010)]
 
 
 def _img_pair(S, orc, order, type_, W, H, D, dims, seed):

@@ -21,7 +21,10 @@ F32, F16, U8N, U16N, S8N, S16N = (cl.CL_FLOAT, cl.CL_HALF_FLOAT, cl.CL_UNORM_INT
 
 FLOAT_FORMATS = [(RGBA, F32), (R, F32), (RGBA, U8N), (BGRA, U8N), (RG, F16), (RGBA, U16N),
                  (R, S8N), (RA, S16N), (A_, U8N), (INT_, U8N), (LUM, F32), (ARGB, U8N),
-                 (RGBA, F16), (RG, U8N)]
+                 (RGBA, F16), (RG, U8N),
+                 # packed formats (NEXT row 4); CL_RGBx: border alpha 0 vs texel alpha 1
+                 (cl.CL_RGB, cl.CL_UNORM_SHORT_565), (cl.CL_RGBx, cl.CL_UNORM_SHORT_555),
+                 (cl.CL_RGBx, cl.CL_UNORM_INT_101010), (cl.CL_RGB, cl.CL_UNORM_INT_101010)]
 INT_FORMATS = [(RGBA, cl.CL_UNSIGNED_INT8), (R, cl.CL_SIGNED_INT16), (RG, cl.CL_UNSIGNED_INT32),
                (RGBA, cl.CL_SIGNED_INT32), (BGRA, cl.CL_SIGNED_INT8), (RA, cl.CL_UNSIGNED_INT16)]
 SHAPES = [(1, (37, 1, 1)), (2, (1, 1, 1)), (2, (3, 5, 1)), (2, (65, 33, 1)), (3, (7, 3, 2)),
@@ -127,6 +130,29 @@ def test_unorm_codes_exhaustive(sess, orc):
         sess.release(img)
 
 
+@pytest.mark.parametrize("order", [cl.CL_RGB, cl.CL_RGBx])
+def test_packed_words_exhaustive(sess, orc, order):
+    """Every 565 / 555 word and 2^16 random 101010 words through read_imagef
+    (NEXT row 4): bit-exact to the oracle, whose fields are pinned to numpy."""
+    g = synth.rng(13)
+    for type_ in (cl.CL_UNORM_SHORT_565, cl.CL_UNORM_SHORT_555, cl.CL_UNORM_INT_101010):
+        if type_ == cl.CL_UNORM_INT_101010:
+            words = g.integers(0, 1 << 32, 1 << 16, dtype=np.uint64).astype(np.uint32)
+        else:
+            words = np.arange(1 << 16, dtype=np.uint16)
+        W, Hh = 256, words.size // 256
+        img = sess.image(order, type_, W, Hh, host=words.reshape(Hh, W, 1))
+        oimg = orc.Image(words.reshape(1, Hh, W, 1).copy(), W, Hh, 1, dims=2, order=order, type=type_)
+        smp = sess.sampler(False, cl.CL_ADDRESS_NONE, cl.CL_FILTER_NEAREST)
+        xs, ys = np.meshgrid(np.arange(W) + 0.5, np.arange(Hh) + 0.5)
+        co = np.stack([xs.ravel(), ys.ravel()], 1).astype(np.float32)
+        got = gpu_read_samples(sess, img, smp, cl.B2CL_RTYPE_FLOAT, co)
+        exp = orc.read_samples(oimg, False, cl.CL_ADDRESS_NONE, cl.CL_FILTER_NEAREST, orc.RT_F, co)
+        assert_parity(got, exp, False, f"packed {hex(order)}/{hex(type_)}")
+        cl.lib().clReleaseSampler(smp)
+        sess.release(img)
+
+
 # ---------------------------------------------------------------- grid mode
 GRID_CASES = [
     # (dims, order, type, img size, sampler, affine-maker, out dims, outc)
@@ -139,6 +165,8 @@ GRID_CASES = [
     (3, RGBA, F16, (12, 10, 9), (1, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR), "rotate3d", (17, 13, 11), 4),
     (2, RGBA, U8N, (64, 64, 1), (0, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_NEAREST), "rotate", (70, 66, 1), 4),
     (2, RG, F32, (33, 21, 1), (1, cl.CL_ADDRESS_NONE, cl.CL_FILTER_LINEAR), "translate", (40, 30, 3), 2),
+    (2, cl.CL_RGBx, cl.CL_UNORM_SHORT_565, (33, 21, 1), (1, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_LINEAR), "rotate", (40, 30, 1), 4),
+    (3, cl.CL_RGB, cl.CL_UNORM_INT_101010, (9, 6, 5), (1, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR), "rotate3d", (11, 7, 6), 4),
     # staged-footprint kernel: separable, non-wrapping, LINEAR (borders, scale != 1)
     (3, R, F32, (30, 20, 12), (1, cl.CL_ADDRESS_CLAMP, cl.CL_FILTER_LINEAR), "stencil", (30, 20, 12), 1),
     (3, R, F32, (30, 20, 12), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "scale2", (33, 21, 9), 1),
@@ -265,6 +293,9 @@ WRITE_FORMATS = [(RGBA, U8N, cl.B2CL_RTYPE_FLOAT), (BGRA, U8N, cl.B2CL_RTYPE_FLO
                  (RGBA, F32, cl.B2CL_RTYPE_FLOAT), (A_, U8N, cl.B2CL_RTYPE_FLOAT),
                  (ARGB, U8N, cl.B2CL_RTYPE_FLOAT), (RA, F16, cl.B2CL_RTYPE_FLOAT),
                  (INT_, F32, cl.B2CL_RTYPE_FLOAT), (LUM, U8N, cl.B2CL_RTYPE_FLOAT),
+                 (cl.CL_RGB, cl.CL_UNORM_SHORT_565, cl.B2CL_RTYPE_FLOAT),
+                 (cl.CL_RGBx, cl.CL_UNORM_SHORT_555, cl.B2CL_RTYPE_FLOAT),
+                 (cl.CL_RGB, cl.CL_UNORM_INT_101010, cl.B2CL_RTYPE_FLOAT),
                  (RGBA, cl.CL_SIGNED_INT8, cl.B2CL_RTYPE_INT), (RG, cl.CL_SIGNED_INT16, cl.B2CL_RTYPE_INT),
                  (R, cl.CL_SIGNED_INT32, cl.B2CL_RTYPE_INT), (RGBA, cl.CL_UNSIGNED_INT8, cl.B2CL_RTYPE_UINT),
                  (RA, cl.CL_UNSIGNED_INT16, cl.B2CL_RTYPE_UINT), (R, cl.CL_UNSIGNED_INT32, cl.B2CL_RTYPE_UINT)]
@@ -308,3 +339,19 @@ def test_write_image(sess, orc, order, type_, rt, dims):
     got = sess.read_image(img, (0, 0, 0), (W, H, D))
     assert np.array_equal(got, oimg.data[:got.size]), f"write {hex(order)}/{hex(type_)}"
     sess.release(img, cbuf, kbuf)
+
+
+def test_supported_formats_match_the_legal_table(sess, orc):
+    """clGetSupportedImageFormats lists exactly the (order, type) pairs the oracle
+    accepts ([CL1.2 §5.3.1.1], packed formats included; CL_Rx / CL_RGx not, A37)."""
+    import ctypes
+    L = cl.lib()
+    n = ctypes.c_uint32()
+    cl.check(L.clGetSupportedImageFormats(sess.ctx, 0, 0x10F1, 0, None, ctypes.byref(n)))
+    fmts = (ctypes.c_uint32 * (2 * n.value))()
+    cl.check(L.clGetSupportedImageFormats(sess.ctx, 0, 0x10F1, n.value, fmts, None))
+    got = {(fmts[2 * i], fmts[2 * i + 1]) for i in range(n.value)}
+    exp = {(o, t) for o in range(0x10B0, 0x10BD) for t in range(0x10D0, 0x10DF)
+           if orc.elem_size(o, t) > 0}
+    assert got == exp
+    assert (cl.CL_RGBx, cl.CL_UNORM_INT_101010) in got and (cl.CL_RGB, cl.CL_UNORM_SHORT_565) in got
