@@ -87,6 +87,8 @@ def lib():
                                        i64, i64, i64, i64, P, i32]
         L.oracle_write_samples.argtypes = [P, i32, P, i64, P, i64]
         L.oracle_convert_texel.argtypes = [u32, u32, i32, P, P]
+        L.oracle_tex_fetch.argtypes = [P, P, P, P]
+        L.oracle_tex1Dfetch.argtypes = [P, u32, ctypes.c_int32, P]
         L.oracle_copy_rect.argtypes = [P, P, sz3, sz3, sz3, ctypes.c_size_t, ctypes.c_size_t,
                                        ctypes.c_size_t, ctypes.c_size_t]
         L.oracle_copy_rect.restype = None
@@ -212,6 +214,44 @@ def convert_texel(order: int, type: int, rtype: int, color) -> bytes:
     out = np.zeros(16, dtype=np.uint8)
     _check(lib().oracle_convert_texel(order, type, rtype, _ptr(col), _ptr(out)))
     return out[:elem_size(order, type)].tobytes()
+
+
+# ---- CUDA texture fetches (oracle.h: NEXT row 3) ----
+TEX_WRAP, TEX_CLAMP, TEX_MIRROR, TEX_BORDER = 0, 1, 2, 3
+TEX_POINT, TEX_LINEAR = 0, 1
+TEX_ELEMENT, TEX_NORMALIZED = 0, 1
+
+
+class _TexDesc(ctypes.Structure):
+    _fields_ = [("address_mode", ctypes.c_uint32 * 3), ("filter_mode", ctypes.c_uint32),
+                ("read_mode", ctypes.c_uint32), ("normalized_coords", ctypes.c_int32)]
+
+
+def tex_fetch(img: Image, address_modes, filter_mode: int, read_mode: int, normalized: bool,
+              coords: np.ndarray) -> np.ndarray:
+    """tex1D/2D/3D (tex*Layered when img.arrayed: the last coordinate is the layer)
+    at each row of coords; returns (n, 4) uint32 bit patterns."""
+    am = list(address_modes) + [0] * (3 - len(address_modes))
+    td = _TexDesc((ctypes.c_uint32 * 3)(*am[:3]), filter_mode, read_mode, int(normalized))
+    coords = np.ascontiguousarray(coords, dtype=np.float32)
+    n = coords.shape[0]
+    out = np.zeros((n, 4), np.uint32)
+    s = img.cstruct()
+    for k in range(n):
+        _check(lib().oracle_tex_fetch(ctypes.byref(s), ctypes.byref(td),
+                                      ctypes.c_void_p(coords[k].ctypes.data),
+                                      ctypes.c_void_p(out[k].ctypes.data)))
+    return out
+
+
+def tex1Dfetch(img: Image, read_mode: int, xs) -> np.ndarray:
+    xs = np.asarray(xs, np.int32)
+    out = np.zeros((xs.size, 4), np.uint32)
+    s = img.cstruct()
+    for k in range(xs.size):
+        _check(lib().oracle_tex1Dfetch(ctypes.byref(s), read_mode, int(xs[k]),
+                                       ctypes.c_void_p(out[k].ctypes.data)))
+    return out
 
 
 def copy_rect(src: np.ndarray, dst: np.ndarray, src_origin, dst_origin, region,

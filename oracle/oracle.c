@@ -547,6 +547,185 @@ int oracle_read_grid(const oracle_image* img, int normalized, uint32_t addressin
 }
 
 /* ------------------------------------------------------------------ */
+/* CUDA texture fetches ([CUDA-PG TF]: the CUDA C Programming Guide,     */
+/* appendix "Texture Fetching"; the source side of P:449)               */
+/* ------------------------------------------------------------------ */
+
+enum { TEX_WRAP = 0, TEX_CLAMP = 1, TEX_MIRROR = 2, TEX_BORDER = 3 };
+enum { TEX_POINT = 0, TEX_LINEAR = 1 };
+enum { TEX_ELEMENT = 0, TEX_NORMALIZED = 1 };
+
+/* stored channel kind: 0 unsigned int, 1 signed int, 2 floating point */
+static int tex_kind(uint32_t type) {
+  switch (type) {
+    case OR_UNORM_INT8: case OR_UNORM_INT16: case OR_UNSIGNED_INT8: case OR_UNSIGNED_INT16:
+    case OR_UNSIGNED_INT32: return 0;
+    case OR_SNORM_INT8: case OR_SNORM_INT16: case OR_SIGNED_INT8: case OR_SIGNED_INT16:
+    case OR_SIGNED_INT32: return 1;
+    default: return 2;
+  }
+}
+
+/* cudaReadModeNormalizedFloat applies to 8- and 16-bit integer channels. */
+static int tex_check(const oracle_image* img, uint32_t read_mode, int filtering_linear) {
+  if (img->order != OR_R && img->order != OR_RG && img->order != OR_RGBA)
+    return OR_IMAGE_FORMAT_NOT_SUPPORTED;                    /* 1, 2 or 4 channels */
+  if (oracle_elem_size(img->order, img->type) < 0) return OR_IMAGE_FORMAT_NOT_SUPPORTED;
+  int kind = tex_kind(img->type), tb = type_bytes(img->type);
+  if (read_mode == TEX_NORMALIZED && (kind == 2 || tb == 4)) return OR_INVALID_VALUE;
+  if (read_mode != TEX_ELEMENT && read_mode != TEX_NORMALIZED) return OR_INVALID_VALUE;
+  /* "linear filtering ... only for textures configured to return floating-point data" */
+  if (filtering_linear && read_mode == TEX_ELEMENT && kind != 2) return OR_INVALID_OPERATION;
+  return OR_SUCCESS;
+}
+
+/* Texel (i,j,k) as the fetch returns it; 0 in every component when `zero`. */
+static void tex_texel(const oracle_image* img, uint32_t read_mode, int64_t i, int64_t j,
+                      int64_t k, int zero, val32* out) {
+  for (int c = 0; c < 4; ++c) out[c].u = 0;
+  if (zero) return;
+  int nc = oracle_channels(img->order), tb = type_bytes(img->type);
+  const uint8_t* p = img->data + k * img->slice_pitch + j * img->row_pitch + i * (int64_t)(nc * tb);
+  for (int c = 0; c < nc; ++c) {
+    int64_t code = load_code(p + c * tb, img->type);
+    int kind = tex_kind(img->type);
+    if (img->type == OR_FLOAT) {
+      out[c].u = (uint32_t)code;
+    } else if (img->type == OR_HALF_FLOAT) {
+      out[c].f = oracle_half_to_float((uint16_t)code);
+    } else if (read_mode == TEX_NORMALIZED) {
+      /* unsigned: c / (2^b - 1); signed: c / (2^(b-1) - 1), the most negative
+         code clamped to -1.0 (reading A42) */
+      float d = kind == 0 ? (float)((1u << (8 * tb)) - 1u) : (float)((1u << (8 * tb - 1)) - 1u);
+      float v = (float)code / d;
+      out[c].f = v < -1.0f ? -1.0f : v;
+    } else {
+      out[c].i = (int32_t)code;                              /* element type */
+    }
+  }
+}
+
+/* One axis of a point fetch: the texel index, or *out = 1 for the border. */
+static int64_t tex_axis_point(float x, int64_t n, int normalized, uint32_t mode, int* out) {
+  float fn = (float)n;
+  *out = 0;
+  if (normalized) {
+    if (mode == TEX_WRAP) x = x - floorf(x);                         /* frac(x) */
+    else if (mode == TEX_MIRROR) {
+      float f = x - floorf(x);
+      x = (fmodf(floorf(x), 2.0f) == 0.0f) ? f : 1.0f - f;           /* floor(x) even / odd */
+    }
+    x = x * fn;
+  }
+  int64_t i = ifloor(x);                                              /* i = floor(x) */
+  switch (mode) {
+    case TEX_WRAP: return ((i % n) + n) % n;   /* frac(x) * N may round to N */
+    case TEX_MIRROR: return i < n - 1 ? i : n - 1;
+    case TEX_CLAMP: return clamp64(i, 0, n - 1);
+    default:
+      if (i < 0 || i >= n) *out = 1;                                  /* border */
+      return i;
+  }
+}
+
+/* One axis of a linear fetch: taps i, i+1 of x_B = x - 0.5 and alpha = frac(x_B). */
+static void tex_axis_linear(float x, int64_t n, int normalized, uint32_t mode, int64_t* t0,
+                            int64_t* t1, int* out0, int* out1, float* alpha) {
+  float fn = (float)n;
+  if (normalized) {
+    if (mode == TEX_WRAP) x = x - floorf(x);
+    else if (mode == TEX_MIRROR) {
+      float f = x - floorf(x);
+      x = (fmodf(floorf(x), 2.0f) == 0.0f) ? f : 1.0f - f;
+    }
+    x = x * fn;
+  }
+  float xb = x - 0.5f;                                                /* x_B = x - 0.5 */
+  int64_t i = ifloor(xb);                                             /* i = floor(x_B) */
+  *alpha = xb - floorf(xb);                                           /* alpha = frac(x_B) */
+  int64_t a = i, b = i + 1;
+  *out0 = *out1 = 0;
+  switch (mode) {
+    case TEX_WRAP: a = ((a % n) + n) % n; b = ((b % n) + n) % n; break;
+    case TEX_MIRROR:                          /* the mirror repeats the edge texel */
+    case TEX_CLAMP: a = clamp64(a, 0, n - 1); b = clamp64(b, 0, n - 1); break;
+    default: *out0 = a < 0 || a >= n; *out1 = b < 0 || b >= n; break;
+  }
+  *t0 = a;
+  *t1 = b;
+}
+
+int oracle_tex_fetch(const oracle_image* img, const oracle_tex_desc* td, const float* coord,
+                     void* out16) {
+  int st = tex_check(img, td->read_mode, td->filter_mode == TEX_LINEAR);
+  if (st != OR_SUCCESS) return st;
+  int dims = img->dims;
+  for (int d = 0; d < dims; ++d) {
+    uint32_t m = td->address_mode[d];
+    if (m > TEX_BORDER) return OR_INVALID_VALUE;
+    if (!td->normalized_coords && (m == TEX_WRAP || m == TEX_MIRROR)) return OR_INVALID_VALUE;
+  }
+  int64_t n[3] = {img->width, img->height, img->depth};
+  /* tex1DLayered / tex2DLayered: the integer layer selects the array slice */
+  int64_t layer = 0;
+  if (img->arrayed) layer = clamp64((int64_t)coord[dims], 0, n[dims] - 1);
+  val32 r[4];
+  if (td->filter_mode == TEX_POINT) {
+    int64_t ix[3] = {0, 0, 0};
+    int out = 0;
+    for (int d = 0; d < dims; ++d) {
+      int o;
+      ix[d] = tex_axis_point(coord[d], n[d], td->normalized_coords, td->address_mode[d], &o);
+      out |= o;
+    }
+    if (img->arrayed) ix[dims] = layer;
+    tex_texel(img, td->read_mode, ix[0], ix[1], ix[2], out, r);
+    memcpy(out16, r, 16);
+    return OR_SUCCESS;
+  }
+  /* tex(x,y,z) = sum over the 2/4/8 taps of the weight products times T,
+     evaluated in fp64 and rounded once (reading O6); weights from the fp32
+     alpha, beta, gamma (reading A41: not the 8-bit fixed point of the
+     texture unit) */
+  int64_t lo[3] = {0, 0, 0}, hi[3] = {0, 0, 0};
+  int olo[3] = {0, 0, 0}, ohi[3] = {0, 0, 0};
+  float w[3] = {0.0f, 0.0f, 0.0f};
+  for (int d = 0; d < dims; ++d)
+    tex_axis_linear(coord[d], n[d], td->normalized_coords, td->address_mode[d], &lo[d], &hi[d],
+                    &olo[d], &ohi[d], &w[d]);
+  if (img->arrayed) lo[dims] = hi[dims] = layer;
+  double acc[4] = {0.0, 0.0, 0.0, 0.0};
+  int nk = dims > 2 ? 2 : 1, nj = dims > 1 ? 2 : 1;
+  for (int kk = 0; kk < nk; ++kk) {
+    double wk = dims > 2 ? (kk ? (double)w[2] : 1.0 - (double)w[2]) : 1.0;
+    for (int jj = 0; jj < nj; ++jj) {
+      double wj = dims > 1 ? (jj ? (double)w[1] : 1.0 - (double)w[1]) : 1.0;
+      for (int ii = 0; ii < 2; ++ii) {
+        double wi = ii ? (double)w[0] : 1.0 - (double)w[0];
+        int out = (ii ? ohi[0] : olo[0]) | (jj ? ohi[1] : olo[1]) | (kk ? ohi[2] : olo[2]);
+        val32 t[4];
+        tex_texel(img, td->read_mode, ii ? hi[0] : lo[0], jj ? hi[1] : lo[1], kk ? hi[2] : lo[2],
+                  out, t);
+        for (int ch = 0; ch < 4; ++ch) acc[ch] += wi * wj * wk * (double)t[ch].f;
+      }
+    }
+  }
+  int nc = oracle_channels(img->order);
+  for (int ch = 0; ch < 4; ++ch) r[ch].f = ch < nc ? (float)acc[ch] : 0.0f;
+  memcpy(out16, r, 16);
+  return OR_SUCCESS;
+}
+
+int oracle_tex1Dfetch(const oracle_image* img, uint32_t read_mode, int32_t x, void* out16) {
+  int st = tex_check(img, read_mode, 0);
+  if (st != OR_SUCCESS) return st;
+  val32 r[4];
+  tex_texel(img, read_mode, x, 0, 0, x < 0 || x >= img->width, r);
+  memcpy(out16, r, 16);
+  return OR_SUCCESS;
+}
+
+/* ------------------------------------------------------------------ */
 /* write_imagef / write_imagei / write_imageui ([CL1.2 §6.12.14.4])     */
 /* ------------------------------------------------------------------ */
 

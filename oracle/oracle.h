@@ -162,6 +162,33 @@ int oracle_write_samples(oracle_image* img, int rtype, const int32_t* icoords,
 int oracle_convert_texel(uint32_t order, uint32_t type, int rtype, const void* color16,
                          uint8_t* texel_out);
 
+/* ---- CUDA texture fetches (NEXT row 3: the CUDA side of the paper's
+ * CUDA-to-OpenCL texture translation) ----
+ * A CUDA texture over the texels of `img` (order R, RG or RGBA = a 1-, 2- or
+ * 4-channel CUDA array or linear memory), fetched as the CUDA C Programming
+ * Guide's "Texture Fetching" appendix defines ([CUDA-PG TF]).  img->type only
+ * says how a channel is STORED -- its bits and signedness (UNORM and
+ * UNSIGNED_INT alike are unsigned integers, SNORM and SIGNED_INT signed,
+ * HALF_FLOAT / FLOAT floating point); read_mode decides the conversion.
+ * out16: the fetched vector as float4 / int4 / uint4 bits, components beyond
+ * the channel count 0.  Returns OR_INVALID_VALUE for what CUDA does not
+ * support (wrap/mirror with unnormalized coordinates, a normalized-float read
+ * of a 32-bit or floating-point channel) and OR_INVALID_OPERATION for linear
+ * filtering of an element-type integer read. */
+typedef struct {
+  uint32_t address_mode[3];  /* cudaTextureAddressMode: 0 wrap, 1 clamp, 2 mirror, 3 border */
+  uint32_t filter_mode;      /* cudaTextureFilterMode: 0 point, 1 linear */
+  uint32_t read_mode;        /* cudaTextureReadMode: 0 element type, 1 normalized float */
+  int32_t normalized_coords;
+} oracle_tex_desc;
+
+/* tex1D / tex2D / tex3D (coord: dims floats) and tex1DLayered / tex2DLayered
+ * (img->arrayed; coord: dims floats then the integer layer as a float). */
+int oracle_tex_fetch(const oracle_image* img, const oracle_tex_desc* td, const float* coord,
+                     void* out16);
+/* tex1Dfetch on linear memory: the texel at integer index x, 0 out of range. */
+int oracle_tex1Dfetch(const oracle_image* img, uint32_t read_mode, int32_t x, void* out16);
+
 /* ---- bulk runtime operations ([CL1.2 §5.2.2-5.3.5]) ----
  * All origins/regions are size_t[3]; rect pitches 0 take the spec defaults. */
 void oracle_copy_rect(const uint8_t* src, uint8_t* dst, const size_t* src_origin,
