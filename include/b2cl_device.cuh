@@ -297,3 +297,89 @@ __device__ __forceinline__ int get_image_width(image2d_array_t im) { return im.i
 __device__ __forceinline__ int get_image_height(image2d_array_t im) { return im.im.h; }
 __device__ __forceinline__ size_t get_image_array_size(image1d_array_t im) { return im.im.h; }
 __device__ __forceinline__ size_t get_image_array_size(image2d_array_t im) { return im.im.d; }
+
+// ---- CUDA texture fetches, as the paper translates them ----
+// A CUDA texture reference becomes an image argument plus a sampler
+// argument (b2clCreateTextureObject makes both from a CUDA-style texture
+// description), and tex1Dfetch / tex1D / tex2D / tex3D become read_imageX;
+// the return type T picks X (f for float T, i for signed, ui for unsigned)
+// and keeps T's components, converted as CUDA returns them (8/16-bit element
+// types narrowed from the int4 / uint4 read).  The fetch is read_imageX
+// exactly: the OpenCL sampler arithmetic of [CL1.2 §8.2] (readings A40, A41
+// and A43 of DESIGN.md record where that differs from a CUDA texture unit).
+namespace b2cl {
+namespace tex {
+template <class T> struct Ret;  // return class and components of T
+#define B2CL_TEX_RET(T, RC, N)                              \
+  template <> struct Ret<T> {                               \
+    static constexpr int rc = RC, n = N;                    \
+  };
+B2CL_TEX_RET(float, dev::R_F, 1) B2CL_TEX_RET(float1, dev::R_F, 1) B2CL_TEX_RET(float2, dev::R_F, 2)
+B2CL_TEX_RET(float4, dev::R_F, 4)
+B2CL_TEX_RET(int, dev::R_I, 1) B2CL_TEX_RET(int1, dev::R_I, 1) B2CL_TEX_RET(int2, dev::R_I, 2)
+B2CL_TEX_RET(int4, dev::R_I, 4)
+B2CL_TEX_RET(unsigned int, dev::R_UI, 1) B2CL_TEX_RET(uint1, dev::R_UI, 1)
+B2CL_TEX_RET(uint2, dev::R_UI, 2) B2CL_TEX_RET(uint4, dev::R_UI, 4)
+B2CL_TEX_RET(signed char, dev::R_I, 1) B2CL_TEX_RET(char1, dev::R_I, 1) B2CL_TEX_RET(char2, dev::R_I, 2)
+B2CL_TEX_RET(char4, dev::R_I, 4)
+B2CL_TEX_RET(unsigned char, dev::R_UI, 1) B2CL_TEX_RET(uchar1, dev::R_UI, 1)
+B2CL_TEX_RET(uchar2, dev::R_UI, 2) B2CL_TEX_RET(uchar4, dev::R_UI, 4)
+B2CL_TEX_RET(short, dev::R_I, 1) B2CL_TEX_RET(short1, dev::R_I, 1) B2CL_TEX_RET(short2, dev::R_I, 2)
+B2CL_TEX_RET(short4, dev::R_I, 4)
+B2CL_TEX_RET(unsigned short, dev::R_UI, 1) B2CL_TEX_RET(ushort1, dev::R_UI, 1)
+B2CL_TEX_RET(ushort2, dev::R_UI, 2) B2CL_TEX_RET(ushort4, dev::R_UI, 4)
+#undef B2CL_TEX_RET
+
+// the first components of the read's 32-bit result v, as T
+template <class T>
+__device__ __forceinline__ T take(uint4 v) {
+  T r;
+  if constexpr (std::is_arithmetic_v<T>) {
+    if constexpr (std::is_same_v<T, float>) r = __uint_as_float(v.x);
+    else r = (T)v.x;
+  } else {
+    using C = decltype(r.x);
+    auto conv = [](uint32_t u) -> C {
+      if constexpr (std::is_same_v<C, float>) return __uint_as_float(u);
+      else return (C)u;
+    };
+    r.x = conv(v.x);
+    if constexpr (Ret<T>::n > 1) r.y = conv(v.y);
+    if constexpr (Ret<T>::n > 2) {
+      r.z = conv(v.z);
+      r.w = conv(v.w);
+    }
+  }
+  return r;
+}
+}  // namespace tex
+}  // namespace b2cl
+
+template <class T>
+__device__ __forceinline__ T tex1Dfetch(image1d_buffer_t im, int x) {
+  return b2cl::tex::take<T>(b2cl::cl_builtin::read_int<1, false>(
+      im.im, b2cl::cl_builtin::kSamplerless, b2cl::tex::Ret<T>::rc, x, 0, 0));
+}
+template <class T>
+__device__ __forceinline__ T tex1D(image1d_t im, sampler_t s, float x) {
+  return b2cl::tex::take<T>(b2cl::cl_builtin::read<1>(im.im, s, b2cl::tex::Ret<T>::rc, x, 0.f, 0.f));
+}
+template <class T>
+__device__ __forceinline__ T tex2D(image2d_t im, sampler_t s, float x, float y) {
+  return b2cl::tex::take<T>(b2cl::cl_builtin::read<2>(im.im, s, b2cl::tex::Ret<T>::rc, x, y, 0.f));
+}
+template <class T>
+__device__ __forceinline__ T tex3D(image3d_t im, sampler_t s, float x, float y, float z) {
+  return b2cl::tex::take<T>(b2cl::cl_builtin::read<3>(im.im, s, b2cl::tex::Ret<T>::rc, x, y, z));
+}
+// layered: the integer layer is the array coordinate (exact as a float below 2^24)
+template <class T>
+__device__ __forceinline__ T tex1DLayered(image1d_array_t im, sampler_t s, float x, int layer) {
+  return b2cl::tex::take<T>(
+      b2cl::cl_builtin::read_array<1>(im.im, s, b2cl::tex::Ret<T>::rc, x, (float)layer, 0.f));
+}
+template <class T>
+__device__ __forceinline__ T tex2DLayered(image2d_array_t im, sampler_t s, float x, float y, int layer) {
+  return b2cl::tex::take<T>(
+      b2cl::cl_builtin::read_array<2>(im.im, s, b2cl::tex::Ret<T>::rc, x, y, (float)layer));
+}

@@ -114,6 +114,81 @@ cl_int b2clEnqueueWriteImageSamples(cl_command_queue command_queue, cl_mem image
                                     cl_uint num_events_in_wait_list,
                                     const cl_event* event_wait_list, cl_event* event);
 
+/* ---- CUDA texture front end ----
+ * The paper's CUDA-to-OpenCL direction translates a texture reference into
+ * an image object and a sampler object added to the kernel's parameters, and
+ * tex1Dfetch() / tex1D() / tex2D() / tex3D() into read_imageX().  A
+ * b2cl_texture is that pair: b2clCreateTextureObject maps a CUDA-style
+ * resource / texture description (the fields and enum values of CUDA's
+ * cudaResourceDesc / cudaTextureDesc) onto an image VIEW of the resource's
+ * storage (no copy: later writes to the storage are seen, as with a CUDA
+ * texture) and a sampler; the device header's tex* functions
+ * (b2cl_device.cuh) take the image and sampler and call the read built-ins.
+ * Mapping (reading A40): wrap -> CLK_ADDRESS_REPEAT, clamp -> CLAMP_TO_EDGE,
+ * mirror -> MIRRORED_REPEAT, border -> CLAMP (border 0 on the texture's
+ * channels); point -> NEAREST, linear -> LINEAR; the channel type of the
+ * view is the stored integer type for element-type reads and the matching
+ * UNORM / SNORM type for normalized-float reads. */
+#define B2CL_RESOURCE_ARRAY 0   /* an image (the translation of a cudaArray) */
+#define B2CL_RESOURCE_LINEAR 2  /* linear memory in a buffer: tex1Dfetch only */
+#define B2CL_RESOURCE_PITCH2D 3 /* pitched 2D memory in a buffer */
+#define B2CL_CHANNEL_SIGNED 0   /* cudaChannelFormatKind */
+#define B2CL_CHANNEL_UNSIGNED 1
+#define B2CL_CHANNEL_FLOAT 2
+#define B2CL_TEX_WRAP 0         /* cudaTextureAddressMode */
+#define B2CL_TEX_CLAMP 1
+#define B2CL_TEX_MIRROR 2
+#define B2CL_TEX_BORDER 3
+#define B2CL_TEX_POINT 0        /* cudaTextureFilterMode */
+#define B2CL_TEX_LINEAR 1
+#define B2CL_READ_ELEMENT_TYPE 0     /* cudaTextureReadMode */
+#define B2CL_READ_NORMALIZED_FLOAT 1
+
+/* cudaChannelFormatDesc: bits per channel x, y, z, w (1, 2 or 4 channels of
+ * equal width: 8/16/32 for integers, 16/32 for floats) and their kind. */
+typedef struct {
+  cl_int x, y, z, w;
+  cl_uint kind;
+} b2cl_channel_format_desc;
+
+typedef struct {
+  cl_uint res_type;                /* B2CL_RESOURCE_* */
+  cl_mem mem;                      /* ARRAY: an image (order R, RG or RGBA, not
+                                      packed, not a shard); LINEAR / PITCH2D: a buffer */
+  size_t offset;                   /* LINEAR / PITCH2D: byte offset into the buffer
+                                      (a multiple of the texel size) */
+  b2cl_channel_format_desc desc;   /* LINEAR / PITCH2D: the texel format */
+  size_t size_in_bytes;            /* LINEAR: bytes of texels (a multiple of the texel size) */
+  size_t width, height, pitch_in_bytes; /* PITCH2D (pitch: a multiple of the texel size) */
+} b2cl_resource_desc;
+
+typedef struct {
+  cl_uint address_mode[3];  /* B2CL_TEX_WRAP..BORDER per axis; the sampled axes must agree */
+  cl_uint filter_mode;      /* B2CL_TEX_POINT / LINEAR */
+  cl_uint read_mode;        /* B2CL_READ_ELEMENT_TYPE / NORMALIZED_FLOAT */
+  cl_int normalized_coords;
+  float border_color[4];    /* must be 0 (OpenCL's border is fixed, reading A40) */
+} b2cl_texture_desc;
+
+typedef struct {
+  cl_mem image;        /* the view (own reference) */
+  cl_sampler sampler;  /* NULL for a LINEAR resource (tex1Dfetch takes none) */
+  b2cl_rtype rtype;    /* read_imagef / i / ui of the view */
+} b2cl_texture;
+
+/* Creates the image view and sampler of a texture.  Errors:
+ * CL_INVALID_CONTEXT / CL_INVALID_MEM_OBJECT for bad handles;
+ * CL_IMAGE_FORMAT_NOT_SUPPORTED for a channel layout CUDA textures do not
+ * have; CL_INVALID_VALUE for a bad resource (range, alignment), disagreeing
+ * address modes on the sampled axes, wrap / mirror with unnormalized
+ * coordinates, a normalized-float read of a 32-bit or float channel, or a
+ * nonzero border colour; CL_INVALID_OPERATION for linear filtering of an
+ * element-type integer read.  On error *tex is untouched. */
+cl_int b2clCreateTextureObject(cl_context context, const b2cl_resource_desc* res_desc,
+                               const b2cl_texture_desc* tex_desc, b2cl_texture* tex);
+/* Releases the view and the sampler of *tex and clears it. */
+cl_int b2clDestroyTextureObject(b2cl_texture* tex);
+
 /* ---- runtime plumbing ---- */
 
 /* A queue on an existing CUDA stream (e.g. torch.cuda.Stream.cuda_stream);
@@ -180,6 +255,21 @@ cl_int b2clValidateSampler(cl_bool normalized_coords, cl_addressing_mode address
 cl_int b2clImageLayout(const cl_image_format* image_format, const cl_image_desc* image_desc,
                        size_t* elem_size, size_t* row_pitch, size_t* slice_pitch,
                        size_t* total_bytes);
+/* The texture mapping of b2clCreateTextureObject: a texture description
+ * over `sampled_dims` axes and the stored format of its resource (for an
+ * ARRAY resource the image's format; otherwise the element-type format of
+ * the channel description) -> the view's format, and the sampler's
+ * normalized flag, addressing and filter mode, and the read's return class.
+ * Same errors as b2clCreateTextureObject. */
+cl_int b2clTextureMapping(const b2cl_texture_desc* tex_desc, cl_uint sampled_dims,
+                          const cl_image_format* stored, cl_image_format* view,
+                          cl_bool* normalized_coords, cl_addressing_mode* addressing_mode,
+                          cl_filter_mode* filter_mode, b2cl_rtype* rtype);
+/* The element-type image format of a cudaChannelFormatDesc (R / RG / RGBA of
+ * SIGNED_INT*, UNSIGNED_INT*, HALF_FLOAT or FLOAT), or
+ * CL_IMAGE_FORMAT_NOT_SUPPORTED. */
+cl_int b2clChannelFormat(const b2cl_channel_format_desc* desc, cl_image_format* format);
+
 /* Errors of an origin / region pixel box on an image of the given type and
  * size ([CL1.2 §5.3.3]). */
 cl_int b2clValidateImageBox(cl_mem_object_type image_type, size_t width, size_t height,

@@ -46,6 +46,12 @@ CL_IMAGE_ARRAY_SIZE, CL_IMAGE_BUFFER = 0x1117, 0x1118
 CL_PROFILING_COMMAND_START, CL_PROFILING_COMMAND_END = 0x1282, 0x1283
 B2CL_RTYPE_FLOAT, B2CL_RTYPE_INT, B2CL_RTYPE_UINT = 0, 1, 2
 B2CL_COORD_FLOAT, B2CL_COORD_INT = 0, 1
+# CUDA texture front end (b2cl_ext.h): cudaResourceDesc / cudaTextureDesc values
+B2CL_RESOURCE_ARRAY, B2CL_RESOURCE_LINEAR, B2CL_RESOURCE_PITCH2D = 0, 2, 3
+B2CL_CHANNEL_SIGNED, B2CL_CHANNEL_UNSIGNED, B2CL_CHANNEL_FLOAT = 0, 1, 2
+B2CL_TEX_WRAP, B2CL_TEX_CLAMP, B2CL_TEX_MIRROR, B2CL_TEX_BORDER = 0, 1, 2, 3
+B2CL_TEX_POINT, B2CL_TEX_LINEAR = 0, 1
+B2CL_READ_ELEMENT_TYPE, B2CL_READ_NORMALIZED_FLOAT = 0, 1
 
 _H = c_void_p
 _P = c_void_p
@@ -142,6 +148,10 @@ PROTOTYPES = {
     "b2clValidateSampler": (_I, [_U, _U, _U]),
     "b2clImageLayout": (_I, [_P, _P, POINTER(_S), POINTER(_S), POINTER(_S), POINTER(_S)]),
     "b2clValidateImageBox": (_I, [_U, _S, _S, _S, _SZ3, _SZ3]),
+    "b2clCreateTextureObject": (_I, [_H, _P, _P, _P]),
+    "b2clDestroyTextureObject": (_I, [_P]),
+    "b2clTextureMapping": (_I, [_P, _U, _P, _P, POINTER(_U), POINTER(_U), POINTER(_U), POINTER(_U)]),
+    "b2clChannelFormat": (_I, [_P, _P]),
 }
 
 
@@ -154,6 +164,32 @@ class ImageDesc(ctypes.Structure):
                 ("image_depth", c_size_t), ("image_array_size", c_size_t),
                 ("image_row_pitch", c_size_t), ("image_slice_pitch", c_size_t),
                 ("num_mip_levels", c_uint32), ("num_samples", c_uint32), ("buffer", c_void_p)]
+
+
+class ChannelFormatDesc(ctypes.Structure):  # b2cl_channel_format_desc
+    _fields_ = [("x", c_int32), ("y", c_int32), ("z", c_int32), ("w", c_int32), ("kind", c_uint32)]
+
+
+class ResourceDesc(ctypes.Structure):  # b2cl_resource_desc
+    _fields_ = [("res_type", c_uint32), ("mem", c_void_p), ("offset", c_size_t),
+                ("desc", ChannelFormatDesc), ("size_in_bytes", c_size_t), ("width", c_size_t),
+                ("height", c_size_t), ("pitch_in_bytes", c_size_t)]
+
+
+class TextureDesc(ctypes.Structure):  # b2cl_texture_desc
+    _fields_ = [("address_mode", c_uint32 * 3), ("filter_mode", c_uint32), ("read_mode", c_uint32),
+                ("normalized_coords", c_int32), ("border_color", c_float * 4)]
+
+
+class Texture(ctypes.Structure):  # b2cl_texture
+    _fields_ = [("image", c_void_p), ("sampler", c_void_p), ("rtype", c_uint32)]
+
+
+def texture_desc(address_modes, filter_mode: int, read_mode: int, normalized: bool,
+                 border=(0.0, 0.0, 0.0, 0.0)) -> TextureDesc:
+    am = list(address_modes) + [B2CL_TEX_WRAP] * (3 - len(address_modes))
+    return TextureDesc((c_uint32 * 3)(*am[:3]), filter_mode, read_mode, int(bool(normalized)),
+                       (c_float * 4)(*border))
 
 
 class CLError(RuntimeError):
@@ -358,6 +394,13 @@ class Session:
                                            halo, None, byref(err))
         check(err.value, "b2clCreateImageShard")
         return m
+
+    def texture(self, res: ResourceDesc, tex_desc: TextureDesc) -> Texture:
+        """b2clCreateTextureObject: the (image view, sampler) pair of a CUDA texture."""
+        t = Texture()
+        check(lib().b2clCreateTextureObject(self.ctx, byref(res), byref(tex_desc), byref(t)),
+              "b2clCreateTextureObject")
+        return t
 
     def sampler(self, normalized: bool, addressing: int, filt: int):
         err = c_int32()

@@ -51,5 +51,9 @@ cl_int validate_sampler(cl_bool norm, cl_addressing_mode am, cl_filter_mode fm);
 cl_int validate_image_box(int dims, size_t w, size_t h, size_t d, const size_t* o,
                           const size_t* r);
 bool image_boxes_overlap(const size_t* a, const size_t* b, const size_t* r);
+cl_int channel_format(const b2cl_channel_format_desc* d, cl_image_format* f);
+cl_int texture_mapping(const b2cl_texture_desc* td, cl_uint dims, const cl_image_format* stored,
+                       cl_image_format* view, cl_bool* norm, cl_addressing_mode* am,
+                       cl_filter_mode* fm, b2cl_rtype* rt);
 
 }  // namespace b2cl

@@ -72,9 +72,11 @@ struct _cl_mem {
   long long shard_ob = 0;
   cl_image_format fmt{};
   cl_image_desc desc{};
-  // a 1D image buffer (CL_MEM_OBJECT_IMAGE1D_BUFFER) owns no storage: its
-  // texels are the bytes of this buffer, which it retains
+  // a 1D image buffer (CL_MEM_OBJECT_IMAGE1D_BUFFER) or a texture's image
+  // view owns no storage: its texels are the bytes of this object (a buffer
+  // or an image) from byte parent_off on, and it retains the object
   cl_mem parent = nullptr;
+  size_t parent_off = 0;
   std::mutex mu;
   std::vector<Store> stores;
   uint64_t valid = 0;                   // bit per ordinal holding valid content
@@ -1001,7 +1003,11 @@ static cl_int enq_end(Enq& E, cudaError_t err) {
 // NVLink (SM copy kernel on the peer pointer) on the queue's stream; the
 // caller's wait list orders it after the producer (OpenCL cross-queue rule).
 static cl_int resident(cl_mem m, cl_command_queue q, bool need_content, char** out) {
-  if (m->parent) m = m->parent;  // a 1D image buffer lives in its buffer
+  size_t off = 0;
+  if (m->parent) {  // a 1D image buffer or a view lives in its parent
+    off = m->parent_off;
+    m = m->parent;
+  }
   std::lock_guard<std::mutex> g(m->mu);
   const int ord = q->dev->ordinal;
   Store* s = nullptr;
@@ -1030,7 +1036,7 @@ static cl_int resident(cl_mem m, cl_command_queue q, bool need_content, char** o
     m->valid |= bit;
   }
   m->users.insert(q);
-  *out = s->ptr;
+  *out = s->ptr + off;
   return CL_SUCCESS;
 }
 
@@ -1050,6 +1056,120 @@ static cl_int check_queue_mem(cl_command_queue q, cl_mem m) {
     cl_int _s = (x);                    \
     if (_s != CL_SUCCESS) return _s;    \
   } while (0)
+
+// ---- CUDA texture front end (b2cl_ext.h, reading A40) ----
+// An image view: layout L over the storage of `parent` (a buffer or an
+// image) from byte `off` on; retains the parent, owns no storage.
+static cl_mem image_view(cl_context c, cl_mem parent, size_t off, cl_mem_object_type type,
+                         const cl_image_format& fmt, const ImageLayout& L) {
+  if (parent->parent) {  // views of views share the root storage
+    off += parent->parent_off;
+    parent = parent->parent;
+  }
+  cl_mem m = new_mem(c, type, parent->flags & (CL_MEM_READ_WRITE | CL_MEM_WRITE_ONLY | CL_MEM_READ_ONLY),
+                     L.bytes);
+  if (!m) return nullptr;
+  m->img = L;
+  m->fmt = fmt;
+  m->desc.image_type = type;
+  m->desc.image_width = L.w;
+  m->desc.image_height = L.arrayed && L.dims == 2 ? 0 : L.h;
+  m->desc.image_depth = L.dims == 3 && !L.arrayed ? L.d : 0;
+  m->desc.image_array_size = L.arrayed ? (L.dims == 2 ? L.h : L.d) : 0;
+  parent->ref++;
+  m->parent = parent;
+  m->parent_off = off;
+  register_mem(m);
+  return m;
+}
+
+extern "C" cl_int b2clCreateTextureObject(cl_context c, const b2cl_resource_desc* rd,
+                                          const b2cl_texture_desc* td, b2cl_texture* tex) {
+  if (!live(g_contexts, c)) return CL_INVALID_CONTEXT;
+  if (!rd || !td || !tex) return CL_INVALID_VALUE;
+  if (!live(g_mems, rd->mem) || rd->mem->ctx != c) return CL_INVALID_MEM_OBJECT;
+  cl_mem src = rd->mem;
+  cl_image_format stored{};
+  ImageLayout L{};
+  cl_mem_object_type vtype = 0;
+  cl_uint sdims = 1;  // sampled axes
+  if (rd->res_type == B2CL_RESOURCE_ARRAY) {
+    if (!is_image(src) || src->shard || src->type == CL_MEM_OBJECT_IMAGE1D_BUFFER)
+      return CL_INVALID_MEM_OBJECT;
+    stored = src->fmt;
+    L = src->img;
+    vtype = src->type;
+    sdims = (cl_uint)(L.dims - L.arrayed);
+  } else if (rd->res_type == B2CL_RESOURCE_LINEAR || rd->res_type == B2CL_RESOURCE_PITCH2D) {
+    if (src->type != CL_MEM_OBJECT_BUFFER) return CL_INVALID_MEM_OBJECT;
+    CHECK(channel_format(&rd->desc, &stored));
+    cl_image_desc d{};
+    const bool lin = rd->res_type == B2CL_RESOURCE_LINEAR;
+    FormatInfo fi;
+    CHECK(format_info(&stored, &fi));
+    d.image_type = lin ? CL_MEM_OBJECT_IMAGE1D_BUFFER : CL_MEM_OBJECT_IMAGE2D;
+    d.image_width = lin ? rd->size_in_bytes / fi.es : rd->width;
+    d.image_height = lin ? 0 : rd->height;
+    d.buffer = lin ? src : nullptr;
+    if (lin && rd->size_in_bytes % fi.es) return CL_INVALID_VALUE;
+    CHECK(image_layout(&stored, &d, &L));
+    if (!lin) {  // the caller's pitch, not the internal one
+      if (rd->pitch_in_bytes < L.w * fi.es || rd->pitch_in_bytes % fi.es) return CL_INVALID_VALUE;
+      L.row_pitch = rd->pitch_in_bytes;
+      L.slice_pitch = L.row_pitch * L.h;
+      L.bytes = L.row_pitch * (L.h - 1) + L.w * fi.es;
+    }
+    // texels naturally aligned (buffers start 256-byte aligned) and inside the buffer
+    if (rd->offset % fi.es || rd->offset > src->size || L.bytes > src->size - rd->offset)
+      return CL_INVALID_VALUE;
+    vtype = d.image_type;
+    sdims = 1 + (lin ? 0 : 1);
+  } else {
+    return CL_INVALID_VALUE;
+  }
+  cl_image_format view{};
+  cl_bool nc;
+  cl_addressing_mode am;
+  cl_filter_mode fm;
+  b2cl_rtype rt;
+  CHECK(texture_mapping(td, sdims, &stored, &view, &nc, &am, &fm, &rt));
+  FormatInfo vfi;
+  CHECK(format_info(&view, &vfi));
+  L.fmt = vfi;  // same bits per texel: only the read conversion changes
+  cl_mem img = nullptr;
+  if (rd->res_type == B2CL_RESOURCE_ARRAY && view.image_channel_data_type == stored.image_channel_data_type) {
+    img = src;  // the image itself
+    src->ref++;
+  } else {
+    img = image_view(c, src, rd->res_type == B2CL_RESOURCE_ARRAY ? 0 : rd->offset, vtype, view, L);
+    if (!img) return CL_OUT_OF_HOST_MEMORY;
+  }
+  cl_sampler smp = nullptr;
+  if (rd->res_type != B2CL_RESOURCE_LINEAR) {  // tex1Dfetch takes no sampler
+    cl_int st = CL_SUCCESS;
+    smp = clCreateSampler(c, nc, am, fm, &st);
+    if (!smp) {
+      clReleaseMemObject(img);
+      return st;
+    }
+  }
+  tex->image = img;
+  tex->sampler = smp;
+  tex->rtype = rt;
+  return CL_SUCCESS;
+}
+
+extern "C" cl_int b2clDestroyTextureObject(b2cl_texture* tex) {
+  if (!tex) return CL_INVALID_VALUE;
+  if (tex->image && !live(g_mems, tex->image)) return CL_INVALID_MEM_OBJECT;
+  if (tex->sampler && !live(g_samplers, tex->sampler)) return CL_INVALID_SAMPLER;
+  if (tex->image) clReleaseMemObject(tex->image);
+  if (tex->sampler) clReleaseSampler(tex->sampler);
+  tex->image = nullptr;
+  tex->sampler = nullptr;
+  return CL_SUCCESS;
+}
+
 
 // Device view of an image.  For the read built-ins (sampling) a shard
 // presents its global extent on the outer axis with the stored window (ob,
@@ -1633,11 +1753,15 @@ extern "C" cl_int b2clGetMemDevicePointer(cl_mem m, cl_device_id d, void** ptr) 
   if (!live(g_mems, m)) return CL_INVALID_MEM_OBJECT;
   if (!valid_device(d) || !ctx_has_device(m->ctx, d)) return CL_INVALID_DEVICE;
   if (!ptr) return CL_INVALID_VALUE;
-  if (m->parent) m = m->parent;  // a 1D image buffer's texels are its buffer's
+  size_t off = 0;
+  if (m->parent) {  // a 1D image buffer's (a view's) texels are its parent's
+    off = m->parent_off;
+    m = m->parent;
+  }
   std::lock_guard<std::mutex> g(m->mu);
   Store* s = nullptr;
   CHECK(ensure_store(m, d->ordinal, nullptr, &s));
-  *ptr = s->ptr;
+  *ptr = s->ptr + off;
   return CL_SUCCESS;
 }
 

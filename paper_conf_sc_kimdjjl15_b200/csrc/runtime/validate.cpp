@@ -11,6 +11,12 @@
 
 namespace b2cl {
 
+#define CHECK_ST(x)                      \
+  do {                                   \
+    cl_int _s = (x);                     \
+    if (_s != CL_SUCCESS) return _s;     \
+  } while (0)
+
 // Khronos channel type / order -> internal codes (dev::TypeCode / OrderCode)
 int type_code(cl_channel_type t) {
   switch (t) {
@@ -235,6 +241,98 @@ cl_int validate_image_box(int dims, size_t w, size_t h, size_t d, const size_t* 
   return CL_SUCCESS;
 }
 
+// ---- CUDA texture front end (reading A40) ----
+cl_int channel_format(const b2cl_channel_format_desc* d, cl_image_format* f) {
+  if (!d || !f) return CL_INVALID_VALUE;
+  const int c[4] = {d->x, d->y, d->z, d->w}, b = d->x;
+  int n = 0;
+  while (n < 4 && c[n] != 0) ++n;
+  for (int k = 0; k < 4; ++k)  // channels of one width, none after an empty one
+    if ((k < n && c[k] != b) || (k >= n && c[k] != 0)) return CL_IMAGE_FORMAT_NOT_SUPPORTED;
+  if (n != 1 && n != 2 && n != 4) return CL_IMAGE_FORMAT_NOT_SUPPORTED;
+  f->image_channel_order = n == 1 ? CL_R : (n == 2 ? CL_RG : CL_RGBA);
+  switch (d->kind) {
+    case B2CL_CHANNEL_SIGNED:
+      if (b == 8) f->image_channel_data_type = CL_SIGNED_INT8;
+      else if (b == 16) f->image_channel_data_type = CL_SIGNED_INT16;
+      else if (b == 32) f->image_channel_data_type = CL_SIGNED_INT32;
+      else return CL_IMAGE_FORMAT_NOT_SUPPORTED;
+      return CL_SUCCESS;
+    case B2CL_CHANNEL_UNSIGNED:
+      if (b == 8) f->image_channel_data_type = CL_UNSIGNED_INT8;
+      else if (b == 16) f->image_channel_data_type = CL_UNSIGNED_INT16;
+      else if (b == 32) f->image_channel_data_type = CL_UNSIGNED_INT32;
+      else return CL_IMAGE_FORMAT_NOT_SUPPORTED;
+      return CL_SUCCESS;
+    case B2CL_CHANNEL_FLOAT:
+      if (b == 16) f->image_channel_data_type = CL_HALF_FLOAT;
+      else if (b == 32) f->image_channel_data_type = CL_FLOAT;
+      else return CL_IMAGE_FORMAT_NOT_SUPPORTED;
+      return CL_SUCCESS;
+    default: return CL_IMAGE_FORMAT_NOT_SUPPORTED;
+  }
+}
+
+cl_int texture_mapping(const b2cl_texture_desc* td, cl_uint dims, const cl_image_format* stored,
+                       cl_image_format* view, cl_bool* norm, cl_addressing_mode* am,
+                       cl_filter_mode* fm, b2cl_rtype* rt) {
+  if (!td || !stored || dims < 1 || dims > 3) return CL_INVALID_VALUE;
+  FormatInfo fi;
+  CHECK_ST(format_info(stored, &fi));
+  // a CUDA texture has 1, 2 or 4 channels in memory order, no packed words
+  if (fi.order != dev::O_R && fi.order != dev::O_RG && fi.order != dev::O_RGBA)
+    return CL_IMAGE_FORMAT_NOT_SUPPORTED;
+  // stored channel: signedness and width (UNORM / UNSIGNED_INT alike)
+  const int t = fi.type;
+  const bool is_float = t == dev::T_HALF || t == dev::T_FLOAT;
+  const bool sgn = t == dev::T_SNORM8 || t == dev::T_SNORM16 || t == dev::T_SINT8 ||
+                   t == dev::T_SINT16 || t == dev::T_SINT32;
+  const int bits = 8 * dev::type_bytes(t);
+  cl_channel_type vt;
+  if (td->read_mode == B2CL_READ_NORMALIZED_FLOAT) {
+    if (is_float || bits == 32) return CL_INVALID_VALUE;  // 8- and 16-bit integers only
+    vt = bits == 8 ? (sgn ? CL_SNORM_INT8 : CL_UNORM_INT8) : (sgn ? CL_SNORM_INT16 : CL_UNORM_INT16);
+  } else if (td->read_mode == B2CL_READ_ELEMENT_TYPE) {
+    if (t == dev::T_HALF) vt = CL_HALF_FLOAT;
+    else if (t == dev::T_FLOAT) vt = CL_FLOAT;
+    else if (bits == 8) vt = sgn ? CL_SIGNED_INT8 : CL_UNSIGNED_INT8;
+    else if (bits == 16) vt = sgn ? CL_SIGNED_INT16 : CL_UNSIGNED_INT16;
+    else vt = sgn ? CL_SIGNED_INT32 : CL_UNSIGNED_INT32;
+  } else {
+    return CL_INVALID_VALUE;
+  }
+  // one OpenCL sampler for all axes: the sampled axes' modes must agree
+  const cl_uint m = td->address_mode[0];
+  for (cl_uint d = 0; d < dims; ++d)
+    if (td->address_mode[d] != m) return CL_INVALID_VALUE;
+  cl_addressing_mode a;
+  switch (m) {
+    case B2CL_TEX_WRAP: a = CL_ADDRESS_REPEAT; break;
+    case B2CL_TEX_CLAMP: a = CL_ADDRESS_CLAMP_TO_EDGE; break;
+    case B2CL_TEX_MIRROR: a = CL_ADDRESS_MIRRORED_REPEAT; break;
+    case B2CL_TEX_BORDER: a = CL_ADDRESS_CLAMP; break;
+    default: return CL_INVALID_VALUE;
+  }
+  if (td->filter_mode != B2CL_TEX_POINT && td->filter_mode != B2CL_TEX_LINEAR) return CL_INVALID_VALUE;
+  for (int c = 0; c < 4; ++c)
+    if (td->border_color[c] != 0.0f) return CL_INVALID_VALUE;
+  const cl_bool nc = td->normalized_coords ? CL_TRUE : CL_FALSE;
+  const cl_filter_mode f = td->filter_mode == B2CL_TEX_LINEAR ? CL_FILTER_LINEAR : CL_FILTER_NEAREST;
+  CHECK_ST(validate_sampler(nc, a, f));  // wrap / mirror need normalized coordinates (A5)
+  const b2cl_rtype r = dev::ret_class(type_code(vt));
+  // "linear filtering ... only for textures configured to return floating-point data"
+  if (f == CL_FILTER_LINEAR && r != B2CL_RTYPE_FLOAT) return CL_INVALID_OPERATION;
+  if (view) {
+    view->image_channel_order = stored->image_channel_order;
+    view->image_channel_data_type = vt;
+  }
+  if (norm) *norm = nc;
+  if (am) *am = a;
+  if (fm) *fm = f;
+  if (rt) *rt = r;
+  return CL_SUCCESS;
+}
+
 bool image_boxes_overlap(const size_t* a, const size_t* b, const size_t* r) {
   for (int k = 0; k < 3; ++k)
     if (!(a[k] < b[k] + r[k] && b[k] < a[k] + r[k])) return false;
@@ -265,6 +363,17 @@ extern "C" cl_int b2clRectOverlap(const size_t* so, const size_t* dso, const siz
 extern "C" cl_int b2clValidateFillBuffer(size_t buffer_size, size_t pattern_size, size_t offset,
                                          size_t size) {
   return validate_fill_buffer(buffer_size, pattern_size, offset, size);
+}
+
+extern "C" cl_int b2clTextureMapping(const b2cl_texture_desc* td, cl_uint dims,
+                                     const cl_image_format* stored, cl_image_format* view,
+                                     cl_bool* norm, cl_addressing_mode* am, cl_filter_mode* fm,
+                                     b2cl_rtype* rt) {
+  return texture_mapping(td, dims, stored, view, norm, am, fm, rt);
+}
+
+extern "C" cl_int b2clChannelFormat(const b2cl_channel_format_desc* d, cl_image_format* f) {
+  return channel_format(d, f);
 }
 
 extern "C" cl_int b2clValidateSampler(cl_bool normalized_coords, cl_addressing_mode am,

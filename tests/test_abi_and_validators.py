@@ -181,3 +181,73 @@ def test_binding_fails_loudly_without_library(monkeypatch, tmp_path):
     monkeypatch.setattr(cl, "_lib", None)
     with pytest.raises(RuntimeError, match="no CPU fallback"):
         cl.lib()
+
+
+# ---------------------------------------------------------------- texture mapping (row 3)
+def _map(L, stored_order, stored_type, modes, filt, rmode, norm, dims, border=(0, 0, 0, 0)):
+    td = cl.texture_desc(modes, filt, rmode, norm, border)
+    st = cl.ImageFormat(stored_order, stored_type)
+    view = cl.ImageFormat()
+    nc, am, fm, rt = ctypes.c_uint32(), ctypes.c_uint32(), ctypes.c_uint32(), ctypes.c_uint32()
+    r = L.b2clTextureMapping(ctypes.byref(td), dims, ctypes.byref(st), ctypes.byref(view),
+                             ctypes.byref(nc), ctypes.byref(am), ctypes.byref(fm), ctypes.byref(rt))
+    return r, (view.image_channel_order, view.image_channel_data_type), nc.value, am.value, fm.value, rt.value
+
+
+def test_texture_mapping_table(L, orc):
+    """The CUDA texture -> (image view, sampler) mapping of P:449 (reading A40): the
+    same table the oracle's translation pin (tests/test_oracle_cuda_tex.py) proves exact."""
+    from tests.test_oracle_cuda_tex import CL_ADDR, CL_FILT, _cl_type
+    stored = [cl.CL_UNSIGNED_INT8, cl.CL_SIGNED_INT8, cl.CL_UNSIGNED_INT16, cl.CL_SIGNED_INT16,
+              cl.CL_UNSIGNED_INT32, cl.CL_SIGNED_INT32, cl.CL_HALF_FLOAT, cl.CL_FLOAT,
+              cl.CL_UNORM_INT8, cl.CL_SNORM_INT16]
+    n = 0
+    for t in stored:
+        for rmode in (0, 1):
+            for mode in range(4):
+                for filt in (0, 1):
+                    for norm in (False, True):
+                        r, view, nc, am, fm, rt = _map(L, cl.CL_RGBA, t, [mode] * 2, filt, rmode, norm, 2)
+                        # what the oracle side expects
+                        raw = {cl.CL_UNORM_INT8: cl.CL_UNSIGNED_INT8, cl.CL_SNORM_INT16: cl.CL_SIGNED_INT16}.get(t, t)
+                        bits32_or_float = raw in (cl.CL_UNSIGNED_INT32, cl.CL_SIGNED_INT32, cl.CL_HALF_FLOAT, cl.CL_FLOAT)
+                        if rmode == 1 and bits32_or_float:
+                            assert r == -30, (hex(t), rmode)
+                            continue
+                        if not norm and mode in (0, 2):
+                            assert r == -30
+                            continue
+                        ctype, ort = _cl_type(orc, raw, rmode)
+                        if filt == 1 and ort != orc.RT_F:
+                            assert r == -59
+                            continue
+                        assert r == 0, (hex(t), rmode, mode, filt, norm, r)
+                        assert view == (cl.CL_RGBA, ctype) and rt == ort
+                        assert (nc, am, fm) == (int(norm), CL_ADDR[mode], CL_FILT[filt])
+                        n += 1
+    assert n > 100
+    # per-axis modes must agree on the sampled axes only
+    assert _map(L, cl.CL_R, cl.CL_FLOAT, [1, 3], 0, 0, True, 2)[0] == -30
+    assert _map(L, cl.CL_R, cl.CL_FLOAT, [1, 3], 0, 0, True, 1)[0] == 0
+    assert _map(L, cl.CL_R, cl.CL_FLOAT, [1, 1, 3], 0, 0, True, 2)[0] == 0
+    # border colour other than 0, orders and packed types CUDA textures do not have
+    assert _map(L, cl.CL_R, cl.CL_FLOAT, [3], 0, 0, True, 1, border=(0, 0, 0, 1))[0] == -30
+    assert _map(L, cl.CL_BGRA, cl.CL_UNORM_INT8, [1], 0, 1, True, 1)[0] == -10
+    assert _map(L, cl.CL_RGB, cl.CL_UNORM_SHORT_565, [1], 0, 1, True, 1)[0] == -10
+
+
+def test_channel_format_desc(L):
+    def fmt(x, y, z, w, kind):
+        d = cl.ChannelFormatDesc(x, y, z, w, kind)
+        f = cl.ImageFormat()
+        r = L.b2clChannelFormat(ctypes.byref(d), ctypes.byref(f))
+        return r, (f.image_channel_order, f.image_channel_data_type)
+    S, U, F = cl.B2CL_CHANNEL_SIGNED, cl.B2CL_CHANNEL_UNSIGNED, cl.B2CL_CHANNEL_FLOAT
+    assert fmt(8, 8, 8, 8, U) == (0, (cl.CL_RGBA, cl.CL_UNSIGNED_INT8))
+    assert fmt(16, 0, 0, 0, S) == (0, (cl.CL_R, cl.CL_SIGNED_INT16))
+    assert fmt(32, 32, 0, 0, F) == (0, (cl.CL_RG, cl.CL_FLOAT))
+    assert fmt(16, 16, 16, 16, F) == (0, (cl.CL_RGBA, cl.CL_HALF_FLOAT))
+    assert fmt(32, 0, 0, 0, U) == (0, (cl.CL_R, cl.CL_UNSIGNED_INT32))
+    for bad in ((8, 8, 8, 0, U), (8, 16, 0, 0, U), (0, 8, 0, 0, U), (8, 0, 8, 0, U), (8, 0, 0, 0, F),
+                (64, 0, 0, 0, S), (8, 0, 0, 0, 7)):
+        assert fmt(*bad)[0] == -10, bad
