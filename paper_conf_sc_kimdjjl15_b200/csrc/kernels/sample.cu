@@ -68,6 +68,11 @@ __global__ void __launch_bounds__(256) k_sample_grid(const SampleParams p) {
   store_out<OUTC>(p, ((uint64_t)z * p.oh + y) * p.ow + x, r);
 }
 
+#ifndef B2CL_SEP_UNROLL
+#define B2CL_SEP_UNROLL 1
+#endif
+constexpr int kSepUnroll = B2CL_SEP_UNROLL;  // rows of a thread in flight together
+
 // Separable maps: block = 32 x 4 threads; tile = (32*XPT) columns x (4*RPW) rows
 // of one output slice.  Lane -> columns lane + 32*t, warp -> RPW consecutive rows.
 template <class C, int OUTC, int XPT, int RPW>
@@ -99,7 +104,7 @@ __global__ void __launch_bounds__(128, (C::type == RT ? 1 : 11)) k_sample_grid_s
     if (lin) az = axis_l<C>(p.smp, s, im.d);
     else nz = axis_n<C>(p.smp, s, im.d);
   }
-#pragma unroll 1
+#pragma unroll kSepUnroll
   for (int r = 0; r < RPW; ++r) {
     const int y = y0 + r;
     if (y >= p.oh) break;
@@ -406,6 +411,136 @@ __global__ void __launch_bounds__(128, B2CL_W4_MINB) k_sample_grid_walk4(const S
   else walk4_run<C, WALK, false>(p, ax, x0, yfix, w0, vst);
 }
 
+// Separable LINEAR maps of 2D RGBA32F images under REPEAT / MIRRORED_REPEAT
+// (every tap in range): the filter footprint of a TW x TH output tile is
+// staged in shared memory once, so L2 serves each texel about once per tile
+// instead of once per tap (the direct kernels issue 4 x 16-byte gathers per
+// sample, and their L1 catches only part of the reuse).
+//   Per axis the taps of consecutive outputs CHAIN upward (i1(x) = i0(x+1):
+//   unit-scale maps, wrap seams included) or downward (i0(x) = i1(x+1): the
+//   reflected half of MIRRORED_REPEAT).  Upward, slot k < TW holds texel
+//   column i0(x0+k) and slot TW holds i1(x0+TW-1): output column t blends
+//   slots (t, t+1).  Downward, slot k holds i1(x0+k), slot TW holds
+//   i0(x0+TW-1): column t blends slots (t+1, t).  Rows likewise.  A tile whose
+//   taps chain neither way on some axis (it contains a mirror fold, or the map
+//   has another scale) reads its taps directly.
+//   Block = 4 warps: warp w takes columns (w & 1)*32 + lane and walks rows
+//   (w >> 1)*TH/2 .. +TH/2, blending x once per row and y from the previous
+//   row's x-blend.  Operations, operands and order are linear_at's: the
+//   results are bit-identical to the other kernels.
+template <class C, int TW, int TH>
+__global__ void __launch_bounds__(128) k_sample_grid_tile(const SampleParams p) {
+  static_assert(C::type == T_FLOAT && C::order == O_RGBA && C::dims == 2 && TW == 64, "2D RGBA32F");
+  static_assert(C::addr == A_REPEAT || C::addr == A_MIRROR, "taps always in range");
+  constexpr int RPW = TH / 2;
+  __shared__ __align__(16) float4 tile[TH + 1][TW + 1];
+  __shared__ int colI0[TW], colI1[TW], rowJ0[TH], rowJ1[TH];
+  __shared__ float colA[TW], colOma[TW], rowA[TH], rowOma[TH];
+  __shared__ int chain[4];  // columns up, columns down, rows up, rows down
+  const Image& im = p.im;
+  const int tid = threadIdx.x;
+  int ty = blockIdx.y;  // MIRRORED: row tiles alternately from both ends (as k_sample_grid_sep)
+  if (C::addr == A_MIRROR) ty = (ty & 1) ? gridDim.y - 1 - (ty >> 1) : (ty >> 1);
+  const int x0 = blockIdx.x * TW, y0 = ty * TH;
+  const uint64_t zoff = (uint64_t)blockIdx.z * p.oh;  // 2D slices of the output repeat (A[2] = 0)
+  // per-axis addressing: threads [0, TW) take the columns, [TW, TW + TH) the rows
+  if (tid < 4) chain[tid] = 1;
+  if (tid < TW) {
+    const AxL ax =
+        axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(p.ox + x0 + tid)), p.A[3]), im.w);
+    colI0[tid] = ax.i0;
+    colI1[tid] = ax.i1;
+    colA[tid] = ax.a;
+    colOma[tid] = ax.oma;
+  } else if (tid < TW + TH) {
+    const int r = tid - TW;
+    const AxL ay =
+        axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(p.oy + y0 + r)), p.A[7]), im.h);
+    rowJ0[r] = ay.i0;
+    rowJ1[r] = ay.i1;
+    rowA[r] = ay.a;
+    rowOma[r] = ay.oma;
+  }
+  __syncthreads();
+  if (tid < TW - 1) {
+    if (colI1[tid] != colI0[tid + 1]) chain[0] = 0;
+    if (colI0[tid] != colI1[tid + 1]) chain[1] = 0;
+  } else if (tid >= TW && tid < TW + TH - 1) {
+    const int r = tid - TW;
+    if (rowJ1[r] != rowJ0[r + 1]) chain[2] = 0;
+    if (rowJ0[r] != rowJ1[r + 1]) chain[3] = 0;
+  }
+  __syncthreads();
+  const bool cup = chain[0], cdn = !cup && chain[1], rup = chain[2], rdn = !rup && chain[3];
+  const int warp = tid >> 5, lane = tid & 31;
+  const int c = (warp & 1) * 32 + lane, r0 = (warp >> 1) * RPW, x = x0 + c;
+  const float a = colA[c], oma = colOma[c];
+  float4* out = reinterpret_cast<float4*>(p.out);
+  if (!(cup || cdn) || !(rup || rdn)) {  // the taps directly (same operations as linear_at)
+    const AxL ax{colI0[c], colI1[c], a, oma, true, true};
+#pragma unroll 1
+    for (int r = r0; r < r0 + RPW; ++r) {
+      const int y = y0 + r;
+      if (y >= p.oh) break;
+      const char* rows[4] = {row_ptr<C>(im, rowJ0[r], 0), row_ptr<C>(im, rowJ1[r], 0), nullptr, nullptr};
+      const bool rok[4] = {true, true, false, false};
+      uint32_t res[4];
+      linear_at<C>(p, rows, rok, ax, rowA[r], rowOma[r], 0.f, 1.f, res, 4);
+      if (x < p.ow)
+        __stcs(out + ((zoff + y) * p.ow + x), make_float4(__uint_as_float(res[0]), __uint_as_float(res[1]),
+                                                           __uint_as_float(res[2]), __uint_as_float(res[3])));
+    }
+    return;
+  }
+  // stage the (TH+1) x (TW+1) footprint with 16-byte async copies (no
+  // register round trip): warp w takes slot rows w, w+4, ...; lane l the slot
+  // columns l and l+32 (lane 0 also slot TW), whose byte offsets are fixed
+  // for the tile -- a copy costs an address add, not an index computation
+  {
+    const int iA = cup ? colI0[lane] : colI1[lane], iB = cup ? colI0[lane + 32] : colI1[lane + 32];
+    const int iC = cup ? colI1[TW - 1] : colI0[TW - 1];
+    const uint64_t oA = (uint64_t)(unsigned)iA * 16u, oB = (uint64_t)(unsigned)iB * 16u,
+                   oC = (uint64_t)(unsigned)iC * 16u;
+    uint32_t dst = static_cast<uint32_t>(__cvta_generic_to_shared(&tile[warp][lane]));
+    for (int r = warp; r <= TH; r += 4, dst += 4 * (TW + 1) * 16) {
+      const int j = r < TH ? (rup ? rowJ0[r] : rowJ1[r]) : (rup ? rowJ1[TH - 1] : rowJ0[TH - 1]);
+      const char* rp = row_ptr<C>(im, j, 0);
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(rp + oA) : "memory");
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst + 32 * 16), "l"(rp + oB) : "memory");
+      if (lane == 0)
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst + TW * 16), "l"(rp + oC) : "memory");
+    }
+  }
+  asm volatile("cp.async.wait_all;" ::: "memory");
+  __syncthreads();
+  // slots of tap i0 / i1 of this column, and of row tap j0 / j1 relative to r
+  const int ci0 = cup ? c : c + 1, ci1 = cup ? c + 1 : c;
+  const int dj0 = rup ? 0 : 1, dj1 = rup ? 1 : 0;
+  auto xblend = [&](int r, float h[4]) {
+    const float4 t0 = tile[r][ci0], t1 = tile[r][ci1];
+    h[0] = lerp1(a, oma, t0.x, t1.x);
+    h[1] = lerp1(a, oma, t0.y, t1.y);
+    h[2] = lerp1(a, oma, t0.z, t1.z);
+    h[3] = lerp1(a, oma, t0.w, t1.w);
+  };
+  float hr[4], hn[4];  // x-blends of slot rows r and r + 1
+  xblend(r0, hr);
+#pragma unroll 4
+  for (int r = r0; r < r0 + RPW; ++r) {
+    xblend(r + 1, hn);
+    const float b = rowA[r], omb = rowOma[r];
+    const float* v0 = dj0 ? hn : hr;  // the x-blend of row j0
+    const float* v1 = dj1 ? hn : hr;  // ... and of row j1
+    const int y = y0 + r;
+    if (x < p.ow && y < p.oh)
+      __stcs(out + ((zoff + y) * p.ow + x),
+             make_float4(lerp1(b, omb, v0[0], v1[0]), lerp1(b, omb, v0[1], v1[1]),
+                         lerp1(b, omb, v0[2], v1[2]), lerp1(b, omb, v0[3], v1[3])));
+#pragma unroll
+    for (int ch = 0; ch < 4; ++ch) hr[ch] = hn[ch];
+  }
+}
+
 template <class C, bool INT_COORD>
 __global__ void __launch_bounds__(256) k_sample_list(const SampleParams p) {
   const uint64_t s = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -476,6 +611,25 @@ static cudaError_t go_walk4(const SampleParams& p, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+#ifndef B2CL_C2M_XPT
+#define B2CL_C2M_XPT 2
+#endif
+#ifndef B2CL_C2M_RPW
+#define B2CL_C2M_RPW 4
+#endif
+#ifndef B2CL_TILE_TH
+#define B2CL_TILE_TH 16
+#endif
+template <class C, int TH>
+static cudaError_t go_tile(const SampleParams& p, cudaStream_t st) {
+  dim3 blk(128, 1, 1);
+  dim3 grd((p.ow + 63) / 64, (p.oh + TH - 1) / TH, p.od);
+  if (is_shard(p)) k_sample_grid_tile<WithShard<C, true>, 64, TH><<<grd, blk, 0, st>>>(p);
+  else k_sample_grid_tile<WithShard<C, false>, 64, TH><<<grd, blk, 0, st>>>(p);
+  count_launch();
+  return cudaGetLastError();
+}
+
 template <class C, int OUTC, int XPT, int RPW>
 static cudaError_t go_sep(const SampleParams& p, cudaStream_t st) {
   dim3 blk(32, 4, 1);
@@ -542,14 +696,18 @@ cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st
     // B2CL_GRID_KERNEL=general|sep|walk|4 forces a kernel family (A/B runs under ncu);
     // the default picks the variant measured fastest on B200 for each hot config
     static const char* force = getenv("B2CL_GRID_KERNEL");
-    const int fk = !force ? 0 : (force[0] == 'g' ? 1 : (force[0] == 's' ? 2 : (force[0] == 'w' ? 3 : (force[0] == '4' ? 4 : 0))));
+    const int fk = !force ? 0 : (force[0] == 'g' ? 1 : (force[0] == 's' ? 2 : (force[0] == 'w' ? 3 : (force[0] == '4' ? 4 : (force[0] == 't' ? 5 : 0)))));
     if (p.arr)  // image arrays: the general kernel, fully run-time format and sampler
       return p.dims == 1 ? go_grid<Layered<Generic<1>>, RT>(p, st) : go_grid<Layered<Generic<2>>, RT>(p, st);
     if (separable(p) && fk != 1) {
       if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_REPEAT, F_LINEAR))
-        return fk == 3 ? go_walk<C2Repeat, 4, 2, 8>(p, st) : go_sep<C2Repeat, 4, 2, 4>(p, st);
+        return fk == 3   ? go_walk<C2Repeat, 4, 2, 8>(p, st)
+               : fk == 2 ? go_sep<C2Repeat, 4, 2, 4>(p, st)
+                         : go_tile<C2Repeat, B2CL_TILE_TH>(p, st);
       if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_MIRROR, F_LINEAR))
-        return fk == 3 ? go_walk<C2Mirror, 4, 2, 8>(p, st) : go_sep<C2Mirror, 4, 2, 4>(p, st);
+        return fk == 3   ? go_walk<C2Mirror, 4, 2, 8>(p, st)
+               : fk == 5 ? go_tile<C2Mirror, B2CL_TILE_TH>(p, st)
+                         : go_sep<C2Mirror, 4, B2CL_C2M_XPT, B2CL_C2M_RPW>(p, st);
       if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR))
         return fk == 2   ? go_sep<C3Cte, 1, 4, 4>(p, st)
                : fk == 3 ? go_walk<C3Cte, 1, B2CL_C3_XPT, B2CL_C3_WALK>(p, st)
