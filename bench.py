@@ -313,7 +313,7 @@ def run_gpu(args):
     A = (ctypes.c_float * 12)(*Af.tolist())
     modes = ("repeat", "mirrored")
     codes = None
-    shard_rows, shard_host = [], []
+    shard_rows, shard_host, shard_begin = [], [], []
     if world == 1:
         codes = c2_codes()
         img = S.image(cl.CL_RGBA, cl.CL_FLOAT, N2D, N2D, host=codes)
@@ -325,6 +325,7 @@ def run_gpu(args):
             begin, count = circular_interval(need, Hg)
             rows = [(begin + s) % Hg for s in range(count)]
             shard_rows.append(count)
+            shard_begin.append(begin)
             shard_host.append(synth.image_rows(cl.CL_RGBA, cl.CL_FLOAT, N2D, rows))
             imgs.append(S.image_shard(cl.CL_RGBA, cl.CL_FLOAT, N2D, Hg, 0, begin, count, 0,
                                       host=shard_host[-1]))
@@ -334,9 +335,10 @@ def run_gpu(args):
             S.sampler(True, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR)]
     origin, region = cl.sz3((0, r0, 0)), cl.sz3((N2D, N2D, 1))
 
-    def launch(k):
-        cl.check(L.b2clEnqueueReadImageGridRegion(S.queue, imgs[k], smps[k], cl.B2CL_RTYPE_FLOAT, A,
-                                                  origin, region, 4, outs[k], 0, 0, None, None),
+    def launch(k, images=None):
+        cl.check(L.b2clEnqueueReadImageGridRegion(S.queue, (images or imgs)[k], smps[k],
+                                                  cl.B2CL_RTYPE_FLOAT, A, origin, region, 4, outs[k],
+                                                  0, 0, None, None),
                  "read grid")
 
     # ---- parity spot check of this exact launch configuration (bench as test) ----
@@ -417,45 +419,91 @@ def run_gpu(args):
         traffic = json.load(open(profs[-1])).get("dram_bytes_per_launch")
 
     # ---- e2e: host buffers through the C-ABI, copies inside the timed region ----
+    # Every step uploads its image(s) from pinned host memory and reads both
+    # outputs back to pinned host memory.  The copies are the step's bound
+    # (256 MiB up, 512 MiB down over the host link per GPU), so the step is
+    # pipelined the way an OpenCL program would: uploads on a second queue
+    # into one of two image copies, so step s+1's upload runs while step s's
+    # results come down; cross-queue order by events only (wait lists).
     e2e = None
     if not args.no_e2e:
-        # the image(s) every step uploads from pinned host memory: the whole
-        # image at N = 1, the two shards (their stored rows) at N > 1
-        uploads = []
-        for k, im in enumerate(imgs[:1] if world == 1 else imgs):
+        q_up = S.queue_for(gpu)
+        hbufs = []
+        for k in range(1 if world == 1 else 2):
             hrows = N2D if world == 1 else shard_rows[k]
             hbuf = torch.empty(hrows * N2D * 16, dtype=torch.uint8).pin_memory()
             src = codes if world == 1 else shard_host[k]
             hbuf.copy_(torch.from_numpy(np.ascontiguousarray(src).reshape(-1).view(np.uint8)))
-            uploads.append((im, hbuf, cl.sz3((N2D, hrows, 1))))
+            hbufs.append((hbuf, cl.sz3((N2D, hrows, 1))))
+        # two device copies of the step's images (copy 0 is the resident one)
+        e2e_imgs = [imgs]
+        if world == 1:
+            im2 = S.image(cl.CL_RGBA, cl.CL_FLOAT, N2D, N2D)
+            e2e_imgs.append([im2, im2])
+        else:
+            e2e_imgs.append([S.image_shard(cl.CL_RGBA, cl.CL_FLOAT, N2D, Hg, 0, shard_begin[k],
+                                           shard_rows[k], 0) for k in range(2)])
         host_out = [torch.empty(nout, dtype=torch.uint8).pin_memory() for _ in range(2)]
         zero3 = cl.sz3((0, 0, 0))
+        done = [None, None]  # marker event of the last step that read image copy b
 
-        def e2e_step():
-            for im, hbuf, reg in uploads:
-                cl.check(L.clEnqueueWriteImage(S.queue, im, 0, zero3, reg, 0, 0,
-                                               ctypes.c_void_p(hbuf.data_ptr()), 0, None, None))
+        def e2e_step(s, first_wait=None):
+            b = s % 2
+            wl = [e for e in (done[b], first_wait) if e]
+            wla = (ctypes.c_void_p * 2)(*wl) if wl else None
+            up = ctypes.c_void_p()
+            targets = e2e_imgs[b][:1] if world == 1 else e2e_imgs[b]
+            for k, (im, (hbuf, reg)) in enumerate(zip(targets, hbufs)):
+                last = k == len(hbufs) - 1
+                cl.check(L.clEnqueueWriteImage(q_up, im, 0, zero3, reg, 0, 0,
+                                               ctypes.c_void_p(hbuf.data_ptr()), len(wl), wla,
+                                               ctypes.byref(up) if last else None))
+            upa = (ctypes.c_void_p * 1)(up)
+            cl.check(L.clEnqueueBarrierWithWaitList(S.queue, 1, upa, None))
+            L.clReleaseEvent(up)
             for k in range(2):
-                launch(k)
+                launch(k, e2e_imgs[b])
                 cl.check(L.clEnqueueReadBuffer(S.queue, outs[k], 0, 0, nout,
                                                ctypes.c_void_p(host_out[k].data_ptr()), 0, None, None))
-            S.finish()
-        for _ in range(2):
-            e2e_step()
+            ev = ctypes.c_void_p()
+            cl.check(L.clEnqueueMarkerWithWaitList(S.queue, 0, None, ctypes.byref(ev)))
+            if done[b]:
+                L.clReleaseEvent(done[b])
+            done[b] = ev.value
+
+        for s in range(2):
+            e2e_step(s)
+        S.finish()
+        cl.check(L.clFinish(q_up))
         if world > 1:
             dist.barrier()
-        steps_e2e = max(3, args.steps // 4)
+        steps_e2e = max(4, args.steps // 4)
         a = T.event()
-        for _ in range(steps_e2e):
-            e2e_step()
-        b = T.event()
+        start = ctypes.c_void_p()  # the first upload starts after the start event
+        cl.check(L.clEnqueueMarkerWithWaitList(S.queue, 0, None, ctypes.byref(start)))
+        for s in range(steps_e2e):
+            e2e_step(s, start.value if s == 0 else None)
+        b_ev = T.event()
         torch.cuda.synchronize(dev)
-        e2e_ms = a.elapsed_time(b) / steps_e2e
+        cl.check(L.clFinish(q_up))
+        L.clReleaseEvent(start)
+        for e in done:
+            if e:
+                L.clReleaseEvent(e)
+        e2e_ms = a.elapsed_time(b_ev) / steps_e2e
         if world > 1:
             e2e_ms = bdist.max_over_ranks(e2e_ms, red_dev)
+        # the downloaded results are this step's: spot-check one row of each pass
+        for k in range(2):
+            dev_row = S.read(outs[k], N2D * 16, np.uint8, offset=N2D * 16 * 777)
+            assert np.array_equal(host_out[k].numpy()[N2D * 16 * 777:N2D * 16 * 778], dev_row)
         e2e = {"value": world * samples_step / (e2e_ms * 1e-3) / 1e9, "unit": "Gsamples/s",
-               "ms_per_step": e2e_ms, "h2d_bytes_per_step": int(sum(u[1].numel() for u in uploads)),
-               "d2h_bytes_per_step": 2 * nout}
+               "ms_per_step": e2e_ms, "h2d_bytes_per_step": int(sum(h[0].numel() for h in hbufs)),
+               "d2h_bytes_per_step": 2 * nout,
+               "pipeline": "uploads on a second queue into two image copies, overlapping the previous "
+                           "step's downloads (event-ordered)"}
+        S.release(*[im for im in set(e2e_imgs[1])])
+        L.clReleaseCommandQueue(q_up)
 
     secondary = None
     if not args.no_secondary:
