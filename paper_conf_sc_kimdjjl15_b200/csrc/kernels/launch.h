@@ -54,6 +54,9 @@ enum RectMode : int { RECT_COPY = 0, RECT_FILL = 1, RECT_FILL_IMAGE = 2, RECT_CO
 cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t stream);
 cudaError_t launch_rect(RectParams& p, int mode, cudaStream_t stream);
 cudaError_t launch_write(const WriteParams& p, cudaStream_t stream);
+// config-3 TMA-staged trilinear kernel (sample_vol.cu); *used = false when
+// the call does not qualify (nothing enqueued)
+cudaError_t launch_sample_vol(const SampleParams& p, cudaStream_t stream, bool* used);
 
 // count of kernels launched by this library
 uint64_t launch_count();

@@ -693,7 +693,7 @@ static bool separable(const SampleParams& p) {
 cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st) {
   if (coord_mode == COORD_GRID) {
     if ((uint64_t)p.ow * p.oh * p.od == 0) return cudaSuccess;
-    // B2CL_GRID_KERNEL=general|sep|walk|4 forces a kernel family (A/B runs under ncu);
+    // B2CL_GRID_KERNEL=general|sep|walk|4|tile forces a kernel family (A/B runs under ncu);
     // the default picks the variant measured fastest on B200 for each hot config
     static const char* force = getenv("B2CL_GRID_KERNEL");
     const int fk = !force ? 0 : (force[0] == 'g' ? 1 : (force[0] == 's' ? 2 : (force[0] == 'w' ? 3 : (force[0] == '4' ? 4 : (force[0] == 't' ? 5 : 0)))));
@@ -708,10 +708,16 @@ cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st
         return fk == 3   ? go_walk<C2Mirror, 4, 2, 8>(p, st)
                : fk == 5 ? go_tile<C2Mirror, B2CL_TILE_TH>(p, st)
                          : go_sep<C2Mirror, 4, B2CL_C2M_XPT, B2CL_C2M_RPW>(p, st);
-      if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR))
+      if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR)) {
+        if (fk == 0 && !is_shard(p)) {
+          bool used = false;
+          const cudaError_t e = launch_sample_vol(p, st, &used);
+          if (used || e != cudaSuccess) return e;
+        }
         return fk == 2   ? go_sep<C3Cte, 1, 4, 4>(p, st)
                : fk == 3 ? go_walk<C3Cte, 1, B2CL_C3_XPT, B2CL_C3_WALK>(p, st)
                          : go_walk4<C3Cte, B2CL_C3_WALK>(p, st);
+      }
       if (p.outc == 4 && matches<2>(p, T_UNORM8, O_RGBA, 0, A_CLAMP, F_NEAREST)) return go_sep<C1Clamp, 4, 2, 4>(p, st);
       switch (p.dims) {
         case 1: return go_sep<Generic<1>, RT, 2, 2>(p, st);

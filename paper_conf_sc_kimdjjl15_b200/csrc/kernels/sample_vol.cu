@@ -1,0 +1,455 @@
+// sample_vol.cu -- TMA-staged trilinear read of one-channel 32-bit float 3D
+// images under separable maps (config 3: 512^3 R32F, CLAMP_TO_EDGE, LINEAR).
+//
+// Steps a3-a7 of the read built-in ([CL1.2 §8.1-8.2]) for every output of a
+// 128 x 16 x WALK box, with the texel fetches (a5: through the
+// CLImage pointer) moved by the Tensor Memory Accelerator:
+//   * a persistent grid of CTAs strides over output tiles; each CTA has one
+//     PRODUCER warp (one elected lane) and four CONSUMER warps;
+//   * per output slice the producer brings the tile's texel footprint in that
+//     slice -- a (132 x 17)-texel box starting at the tile's first tap (i0 of
+//     its first column, rounded down to 16 bytes as TMA requires, and of its
+//     first row) -- into a shared-memory ring with one
+//     cp.async.bulk.tensor.3d (out-of-image box parts arrive as zeros, which
+//     is the border texel, A8), completing on a `full` mbarrier;
+//   * consumers x-blend each staged texel row once, y-blend neighbouring rows,
+//     keep the (x,y)-blended slice in registers and z-blend it with the next
+//     one, then release the stage on an `empty` mbarrier.
+// Bytes in flight are the ring (STAGES x 8.9 KB per CTA), independent of
+// registers -- the limit of the register-pipelined walk kernels.
+//
+// Exactness.  Every output is computed with the operations and operands of
+// linear_at (read.cuh): per texel row lerp1(a, 1-a, T[i0], T[i1]), then
+// lerp1(b, ..) of the rows j0, j1, then lerp1(g, ..) of the slices k0, k1,
+// with the per-axis AxL of axis_l -- so the results are bit-identical to the
+// other grid kernels (the parity tests run all of them).  A thread whose taps
+// fall outside the staged box (non-unit maps, fp rounding at a tile edge)
+// fetches those samples from global memory instead, still in lock-step with
+// the ring.  Slices are consumed in walk order: the map's z coordinate must
+// be non-decreasing in the output z (A[10] >= 0, host check), so with the
+// monotone CLAMP_TO_EDGE addressing the slice pair (k0, k1) only moves
+// forward and each slice is staged once per tile.
+#include <cudaTypedefs.h>
+
+#include <mutex>
+
+#include "../device/read.cuh"
+#include "launch.h"
+
+namespace b2cl {
+using namespace dev;
+
+#ifndef B2CL_VOL_NS
+#define B2CL_VOL_NS 4
+#endif
+#ifndef B2CL_VOL_MIN_STEPS
+#define B2CL_VOL_MIN_STEPS 8
+#endif
+#ifndef B2CL_VOL_MINB
+#define B2CL_VOL_MINB 4
+#endif
+constexpr int VT_W = 128;                 // output columns per tile (32 lanes x 4)
+constexpr int VT_H = 16;                  // output rows per tile (4 warps x 4)
+constexpr int VB_W = 132;                 // staged texel columns (TW + 1, rounded to 16 B)
+constexpr int VB_H = VT_H + 1;            // staged texel rows
+constexpr int VB_BYTES = VB_W * VB_H * 4; // one TMA box
+constexpr int VB_STRIDE = (VB_BYTES + 127) / 128 * 128;
+constexpr int VOL_NS = B2CL_VOL_NS;       // ring stages
+constexpr int VOL_MIN_STEPS = B2CL_VOL_MIN_STEPS;  // fewest column steps per CTA
+constexpr int VOL_THREADS = 160;          // 4 consumer warps + 1 producer warp
+
+struct VolTiles {
+  int ntx, nty, nzc;  // tiles along x and y, slice chunks along z
+  int walk;           // output slices per chunk
+  int vst;            // 1: 16-byte output stores allowed (ow % 4 == 0, out 16-B aligned)
+};
+
+__device__ __forceinline__ uint32_t vol_smem(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+#ifndef B2CL_VOL_HINT
+#define B2CL_VOL_HINT 0
+#endif
+__device__ __forceinline__ void vol_wait(uint64_t* bar, uint32_t parity) {
+  const uint32_t b = vol_smem(bar);
+  uint32_t done;
+  do {
+#if B2CL_VOL_HINT
+    asm volatile(
+        "{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2, %3; selp.u32 %0, 1, 0, P; }"
+        : "=r"(done)
+        : "r"(b), "r"(parity), "r"(B2CL_VOL_HINT)
+        : "memory");
+#else
+    asm volatile(
+        "{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2; selp.u32 %0, 1, 0, P; }"
+        : "=r"(done)
+        : "r"(b), "r"(parity)
+        : "memory");
+#endif
+  } while (!done);
+}
+
+template <class C>
+__device__ __forceinline__ AxL vol_axis(const SampleParams& p, int a, int o, int idx, int n) {
+  // coordinate of output index `idx` (region origin o) on a separable axis:
+  // A[a] * idx + A[a + 2 or 3]: the same two ops as k_sample_grid_sep
+  return axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[a], __int2float_rn(o + idx)), p.A[a == 0 ? 3 : (a == 5 ? 7 : 11)]), n);
+}
+
+// Do the taps of columns xc..xc+3 and of row yr (those inside the output
+// region) fall inside the box staged at (xb, yb)?  A tile is staged only if
+// this holds for all its columns and rows (decided identically by the
+// producer warp and the consumer warps).
+template <class C>
+__device__ __forceinline__ bool vol_in_window(const SampleParams& p, int xc, int yr, int xb, int yb) {
+  bool ok = true;
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    if (xc + u < p.ow) {
+      const AxL a = vol_axis<C>(p, 0, p.ox, xc + u, p.im.w);
+      ok = ok && a.i0 - xb >= 0 && a.i0 - xb < VB_W && a.i1 - xb >= 0 && a.i1 - xb < VB_W;
+    }
+  }
+  if (yr < p.oh) {
+    const AxL a = vol_axis<C>(p, 5, p.oy, yr, p.im.h);
+    ok = ok && a.i0 - yb >= 0 && a.i0 - yb < VB_H && a.i1 - yb >= 0 && a.i1 - yb < VB_H;
+  }
+  return ok;
+}
+
+// Work split.  Tiles are (tx, ty, zc): 128 x 16 output columns/rows and a
+// chunk of `walk` output slices, ordered tx fastest, then ty, then zc, and
+// dealt round-robin to a persistent grid, so the CTAs resident at any time
+// read neighbouring boxes of the same slices (DRAM pages and the shared halo
+// rows stay hot).  The host picks the chunk count as a multiple of
+// G / gcd(G, tiles per slice plane) so every CTA gets the same number of tiles.
+struct VolSeg {
+  int tx, ty, w0, nst;  // tile column, first output slice, steps
+};
+
+__device__ __forceinline__ VolSeg vol_seg(const SampleParams& p, const VolTiles& tl, int t) {
+  VolSeg q;
+  q.tx = t % tl.ntx;
+  const int r = t / tl.ntx;
+  q.ty = r % tl.nty;
+  q.w0 = (r / tl.nty) * tl.walk;
+  q.nst = min(tl.walk, p.od - q.w0);
+  return q;
+}
+
+template <class C>
+__global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
+    k_sample_grid_vol(const SampleParams p, const VolTiles tl, const __grid_constant__ CUtensorMap tmap) {
+  static_assert(C::dims == 3 && C::nch == 1 && C::type == T_FLOAT, "R32F-type 3D images");
+  extern __shared__ __align__(128) unsigned char vol_buf[];
+  __shared__ uint64_t full[VOL_NS], empty[VOL_NS];
+  __shared__ float4 rowtab[4][4];  // per consumer warp and row: {b, 1-b, slot j0, slot j1}
+  const Image& im = p.im;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < VOL_NS; ++s) {
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(vol_smem(&full[s])) : "memory");
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 4;" ::"r"(vol_smem(&empty[s])) : "memory");
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  __syncthreads();
+  const int ntiles = tl.ntx * tl.nty * tl.nzc;
+  constexpr int NONE = -2147483647 - 1;
+
+  if (warp == 4) {  // ------------------------------------------------ producer
+    if (lane == 0) asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmap)) : "memory");
+    int s = 0;
+    uint32_t ph = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      const VolSeg q = vol_seg(p, tl, t);
+      const int xb = vol_axis<C>(p, 0, p.ox, q.tx * VT_W, im.w).i0 & ~3;  // 16-B aligned box start
+      const int yb = vol_axis<C>(p, 5, p.oy, q.ty * VT_H, im.h).i0;
+      // the consumers' tile decision, evaluated the same way by this warp
+      if (!__all_sync(0xffffffffu, vol_in_window<C>(p, q.tx * VT_W + 4 * lane, q.ty * VT_H + (lane & 15), xb, yb)))
+        continue;
+      if (lane != 0) continue;
+      int kA = NONE, kB = NONE;
+      for (int w = 0; w < q.nst; ++w) {
+        const AxL az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
+        // the slices a step stages: lo unless held, then hi unless held
+        const bool need0 = !(az.i0 == kA || az.i0 == kB);
+        const bool need1 = !(az.i1 == az.i0 || az.i1 == kB);
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          if (!(h ? need1 : need0)) continue;
+          const int k = h ? az.i1 : az.i0;
+          vol_wait(&empty[s], ph ^ 1u);
+          const uint32_t fb = vol_smem(&full[s]);
+          asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(VB_BYTES)
+                       : "memory");
+          asm volatile(
+              "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+              " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(vol_smem(vol_buf + s * VB_STRIDE)),
+              "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(xb), "r"(yb), "r"(k), "r"(fb)
+              : "memory");
+          if (++s == VOL_NS) { s = 0; ph ^= 1u; }
+        }
+        kA = az.i0;
+        kB = az.i1;
+      }
+    }
+    return;
+  }
+
+  // --------------------------------------------------------------- consumers
+  int s = 0;
+  uint32_t ph = 0;
+  for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    const VolSeg q = vol_seg(p, tl, t);
+    const int xt = q.tx * VT_W, yt = q.ty * VT_H;
+    const int xb = vol_axis<C>(p, 0, p.ox, xt, im.w).i0 & ~3;  // as the producer's
+    const int yb = vol_axis<C>(p, 5, p.oy, yt, im.h).i0;
+    // this thread: columns xt + 4*lane + (0..3), rows yt + 4*warp + (0..3)
+    const int xc = xt + 4 * lane, yr = yt + 4 * warp;
+    // tile decision: every consumer thread tests its columns and row
+    // threadIdx.x & 15 (so the 128 threads cover the 16 rows as the producer's lanes do)
+    int fast = vol_in_window<C>(p, xc, yt + (threadIdx.x & 15), xb, yb);
+    asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, 128, P; selp.s32 %0, 1, 0, Q; }"
+                 : "=r"(fast) : "r"(fast) : "memory");
+    if (!fast) {  // the taps directly (linear_at), no staging for this tile
+#pragma unroll 1
+      for (int w = 0; w < q.nst; ++w) {
+        const int z = q.w0 + w;
+        const AxL az = vol_axis<C>(p, 10, p.oz, z, im.d);
+#pragma unroll 1
+        for (int r = 0; r < 4; ++r) {
+          const int y = yr + r;
+          if (y >= p.oh) break;
+          const AxL ay = vol_axis<C>(p, 5, p.oy, y, im.h);
+          const char* rows[4] = {row_ptr<C>(im, ay.i0, az.i0), row_ptr<C>(im, ay.i1, az.i0),
+                                 row_ptr<C>(im, ay.i0, az.i1), row_ptr<C>(im, ay.i1, az.i1)};
+          const bool rok[4] = {ay.ok0 && az.ok0, ay.ok1 && az.ok0, ay.ok0 && az.ok1, ay.ok1 && az.ok1};
+#pragma unroll 1
+          for (int u = 0; u < 4; ++u) {
+            if (xc + u >= p.ow) break;
+            uint32_t res[4];
+            linear_at<C>(p, rows, rok, vol_axis<C>(p, 0, p.ox, xc + u, im.w), ay.a, ay.oma, az.a, az.oma, res, 1);
+            __stcs(reinterpret_cast<float*>(p.out) + ((uint64_t)z * p.oh + y) * p.ow + xc + u,
+                   __uint_as_float(res[0]));
+          }
+        }
+      }
+      continue;
+    }
+    // x axis per thread; the warp's 4 rows (warp-uniform) in shared memory
+    AxL ax[4];
+    int sl[4];  // staged column slots of tap i0 | i1 << 16
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      ax[u] = vol_axis<C>(p, 0, p.ox, xc + u, im.w);
+      // (columns / rows outside the output region: slots clamped, never stored)
+      sl[u] = min(max(ax[u].i0 - xb, 0), VB_W - 1) | min(max(ax[u].i1 - xb, 0), VB_W - 1) << 16;
+    }
+    __syncwarp();  // the previous segment's row table is no longer read
+    if (lane < 4) {
+      const AxL ay = vol_axis<C>(p, 5, p.oy, yr + lane, im.h);
+      rowtab[warp][lane] = make_float4(ay.a, ay.oma, __int_as_float(min(max(ay.i0 - yb, 0), VB_H - 1)),
+                                       __int_as_float(min(max(ay.i1 - yb, 0), VB_H - 1)));
+    }
+    __syncwarp();
+    // 16-byte row segments: four unit-stride column taps starting 16-B aligned
+    const int c0 = sl[0] & 0xffff;
+    bool vecx = (c0 & 3) == 0 && c0 + 4 < VB_W;
+#pragma unroll
+    for (int u = 0; u < 4; ++u) vecx = vecx && sl[u] == ((c0 + u) | (c0 + u + 1) << 16);
+    // the 4 rows of the warp chain (j1 of row r is j0 of row r+1): 5 texel rows
+    bool rchain = true;
+#pragma unroll
+    for (int r = 0; r < 3; ++r) rchain = rchain && rowtab[warp][r].w == rowtab[warp][r + 1].z;
+
+    // x-blend of staged texel row j for the 4 columns
+    auto xblend = [&](const float* buf, float jf, float h[4]) {
+      const float* row = buf + __float_as_int(jf) * VB_W;
+      float T0[4], T1[4];
+      if (vecx) {
+        const float4 v = *reinterpret_cast<const float4*>(row + c0);
+        T0[0] = v.x; T0[1] = v.y; T0[2] = v.z; T0[3] = v.w;
+        T1[0] = v.y; T1[1] = v.z; T1[2] = v.w; T1[3] = row[c0 + 4];
+      } else {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) { T0[u] = row[sl[u] & 0xffff]; T1[u] = row[sl[u] >> 16]; }
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) h[u] = lerp1(ax[u].a, ax[u].oma, T0[u], T1[u]);
+    };
+    // the (x,y)-blended slice of the next ring stage: V[row][column]
+    auto slice = [&](float V[4][4]) {
+      vol_wait(&full[s], ph);
+      const float* buf = reinterpret_cast<const float*>(vol_buf + s * VB_STRIDE);
+      float Hp[4], Hn[4];
+      if (rchain) {
+        xblend(buf, rowtab[warp][0].z, Hp);
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+          const float4 ry = rowtab[warp][r];
+          xblend(buf, ry.w, Hn);
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            V[r][u] = lerp1(ry.x, ry.y, Hp[u], Hn[u]);
+            Hp[u] = Hn[u];
+          }
+        }
+      } else {
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+          const float4 ry = rowtab[warp][r];
+          xblend(buf, ry.z, Hp);
+          xblend(buf, ry.w, Hn);
+#pragma unroll
+          for (int u = 0; u < 4; ++u) V[r][u] = lerp1(ry.x, ry.y, Hp[u], Hn[u]);
+        }
+      }
+      __syncwarp();
+      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(vol_smem(&empty[s])) : "memory");
+      if (++s == VOL_NS) { s = 0; ph ^= 1u; }
+    };
+    auto copy = [](float D[4][4], const float S[4][4]) {
+#pragma unroll
+      for (int r = 0; r < 4; ++r)
+#pragma unroll
+        for (int u = 0; u < 4; ++u) D[r][u] = S[r][u];
+    };
+    // output rows of the thread (a row outside the region is not stored)
+    const bool vst = tl.vst && xc + 3 < p.ow;
+    int rmask = 0;
+#pragma unroll
+    for (int r = 0; r < 4; ++r) rmask |= (yr + r < p.oh) << r;
+    float* orow = reinterpret_cast<float*>(p.out) + ((uint64_t)(q.w0) * p.oh + yr) * p.ow + xc;
+    const uint64_t zstride = (uint64_t)p.oh * p.ow;
+    int kA = NONE, kB = NONE;
+    // One step with X holding slice kA and Y slice kB (the previous step's lo,
+    // hi); it leaves lo in Y and hi in X, so the next step swaps the roles --
+    // the common unit-stride step (lo = previous hi, one new hi) copies nothing.
+    auto step = [&](int w, float X[4][4], float Y[4][4]) {
+      const AxL az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
+      if (az.i0 == kA && az.i1 == kB && az.i0 != az.i1) {  // both held, in place: swap
+#pragma unroll
+        for (int r = 0; r < 4; ++r)
+#pragma unroll
+          for (int u = 0; u < 4; ++u) { const float t = X[r][u]; X[r][u] = Y[r][u]; Y[r][u] = t; }
+      } else {
+        if (az.i0 == kB) {
+        } else if (az.i0 == kA) {
+          copy(Y, X);
+        } else {
+          slice(Y);
+        }
+        if (az.i1 == az.i0) copy(X, Y);
+        else slice(X);
+      }
+      kA = az.i0;
+      kB = az.i1;
+#pragma unroll
+      for (int r = 0; r < 4; ++r) {
+        if (!(rmask >> r & 1)) break;
+        float o[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) o[u] = lerp1(az.a, az.oma, Y[r][u], X[r][u]);
+        float* op = orow + (uint64_t)r * p.ow;
+        if (vst) {
+          __stcs(reinterpret_cast<float4*>(op), make_float4(o[0], o[1], o[2], o[3]));
+        } else {
+#pragma unroll
+          for (int u = 0; u < 4; ++u)
+            if (xc + u < p.ow) __stcs(op + u, o[u]);
+        }
+      }
+      orow += zstride;
+    };
+    float VA[4][4], VB[4][4];
+#pragma unroll 1
+    for (int w = 0; w < q.nst; w += 2) {
+      step(w, VA, VB);
+      if (w + 1 < q.nst) step(w + 1, VB, VA);
+    }
+  }
+}
+
+// ------------------------------------------------------------------ host
+static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
+  });
+  return fn;
+}
+
+// the image's texels as a 3D fp32 tensor (w, h, d) with its pitches, read in
+// (VB_W x VB_H x 1) boxes; out-of-range box elements are filled with zeros
+static bool vol_tensor_map(const Image& im, CUtensorMap* m) {
+  auto enc = encode_fn();
+  if (!enc) return false;
+  if ((reinterpret_cast<uintptr_t>(im.ptr) & 15) || (im.rp & 15) || (im.sp & 15)) return false;
+  const cuuint64_t dims[3] = {(cuuint64_t)im.w, (cuuint64_t)im.h, (cuuint64_t)im.d};
+  const cuuint64_t strides[2] = {im.rp, im.sp};
+  const cuuint32_t box[3] = {VB_W, VB_H, 1};
+  const cuuint32_t es[3] = {1, 1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, im.ptr, dims, strides, box, es,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// Launch the TMA kernel for config C if the call qualifies (plain image,
+// non-decreasing z map, encodable tensor); *used = false otherwise.
+template <class C>
+static cudaError_t go_vol(const SampleParams& p, cudaStream_t st, bool* used) {
+  *used = false;
+  if (!(p.A[10] >= 0.0f)) return cudaSuccess;
+  CUtensorMap tm;
+  if (!vol_tensor_map(p.im, &tm)) return cudaSuccess;
+  static int sms[64] = {0}, occ = 0;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const size_t smem = (size_t)VOL_NS * VB_STRIDE;
+  if (dev < 0 || dev >= 64) return cudaSuccess;
+  if (!sms[dev]) {
+    cudaFuncSetAttribute(k_sample_grid_vol<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaDeviceGetAttribute(&sms[dev], cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sample_grid_vol<C>, VOL_THREADS, smem);
+    if (occ < 1) occ = 1;
+  }
+  VolTiles tl;
+  tl.ntx = (p.ow + VT_W - 1) / VT_W;
+  tl.nty = (p.oh + VT_H - 1) / VT_H;
+  tl.vst = (p.ow & 3) == 0 && (reinterpret_cast<uintptr_t>(p.out) & 15) == 0;
+  // one CTA per resident slot; chunks: a multiple of G / gcd(G, ntx*nty) so
+  // the tiles split evenly, each chunk at least VOL_MIN_STEPS slices long
+  const long long plane = (long long)tl.ntx * tl.nty;
+  if (plane * p.od > 0x7fffffffLL) return cudaSuccess;
+  long long G = (long long)sms[dev] * occ;
+  long long a = G, b = plane;
+  while (b) { const long long t = a % b; a = b; b = t; }
+  const long long unit = G / a;  // chunks per balanced round
+  long long nzc = unit;
+  while (nzc * 2 <= p.od / VOL_MIN_STEPS && nzc * 2 <= 4 * unit) nzc *= 2;
+  if ((p.od + nzc - 1) / nzc < VOL_MIN_STEPS) nzc = std::max<long long>(1, p.od / VOL_MIN_STEPS);
+  tl.walk = (int)((p.od + nzc - 1) / nzc);
+  tl.nzc = (p.od + tl.walk - 1) / tl.walk;
+  const int grid = (int)std::max<long long>(1, std::min<long long>(G, plane * tl.nzc));
+  k_sample_grid_vol<C><<<grid, VOL_THREADS, smem, st>>>(p, tl, tm);
+  count_launch();
+  *used = true;
+  return cudaGetLastError();
+}
+
+using C3CteV = WithShard<Cfg<3, T_FLOAT, O_R, 1, A_CTE, F_LINEAR, R_F>, false>;
+
+cudaError_t launch_sample_vol(const SampleParams& p, cudaStream_t st, bool* used) {
+  return go_vol<C3CteV>(p, st, used);
+}
+
+}  // namespace b2cl

@@ -186,6 +186,14 @@ GRID_CASES = [
     # texel of the last lane comes from the next 16 bytes), output width not /4
     (3, R, F32, (260, 4, 19), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "stencil+1", (258, 4, 19), 1),
     (3, R, F32, (260, 4, 19), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "stencil+4", (250, 4, 19), 1),
+    # config-3 TMA kernel (k_sample_grid_vol): ragged tiles on every axis; a
+    # 2x magnification (taps shared by neighbouring outputs and slices: scalar
+    # slots, unchained rows, repeated z pairs); 2x minification (taps outside
+    # the staged box: direct tiles); a z map running backwards (other kernel)
+    (3, R, F32, (300, 37, 40), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "stencil", (300, 37, 40), 1),
+    (3, R, F32, (70, 45, 30), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "magnify", (150, 40, 50), 1),
+    (3, R, F32, (300, 60, 40), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "scale2", (150, 33, 21), 1),
+    (3, R, F32, (140, 20, 24), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "stencil-zneg", (140, 20, 24), 1),
 ]
 
 
@@ -200,6 +208,17 @@ def _affine(kind, size, out):
         A[0], A[3] = 2.0 / W, -0.3 / W
         A[5], A[7] = 2.0 / H, 0.45 / H
         A[10], A[11] = 2.0 / D, -0.2 / D
+        return A
+    if kind == "magnify":  # 2x magnification, separable, offset by a fraction of a texel
+        A = np.zeros(12, np.float32)
+        A[0], A[3] = 0.5 / W, 0.37 / W
+        A[5], A[7] = 0.5 / H, 0.81 / H
+        A[10], A[11] = 0.5 / D, 0.13 / D
+        return A
+    if kind == "stencil-zneg":  # z runs backwards through the volume
+        A = synth.affine_stencil_3d(W)
+        A[5], A[7] = 1.0 / H, (0.5 + 0.6) / H
+        A[10], A[11] = -1.0 / D, (D - 0.5 + 0.2) / D
         return A
     if kind == "rotate3d":
         return synth.affine_rotate_3d(W, 20.0)
