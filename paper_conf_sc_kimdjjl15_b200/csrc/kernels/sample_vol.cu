@@ -2,20 +2,21 @@
 // images under separable maps (config 3: 512^3 R32F, CLAMP_TO_EDGE, LINEAR).
 //
 // Steps a3-a7 of the read built-in ([CL1.2 §8.1-8.2]) for every output of a
-// 128 x 16 x WALK box, with the texel fetches (a5: through the
-// CLImage pointer) moved by the Tensor Memory Accelerator:
+// 256 x 8 x walk box, with the texel fetches (a5: through the CLImage
+// pointer) moved by the TMA engine:
 //   * a persistent grid of CTAs strides over output tiles; each CTA has one
-//     PRODUCER warp (one elected lane) and four CONSUMER warps;
-//   * per output slice the producer brings the tile's texel footprint in that
-//     slice -- a (132 x 17)-texel box starting at the tile's first tap (i0 of
-//     its first column, rounded down to 16 bytes as TMA requires, and of its
-//     first row) -- into a shared-memory ring with one
-//     cp.async.bulk.tensor.3d (out-of-image box parts arrive as zeros, which
-//     is the border texel, A8), completing on a `full` mbarrier;
+//     PRODUCER warp and four CONSUMER warps;
+//   * per output slice the producer stages the tile's texel footprint in that
+//     slice -- a (260 x 9)-texel box starting at the tile's first tap (i0 of
+//     its first column rounded down to 16 bytes, and of its first row) -- in a
+//     shared-memory ring: one cp.async.bulk per box row (one per lane),
+//     completing on a `full` mbarrier.  (B2CL_VOL_BULK=0 builds the 132 x 17
+//     variant that moves each box with one cp.async.bulk.tensor.3d; on B200
+//     it measured 196 us against 189 us for the row copies at config 3.)
 //   * consumers x-blend each staged texel row once, y-blend neighbouring rows,
 //     keep the (x,y)-blended slice in registers and z-blend it with the next
 //     one, then release the stage on an `empty` mbarrier.
-// Bytes in flight are the ring (STAGES x 8.9 KB per CTA), independent of
+// Bytes in flight are the ring (STAGES x 9.4 KB per CTA), independent of
 // registers -- the limit of the register-pipelined walk kernels.
 //
 // Exactness.  Every output is computed with the operations and operands of
@@ -31,6 +32,7 @@
 // forward and each slice is staged once per tile.
 #include <cudaTypedefs.h>
 
+#include <cstring>
 #include <mutex>
 
 #include "../device/read.cuh"
@@ -39,8 +41,11 @@
 namespace b2cl {
 using namespace dev;
 
+#ifndef B2CL_VOL_BULK
+#define B2CL_VOL_BULK 1
+#endif
 #ifndef B2CL_VOL_NS
-#define B2CL_VOL_NS 4
+#define B2CL_VOL_NS 3
 #endif
 #ifndef B2CL_VOL_MIN_STEPS
 #define B2CL_VOL_MIN_STEPS 8
@@ -48,9 +53,14 @@ using namespace dev;
 #ifndef B2CL_VOL_MINB
 #define B2CL_VOL_MINB 4
 #endif
-constexpr int VT_W = 128;                 // output columns per tile (32 lanes x 4)
-constexpr int VT_H = 16;                  // output rows per tile (4 warps x 4)
-constexpr int VB_W = 132;                 // staged texel columns (TW + 1, rounded to 16 B)
+#ifndef B2CL_VOL_XW
+#define B2CL_VOL_XW 2
+#endif
+constexpr int VOL_XW = B2CL_VOL_XW;       // consumer warps across x (1: TMA boxes; 4: row copies)
+static_assert(VOL_XW == 1 || B2CL_VOL_BULK, "a TMA box is at most 256 texels wide");
+constexpr int VT_W = 128 * VOL_XW;        // output columns per tile (32 lanes x 4 per warp)
+constexpr int VT_H = 16 / VOL_XW;         // output rows per tile (4 per warp)
+constexpr int VB_W = VT_W + 4;            // staged texel columns (TW + 1, from a 16-B aligned start)
 constexpr int VB_H = VT_H + 1;            // staged texel rows
 constexpr int VB_BYTES = VB_W * VB_H * 4; // one TMA box
 constexpr int VB_STRIDE = (VB_BYTES + 127) / 128 * 128;
@@ -143,6 +153,8 @@ template <class C>
 __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
     k_sample_grid_vol(const SampleParams p, const VolTiles tl, const __grid_constant__ CUtensorMap tmap) {
   static_assert(C::dims == 3 && C::nch == 1 && C::type == T_FLOAT, "R32F-type 3D images");
+  // row copies stage only texels inside the image: exact when no tap leaves it
+  static_assert(!B2CL_VOL_BULK || C::addr == A_CTE, "row copies need CLAMP_TO_EDGE");
   extern __shared__ __align__(128) unsigned char vol_buf[];
   __shared__ uint64_t full[VOL_NS], empty[VOL_NS];
   __shared__ float4 rowtab[4][4];  // per consumer warp and row: {b, 1-b, slot j0, slot j1}
@@ -169,9 +181,14 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
       const int xb = vol_axis<C>(p, 0, p.ox, q.tx * VT_W, im.w).i0 & ~3;  // 16-B aligned box start
       const int yb = vol_axis<C>(p, 5, p.oy, q.ty * VT_H, im.h).i0;
       // the consumers' tile decision, evaluated the same way by this warp
-      if (!__all_sync(0xffffffffu, vol_in_window<C>(p, q.tx * VT_W + 4 * lane, q.ty * VT_H + (lane & 15), xb, yb)))
-        continue;
+      bool win = true;
+#pragma unroll
+      for (int m = 0; m < VOL_XW; ++m)
+        win = win && vol_in_window<C>(p, q.tx * VT_W + 128 * m + 4 * lane, q.ty * VT_H + lane % VT_H, xb, yb);
+      if (!__all_sync(0xffffffffu, win)) continue;
+#if !B2CL_VOL_BULK
       if (lane != 0) continue;
+#endif
       int kA = NONE, kB = NONE;
       for (int w = 0; w < q.nst; ++w) {
         const AxL az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
@@ -182,8 +199,27 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
         for (int h = 0; h < 2; ++h) {
           if (!(h ? need1 : need0)) continue;
           const int k = h ? az.i1 : az.i0;
-          vol_wait(&empty[s], ph ^ 1u);
           const uint32_t fb = vol_smem(&full[s]);
+#if B2CL_VOL_BULK
+          // one plain bulk copy per box row (lanes 0..16), rows inside the
+          // image only, each clipped to its row pitch (CLAMP_TO_EDGE: the
+          // taps never reach the unfilled parts)
+          const int nrow = min(VB_H, im.h - yb);
+          const uint32_t rb = (uint32_t)min((uint64_t)VB_W * 4u, im.rp - (uint64_t)xb * 4u);
+          if (lane == 0) {
+            vol_wait(&empty[s], ph ^ 1u);
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(rb * nrow)
+                         : "memory");
+          }
+          __syncwarp();
+          if (lane < nrow)
+            asm volatile(
+                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                    vol_smem(vol_buf + s * VB_STRIDE + lane * VB_W * 4)),
+                "l"(im.ptr + (uint64_t)k * im.sp + (uint64_t)(yb + lane) * im.rp + (uint64_t)xb * 4u), "r"(rb), "r"(fb)
+                : "memory");
+#else
+          vol_wait(&empty[s], ph ^ 1u);
           asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(VB_BYTES)
                        : "memory");
           asm volatile(
@@ -191,6 +227,7 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
               " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(vol_smem(vol_buf + s * VB_STRIDE)),
               "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(xb), "r"(yb), "r"(k), "r"(fb)
               : "memory");
+#endif
           if (++s == VOL_NS) { s = 0; ph ^= 1u; }
         }
         kA = az.i0;
@@ -209,10 +246,10 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
     const int xb = vol_axis<C>(p, 0, p.ox, xt, im.w).i0 & ~3;  // as the producer's
     const int yb = vol_axis<C>(p, 5, p.oy, yt, im.h).i0;
     // this thread: columns xt + 4*lane + (0..3), rows yt + 4*warp + (0..3)
-    const int xc = xt + 4 * lane, yr = yt + 4 * warp;
+    const int xc = xt + 128 * (warp % VOL_XW) + 4 * lane, yr = yt + 4 * (warp / VOL_XW);
     // tile decision: every consumer thread tests its columns and row
-    // threadIdx.x & 15 (so the 128 threads cover the 16 rows as the producer's lanes do)
-    int fast = vol_in_window<C>(p, xc, yt + (threadIdx.x & 15), xb, yb);
+    // threadIdx.x % VT_H (so the 128 threads cover the tile's rows as the producer's lanes do)
+    int fast = vol_in_window<C>(p, xc, yt + threadIdx.x % VT_H, xb, yb);
     asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, 128, P; selp.s32 %0, 1, 0, Q; }"
                  : "=r"(fast) : "r"(fast) : "memory");
     if (!fast) {  // the taps directly (linear_at), no staging for this tile
@@ -286,7 +323,11 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
       vol_wait(&full[s], ph);
       const float* buf = reinterpret_cast<const float*>(vol_buf + s * VB_STRIDE);
       float Hp[4], Hn[4];
+#ifdef B2CL_VOL_NOCOMPUTE  // A/B experiment only: the ring without the blends
+      if (buf[lane] == 12345.f) {
+#else
       if (rchain) {
+#endif
         xblend(buf, rowtab[warp][0].z, Hp);
 #pragma unroll
         for (int r = 0; r < 4; ++r) {
@@ -326,35 +367,18 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
     float* orow = reinterpret_cast<float*>(p.out) + ((uint64_t)(q.w0) * p.oh + yr) * p.ow + xc;
     const uint64_t zstride = (uint64_t)p.oh * p.ow;
     int kA = NONE, kB = NONE;
-    // One step with X holding slice kA and Y slice kB (the previous step's lo,
-    // hi); it leaves lo in Y and hi in X, so the next step swaps the roles --
-    // the common unit-stride step (lo = previous hi, one new hi) copies nothing.
-    auto step = [&](int w, float X[4][4], float Y[4][4]) {
-      const AxL az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
-      if (az.i0 == kA && az.i1 == kB && az.i0 != az.i1) {  // both held, in place: swap
-#pragma unroll
-        for (int r = 0; r < 4; ++r)
-#pragma unroll
-          for (int u = 0; u < 4; ++u) { const float t = X[r][u]; X[r][u] = Y[r][u]; Y[r][u] = t; }
-      } else {
-        if (az.i0 == kB) {
-        } else if (az.i0 == kA) {
-          copy(Y, X);
-        } else {
-          slice(Y);
-        }
-        if (az.i1 == az.i0) copy(X, Y);
-        else slice(X);
-      }
-      kA = az.i0;
-      kB = az.i1;
+    // z-blend of the held slices lo (L) and hi (H) into the 4 output rows
+    auto emit = [&](const AxL& az, const float L[4][4], const float H[4][4]) {
 #pragma unroll
       for (int r = 0; r < 4; ++r) {
         if (!(rmask >> r & 1)) break;
         float o[4];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) o[u] = lerp1(az.a, az.oma, Y[r][u], X[r][u]);
+        for (int u = 0; u < 4; ++u) o[u] = lerp1(az.a, az.oma, L[r][u], H[r][u]);
         float* op = orow + (uint64_t)r * p.ow;
+#ifdef B2CL_VOL_NOSTORE  // A/B experiment only: read side alone
+        if (o[0] != 12345.f) continue;
+#endif
         if (vst) {
           __stcs(reinterpret_cast<float4*>(op), make_float4(o[0], o[1], o[2], o[3]));
         } else {
@@ -365,11 +389,60 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
       }
       orow += zstride;
     };
+    // VA holds slice kA (the previous step's lo), VB slice kB (its hi).  The
+    // common unit-stride step -- lo = the previous hi, one new hi -- stages
+    // the new slice over the old lo and swaps the roles; two such steps
+    // restore them, so a run of common steps copies nothing.  Any other step
+    // (the first of a tile, clamped or repeated indices) goes through the
+    // general step, which keeps the roles; the producer stages the same
+    // slices in the same order (lo unless held, then hi unless held).
     float VA[4][4], VB[4][4];
+    int w = 0;
 #pragma unroll 1
-    for (int w = 0; w < q.nst; w += 2) {
-      step(w, VA, VB);
-      if (w + 1 < q.nst) step(w + 1, VB, VA);
+    while (w < q.nst) {
+      AxL az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
+      if (az.i0 == kB && az.i1 != az.i0) {
+        slice(VA);
+        emit(az, VB, VA);
+        kA = az.i0;
+        kB = az.i1;
+        if (++w < q.nst) {
+          az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
+          if (az.i0 == kB && az.i1 != az.i0) {
+            slice(VB);
+            emit(az, VA, VB);
+            kA = az.i0;
+            kB = az.i1;
+            ++w;
+            continue;
+          }
+        }
+#pragma unroll
+        for (int r = 0; r < 4; ++r)
+#pragma unroll
+          for (int u = 0; u < 4; ++u) { const float t = VA[r][u]; VA[r][u] = VB[r][u]; VB[r][u] = t; }
+        if (w >= q.nst) break;
+      }
+      // general step: lo into VA, hi into VB, staging only what is not held
+      int hb = kB;  // slice held in VB
+#pragma unroll 1
+      for (int h = 0; h < 2; ++h) {
+        const int k = h ? az.i1 : az.i0;
+        if (h == 0) {
+          if (k == kA) continue;
+          if (k == kB) { copy(VA, VB); continue; }
+        } else {
+          if (k == hb) continue;
+          if (k == az.i0) { copy(VB, VA); continue; }
+        }
+        slice(VB);
+        hb = k;
+        if (h == 0) copy(VA, VB);
+      }
+      kA = az.i0;
+      kB = az.i1;
+      emit(az, VA, VB);
+      ++w;
     }
   }
 }
@@ -410,7 +483,12 @@ static cudaError_t go_vol(const SampleParams& p, cudaStream_t st, bool* used) {
   *used = false;
   if (!(p.A[10] >= 0.0f)) return cudaSuccess;
   CUtensorMap tm;
-  if (!vol_tensor_map(p.im, &tm)) return cudaSuccess;
+  if (B2CL_VOL_BULK) {  // row copies: no tensor map (16-B aligned rows needed)
+    memset(&tm, 0, sizeof(tm));
+    if ((reinterpret_cast<uintptr_t>(p.im.ptr) & 15) || (p.im.rp & 15) || (p.im.sp & 15)) return cudaSuccess;
+  } else if (!vol_tensor_map(p.im, &tm)) {
+    return cudaSuccess;
+  }
   static int sms[64] = {0}, occ = 0;
   int dev = 0;
   cudaGetDevice(&dev);
