@@ -41,6 +41,14 @@ __device__ __forceinline__ int layer_of(float c, int n) {
   return min(max(__float2int_rn(c), 0), n - 1);
 }
 
+// coordinate of output (x,y,z) under the affine map: ((A0*x + A1*y) + A2*z) + A3
+__device__ __forceinline__ float affine_coord(const float* A, float x, float y, float z) {
+  float v = __fmul_rn(A[0], x);
+  v = __fadd_rn(v, __fmul_rn(A[1], y));
+  v = __fadd_rn(v, __fmul_rn(A[2], z));
+  return __fadd_rn(v, A[3]);
+}
+
 struct AxN {  // NEAREST, one axis
   int i;
   bool ok;

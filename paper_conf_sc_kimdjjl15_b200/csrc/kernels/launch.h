@@ -57,6 +57,8 @@ cudaError_t launch_write(const WriteParams& p, cudaStream_t stream);
 // config-3 TMA-staged trilinear kernel (sample_vol.cu); *used = false when
 // the call does not qualify (nothing enqueued)
 cudaError_t launch_sample_vol(const SampleParams& p, cudaStream_t stream, bool* used);
+// ... and its rotated-map variant (x, y any affine in the output x, y; z separable)
+cudaError_t launch_sample_volr(const SampleParams& p, cudaStream_t stream, bool* used);
 
 // count of kernels launched by this library
 uint64_t launch_count();

@@ -28,14 +28,6 @@
 namespace b2cl {
 using namespace dev;
 
-// coordinate of output (x,y,z) under the affine map: ((A0*x + A1*y) + A2*z) + A3
-__device__ __forceinline__ float affine_coord(const float* A, float x, float y, float z) {
-  float v = __fmul_rn(A[0], x);
-  v = __fadd_rn(v, __fmul_rn(A[1], y));
-  v = __fadd_rn(v, __fmul_rn(A[2], z));
-  return __fadd_rn(v, A[3]);
-}
-
 template <int OUTC>
 __device__ __forceinline__ void store_out(const SampleParams& p, uint64_t idx, const uint32_t r[4]) {
   const int outc = OUTC == RT ? p.outc : OUTC;
@@ -727,7 +719,14 @@ cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st
     }
     if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_REPEAT, F_LINEAR)) return go_grid<C2Repeat, 4>(p, st);
     if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_MIRROR, F_LINEAR)) return go_grid<C2Mirror, 4>(p, st);
-    if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR)) return go_grid<C3Cte, 1>(p, st);
+    if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR)) {
+      if (fk == 0 && !is_shard(p)) {
+        bool used = false;
+        const cudaError_t e = launch_sample_volr(p, st, &used);
+        if (used || e != cudaSuccess) return e;
+      }
+      return go_grid<C3Cte, 1>(p, st);
+    }
     switch (p.dims) {
       case 1: return go_grid<Generic<1>, RT>(p, st);
       case 2: return go_grid<Generic<2>, RT>(p, st);

@@ -32,6 +32,7 @@
 // forward and each slice is staged once per tile.
 #include <cudaTypedefs.h>
 
+#include <cmath>
 #include <cstring>
 #include <mutex>
 
@@ -447,6 +448,245 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
   }
 }
 
+// ===================================================================
+// Rotated maps (config 3 map B, volume rendering): the x and y coordinates
+// are any affine function of the output (x, y) and the z coordinate depends
+// on the output z alone (A[2] = A[6] = A[8] = A[9] = 0).  The z axis is then
+// walked exactly as above -- (x,y)-blended slices held in registers, one new
+// slice per common step -- while the (x,y) footprint of a 64 x 32 output tile
+// is the bounding box of the taps of its four corners (the fp32 coordinate is
+// monotone in x and in y separately, and so are the axis indices): at most
+// RB_W x RB_H texels, staged per slice by one cp.async.bulk per box row.  Each
+// sample keeps its own tap offsets and weights (8 samples per thread, one
+// column and 8 rows), the blend order is linear_at's: bit-identical results.
+#ifndef B2CL_VOLR_NS
+#define B2CL_VOLR_NS 3
+#endif
+#ifndef B2CL_VOLR_MINB
+#define B2CL_VOLR_MINB 2
+#endif
+constexpr int RT_W = 64, RT_H = 32;           // output tile
+constexpr int RB_MAXW = 128, RB_MAXH = 128;   // largest staged box (texels)
+constexpr int VOLR_NS = B2CL_VOLR_NS;
+constexpr int VOLR_THREADS = 288;             // 8 consumer warps + 1 producer warp
+constexpr int VOLR_S = 8;                     // samples (rows) per consumer thread
+
+struct VolrBox {
+  int xb, yb;    // first staged texel column (16-B aligned) and row
+  int ok;        // 0: the footprint exceeds the launch's box (bw x bh)
+};
+
+struct VolrGeom {
+  int bw, bh;    // staged box (texels), chosen per launch from the map's footprint
+  int stride;    // bytes per ring stage (128-B multiple)
+};
+
+// the tile's staged box from its corners' taps (identical in every warp)
+template <class C>
+__device__ __forceinline__ VolrBox volr_box(const SampleParams& p, const VolrGeom& g, int x0, int y0, int z,
+                                            int lane) {
+  const int x1 = min(x0 + RT_W, p.ow) - 1, y1 = min(y0 + RT_H, p.oh) - 1;
+  const int cx = (lane & 1) ? x1 : x0, cy = (lane & 2) ? y1 : y0;
+  const float xf = __int2float_rn(p.ox + cx), yf = __int2float_rn(p.oy + cy), zf = __int2float_rn(p.oz + z);
+  const AxL ax = axis_l<C>(p.smp, affine_coord(p.A, xf, yf, zf), p.im.w);
+  const AxL ay = axis_l<C>(p.smp, affine_coord(p.A + 4, xf, yf, zf), p.im.h);
+  int xmin = min(ax.i0, ax.i1), xmax = max(ax.i0, ax.i1), ymin = min(ay.i0, ay.i1), ymax = max(ay.i0, ay.i1);
+#pragma unroll
+  for (int o = 1; o < 4; o <<= 1) {
+    xmin = min(xmin, __shfl_xor_sync(0xffffffffu, xmin, o));
+    xmax = max(xmax, __shfl_xor_sync(0xffffffffu, xmax, o));
+    ymin = min(ymin, __shfl_xor_sync(0xffffffffu, ymin, o));
+    ymax = max(ymax, __shfl_xor_sync(0xffffffffu, ymax, o));
+  }
+  VolrBox b;
+  b.xb = __shfl_sync(0xffffffffu, xmin, 0) & ~3;
+  b.yb = __shfl_sync(0xffffffffu, ymin, 0);
+  b.ok = __shfl_sync(0xffffffffu, xmax, 0) - b.xb < g.bw && __shfl_sync(0xffffffffu, ymax, 0) - b.yb < g.bh;
+  return b;
+}
+
+template <class C>
+__global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
+    k_sample_grid_volr(const SampleParams p, const VolTiles tl, const VolrGeom g,
+                       const __grid_constant__ CUtensorMap tmap) {
+  static_assert(C::dims == 3 && C::nch == 1 && C::type == T_FLOAT && C::addr == A_CTE, "R32F, CLAMP_TO_EDGE");
+  extern __shared__ __align__(128) unsigned char volr_buf[];
+  __shared__ uint64_t full[VOLR_NS], empty[VOLR_NS];
+  const Image& im = p.im;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < VOLR_NS; ++s) {
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(vol_smem(&full[s])) : "memory");
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 8;" ::"r"(vol_smem(&empty[s])) : "memory");
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  __syncthreads();
+  const int ntiles = tl.ntx * tl.nty * tl.nzc;
+  constexpr int NONE = -2147483647 - 1;
+
+  if (warp == 8) {  // ------------------------------------------------ producer
+    int s = 0;
+    uint32_t ph = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      const VolSeg q = vol_seg(p, tl, t);
+      const VolrBox bx = volr_box<C>(p, g, q.tx * RT_W, q.ty * RT_H, q.w0, lane);
+      if (!bx.ok || lane != 0) continue;  // (not ok: the consumers read this tile directly)
+      int kA = NONE, kB = NONE;
+      for (int w = 0; w < q.nst; ++w) {
+        const AxL az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
+        const bool need0 = !(az.i0 == kA || az.i0 == kB);
+        const bool need1 = !(az.i1 == az.i0 || az.i1 == kB);
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          if (!(h ? need1 : need0)) continue;
+          const int k = h ? az.i1 : az.i0;
+          const uint32_t fb = vol_smem(&full[s]);
+          vol_wait(&empty[s], ph ^ 1u);
+          asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(g.bw * g.bh * 4)
+                       : "memory");
+          asm volatile(
+              "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+              " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(vol_smem(volr_buf + s * g.stride)),
+              "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(bx.xb), "r"(bx.yb), "r"(k), "r"(fb)
+              : "memory");
+          if (++s == VOLR_NS) { s = 0; ph ^= 1u; }
+        }
+        kA = az.i0;
+        kB = az.i1;
+      }
+    }
+    return;
+  }
+
+  // --------------------------------------------------------------- consumers
+  int s = 0;
+  uint32_t ph = 0;
+  const int col = threadIdx.x & (RT_W - 1), rg = threadIdx.x / RT_W;  // column, row group of 8
+  for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    const VolSeg q = vol_seg(p, tl, t);
+    const int x = q.tx * RT_W + col, y0 = q.ty * RT_H + rg * VOLR_S;
+    const VolrBox bx = volr_box<C>(p, g, q.tx * RT_W, q.ty * RT_H, q.w0, lane);
+    // per sample: packed staged offset of tap (j0, i0) | (i1 - i0) << 16 | (j1 != j0) << 17, and the weights
+    int off[VOLR_S];
+    float wa[VOLR_S], wb[VOLR_S];
+    int in = bx.ok;
+    const float xf = __int2float_rn(p.ox + x), zf = __int2float_rn(p.oz + q.w0);
+#pragma unroll
+    for (int r = 0; r < VOLR_S; ++r) {
+      const float yf = __int2float_rn(p.oy + y0 + r);
+      const AxL ax = axis_l<C>(p.smp, affine_coord(p.A, xf, yf, zf), im.w);
+      const AxL ay = axis_l<C>(p.smp, affine_coord(p.A + 4, xf, yf, zf), im.h);
+      const int sx0 = ax.i0 - bx.xb, sx1 = ax.i1 - bx.xb, sy0 = ay.i0 - bx.yb, sy1 = ay.i1 - bx.yb;
+      const bool v = x < p.ow && y0 + r < p.oh;
+      const bool ok = sx0 >= 0 && sx1 >= sx0 && sx1 - sx0 <= 1 && sx1 < g.bw && sy0 >= 0 && sy1 >= sy0 &&
+                      sy1 - sy0 <= 1 && sy1 < g.bh;
+      in = in && (ok || !v);
+      off[r] = ok ? (sy0 * g.bw + sx0) | (sx1 - sx0) << 16 | (sy1 - sy0) << 17 : 0;
+      wa[r] = ax.a;
+      wb[r] = ay.a;
+    }
+    int fast;
+    asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, 256, P; selp.s32 %0, 1, 0, Q; }"
+                 : "=r"(fast) : "r"(in) : "memory");
+    if (!fast) {  // the taps directly (read_image, the general kernel's coordinates)
+#pragma unroll 1
+      for (int w = 0; w < q.nst; ++w) {
+        const int z = q.w0 + w;
+#pragma unroll 1
+        for (int r = 0; r < VOLR_S; ++r) {
+          const int y = y0 + r;
+          if (x >= p.ow || y >= p.oh) break;
+          const float xf2 = __int2float_rn(p.ox + x), yf2 = __int2float_rn(p.oy + y), zf2 = __int2float_rn(p.oz + z);
+          const float c[3] = {affine_coord(p.A, xf2, yf2, zf2), affine_coord(p.A + 4, xf2, yf2, zf2),
+                              affine_coord(p.A + 8, xf2, yf2, zf2)};
+          uint32_t res[4];
+          read_image<C>(p, c, res, 1);
+          __stcs(reinterpret_cast<float*>(p.out) + ((uint64_t)z * p.oh + y) * p.ow + x, __uint_as_float(res[0]));
+        }
+      }
+      continue;
+    }
+    auto slice = [&](float V[VOLR_S]) {
+      vol_wait(&full[s], ph);
+      const float* buf = reinterpret_cast<const float*>(volr_buf + s * g.stride);
+#pragma unroll
+      for (int r = 0; r < VOLR_S; ++r) {
+        const float* t0 = buf + (off[r] & 0xffff);
+        const int dx = off[r] >> 16 & 1, dy = (off[r] >> 17) * g.bw;
+        const float oma = __fsub_rn(1.0f, wa[r]), omb = __fsub_rn(1.0f, wb[r]);
+        const float h0 = lerp1(wa[r], oma, t0[0], t0[dx]);
+        const float h1 = lerp1(wa[r], oma, t0[dy], t0[dy + dx]);
+        V[r] = lerp1(wb[r], omb, h0, h1);
+      }
+      __syncwarp();
+      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(vol_smem(&empty[s])) : "memory");
+      if (++s == VOLR_NS) { s = 0; ph ^= 1u; }
+    };
+    float* orow = reinterpret_cast<float*>(p.out) + ((uint64_t)q.w0 * p.oh + y0) * p.ow + x;
+    const uint64_t zstride = (uint64_t)p.oh * p.ow;
+    int nrow = x < p.ow ? min(VOLR_S, p.oh - y0) : 0;
+    auto emit = [&](const AxL& az, const float L[VOLR_S], const float H[VOLR_S]) {
+#pragma unroll
+      for (int r = 0; r < VOLR_S; ++r)
+        if (r < nrow) __stcs(orow + (uint64_t)r * p.ow, lerp1(az.a, az.oma, L[r], H[r]));
+      orow += zstride;
+    };
+    auto copy = [](float D[VOLR_S], const float S[VOLR_S]) {
+#pragma unroll
+      for (int r = 0; r < VOLR_S; ++r) D[r] = S[r];
+    };
+    // the z walk of k_sample_grid_vol (same roles, same staging order)
+    float VA[VOLR_S], VB[VOLR_S];
+    int kA = NONE, kB = NONE;
+    int w = 0;
+#pragma unroll 1
+    while (w < q.nst) {
+      AxL az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
+      if (az.i0 == kB && az.i1 != az.i0) {
+        slice(VA);
+        emit(az, VB, VA);
+        kA = az.i0;
+        kB = az.i1;
+        if (++w < q.nst) {
+          az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
+          if (az.i0 == kB && az.i1 != az.i0) {
+            slice(VB);
+            emit(az, VA, VB);
+            kA = az.i0;
+            kB = az.i1;
+            ++w;
+            continue;
+          }
+        }
+#pragma unroll
+        for (int r = 0; r < VOLR_S; ++r) { const float tt = VA[r]; VA[r] = VB[r]; VB[r] = tt; }
+        if (w >= q.nst) break;
+      }
+      int hb = kB;
+#pragma unroll 1
+      for (int h = 0; h < 2; ++h) {
+        const int k = h ? az.i1 : az.i0;
+        if (h == 0) {
+          if (k == kA) continue;
+          if (k == kB) { copy(VA, VB); continue; }
+        } else {
+          if (k == hb) continue;
+          if (k == az.i0) { copy(VB, VA); continue; }
+        }
+        slice(VB);
+        hb = k;
+        if (h == 0) copy(VA, VB);
+      }
+      kA = az.i0;
+      kB = az.i1;
+      emit(az, VA, VB);
+      ++w;
+    }
+  }
+}
+
 // ------------------------------------------------------------------ host
 static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
@@ -476,6 +716,40 @@ static bool vol_tensor_map(const Image& im, CUtensorMap* m) {
              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// Persistent-grid plan shared by the staged kernels: one CTA per resident
+// slot; z chunks: a multiple of G / gcd(G, tiles per plane) so the tiles
+// split evenly over the CTAs, each chunk at least VOL_MIN_STEPS slices long.
+static bool vol_plan(const SampleParams& p, int tw, int th, const void* fn, int threads, size_t smem, int* occ,
+                     VolTiles* tl, int* grid) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) return false;
+  static int sms[64] = {0};
+  if (!occ[dev]) {
+    cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaDeviceGetAttribute(&sms[dev], cudaDevAttrMultiProcessorCount, dev);
+    int o = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, fn, threads, smem);
+    occ[dev] = o < 1 ? 1 : o;
+  }
+  tl->ntx = (p.ow + tw - 1) / tw;
+  tl->nty = (p.oh + th - 1) / th;
+  tl->vst = (p.ow & 3) == 0 && (reinterpret_cast<uintptr_t>(p.out) & 15) == 0;
+  const long long plane = (long long)tl->ntx * tl->nty;
+  if (plane * p.od > 0x7fffffffLL) return false;
+  const long long G = (long long)sms[dev] * occ[dev];
+  long long a = G, b = plane;
+  while (b) { const long long t = a % b; a = b; b = t; }
+  const long long unit = G / a;  // chunks per balanced round
+  long long nzc = unit;
+  while (nzc * 2 <= p.od / VOL_MIN_STEPS && nzc * 2 <= 4 * unit) nzc *= 2;
+  if ((p.od + nzc - 1) / nzc < VOL_MIN_STEPS) nzc = std::max<long long>(1, p.od / VOL_MIN_STEPS);
+  tl->walk = (int)((p.od + nzc - 1) / nzc);
+  tl->nzc = (p.od + tl->walk - 1) / tl->walk;
+  *grid = (int)std::max<long long>(1, std::min<long long>(G, plane * tl->nzc));
+  return true;
+}
+
 // Launch the TMA kernel for config C if the call qualifies (plain image,
 // non-decreasing z map, encodable tensor); *used = false otherwise.
 template <class C>
@@ -489,36 +763,57 @@ static cudaError_t go_vol(const SampleParams& p, cudaStream_t st, bool* used) {
   } else if (!vol_tensor_map(p.im, &tm)) {
     return cudaSuccess;
   }
-  static int sms[64] = {0}, occ = 0;
-  int dev = 0;
-  cudaGetDevice(&dev);
+  static int occ[64] = {0};
   const size_t smem = (size_t)VOL_NS * VB_STRIDE;
-  if (dev < 0 || dev >= 64) return cudaSuccess;
-  if (!sms[dev]) {
-    cudaFuncSetAttribute(k_sample_grid_vol<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    cudaDeviceGetAttribute(&sms[dev], cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sample_grid_vol<C>, VOL_THREADS, smem);
-    if (occ < 1) occ = 1;
-  }
   VolTiles tl;
-  tl.ntx = (p.ow + VT_W - 1) / VT_W;
-  tl.nty = (p.oh + VT_H - 1) / VT_H;
-  tl.vst = (p.ow & 3) == 0 && (reinterpret_cast<uintptr_t>(p.out) & 15) == 0;
-  // one CTA per resident slot; chunks: a multiple of G / gcd(G, ntx*nty) so
-  // the tiles split evenly, each chunk at least VOL_MIN_STEPS slices long
-  const long long plane = (long long)tl.ntx * tl.nty;
-  if (plane * p.od > 0x7fffffffLL) return cudaSuccess;
-  long long G = (long long)sms[dev] * occ;
-  long long a = G, b = plane;
-  while (b) { const long long t = a % b; a = b; b = t; }
-  const long long unit = G / a;  // chunks per balanced round
-  long long nzc = unit;
-  while (nzc * 2 <= p.od / VOL_MIN_STEPS && nzc * 2 <= 4 * unit) nzc *= 2;
-  if ((p.od + nzc - 1) / nzc < VOL_MIN_STEPS) nzc = std::max<long long>(1, p.od / VOL_MIN_STEPS);
-  tl.walk = (int)((p.od + nzc - 1) / nzc);
-  tl.nzc = (p.od + tl.walk - 1) / tl.walk;
-  const int grid = (int)std::max<long long>(1, std::min<long long>(G, plane * tl.nzc));
+  int grid = 0;
+  if (!vol_plan(p, VT_W, VT_H, reinterpret_cast<const void*>(k_sample_grid_vol<C>), VOL_THREADS, smem, occ, &tl,
+                &grid))
+    return cudaSuccess;
   k_sample_grid_vol<C><<<grid, VOL_THREADS, smem, st>>>(p, tl, tm);
+  count_launch();
+  *used = true;
+  return cudaGetLastError();
+}
+
+template <class C>
+static cudaError_t go_volr(const SampleParams& p, cudaStream_t st, bool* used) {
+  *used = false;
+  const float* A = p.A;
+  if (!(A[2] == 0.0f && A[6] == 0.0f && A[8] == 0.0f && A[9] == 0.0f && A[10] >= 0.0f)) return cudaSuccess;
+  // the box: the footprint of a tile, |d(texel)/d(output)| summed over the
+  // tile's extent, plus the LINEAR neighbour, 2 texels of rounding and the
+  // 16-byte alignment of its start (the kernel checks every tile against it)
+  const double sx = (p.smp.norm ? (double)p.im.w : 1.0), sy = (p.smp.norm ? (double)p.im.h : 1.0);
+  const double fw = (std::fabs((double)A[0]) * (RT_W - 1) + std::fabs((double)A[1]) * (RT_H - 1)) * sx;
+  const double fh = (std::fabs((double)A[4]) * (RT_W - 1) + std::fabs((double)A[5]) * (RT_H - 1)) * sy;
+  if (!(fw < RB_MAXW && fh < RB_MAXH)) return cudaSuccess;
+  VolrGeom g;
+  g.bw = std::min(RB_MAXW, ((int)std::ceil(fw) + 1 + 2 + 3 + 3) & ~3);
+  g.bh = std::min(RB_MAXH, (int)std::ceil(fh) + 1 + 2);
+  g.stride = (g.bw * g.bh * 4 + 127) & ~127;
+  auto enc = encode_fn();
+  if (!enc) return cudaSuccess;
+  const Image& im = p.im;
+  if ((reinterpret_cast<uintptr_t>(im.ptr) & 15) || (im.rp & 15) || (im.sp & 15)) return cudaSuccess;
+  CUtensorMap tm;
+  const cuuint64_t dims[3] = {(cuuint64_t)im.w, (cuuint64_t)im.h, (cuuint64_t)im.d};
+  const cuuint64_t strides[2] = {im.rp, im.sp};
+  const cuuint32_t box[3] = {(cuuint32_t)g.bw, (cuuint32_t)g.bh, 1};
+  const cuuint32_t es[3] = {1, 1, 1};
+  if (enc(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, im.ptr, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+          CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    return cudaSuccess;
+  int occ[64] = {0};  // (occupancy depends on this launch's box)
+  const size_t smem = (size_t)VOLR_NS * g.stride;
+  if (smem > 200 * 1024) return cudaSuccess;
+  VolTiles tl;
+  int grid = 0;
+  if (!vol_plan(p, RT_W, RT_H, reinterpret_cast<const void*>(k_sample_grid_volr<C>), VOLR_THREADS, smem, occ, &tl,
+                &grid))
+    return cudaSuccess;
+  k_sample_grid_volr<C><<<grid, VOLR_THREADS, smem, st>>>(p, tl, g, tm);
   count_launch();
   *used = true;
   return cudaGetLastError();
@@ -528,6 +823,10 @@ using C3CteV = WithShard<Cfg<3, T_FLOAT, O_R, 1, A_CTE, F_LINEAR, R_F>, false>;
 
 cudaError_t launch_sample_vol(const SampleParams& p, cudaStream_t st, bool* used) {
   return go_vol<C3CteV>(p, st, used);
+}
+
+cudaError_t launch_sample_volr(const SampleParams& p, cudaStream_t st, bool* used) {
+  return go_volr<C3CteV>(p, st, used);
 }
 
 }  // namespace b2cl

@@ -194,6 +194,12 @@ GRID_CASES = [
     (3, R, F32, (70, 45, 30), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "magnify", (150, 40, 50), 1),
     (3, R, F32, (300, 60, 40), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "scale2", (150, 33, 21), 1),
     (3, R, F32, (140, 20, 24), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "stencil-zneg", (140, 20, 24), 1),
+    # rotated-map staged kernel (k_sample_grid_volr): ragged tiles, the corners
+    # clamped to the edges; 3x minification (footprint larger than the box:
+    # direct tiles); z at half scale (repeated slice pairs)
+    (3, R, F32, (90, 90, 21), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d", (100, 70, 25), 1),
+    (3, R, F32, (90, 90, 21), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d-min", (70, 66, 9), 1),
+    (3, R, F32, (90, 90, 21), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d-zhalf", (130, 33, 30), 1),
 ]
 
 
@@ -219,6 +225,13 @@ def _affine(kind, size, out):
         A = synth.affine_stencil_3d(W)
         A[5], A[7] = 1.0 / H, (0.5 + 0.6) / H
         A[10], A[11] = -1.0 / D, (D - 0.5 + 0.2) / D
+        return A
+    if kind.startswith("rotate3d-"):
+        A = synth.affine_rotate_3d(W, 20.0)
+        if kind.endswith("min"):
+            A[[0, 1, 4, 5]] *= 3.0
+        else:
+            A[10] *= 0.5
         return A
     if kind == "rotate3d":
         return synth.affine_rotate_3d(W, 20.0)

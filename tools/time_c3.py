@@ -1,6 +1,6 @@
 """Time the config-3 read (512^3 R32F trilinear, stencil map) with CUDA events.
 
-    python tools/time_c3.py   (kernel variant chosen by the library's B2CL_TUNE env)
+    python tools/time_c3.py [rot]   (rot: the volume-render rotation, map B)
 """
 import ctypes
 import os
@@ -23,7 +23,8 @@ def main():
                   host=synth.image_codes(synth.rng(3), cl.CL_R, cl.CL_FLOAT, n, n, n))
     out = S.buffer(n ** 3 * 4)
     smp = S.sampler(True, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR)
-    A = (ctypes.c_float * 12)(*synth.affine_stencil_3d(n).tolist())
+    rot = len(sys.argv) > 1 and sys.argv[1] == "rot"
+    A = (ctypes.c_float * 12)(*(synth.affine_rotate_3d(n, 20.0) if rot else synth.affine_stencil_3d(n)).tolist())
     d = cl.sz3((n, n, n))
 
     def go():
@@ -37,7 +38,7 @@ def main():
     e1.record(st)
     torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / 20
-    print(f"variant {os.environ.get('B2CL_TUNE', '0')}: {ms * 1e3:.1f} us, "
+    print(f"{'rotated' if rot else 'stencil'}  {os.environ.get('B2CL_TUNE', '0')}: {ms * 1e3:.1f} us, "
           f"{n ** 3 / ms / 1e6:.1f} Gsamples/s, {2 * n ** 3 * 4 / ms / 1e6:.0f} GB/s")
 
 
