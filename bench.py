@@ -633,12 +633,19 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
         S.queue, vol, smp3, 0, A3, d3, 1, out3, 0, 0, None, None)), 10)
     byt = 2 * n3 ** 3 * 4
     res["c3_trilinear_512"] = {"Gsamples/s": n3 ** 3 / ms / 1e6, "ms": ms, "GB/s": byt / ms / 1e6,
-                               "hbm_frac": byt / ms / 1e6 / hbm_peak, "map": "stencil (A)"}
+                               "hbm_frac": byt / ms / 1e6 / hbm_peak, "map": "stencil (A)",
+                               "kernel": "k_sample_grid_vol (256x8 tiles, per-row cp.async.bulk ring)",
+                               "algorithmic_bytes": byt}
     A3b = (ctypes.c_float * 12)(*synth.affine_rotate_3d(n3, 20.0).tolist())
     ms = _time_launches(T, torch, dev, lambda: cl.check(L.b2clEnqueueReadImageGrid(
         S.queue, vol, smp3, 0, A3b, d3, 1, out3, 0, 0, None, None)), 10)
-    res["c3_trilinear_512_rotated"] = {"Gsamples/s": n3 ** 3 / ms / 1e6, "ms": ms,
-                                       "map": "volume-render rotation (B), 20 deg about z"}
+    # map (B): every texel whose tap weight is non-zero is read once (the
+    # rotated grid covers the volume's interior; clamped corners re-read edge
+    # texels) -- algorithmic bytes counted as 4 B in + 4 B out per sample
+    res["c3_trilinear_512_rotated"] = {"Gsamples/s": n3 ** 3 / ms / 1e6, "ms": ms, "GB/s": byt / ms / 1e6,
+                                       "hbm_frac": byt / ms / 1e6 / hbm_peak,
+                                       "map": "volume-render rotation (B), 20 deg about z",
+                                       "kernel": "k_sample_grid_volr (64x32 tiles, tensor-TMA footprint box)"}
     S.release(vol, out3)
     L.clReleaseSampler(smp3)
     # config 4: 8 GiB pitched CopyBufferRect (src padded, dst tight) and a misaligned variant

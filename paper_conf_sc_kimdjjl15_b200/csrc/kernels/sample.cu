@@ -21,6 +21,7 @@
 // time): the fully run-time instance covers every format x sampler; the
 // compile-time instances are the hot configurations of BASELINE.json.
 #include <atomic>
+#include <type_traits>
 
 #include "../device/read.cuh"
 #include "launch.h"
@@ -428,6 +429,7 @@ __global__ void __launch_bounds__(128) k_sample_grid_tile(const SampleParams p) 
   __shared__ __align__(16) float4 tile[TH + 1][TW + 1];
   __shared__ int colI0[TW], colI1[TW], rowJ0[TH], rowJ1[TH];
   __shared__ float colA[TW], colOma[TW], rowA[TH], rowOma[TH];
+  __shared__ float2 rowW[TH];  // (b, 1 - b) of each row, for the staged walk
   __shared__ int chain[4];  // columns up, columns down, rows up, rows down
   const Image& im = p.im;
   const int tid = threadIdx.x;
@@ -452,6 +454,7 @@ __global__ void __launch_bounds__(128) k_sample_grid_tile(const SampleParams p) 
     rowJ1[r] = ay.i1;
     rowA[r] = ay.a;
     rowOma[r] = ay.oma;
+    rowW[r] = make_float2(ay.a, ay.oma);
   }
   __syncthreads();
   if (tid < TW - 1) {
@@ -505,32 +508,41 @@ __global__ void __launch_bounds__(128) k_sample_grid_tile(const SampleParams p) 
   }
   asm volatile("cp.async.wait_all;" ::: "memory");
   __syncthreads();
-  // slots of tap i0 / i1 of this column, and of row tap j0 / j1 relative to r
+  // slots of tap i0 / i1 of this column; the row taps are slot rows r, r + 1
+  // (upward chain: j0 = r; downward: j1 = r).  One instance of the row walk
+  // per chain direction, so no per-sample selects.
   const int ci0 = cup ? c : c + 1, ci1 = cup ? c + 1 : c;
-  const int dj0 = rup ? 0 : 1, dj1 = rup ? 1 : 0;
-  auto xblend = [&](int r, float h[4]) {
-    const float4 t0 = tile[r][ci0], t1 = tile[r][ci1];
-    h[0] = lerp1(a, oma, t0.x, t1.x);
-    h[1] = lerp1(a, oma, t0.y, t1.y);
-    h[2] = lerp1(a, oma, t0.z, t1.z);
-    h[3] = lerp1(a, oma, t0.w, t1.w);
-  };
-  float hr[4], hn[4];  // x-blends of slot rows r and r + 1
-  xblend(r0, hr);
+  const int nrow = x < p.ow ? min(RPW, p.oh - (y0 + r0)) : 0;
+  float4* orow = out + ((zoff + y0 + r0) * p.ow + x);
+  auto walk = [&](auto up) {
+    constexpr bool UP = decltype(up)::value;
+    const float4* trow = &tile[r0][0];
+    auto xblend = [&](const float4* t, float h[4]) {
+      const float4 t0 = t[ci0], t1 = t[ci1];
+      h[0] = lerp1(a, oma, t0.x, t1.x);
+      h[1] = lerp1(a, oma, t0.y, t1.y);
+      h[2] = lerp1(a, oma, t0.z, t1.z);
+      h[3] = lerp1(a, oma, t0.w, t1.w);
+    };
+    float hr[4], hn[4];  // x-blends of slot rows r and r + 1
+    xblend(trow, hr);
 #pragma unroll 4
-  for (int r = r0; r < r0 + RPW; ++r) {
-    xblend(r + 1, hn);
-    const float b = rowA[r], omb = rowOma[r];
-    const float* v0 = dj0 ? hn : hr;  // the x-blend of row j0
-    const float* v1 = dj1 ? hn : hr;  // ... and of row j1
-    const int y = y0 + r;
-    if (x < p.ow && y < p.oh)
-      __stcs(out + ((zoff + y) * p.ow + x),
-             make_float4(lerp1(b, omb, v0[0], v1[0]), lerp1(b, omb, v0[1], v1[1]),
-                         lerp1(b, omb, v0[2], v1[2]), lerp1(b, omb, v0[3], v1[3])));
+    for (int r = 0; r < RPW; ++r) {
+      trow += TW + 1;
+      xblend(trow, hn);
+      const float2 bw = rowW[r0 + r];  // (b, 1 - b)
+      const float* v0 = UP ? hr : hn;  // the x-blend of row j0
+      const float* v1 = UP ? hn : hr;  // ... and of row j1
+      if (r < nrow)
+        __stcs(orow, make_float4(lerp1(bw.x, bw.y, v0[0], v1[0]), lerp1(bw.x, bw.y, v0[1], v1[1]),
+                                 lerp1(bw.x, bw.y, v0[2], v1[2]), lerp1(bw.x, bw.y, v0[3], v1[3])));
+      orow += p.ow;
 #pragma unroll
-    for (int ch = 0; ch < 4; ++ch) hr[ch] = hn[ch];
-  }
+      for (int ch = 0; ch < 4; ++ch) hr[ch] = hn[ch];
+    }
+  };
+  if (rup) walk(std::true_type{});
+  else walk(std::false_type{});
 }
 
 template <class C, bool INT_COORD>

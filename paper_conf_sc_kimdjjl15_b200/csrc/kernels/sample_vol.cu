@@ -195,7 +195,7 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
         const AxL az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
         // the slices a step stages: lo unless held, then hi unless held
         const bool need0 = !(az.i0 == kA || az.i0 == kB);
-        const bool need1 = !(az.i1 == az.i0 || az.i1 == kB);
+        const bool need1 = !(az.i1 == az.i0 || (!need0 && az.i1 == kB));  // the consumers' rule
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           if (!(h ? need1 : need0)) continue;
@@ -537,7 +537,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
       for (int w = 0; w < q.nst; ++w) {
         const AxL az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
         const bool need0 = !(az.i0 == kA || az.i0 == kB);
-        const bool need1 = !(az.i1 == az.i0 || az.i1 == kB);
+        const bool need1 = !(az.i1 == az.i0 || (!need0 && az.i1 == kB));  // the consumers' rule
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           if (!(h ? need1 : need0)) continue;
