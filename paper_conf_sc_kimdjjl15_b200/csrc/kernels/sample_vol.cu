@@ -2,21 +2,21 @@
 // images under separable maps (config 3: 512^3 R32F, CLAMP_TO_EDGE, LINEAR).
 //
 // Steps a3-a7 of the read built-in ([CL1.2 §8.1-8.2]) for every output of a
-// 256 x 8 x walk box, with the texel fetches (a5: through the CLImage
+// 256 x 16 x walk box, with the texel fetches (a5: through the CLImage
 // pointer) moved by the TMA engine:
 //   * a persistent grid of CTAs strides over output tiles; each CTA has one
-//     PRODUCER warp and four CONSUMER warps;
+//     PRODUCER warp and eight CONSUMER warps (2 across x, 4 down y);
 //   * per output slice the producer stages the tile's texel footprint in that
-//     slice -- a (260 x 9)-texel box starting at the tile's first tap (i0 of
+//     slice -- a (260 x 17)-texel box starting at the tile's first tap (i0 of
 //     its first column rounded down to 16 bytes, and of its first row) -- in a
 //     shared-memory ring: one cp.async.bulk per box row (one per lane),
 //     completing on a `full` mbarrier.  (B2CL_VOL_BULK=0 builds the 132 x 17
-//     variant that moves each box with one cp.async.bulk.tensor.3d; on B200
-//     it measured 196 us against 189 us for the row copies at config 3.)
+//     variant (with B2CL_VOL_XW=1) that moves each box with one cp.async.bulk.tensor.3d; on B200
+//     it measured 196 us against 186 us for the row copies at config 3.)
 //   * consumers x-blend each staged texel row once, y-blend neighbouring rows,
 //     keep the (x,y)-blended slice in registers and z-blend it with the next
 //     one, then release the stage on an `empty` mbarrier.
-// Bytes in flight are the ring (STAGES x 9.4 KB per CTA), independent of
+// Bytes in flight are the ring (STAGES x 17.7 KB per CTA), independent of
 // registers -- the limit of the register-pipelined walk kernels.
 //
 // Exactness.  Every output is computed with the operations and operands of
@@ -52,7 +52,7 @@ using namespace dev;
 #define B2CL_VOL_MIN_STEPS 8
 #endif
 #ifndef B2CL_VOL_MINB
-#define B2CL_VOL_MINB 4
+#define B2CL_VOL_MINB 2
 #endif
 #ifndef B2CL_VOL_XW
 #define B2CL_VOL_XW 2
@@ -60,14 +60,20 @@ using namespace dev;
 constexpr int VOL_XW = B2CL_VOL_XW;       // consumer warps across x (1: TMA boxes; 4: row copies)
 static_assert(VOL_XW == 1 || B2CL_VOL_BULK, "a TMA box is at most 256 texels wide");
 constexpr int VT_W = 128 * VOL_XW;        // output columns per tile (32 lanes x 4 per warp)
-constexpr int VT_H = 16 / VOL_XW;         // output rows per tile (4 per warp)
+#ifndef B2CL_VOL_YW
+#define B2CL_VOL_YW 4
+#endif
+constexpr int VOL_YW = B2CL_VOL_YW;       // consumer warps down y
+constexpr int VOL_CW = VOL_XW * VOL_YW;   // consumer warps
+constexpr int VT_H = 4 * VOL_YW;          // output rows per tile (4 per warp)
 constexpr int VB_W = VT_W + 4;            // staged texel columns (TW + 1, from a 16-B aligned start)
 constexpr int VB_H = VT_H + 1;            // staged texel rows
 constexpr int VB_BYTES = VB_W * VB_H * 4; // one TMA box
 constexpr int VB_STRIDE = (VB_BYTES + 127) / 128 * 128;
 constexpr int VOL_NS = B2CL_VOL_NS;       // ring stages
 constexpr int VOL_MIN_STEPS = B2CL_VOL_MIN_STEPS;  // fewest column steps per CTA
-constexpr int VOL_THREADS = 160;          // 4 consumer warps + 1 producer warp
+constexpr int VOL_THREADS = 32 * (VOL_CW + 1);  // consumer warps + 1 producer warp
+static_assert(VT_H < 32, "the producer's lanes cover the tile's rows");
 
 struct VolTiles {
   int ntx, nty, nzc;  // tiles along x and y, slice chunks along z
@@ -158,13 +164,13 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
   static_assert(!B2CL_VOL_BULK || C::addr == A_CTE, "row copies need CLAMP_TO_EDGE");
   extern __shared__ __align__(128) unsigned char vol_buf[];
   __shared__ uint64_t full[VOL_NS], empty[VOL_NS];
-  __shared__ float4 rowtab[4][4];  // per consumer warp and row: {b, 1-b, slot j0, slot j1}
+  __shared__ float4 rowtab[VOL_CW][4];  // per consumer warp and row: {b, 1-b, slot j0, slot j1}
   const Image& im = p.im;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < VOL_NS; ++s) {
       asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(vol_smem(&full[s])) : "memory");
-      asm volatile("mbarrier.init.shared::cta.b64 [%0], 4;" ::"r"(vol_smem(&empty[s])) : "memory");
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(vol_smem(&empty[s])), "r"(VOL_CW) : "memory");
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -173,7 +179,7 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
   const int ntiles = tl.ntx * tl.nty * tl.nzc;
   constexpr int NONE = -2147483647 - 1;
 
-  if (warp == 4) {  // ------------------------------------------------ producer
+  if (warp == VOL_CW) {  // ------------------------------------------------ producer
     if (lane == 0) asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmap)) : "memory");
     int s = 0;
     uint32_t ph = 0;
@@ -249,10 +255,10 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
     // this thread: columns xt + 4*lane + (0..3), rows yt + 4*warp + (0..3)
     const int xc = xt + 128 * (warp % VOL_XW) + 4 * lane, yr = yt + 4 * (warp / VOL_XW);
     // tile decision: every consumer thread tests its columns and row
-    // threadIdx.x % VT_H (so the 128 threads cover the tile's rows as the producer's lanes do)
+    // threadIdx.x % VT_H (so the consumer threads cover the tile's rows as the producer's lanes do)
     int fast = vol_in_window<C>(p, xc, yt + threadIdx.x % VT_H, xb, yb);
-    asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, 128, P; selp.s32 %0, 1, 0, Q; }"
-                 : "=r"(fast) : "r"(fast) : "memory");
+    asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, %2, P; selp.s32 %0, 1, 0, Q; }"
+                 : "=r"(fast) : "r"(fast), "n"(32 * VOL_CW) : "memory");
     if (!fast) {  // the taps directly (linear_at), no staging for this tile
 #pragma unroll 1
       for (int w = 0; w < q.nst; ++w) {
