@@ -309,3 +309,57 @@ def test_validation_has_no_side_effects(sess):
     assert np.array_equal(sess.read(b, 4096), data)
     sess.release(b, img, uimg)
     cl.lib().clReleaseSampler(smp)
+
+
+def test_config4_full_size_sampled(sess, orc):
+    """BASELINE config 4 at full size, in the launch configuration bench.py
+    times: the 8 GiB pitched CopyBufferRect (region {16384 B, 2048, 256}, source
+    row pitch 16512, slice pitch 2056 * 16512, tight destination), its
+    misaligned variant (source origin x = 3, pitch 16387) and the 8 GiB
+    FillBuffer; every byte of sampled rows (first / middle / last slices and
+    rows, both ragged ends) against the oracle applied to those rows."""
+    region = (16384, 2048, 256)
+    srp, ssp = 16512, 2056 * 16512
+    nsrc = ssp * region[2]
+    S_bytes = region[0] * region[1] * region[2]
+    src = sess.buffer(nsrc)
+    # seeded source contents, one slice at a time (the host never holds 8 GiB)
+    for z in range(region[2]):
+        sess.write(src, _rand_bytes(synth.rng(4000 + z), ssp), offset=z * ssp)
+    dst = sess.buffer(S_bytes)
+    zero = cl.sz3((0, 0, 0))
+    samples = [(z, y) for z in (0, 1, 127, 253, 254, 255) for y in (0, 1, 1023, 2046, 2047)]
+
+    def src_row(off, n):
+        z, r = divmod(off, ssp)
+        full = _rand_bytes(synth.rng(4000 + z), ssp)
+        row = full[r:r + n]
+        if len(row) < n:  # the row continues into the next slice
+            row = np.concatenate([row, _rand_bytes(synth.rng(4001 + z), ssp)[:n - len(row)]])
+        return row
+
+    def check_rows(so, rp, sp, drp, dsp, reg):
+        R0 = reg[0]
+        for z, y in samples:
+            if z >= reg[2] or y >= reg[1]:
+                continue
+            s_off = so + z * sp + y * rp
+            exp = np.zeros(R0, np.uint8)
+            orc.copy_rect(src_row(s_off, R0), exp, (0, 0, 0), (0, 0, 0), (R0, 1, 1), R0, R0, R0, R0)
+            got = sess.read(dst, R0, offset=z * dsp + y * drp)
+            assert np.array_equal(got, exp), (so, z, y)
+
+    cl.check(cl.lib().clEnqueueCopyBufferRect(sess.queue, src, dst, zero, zero, cl.sz3(region), srp, ssp,
+                                              0, 0, 0, None, None))
+    check_rows(0, srp, ssp, region[0], region[0] * region[1], region)
+    reg2 = (16384, 2048, 255)
+    cl.check(cl.lib().clEnqueueCopyBufferRect(sess.queue, src, dst, cl.sz3((3, 0, 0)), zero, cl.sz3(reg2), 16387,
+                                              16387 * 2056, 0, 0, 0, None, None))
+    check_rows(3, 16387, 16387 * 2056, reg2[0], reg2[0] * reg2[1], reg2)
+    pat = np.arange(16, dtype=np.uint8)
+    cl.check(cl.lib().clEnqueueFillBuffer(sess.queue, dst, pat.ctypes.data, 16, 0, S_bytes, 0, None, None))
+    for off in (0, S_bytes // 2 - 4096, S_bytes - 8192):
+        exp = np.zeros(8192, np.uint8)
+        orc.fill_buffer(exp, pat.tobytes(), 0, 8192)
+        assert np.array_equal(sess.read(dst, 8192, offset=off), exp), off
+    sess.release(src, dst)
