@@ -633,10 +633,17 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
     float* orow = reinterpret_cast<float*>(p.out) + ((uint64_t)q.w0 * p.oh + y0) * p.ow + x;
     const uint64_t zstride = (uint64_t)p.oh * p.ow;
     int nrow = x < p.ow ? min(VOLR_S, p.oh - y0) : 0;
+    const int ow = p.ow;
     auto emit = [&](const AxL& az, const float L[VOLR_S], const float H[VOLR_S]) {
+      float* o = orow;
+      if (nrow == VOLR_S) {
 #pragma unroll
-      for (int r = 0; r < VOLR_S; ++r)
-        if (r < nrow) __stcs(orow + (uint64_t)r * p.ow, lerp1(az.a, az.oma, L[r], H[r]));
+        for (int r = 0; r < VOLR_S; ++r, o += ow) __stcs(o, lerp1(az.a, az.oma, L[r], H[r]));
+      } else {
+#pragma unroll
+        for (int r = 0; r < VOLR_S; ++r, o += ow)
+          if (r < nrow) __stcs(o, lerp1(az.a, az.oma, L[r], H[r]));
+      }
       orow += zstride;
     };
     auto copy = [](float D[VOLR_S], const float S[VOLR_S]) {
