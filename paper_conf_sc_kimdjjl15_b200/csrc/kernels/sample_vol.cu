@@ -597,6 +597,26 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
     asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, 256, P; selp.s32 %0, 1, 0, Q; }"
                  : "=r"(fast) : "r"(in) : "memory");
     if (!fast) {  // the taps directly (read_image, the general kernel's coordinates)
+      // (CLAMP_TO_EDGE indices are monotone in x and y, so every tap of a tile
+      // whose corner box fits lies in it and this does not happen; should it,
+      // the slices the producer staged are released unread, in its order)
+      if (bx.ok) {
+        int kA = NONE, kB = NONE;
+#pragma unroll 1
+        for (int w = 0; w < q.nst; ++w) {
+          const AxL az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
+          const bool need0 = !(az.i0 == kA || az.i0 == kB);
+          const bool need1 = !(az.i1 == az.i0 || (!need0 && az.i1 == kB));
+          for (int h = 0; h < (int)need0 + (int)need1; ++h) {
+            vol_wait(&full[s], ph);
+            __syncwarp();
+            if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(vol_smem(&empty[s])) : "memory");
+            if (++s == VOLR_NS) { s = 0; ph ^= 1u; }
+          }
+          kA = az.i0;
+          kB = az.i1;
+        }
+      }
 #pragma unroll 1
       for (int w = 0; w < q.nst; ++w) {
         const int z = q.w0 + w;
