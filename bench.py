@@ -620,6 +620,29 @@ def _time_launches(T, torch, dev, fn, iters):
 def run_secondary(S, L, T, torch, dev, hbm_peak, args):
     from paper_conf_sc_kimdjjl15_b200 import cl, synth
     res = {}
+    # config 2 map (B): 30 deg rotation about the centre, unit scale (the general
+    # kernel, warps on 8 x 4 output patches).  REPEAT wraps the rotated square
+    # onto the torus with density ~1, so about every texel is read once:
+    # algorithmic bytes ~ 16 B in + 16 B out per sample (stated, not counted)
+    n2 = 4096
+    img2 = S.image(cl.CL_RGBA, cl.CL_FLOAT, n2, n2,
+                   host=synth.image_codes(synth.rng(2), cl.CL_RGBA, cl.CL_FLOAT, n2, n2))
+    out2 = S.buffer(n2 * n2 * 16)
+    A2 = (ctypes.c_float * 12)(*synth.affine_rotate_2d(n2, n2, 30.0).tolist())
+    d2 = cl.sz3((n2, n2, 1))
+    for name, addr in (("repeat", cl.CL_ADDRESS_REPEAT), ("mirrored", cl.CL_ADDRESS_MIRRORED_REPEAT)):
+        smp2 = S.sampler(True, addr, cl.CL_FILTER_LINEAR)
+        ms = _time_launches(T, torch, dev, lambda: cl.check(L.b2clEnqueueReadImageGrid(
+            S.queue, img2, smp2, 0, A2, d2, 4, out2, 0, 0, None, None)), 10)
+        e = {"Gsamples/s": n2 * n2 / ms / 1e6, "ms": ms, "map": "rotation 30 deg (B)",
+             "kernel": "k_sample_grid (8x4 output patch per warp)"}
+        if name == "repeat":
+            b2 = 32 * n2 * n2
+            e.update({"GB/s": b2 / ms / 1e6, "hbm_frac": b2 / ms / 1e6 / hbm_peak,
+                      "algorithmic_bytes": b2})
+        res[f"c2_map_b_{name}"] = e
+        L.clReleaseSampler(smp2)
+    S.release(img2, out2)
     # config 3: 512^3 R32F trilinear, stencil map, CLAMP_TO_EDGE
     n3 = 512
     g = synth.rng(3)

@@ -46,8 +46,24 @@ __device__ __forceinline__ void store_out(const SampleParams& p, uint64_t idx, c
 
 template <class C, int OUTC>
 __global__ void __launch_bounds__(256) k_sample_grid(const SampleParams p) {
+#ifndef B2CL_GRID_PATCH
+#define B2CL_GRID_PATCH 1
+#endif
+#if B2CL_GRID_PATCH
+  // block = 32 x 8 outputs; each warp takes an 8 x 4 patch of them (not one
+  // 32-wide row), so under rotations and other non-axis-aligned maps a
+  // warp's taps fall in a compact texel region: fewer cache lines per load
+#ifndef B2CL_GRID_PW
+#define B2CL_GRID_PW 8
+#endif
+  constexpr int PW = B2CL_GRID_PW, PH = 32 / PW;  // warp patch (PW x PH outputs)
+  const int lane = threadIdx.x, w = threadIdx.y;
+  const int x = blockIdx.x * 32 + (w % (32 / PW)) * PW + (lane % PW);
+  const int y = blockIdx.y * 8 + (w / (32 / PW)) * PH + (lane / PW);
+#else
   const int x = blockIdx.x * blockDim.x + threadIdx.x;
   const int y = blockIdx.y * blockDim.y + threadIdx.y;
+#endif
   const int z = blockIdx.z;
   if (x >= p.ow || y >= p.oh) return;
   const float xf = __int2float_rn(p.ox + x), yf = __int2float_rn(p.oy + y),
