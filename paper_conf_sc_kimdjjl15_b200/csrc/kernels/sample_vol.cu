@@ -471,11 +471,14 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
 #ifndef B2CL_VOLR_MINB
 #define B2CL_VOLR_MINB 2
 #endif
-constexpr int RT_W = 64, RT_H = 32;           // output tile
+#ifndef B2CL_VOLR_S
+#define B2CL_VOLR_S 8
+#endif
+constexpr int VOLR_S = B2CL_VOLR_S;           // samples (rows) per consumer thread
+constexpr int RT_W = 64, RT_H = 4 * VOLR_S;   // output tile (256 consumer threads: 64 columns x 4 row groups)
 constexpr int RB_MAXW = 128, RB_MAXH = 128;   // largest staged box (texels)
 constexpr int VOLR_NS = B2CL_VOLR_NS;
 constexpr int VOLR_THREADS = 288;             // 8 consumer warps + 1 producer warp
-constexpr int VOLR_S = 8;                     // samples (rows) per consumer thread
 
 struct VolrBox {
   int xb, yb;    // first staged texel column (16-B aligned) and row
@@ -569,7 +572,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
   // --------------------------------------------------------------- consumers
   int s = 0;
   uint32_t ph = 0;
-  const int col = threadIdx.x & (RT_W - 1), rg = threadIdx.x / RT_W;  // column, row group of 8
+  const int col = threadIdx.x & (RT_W - 1), rg = threadIdx.x / RT_W;  // column, row group of VOLR_S
   for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
     const VolSeg q = vol_seg(p, tl, t);
     const int x = q.tx * RT_W + col, y0 = q.ty * RT_H + rg * VOLR_S;
