@@ -642,7 +642,33 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
                       "algorithmic_bytes": b2})
         res[f"c2_map_b_{name}"] = e
         L.clReleaseSampler(smp2)
+    # config 5's image on one GPU (the N = 1 point of its row-sharded scaling):
+    # 32768^2 RGBA32F, 16 GiB, map (A), both samplers.  Its rows are the
+    # 4096-row seeded band above copied 8 times (device copies; the texel
+    # addresses, and so the traffic, are those of a 16 GiB image)
+    n5 = 32768
+    img5 = S.image(cl.CL_RGBA, cl.CL_FLOAT, n5, n5)
+    for by in range(0, n5, n2):
+        for bx in range(0, n5, n2):
+            cl.check(L.clEnqueueCopyImage(S.queue, img2, img5, cl.sz3((0, 0, 0)), cl.sz3((bx, by, 0)),
+                                          cl.sz3((n2, n2, 1)), 0, None, None))
     S.release(img2, out2)
+    out5 = S.buffer(n5 * n5 * 16)
+    A5 = (ctypes.c_float * 12)(*synth.affine_translate_2d(n5, n5).tolist())
+    d5 = cl.sz3((n5, n5, 1))
+    smp5 = [S.sampler(True, a, cl.CL_FILTER_LINEAR)
+            for a in (cl.CL_ADDRESS_REPEAT, cl.CL_ADDRESS_MIRRORED_REPEAT)]
+
+    def step5():
+        for k in range(2):
+            cl.check(L.b2clEnqueueReadImageGrid(S.queue, img5, smp5[k], 0, A5, d5, 4, out5, 0, 0, None, None))
+    ms = _time_launches(T, torch, dev, step5, 3)
+    res["c5_image_32768_1gpu"] = {"Gsamples/s": 2 * n5 * n5 / ms / 1e6, "ms_per_step": ms,
+                                  "step": "REPEAT + MIRRORED_REPEAT reads of map (A), 2 x 1.07 G samples",
+                                  "image": "32768x32768 RGBA32F (16 GiB)"}
+    for smp in smp5:
+        L.clReleaseSampler(smp)
+    S.release(img5, out5)
     # config 3: 512^3 R32F trilinear, stencil map, CLAMP_TO_EDGE
     n3 = 512
     g = synth.rng(3)
