@@ -10,9 +10,10 @@
 //     slice -- a (260 x 17)-texel box starting at the tile's first tap (i0 of
 //     its first column rounded down to 16 bytes, and of its first row) -- in a
 //     shared-memory ring: one cp.async.bulk per box row (one per lane),
-//     completing on a `full` mbarrier.  (B2CL_VOL_BULK=0 builds the 132 x 17
-//     variant (with B2CL_VOL_XW=1) that moves each box with one cp.async.bulk.tensor.3d; on B200
-//     it measured 196 us against 186 us for the row copies at config 3.)
+//     completing on a `full` mbarrier.  (B2CL_VOL_BULK=0 B2CL_VOL_XW=1
+//     builds the 132 x 17 variant that moves each box with one
+//     cp.async.bulk.tensor.3d; on B200 it measured 196 us against 186 us
+//     for the row copies at config 3.)
 //   * consumers x-blend each staged texel row once, y-blend neighbouring rows,
 //     keep the (x,y)-blended slice in registers and z-blend it with the next
 //     one, then release the stage on an `empty` mbarrier.
@@ -23,10 +24,11 @@
 // linear_at (read.cuh): per texel row lerp1(a, 1-a, T[i0], T[i1]), then
 // lerp1(b, ..) of the rows j0, j1, then lerp1(g, ..) of the slices k0, k1,
 // with the per-axis AxL of axis_l -- so the results are bit-identical to the
-// other grid kernels (the parity tests run all of them).  A thread whose taps
-// fall outside the staged box (non-unit maps, fp rounding at a tile edge)
-// fetches those samples from global memory instead, still in lock-step with
-// the ring.  Slices are consumed in walk order: the map's z coordinate must
+// other grid kernels (the parity tests run all of them).  A tile with a tap
+// outside its box (non-unit maps, fp rounding at a tile edge) is not staged:
+// the producer warp and the consumer warps test the same columns and rows
+// (vol_in_window) and agree, and the consumers read that tile's taps from
+// global memory (linear_at).  Slices are consumed in walk order: the map's z coordinate must
 // be non-decreasing in the output z (A[10] >= 0, host check), so with the
 // monotone CLAMP_TO_EDGE addressing the slice pair (k0, k1) only moves
 // forward and each slice is staged once per tile.
@@ -66,7 +68,7 @@ constexpr int VT_W = 128 * VOL_XW;        // output columns per tile (32 lanes x
 constexpr int VOL_YW = B2CL_VOL_YW;       // consumer warps down y
 constexpr int VOL_CW = VOL_XW * VOL_YW;   // consumer warps
 constexpr int VT_H = 4 * VOL_YW;          // output rows per tile (4 per warp)
-constexpr int VB_W = VT_W + 4;            // staged texel columns (TW + 1, from a 16-B aligned start)
+constexpr int VB_W = VT_W + 4;            // staged texel columns (TW + 1 taps + up to 3 of 16-B alignment)
 constexpr int VB_H = VT_H + 1;            // staged texel rows
 constexpr int VB_BYTES = VB_W * VB_H * 4; // one TMA box
 constexpr int VB_STRIDE = (VB_BYTES + 127) / 128 * 128;
