@@ -121,9 +121,29 @@ __device__ __forceinline__ AxL vol_axis(const SampleParams& p, int a, int o, int
 // region) fall inside the box staged at (xb, yb)?  A tile is staged only if
 // this holds for all its columns and rows (decided identically by the
 // producer warp and the consumer warps).
+#ifndef B2CL_VOL_FASTONLY
+#define B2CL_VOL_FASTONLY 1
+#endif
 template <class C>
-__device__ __forceinline__ bool vol_in_window(const SampleParams& p, int xc, int yr, int xb, int yb) {
+__device__ __forceinline__ bool vol_in_window(const SampleParams& p, int xc, int yr, int xb, int yb, bool chain_next) {
   bool ok = true;
+#if B2CL_VOL_FASTONLY
+  // the staged path's only form: the 4 columns' i0 are unit-stride from a
+  // 16-byte aligned slot and i1 = i0 + 1 for the first three (the fourth
+  // column's i1 is read from its own slot), the warp's rows chain (j1 of a
+  // row is j0 of the next), every tap inside the box
+  AxL a[4];
+#pragma unroll
+  for (int u = 0; u < 4; ++u) a[u] = vol_axis<C>(p, 0, p.ox, xc + u, p.im.w);
+  const int c0 = a[0].i0 - xb;
+  ok = c0 >= 0 && (c0 & 3) == 0 && c0 + 3 < VB_W && a[3].i1 - xb >= 0 && a[3].i1 - xb < VB_W;
+#pragma unroll
+  for (int u = 0; u < 4; ++u) ok = ok && a[u].i0 == a[0].i0 + u && (u == 3 || a[u].i1 == a[u].i0 + 1);
+  const AxL r0 = vol_axis<C>(p, 5, p.oy, yr, p.im.h);
+  ok = ok && r0.i0 - yb >= 0 && r0.i0 - yb < VB_H && r0.i1 - yb >= 0 && r0.i1 - yb < VB_H;
+  if (chain_next) ok = ok && vol_axis<C>(p, 5, p.oy, yr + 1, p.im.h).i0 == r0.i1;
+#else
+  (void)chain_next;
 #pragma unroll
   for (int u = 0; u < 4; ++u) {
     if (xc + u < p.ow) {
@@ -135,6 +155,7 @@ __device__ __forceinline__ bool vol_in_window(const SampleParams& p, int xc, int
     const AxL a = vol_axis<C>(p, 5, p.oy, yr, p.im.h);
     ok = ok && a.i0 - yb >= 0 && a.i0 - yb < VB_H && a.i1 - yb >= 0 && a.i1 - yb < VB_H;
   }
+#endif
   return ok;
 }
 
@@ -193,7 +214,8 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
       bool win = true;
 #pragma unroll
       for (int m = 0; m < VOL_XW; ++m)
-        win = win && vol_in_window<C>(p, q.tx * VT_W + 128 * m + 4 * lane, q.ty * VT_H + lane % VT_H, xb, yb);
+        win = win && vol_in_window<C>(p, q.tx * VT_W + 128 * m + 4 * lane, q.ty * VT_H + lane % VT_H, xb, yb,
+                                      (lane % VT_H & 3) != 3);
       if (!__all_sync(0xffffffffu, win)) continue;
 #if !B2CL_VOL_BULK
       if (lane != 0) continue;
@@ -258,7 +280,7 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
     const int xc = xt + 128 * (warp % VOL_XW) + 4 * lane, yr = yt + 4 * (warp / VOL_XW);
     // tile decision: every consumer thread tests its columns and row
     // threadIdx.x % VT_H (so the consumer threads cover the tile's rows as the producer's lanes do)
-    int fast = vol_in_window<C>(p, xc, yt + threadIdx.x % VT_H, xb, yb);
+    int fast = vol_in_window<C>(p, xc, yt + threadIdx.x % VT_H, xb, yb, (threadIdx.x % VT_H & 3) != 3);
     asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, %2, P; selp.s32 %0, 1, 0, Q; }"
                  : "=r"(fast) : "r"(fast), "n"(32 * VOL_CW) : "memory");
     if (!fast) {  // the taps directly (linear_at), no staging for this tile
@@ -304,6 +326,34 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
     __syncwarp();
     // 16-byte row segments: four unit-stride column taps starting 16-B aligned
     const int c0 = sl[0] & 0xffff;
+#if B2CL_VOL_FASTONLY
+    const int c4 = sl[3] >> 16;  // the fourth column's i1 slot (c0 + 4, or c0 + 3 clamped)
+    // x-blend of staged texel row j for the 4 columns (the tile passed vol_in_window)
+    auto xblend = [&](const float* buf, float jf, float h[4]) {
+      const float* row = buf + __float_as_int(jf) * VB_W;
+      const float4 v = *reinterpret_cast<const float4*>(row + c0);
+      const float T0[4] = {v.x, v.y, v.z, v.w}, T1[4] = {v.y, v.z, v.w, row[c4]};
+#pragma unroll
+      for (int u = 0; u < 4; ++u) h[u] = lerp1(ax[u].a, ax[u].oma, T0[u], T1[u]);
+    };
+    // the (x,y)-blended slice of the next ring stage: V[row][column]; the
+    // warp's rows chain, so 5 staged texel rows give its 4 output rows
+    auto slice = [&](float V[4][4]) {
+      vol_wait(&full[s], ph);
+      const float* buf = reinterpret_cast<const float*>(vol_buf + s * VB_STRIDE);
+      float Hp[4], Hn[4];
+      xblend(buf, rowtab[warp][0].z, Hp);
+#pragma unroll
+      for (int r = 0; r < 4; ++r) {
+        const float4 ry = rowtab[warp][r];
+        xblend(buf, ry.w, Hn);
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          V[r][u] = lerp1(ry.x, ry.y, Hp[u], Hn[u]);
+          Hp[u] = Hn[u];
+        }
+      }
+#else
     bool vecx = (c0 & 3) == 0 && c0 + 4 < VB_W;
 #pragma unroll
     for (int u = 0; u < 4; ++u) vecx = vecx && sl[u] == ((c0 + u) | (c0 + u + 1) << 16);
@@ -358,6 +408,7 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
           for (int u = 0; u < 4; ++u) V[r][u] = lerp1(ry.x, ry.y, Hp[u], Hn[u]);
         }
       }
+#endif
       __syncwarp();
       if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(vol_smem(&empty[s])) : "memory");
       if (++s == VOL_NS) { s = 0; ph ^= 1u; }
