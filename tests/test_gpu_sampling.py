@@ -387,3 +387,31 @@ def test_supported_formats_match_the_legal_table(sess, orc):
            if orc.elem_size(o, t) > 0}
     assert got == exp
     assert (cl.CL_RGBx, cl.CL_UNORM_INT_101010) in got and (cl.CL_RGB, cl.CL_UNORM_SHORT_565) in got
+
+
+@pytest.mark.parametrize("case", ["inf_x", "nan_y", "huge_z", "zero_scale", "neg_zero"])
+def test_config3_kernels_degenerate_maps(sess, orc, case):
+    """The config-3 format and sampler with degenerate separable and rotated
+    maps (infinite / NaN / huge coefficients, zero scale, -0): whichever kernel
+    the library picks (staged, walk or general) agrees with the oracle."""
+    W, H, D = 70, 20, 12
+    img, oimg, _ = make_images(sess, orc, R, F32, W, H, D, 3, seed=99)
+    smp = sess.sampler(True, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR)
+    for rotated in (False, True):
+        A = synth.affine_rotate_3d(W, 20.0) if rotated else _affine("stencil", (W, H, D), (W, H, D))
+        A = A.copy()
+        if case == "inf_x":
+            A[0] = np.float32(np.inf)
+        elif case == "nan_y":
+            A[7] = np.float32(np.nan)
+        elif case == "huge_z":
+            A[11] = np.float32(3e9)
+        elif case == "zero_scale":
+            A[0] = A[5] = A[10] = np.float32(0.0)
+        else:
+            A[10] = np.float32(-0.0)
+        out = (W, H, D)
+        got = gpu_read_grid(sess, img, smp, cl.B2CL_RTYPE_FLOAT, A, out, 1)
+        exp = orc.read_grid(oimg, True, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR, orc.RT_F, A, out, 1)
+        assert_parity(got, exp, True, f"{case} rotated={rotated}")
+    sess.release(img)
