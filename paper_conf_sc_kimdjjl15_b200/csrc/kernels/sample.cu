@@ -85,7 +85,10 @@ constexpr int kSepUnroll = B2CL_SEP_UNROLL;  // rows of a thread in flight toget
 // Separable maps: block = 32 x 4 threads; tile = (32*XPT) columns x (4*RPW) rows
 // of one output slice.  Lane -> columns lane + 32*t, warp -> RPW consecutive rows.
 template <class C, int OUTC, int XPT, int RPW>
-__global__ void __launch_bounds__(128, (C::type == RT ? 1 : 11)) k_sample_grid_sep(const SampleParams p) {
+#ifndef B2CL_SEP_MINB
+#define B2CL_SEP_MINB 11
+#endif
+__global__ void __launch_bounds__(128, (C::type == RT ? 1 : B2CL_SEP_MINB)) k_sample_grid_sep(const SampleParams p) {
   const Image& im = p.im;
   const int z = blockIdx.z;
   const int x0 = blockIdx.x * (32 * XPT) + threadIdx.x;
