@@ -191,6 +191,44 @@ def _axis_taps(coef, offset, n_out, n, mode, start=0):
     return np.unique(np.concatenate([i0[a != 1], i1[a != 0]]))
 
 
+def _distinct_texels_2d(A, W, H, mode, chunk=256):
+    """Number of distinct texels a LINEAR read of the 2D affine map A (output
+    W x H, image W x H, normalized, z = 0) touches with a non-zero tap weight,
+    under REPEAT or MIRRORED_REPEAT ([CL1.2 §8.2] in numpy float32, one RN op
+    per step as the kernels and the oracle; measurement bookkeeping only)."""
+    f32 = np.float32
+    seen = np.zeros((H, W), dtype=bool)
+    x = np.arange(W, dtype=f32)[None, :]
+
+    def axis(c, n):
+        fn = f32(n)
+        if mode == "repeat":
+            u = ((c - np.floor(c)).astype(f32) * fn).astype(f32)
+        else:
+            sp = (f32(2.0) * np.rint((f32(0.5) * c).astype(f32))).astype(f32)
+            u = (np.abs((c - sp).astype(f32)) * fn).astype(f32)
+        t = (u - f32(0.5)).astype(f32)
+        b = np.floor(t).astype(np.int64)
+        a = (t - np.floor(t)).astype(f32)
+        if mode == "repeat":
+            return np.where(b < 0, b + n, b), np.where(b + 1 > n - 1, b + 1 - n, b + 1), a
+        return np.maximum(b, 0), np.minimum(b + 1, n - 1), a
+
+    for y0 in range(0, H, chunk):
+        y = np.arange(y0, min(H, y0 + chunk), dtype=f32)[:, None]
+        cs = []
+        for r in range(2):
+            v = (f32(A[4 * r]) * x).astype(f32) + (f32(A[4 * r + 1]) * y).astype(f32)
+            v = (v.astype(f32) + (f32(A[4 * r + 2]) * f32(0.0))).astype(f32)
+            cs.append((v + f32(A[4 * r + 3])).astype(f32))
+        i0, i1, a = axis(cs[0], W)
+        j0, j1, b = axis(cs[1], H)
+        for jj, ii, m in ((j0, i0, (a != 1) & (b != 1)), (j0, i1, (a != 0) & (b != 1)),
+                          (j1, i0, (a != 1) & (b != 0)), (j1, i1, (a != 0) & (b != 0))):
+            seen[jj[m], ii[m]] = True
+    return int(seen.sum())
+
+
 def circular_interval(idx, n):
     """Smallest (begin, count) whose circular range {(begin+s) mod n} covers idx."""
     rows = np.unique(np.asarray(idx, dtype=np.int64))
@@ -621,9 +659,8 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
     from paper_conf_sc_kimdjjl15_b200 import cl, synth
     res = {}
     # config 2 map (B): 30 deg rotation about the centre, unit scale (the general
-    # kernel, warps on 8 x 4 output patches).  REPEAT wraps the rotated square
-    # onto the torus with density ~1, so about every texel is read once:
-    # algorithmic bytes ~ 16 B in + 16 B out per sample (stated, not counted)
+    # kernel, warps on 8 x 4 output patches); algorithmic bytes = the distinct
+    # texels with a non-zero tap weight (counted on the host) x 16 B + 16 B out
     n2 = 4096
     img2 = S.image(cl.CL_RGBA, cl.CL_FLOAT, n2, n2,
                    host=synth.image_codes(synth.rng(2), cl.CL_RGBA, cl.CL_FLOAT, n2, n2))
@@ -636,10 +673,10 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
             S.queue, img2, smp2, 0, A2, d2, 4, out2, 0, 0, None, None)), 10)
         e = {"Gsamples/s": n2 * n2 / ms / 1e6, "ms": ms, "map": "rotation 30 deg (B)",
              "kernel": "k_sample_grid (8x4 output patch per warp)"}
-        if name == "repeat":
-            b2 = 32 * n2 * n2
-            e.update({"GB/s": b2 / ms / 1e6, "hbm_frac": b2 / ms / 1e6 / hbm_peak,
-                      "algorithmic_bytes": b2})
+        texels = _distinct_texels_2d(synth.affine_rotate_2d(n2, n2, 30.0), n2, n2, name)
+        b2 = 16 * texels + 16 * n2 * n2
+        e.update({"GB/s": b2 / ms / 1e6, "hbm_frac": b2 / ms / 1e6 / hbm_peak, "algorithmic_bytes": b2,
+                  "distinct_texels": texels})
         res[f"c2_map_b_{name}"] = e
         L.clReleaseSampler(smp2)
     # config 5's image on one GPU (the N = 1 point of its row-sharded scaling):
