@@ -178,6 +178,8 @@ def _axis_taps(coef, offset, n_out, n, mode, start=0):
     fn = f32(n)
     if mode == "repeat":
         u = ((s - np.floor(s)).astype(f32) * fn).astype(f32)
+    elif mode == "clamp_to_edge":
+        u = (s * fn).astype(f32)
     else:
         sp = (f32(2.0) * np.rint((f32(0.5) * s).astype(f32))).astype(f32)
         u = (np.abs((s - sp).astype(f32)) * fn).astype(f32)
@@ -186,6 +188,8 @@ def _axis_taps(coef, offset, n_out, n, mode, start=0):
     a = (t - np.floor(t)).astype(f32)
     if mode == "repeat":
         i0, i1 = np.where(b < 0, b + n, b), np.where(b + 1 > n - 1, b + 1 - n, b + 1)
+    elif mode == "clamp_to_edge":
+        i0, i1 = np.clip(b, 0, n - 1), np.clip(b + 1, 0, n - 1)
     else:
         i0, i1 = np.maximum(b, 0), np.minimum(b + 1, n - 1)
     return np.unique(np.concatenate([i0[a != 1], i1[a != 0]]))
@@ -194,7 +198,7 @@ def _axis_taps(coef, offset, n_out, n, mode, start=0):
 def _distinct_texels_2d(A, W, H, mode, chunk=256):
     """Number of distinct texels a LINEAR read of the 2D affine map A (output
     W x H, image W x H, normalized, z = 0) touches with a non-zero tap weight,
-    under REPEAT or MIRRORED_REPEAT ([CL1.2 §8.2] in numpy float32, one RN op
+    under REPEAT, MIRRORED_REPEAT or CLAMP_TO_EDGE ([CL1.2 §8.2] in numpy float32, one RN op
     per step as the kernels and the oracle; measurement bookkeeping only)."""
     f32 = np.float32
     seen = np.zeros((H, W), dtype=bool)
@@ -204,6 +208,8 @@ def _distinct_texels_2d(A, W, H, mode, chunk=256):
         fn = f32(n)
         if mode == "repeat":
             u = ((c - np.floor(c)).astype(f32) * fn).astype(f32)
+        elif mode == "clamp_to_edge":
+            u = (c * fn).astype(f32)
         else:
             sp = (f32(2.0) * np.rint((f32(0.5) * c).astype(f32))).astype(f32)
             u = (np.abs((c - sp).astype(f32)) * fn).astype(f32)
@@ -212,6 +218,8 @@ def _distinct_texels_2d(A, W, H, mode, chunk=256):
         a = (t - np.floor(t)).astype(f32)
         if mode == "repeat":
             return np.where(b < 0, b + n, b), np.where(b + 1 > n - 1, b + 1 - n, b + 1), a
+        if mode == "clamp_to_edge":
+            return np.clip(b, 0, n - 1), np.clip(b + 1, 0, n - 1), a
         return np.maximum(b, 0), np.minimum(b + 1, n - 1), a
 
     for y0 in range(0, H, chunk):
@@ -725,11 +733,15 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
     A3b = (ctypes.c_float * 12)(*synth.affine_rotate_3d(n3, 20.0).tolist())
     ms = _time_launches(T, torch, dev, lambda: cl.check(L.b2clEnqueueReadImageGrid(
         S.queue, vol, smp3, 0, A3b, d3, 1, out3, 0, 0, None, None)), 10)
-    # map (B): every texel whose tap weight is non-zero is read once (the
-    # rotated grid covers the volume's interior; clamped corners re-read edge
-    # texels) -- algorithmic bytes counted as 4 B in + 4 B out per sample
-    res["c3_trilinear_512_rotated"] = {"Gsamples/s": n3 ** 3 / ms / 1e6, "ms": ms, "GB/s": byt / ms / 1e6,
-                                       "hbm_frac": byt / ms / 1e6 / hbm_peak,
+    # map (B) is a rotation about z: the texels it taps with a non-zero weight
+    # are (the xy taps of one slice) x (the z taps), counted on the host
+    Arot = synth.affine_rotate_3d(n3, 20.0)
+    txy = _distinct_texels_2d(Arot, n3, n3, "clamp_to_edge")
+    tz = _axis_taps(Arot[10], Arot[11], n3, n3, "clamp_to_edge").size
+    bytr = 4 * txy * tz + 4 * n3 ** 3
+    res["c3_trilinear_512_rotated"] = {"Gsamples/s": n3 ** 3 / ms / 1e6, "ms": ms, "GB/s": bytr / ms / 1e6,
+                                       "hbm_frac": bytr / ms / 1e6 / hbm_peak, "algorithmic_bytes": bytr,
+                                       "distinct_texels": txy * tz,
                                        "map": "volume-render rotation (B), 20 deg about z",
                                        "kernel": "k_sample_grid_volr (64x32 tiles, tensor-TMA footprint box)"}
     S.release(vol, out3)
