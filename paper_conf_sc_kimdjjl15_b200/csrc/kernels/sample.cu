@@ -21,6 +21,7 @@
 // time): the fully run-time instance covers every format x sampler; the
 // compile-time instances are the hot configurations of BASELINE.json.
 #include <atomic>
+#include <cmath>
 #include <type_traits>
 
 #include "../device/read.cuh"
@@ -564,6 +565,193 @@ __global__ void __launch_bounds__(128) k_sample_grid_tile(const SampleParams p) 
   else walk(std::false_type{});
 }
 
+// MIRRORED_REPEAT folds: an output column x and its mirror image Mx - x tap
+// (nearly) the same texel columns, and likewise rows.  k_sample_grid_fold
+// stages ONE texel box per block -- the union of the taps of a 64 x 16 tile
+// of "primary" outputs and of its three mirror images -- and blends all four
+// output tiles from it: a quarter of the staging of k_sample_grid_tile per
+// output.  The pairing (Mx, My) is the host's guess; every tap is checked
+// against the staged box and a tile that does not fit reads its taps
+// directly, so results are always linear_at's (bit-identical).
+//   Primary columns: xp in [0, Px) maps to x = xp for xp < Ax, else
+//   Mx + 1 + (xp - Ax) (the columns whose mirror image is outside the
+//   output); column x's partner Mx - x is used when inside [0, ow) and != x.
+#ifndef B2CL_FOLD_UNROLL
+#define B2CL_FOLD_UNROLL 1
+#endif
+constexpr int kFoldUnroll = B2CL_FOLD_UNROLL;  // output tiles of a block in flight together
+
+struct FoldMap {
+  int Mx, Ax, Px;  // columns
+  int My, Ay, Py;  // rows
+};
+
+__device__ __forceinline__ int fold_prim(int pi, int M, int A) { return pi < A ? pi : M + 1 + (pi - A); }
+
+template <class C>
+__global__ void __launch_bounds__(128) k_sample_grid_fold(const SampleParams p, const FoldMap fm) {
+  static_assert(C::type == T_FLOAT && C::order == O_RGBA && C::dims == 2, "2D RGBA32F");
+  static_assert(C::addr == A_REPEAT || C::addr == A_MIRROR, "taps always in range");
+#ifndef B2CL_FOLD_PAD
+#define B2CL_FOLD_PAD 6
+#endif
+  // the staged box: the tile's taps plus room for the mirror images' offsets
+  constexpr int TW = 64, TH = 16, BW = TW + B2CL_FOLD_PAD, BH = TH + B2CL_FOLD_PAD;
+  __shared__ __align__(16) float4 box[BH][BW];
+  __shared__ int cI0[2][TW], cI1[2][TW], cX[2][TW], rY[2][TH];
+  __shared__ float cA[2][TW], cOma[2][TW];
+  __shared__ float4 rT[2][TH];  // per row: {b, 1 - b, j0 bits, j1 bits}
+  __shared__ int bb[4];         // column min, max, row min, max of the staged box
+  const Image& im = p.im;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int xp0 = blockIdx.x * TW, yp0 = blockIdx.y * TH;
+  if (tid == 0) { bb[0] = 0x7fffffff; bb[1] = -1; bb[2] = 0x7fffffff; bb[3] = -1; }
+  __syncthreads();
+  // tables: [0] primary, [1] partner; x / y = -1 marks an absent output
+  {
+    const int h = tid >> 6, c = tid & 63;  // 128 threads: 64 columns x {primary, partner}
+    const int xp = xp0 + c;
+    int x = xp < fm.Px ? fold_prim(xp, fm.Mx, fm.Ax) : -1;
+    if (h == 1 && x >= 0) {
+      const int xm = fm.Mx - x;
+      x = (xm >= 0 && xm < p.ow && xm != x) ? xm : -1;
+    }
+    cX[h][c] = x;
+    if (x >= 0) {
+      const AxL ax = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(p.ox + x)), p.A[3]), im.w);
+      cI0[h][c] = ax.i0; cI1[h][c] = ax.i1; cA[h][c] = ax.a; cOma[h][c] = ax.oma;
+      atomicMin(&bb[0], min(ax.i0, ax.i1));
+      atomicMax(&bb[1], max(ax.i0, ax.i1));
+    } else {
+      cI0[h][c] = cI1[h][c] = 0x3fffffff;  // (never staged, never stored)
+      cA[h][c] = 0.f; cOma[h][c] = 1.f;
+    }
+    if (tid < 2 * TH) {
+      const int hr = tid / TH, r = tid % TH;
+      const int yp = yp0 + r;
+      int y = yp < fm.Py ? fold_prim(yp, fm.My, fm.Ay) : -1;
+      if (hr == 1 && y >= 0) {
+        const int ym = fm.My - y;
+        y = (ym >= 0 && ym < p.oh && ym != y) ? ym : -1;
+      }
+      rY[hr][r] = y;
+      if (y >= 0) {
+        const AxL ay = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(p.oy + y)), p.A[7]), im.h);
+        rT[hr][r] = make_float4(ay.a, ay.oma, __int_as_float(ay.i0), __int_as_float(ay.i1));
+        atomicMin(&bb[2], min(ay.i0, ay.i1));
+        atomicMax(&bb[3], max(ay.i0, ay.i1));
+      }
+    }
+  }
+  __syncthreads();
+  const int c0 = bb[0], r0 = bb[2];
+  const bool staged = bb[1] >= c0 && bb[1] - c0 < BW && bb[3] >= r0 && bb[3] - r0 < BH;
+  const uint64_t zoff = (uint64_t)blockIdx.z * p.oh;
+  float4* out = reinterpret_cast<float4*>(p.out) + zoff * p.ow;
+  if (staged) {  // the union box: warp w copies box rows w, w + 4, ...; 16-byte async copies
+    const int nc = bb[1] - c0 + 1, nr = bb[3] - r0 + 1;
+    for (int rr = warp; rr < nr; rr += 4) {
+      const char* src = row_ptr<C>(im, r0 + rr, 0) + (uint64_t)(unsigned)c0 * 16u;
+      const uint32_t dst = static_cast<uint32_t>(__cvta_generic_to_shared(&box[rr][0]));
+      for (int cc = lane; cc < nc; cc += 32)
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst + cc * 16), "l"(src + cc * 16)
+                     : "memory");
+    }
+    asm volatile("cp.async.wait_all;" ::: "memory");
+  }
+  __syncthreads();
+  // warp w: columns (w & 1)*32 + lane, rows (w >> 1)*8 .. +8, for each of the
+  // four (column set, row set) combinations
+  const int c = (warp & 1) * 32 + lane, rb = (warp >> 1) * (TH / 2);
+#pragma unroll kFoldUnroll
+  for (int combo = 0; combo < 4; ++combo) {
+    const int hc = combo & 1, hr = combo >> 1;
+    const int x = cX[hc][c];
+    const int i0 = cI0[hc][c], i1 = cI1[hc][c];
+    const float a = cA[hc][c], oma = cOma[hc][c];
+    if (!staged) {  // the taps directly
+      if (x < 0) continue;
+      const AxL ax{i0, i1, a, oma, true, true};
+#pragma unroll 1
+      for (int r = rb; r < rb + TH / 2; ++r) {
+        const int y = rY[hr][r];
+        if (y < 0) continue;
+        const float4 ry = rT[hr][r];
+        const char* rows[4] = {row_ptr<C>(im, __float_as_int(ry.z), 0), row_ptr<C>(im, __float_as_int(ry.w), 0),
+                               nullptr, nullptr};
+        const bool rok[4] = {true, true, false, false};
+        uint32_t res[4];
+        linear_at<C>(p, rows, rok, ax, ry.x, ry.y, 0.f, 1.f, res, 4);
+        __stcs(out + ((uint64_t)y * p.ow + x), make_float4(__uint_as_float(res[0]), __uint_as_float(res[1]),
+                                                             __uint_as_float(res[2]), __uint_as_float(res[3])));
+      }
+      continue;
+    }
+    // byte offsets of this column's two taps within a staged row (absent
+    // columns read slot 0 and store nothing)
+    const uint32_t o0 = x >= 0 ? (uint32_t)(i0 - c0) * 16u : 0u, o1 = x >= 0 ? (uint32_t)(i1 - c0) * 16u : 0u;
+    const char* bbase = reinterpret_cast<const char*>(&box[0][0]);
+    auto xblend = [&](int j, float4& h) {
+      const char* row = bbase + (uint32_t)(j - r0) * (BW * 16);
+      const float4 t0 = *reinterpret_cast<const float4*>(row + o0);
+      const float4 t1 = *reinterpret_cast<const float4*>(row + o1);
+      h = make_float4(lerp1(a, oma, t0.x, t1.x), lerp1(a, oma, t0.y, t1.y), lerp1(a, oma, t0.z, t1.z),
+                      lerp1(a, oma, t0.w, t1.w));
+    };
+    auto emit = [&](int y, const float4& ry, const float4& n0, const float4& n1) {
+      if (x >= 0)
+        __stcs(out + ((uint64_t)y * p.ow + x), make_float4(lerp1(ry.x, ry.y, n0.x, n1.x), lerp1(ry.x, ry.y, n0.y, n1.y),
+                                                           lerp1(ry.x, ry.y, n0.z, n1.z), lerp1(ry.x, ry.y, n0.w, n1.w)));
+    };
+    // the warp's 8 rows of this row set: all present and chained one way
+    // (j1 of a row = j0 of the next: UP; j0 = j1 of the next: DOWN), so each
+    // texel row is x-blended once; otherwise both taps per row
+    bool all = true, up = true, dn = true;
+#pragma unroll
+    for (int r = rb; r < rb + TH / 2; ++r) {
+      all = all && rY[hr][r] >= 0;
+      if (r + 1 < rb + TH / 2) {
+        const float4 ra = rT[hr][r], rn = rT[hr][r + 1];
+        up = up && __float_as_int(ra.w) == __float_as_int(rn.z);
+        dn = dn && __float_as_int(ra.z) == __float_as_int(rn.w);
+      }
+    }
+    auto walk = [&](auto upc) {
+      constexpr bool UP = decltype(upc)::value;
+      float4 hp;  // x-blend of the texel row shared with the previous output row
+      {
+        const float4 ry = rT[hr][rb];
+        xblend(__float_as_int(UP ? ry.z : ry.w), hp);
+      }
+#pragma unroll 4
+      for (int r = rb; r < rb + TH / 2; ++r) {
+        const float4 ry = rT[hr][r];
+        float4 hn;
+        xblend(__float_as_int(UP ? ry.w : ry.z), hn);
+        if (UP) emit(rY[hr][r], ry, hp, hn);
+        else emit(rY[hr][r], ry, hn, hp);
+        hp = hn;
+      }
+    };
+    if (all && up) {
+      walk(std::true_type{});
+    } else if (all && dn) {
+      walk(std::false_type{});
+    } else {
+#pragma unroll 1
+      for (int r = rb; r < rb + TH / 2; ++r) {
+        const int y = rY[hr][r];
+        if (y < 0) continue;  // (warp-uniform)
+        const float4 ry = rT[hr][r];
+        float4 n0, n1;
+        xblend(__float_as_int(ry.z), n0);
+        xblend(__float_as_int(ry.w), n1);
+        emit(y, ry, n0, n1);
+      }
+    }
+  }
+}
+
 template <class C, bool INT_COORD>
 __global__ void __launch_bounds__(256) k_sample_list(const SampleParams p) {
   const uint64_t s = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -653,6 +841,41 @@ static cudaError_t go_tile(const SampleParams& p, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+// the mirror pairing of one output axis under MIRRORED_REPEAT: the fold point
+// (an integer of the coordinate) inside the region, and the index sum M with
+// s(x) + s(M - x) = 2 * fold (double arithmetic: a guess the kernel checks)
+static bool fold_axis(double a, double c, int o, int n, int* M, int* A, int* P) {
+  if (!(a != 0.0) || !std::isfinite(a) || !std::isfinite(c) || n < 64) return false;
+  const double s0 = a * o + c, s1 = a * (o + n - 1) + c;
+  const double lo = std::min(s0, s1), hi = std::max(s0, s1);
+  const double f = std::ceil(lo);
+  if (!(f < hi) || f + 1.0 < hi) return false;  // exactly one fold point inside
+  const double m = (2.0 * f - 2.0 * c) / a - 2.0 * o;
+  if (!(std::fabs(m) < 1e9)) return false;
+  const long long Mi = std::llround(m);
+  // primary indices: [0, Mi/2] and (Mi, n)
+  const long long A1 = std::min<long long>(n, std::max<long long>(0, Mi / 2 + 1));
+  const long long A2 = std::max<long long>(0, n - 1 - std::max<long long>(Mi, -1));
+  *M = (int)Mi;
+  *A = (int)A1;
+  *P = (int)(A1 + A2);
+  return *P > 0 && *P < n;  // a real fold pairs something
+}
+
+template <class C>
+static bool go_fold(const SampleParams& p, cudaStream_t st, cudaError_t* err) {
+  FoldMap fm;
+  if (!p.smp.norm) return false;
+  if (!fold_axis((double)p.A[0], (double)p.A[3], p.ox, p.ow, &fm.Mx, &fm.Ax, &fm.Px)) return false;
+  if (!fold_axis((double)p.A[5], (double)p.A[7], p.oy, p.oh, &fm.My, &fm.Ay, &fm.Py)) return false;
+  dim3 grd((fm.Px + 63) / 64, (fm.Py + 15) / 16, p.od);
+  if (is_shard(p)) k_sample_grid_fold<WithShard<C, true>><<<grd, 128, 0, st>>>(p, fm);
+  else k_sample_grid_fold<WithShard<C, false>><<<grd, 128, 0, st>>>(p, fm);
+  count_launch();
+  *err = cudaGetLastError();
+  return true;
+}
+
 template <class C, int OUTC, int XPT, int RPW>
 static cudaError_t go_sep(const SampleParams& p, cudaStream_t st) {
   dim3 blk(32, 4, 1);
@@ -661,6 +884,13 @@ static cudaError_t go_sep(const SampleParams& p, cudaStream_t st) {
   else k_sample_grid_sep<WithShard<C, false>, OUTC, XPT, RPW><<<grd, blk, 0, st>>>(p);
   count_launch();
   return cudaGetLastError();
+}
+
+template <class C>
+static cudaError_t fold_or_sep(const SampleParams& p, cudaStream_t st) {
+  cudaError_t e = cudaSuccess;
+  if (go_fold<C>(p, st, &e)) return e;
+  return go_sep<C, 4, B2CL_C2M_XPT, B2CL_C2M_RPW>(p, st);
 }
 
 template <class C>
@@ -730,7 +960,8 @@ cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st
       if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_MIRROR, F_LINEAR))
         return fk == 3   ? go_walk<C2Mirror, 4, 2, 8>(p, st)
                : fk == 5 ? go_tile<C2Mirror, B2CL_TILE_TH>(p, st)
-                         : go_sep<C2Mirror, 4, B2CL_C2M_XPT, B2CL_C2M_RPW>(p, st);
+               : fk == 2 ? go_sep<C2Mirror, 4, B2CL_C2M_XPT, B2CL_C2M_RPW>(p, st)
+               : fold_or_sep<C2Mirror>(p, st);
       if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR)) {
         if (fk == 0 && !is_shard(p)) {
           bool used = false;

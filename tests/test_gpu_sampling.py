@@ -194,6 +194,13 @@ GRID_CASES = [
     (3, R, F32, (70, 45, 30), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "magnify", (150, 40, 50), 1),
     (3, R, F32, (300, 60, 40), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "scale2", (150, 33, 21), 1),
     (3, R, F32, (140, 20, 24), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "stencil-zneg", (140, 20, 24), 1),
+    # mirror-fold kernel (k_sample_grid_fold, MIRRORED_REPEAT with one fold per
+    # axis): ragged primary tiles, unpaired columns past the mirror sum, an
+    # exact and an inexact mirror, the fold near an edge, a 3-slice output
+    (2, RGBA, F32, (300, 130, 1), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "translate", (300, 130, 1), 4),
+    (2, RGBA, F32, (257, 129, 1), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "fold-exact", (257, 129, 1), 4),
+    (2, RGBA, F32, (200, 150, 1), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "fold-edge", (200, 150, 1), 4),
+    (2, RGBA, F32, (160, 96, 1), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "translate", (160, 96, 3), 4),
     # rotated-map staged kernel (k_sample_grid_volr): ragged tiles, the corners
     # clamped to the edges; 3x minification (footprint larger than the box:
     # direct tiles); z at half scale (repeated slice pairs)
@@ -215,6 +222,10 @@ def _affine(kind, size, out):
         A[5], A[7] = 2.0 / H, 0.45 / H
         A[10], A[11] = 2.0 / D, -0.2 / D
         return A
+    if kind == "fold-exact":  # mirror sum an integer: partners tap the same texels
+        return synth.affine_translate_2d(W, H, dx=0.5, dy=0.5)
+    if kind == "fold-edge":  # the fold 10 / 7 outputs from the right / bottom edge
+        return synth.affine_translate_2d(W, H, dx=-10.3, dy=-7.6)
     if kind == "magnify":  # 2x magnification, separable, offset by a fraction of a texel
         A = np.zeros(12, np.float32)
         A[0], A[3] = 0.5 / W, 0.37 / W
