@@ -580,6 +580,10 @@ __global__ void __launch_bounds__(128) k_sample_grid_tile(const SampleParams p) 
 #define B2CL_FOLD_UNROLL 1
 #endif
 constexpr int kFoldUnroll = B2CL_FOLD_UNROLL;  // output tiles of a block in flight together
+#ifndef B2CL_FOLD_WALK_UNROLL
+#define B2CL_FOLD_WALK_UNROLL 8
+#endif
+constexpr int kFoldWalkUnroll = B2CL_FOLD_WALK_UNROLL;  // rows of the walk unrolled
 
 struct FoldMap {
   int Mx, Ax, Px;  // columns
@@ -723,7 +727,7 @@ __global__ void __launch_bounds__(128) k_sample_grid_fold(const SampleParams p, 
         const float4 ry = rT[hr][rb];
         xblend(__float_as_int(UP ? ry.z : ry.w), hp);
       }
-#pragma unroll 4
+#pragma unroll kFoldWalkUnroll
       for (int r = rb; r < rb + TH / 2; ++r) {
         const float4 ry = rT[hr][r];
         float4 hn;
