@@ -592,8 +592,11 @@ struct FoldMap {
 
 __device__ __forceinline__ int fold_prim(int pi, int M, int A) { return pi < A ? pi : M + 1 + (pi - A); }
 
+#ifndef B2CL_FOLD_MINB
+#define B2CL_FOLD_MINB 1
+#endif
 template <class C>
-__global__ void __launch_bounds__(128) k_sample_grid_fold(const SampleParams p, const FoldMap fm) {
+__global__ void __launch_bounds__(128, B2CL_FOLD_MINB) k_sample_grid_fold(const SampleParams p, const FoldMap fm) {
   static_assert(C::type == T_FLOAT && C::order == O_RGBA && C::dims == 2, "2D RGBA32F");
   static_assert(C::addr == A_REPEAT || C::addr == A_MIRROR, "taps always in range");
 #ifndef B2CL_FOLD_PAD
