@@ -381,11 +381,27 @@ def run_gpu(args):
             S.sampler(True, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR)]
     origin, region = cl.sz3((0, r0, 0)), cl.sz3((N2D, N2D, 1))
 
-    def launch(k, images=None):
-        cl.check(L.b2clEnqueueReadImageGridRegion(S.queue, (images or imgs)[k], smps[k],
+    def launch(k, images=None, queue=None, nwait=0, wait=None, ev=None):
+        cl.check(L.b2clEnqueueReadImageGridRegion(queue or S.queue, (images or imgs)[k], smps[k],
                                                   cl.B2CL_RTYPE_FLOAT, A, origin, region, 4, outs[k],
-                                                  0, 0, None, None),
+                                                  0, nwait, wait, ev),
                  "read grid")
+
+    # The step: the two reads are independent (one image, two samplers, two
+    # outputs), so the program issues them on two command queues of the
+    # device, as an OpenCL program would, and joins them with events: the
+    # second queue starts after a marker of the first (the previous step is
+    # complete) and the first queue's barrier waits for the second read.
+    q_two = S.queue_for(gpu)
+
+    def step():
+        mk, e1 = ctypes.c_void_p(), ctypes.c_void_p()
+        cl.check(L.clEnqueueMarkerWithWaitList(S.queue, 0, None, ctypes.byref(mk)))
+        launch(1, queue=q_two, nwait=1, wait=(ctypes.c_void_p * 1)(mk), ev=ctypes.byref(e1))
+        launch(0)
+        cl.check(L.clEnqueueBarrierWithWaitList(S.queue, 1, (ctypes.c_void_p * 1)(e1), None))
+        L.clReleaseEvent(mk)
+        L.clReleaseEvent(e1)
 
     # ---- parity spot check of this exact launch configuration (bench as test) ----
     launch(0)
@@ -417,8 +433,7 @@ def run_gpu(args):
 
     # ---- warmup + timed steps ----
     for _ in range(args.warmup):
-        launch(0)
-        launch(1)
+        step()
     torch.cuda.synchronize(dev)
     if world > 1:
         dist.barrier()
@@ -429,8 +444,7 @@ def run_gpu(args):
     n_launch0 = cl.launch_count()
     t_start = T.event()
     for _ in range(args.steps):
-        launch(0)
-        launch(1)
+        step()
     t_end = T.event()
     torch.cuda.synchronize(dev)
     gpu_launches = cl.launch_count() - n_launch0
@@ -579,6 +593,8 @@ def run_gpu(args):
                        "samples_per_step": samples_step, "launches_per_step": 2,
                        "timing": ("step: K steps between two events; kernel_ms: K back-to-back "
                                   "launches of that kernel between two events, right after"),
+                       "step": ("REPEAT read on the queue, MIRRORED read on a second queue of "
+                                "the device, joined by a marker and a barrier every step"),
                        "parallelism": ("single GPU" if world == 1 else
                                        f"row-sharded x{world}: global {Hg}x{N2D} image, "
                                        f"4096 output rows per GPU from shards of "
@@ -598,6 +614,7 @@ def run_gpu(args):
             "secondary": secondary,
         }
         print(json.dumps(line), flush=True)
+    L.clReleaseCommandQueue(q_two)
     S.release(*set(imgs), *outs)
     for s in smps:
         L.clReleaseSampler(s)
