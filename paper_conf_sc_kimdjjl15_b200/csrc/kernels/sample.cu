@@ -59,8 +59,20 @@ __global__ void __launch_bounds__(256) k_sample_grid(const SampleParams p) {
 #endif
   constexpr int PW = B2CL_GRID_PW, PH = 32 / PW;  // warp patch (PW x PH outputs)
   const int lane = threadIdx.x, w = threadIdx.y;
-  const int x = blockIdx.x * 32 + (w % (32 / PW)) * PW + (lane % PW);
-  const int y = blockIdx.y * 8 + (w / (32 / PW)) * PH + (lane / PW);
+#ifndef B2CL_GRID_QW
+#define B2CL_GRID_QW 0
+#endif
+#if B2CL_GRID_QW && B2CL_GRID_PW == 8
+  // each quarter-warp (8 lanes: one L1 wavefront group of 16-B loads) takes a
+  // QW x (8/QW) block of the 8 x 4 patch instead of one 8-wide row
+  constexpr int QW = B2CL_GRID_QW, QH = 8 / QW;
+  const int qq = lane >> 3, qr = lane & 7;
+  const int lx = (qq % (PW / QW)) * QW + qr % QW, ly = (qq / (PW / QW)) * QH + qr / QW;
+#else
+  const int lx = lane % PW, ly = lane / PW;
+#endif
+  const int x = blockIdx.x * 32 + (w % (32 / PW)) * PW + lx;
+  const int y = blockIdx.y * 8 + (w / (32 / PW)) * PH + ly;
 #else
   const int x = blockIdx.x * blockDim.x + threadIdx.x;
   const int y = blockIdx.y * blockDim.y + threadIdx.y;
