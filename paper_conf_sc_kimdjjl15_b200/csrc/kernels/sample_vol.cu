@@ -519,7 +519,7 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
 // sample keeps its own tap offsets and weights (8 samples per thread, one
 // column and 8 rows), the blend order is linear_at's: bit-identical results.
 #ifndef B2CL_VOLR_NS
-#define B2CL_VOLR_NS 3
+#define B2CL_VOLR_NS 4
 #endif
 #ifndef B2CL_VOLR_MINB
 #define B2CL_VOLR_MINB 2
