@@ -37,6 +37,8 @@ RT_F, RT_I, RT_UI = 0, 1, 2
 
 def build(force: bool = False) -> str:
     """Compile liboracle.so with gcc (-ffp-contract=off, no fast-math)."""
+    if os.environ.get("B2CL_ORACLE_LIB"):
+        return os.environ["B2CL_ORACLE_LIB"]
     if (not force and os.path.exists(_LIB)
             and os.path.getmtime(_LIB) >= max(os.path.getmtime(_SRC), os.path.getmtime(_HDR))):
         return _LIB
@@ -63,7 +65,9 @@ _lib = None
 def lib():
     global _lib
     if _lib is None:
-        L = ctypes.CDLL(build())
+        # B2CL_ORACLE_LIB: a prebuilt oracle library (tools/mutate_oracle.py
+        # loads deliberately mutated copies through it to prove the pins bite)
+        L = ctypes.CDLL(os.environ.get("B2CL_ORACLE_LIB") or build())
         sz3 = ctypes.POINTER(ctypes.c_size_t)
         P = ctypes.c_void_p
         i64, u32, i32 = ctypes.c_int64, ctypes.c_uint32, ctypes.c_int
