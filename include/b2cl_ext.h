@@ -230,6 +230,13 @@ cl_mem b2clCreateBufferFromIpcHandle(cl_context context, cl_device_id device,
 /* Number of b2cl kernels launched by this process so far (bench evidence). */
 cl_ulong b2clGetKernelLaunchCount(void);
 
+/* Name of the kernel the library's most recent launch from THIS host thread
+ * used (e.g. "k_sample_grid_tile"): the enqueue calls pick one kernel family
+ * per call (csrc/kernels/sample.cu launch_sample), and the bench reports which.
+ * Returns a static NUL-terminated string owned by the library ("" before the
+ * first launch); never NULL.  No side effects. */
+const char* b2clGetLastKernelName(void);
+
 /* ---- pure host validators (no GPU needed; the enqueue calls use them) ---- */
 
 /* Errors of clEnqueueCopyBufferRect for buffers of src_size / dst_size

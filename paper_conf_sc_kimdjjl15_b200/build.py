@@ -22,7 +22,7 @@ BUILD = os.path.join(ROOT, "build", "b2cl")
 LIB = os.path.join(HERE, "libb2cl.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
-SOURCES = ["kernels/sample.cu", "kernels/sample_vol.cu", "kernels/rect.cu", "runtime/runtime.cpp", "runtime/validate.cpp"]
+SOURCES = ["kernels/sample.cu", "kernels/sample_vol.cu", "kernels/sample_box.cu", "kernels/rect.cu", "runtime/runtime.cpp", "runtime/validate.cpp"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
          "-I" + os.path.join(ROOT, "include"), "-Xptxas", "-warn-spills"]

@@ -142,6 +142,7 @@ PROTOTYPES = {
     "b2clGetMemIpcHandle": (_I, [_H, _P]),
     "b2clCreateBufferFromIpcHandle": (_H, [_H, _H, _P, _S, _PI]),
     "b2clGetKernelLaunchCount": (_L, []),
+    "b2clGetLastKernelName": (ctypes.c_char_p, []),
     "b2clValidateCopyBufferRect": (_I, [_S, _S, _I, _SZ3, _SZ3, _SZ3, _S, _S, _S, _S]),
     "b2clRectOverlap": (_I, [_SZ3, _SZ3, _SZ3, _S, _S]),
     "b2clValidateFillBuffer": (_I, [_S, _S, _S, _S]),
@@ -242,6 +243,11 @@ def _ptr(a: np.ndarray) -> c_void_p:
 
 def launch_count() -> int:
     return int(lib().b2clGetKernelLaunchCount())
+
+
+def last_kernel() -> str:
+    """The kernel the library's last launch from this thread used."""
+    return lib().b2clGetLastKernelName().decode()
 
 
 # ---- torch allocator hook (device memory from PyTorch's caching allocator) ----

@@ -60,8 +60,13 @@ cudaError_t launch_sample_vol(const SampleParams& p, cudaStream_t stream, bool* 
 // ... and its rotated-map variant (x, y any affine in the output x, y; z separable)
 cudaError_t launch_sample_volr(const SampleParams& p, cudaStream_t stream, bool* used);
 
-// count of kernels launched by this library
+// ... and 2D RGBA32F LINEAR reads under any affine map (sample_box.cu)
+cudaError_t launch_sample_box(const SampleParams& p, cudaStream_t stream, bool* used);
+
+// count of kernels launched by this library; the name of the last kernel this
+// host thread launched (b2clGetLastKernelName: the bench reports it)
 uint64_t launch_count();
-void count_launch();
+void count_launch(const char* kernel);
+const char* last_kernel();
 
 }  // namespace b2cl

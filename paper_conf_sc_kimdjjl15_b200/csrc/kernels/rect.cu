@@ -323,7 +323,7 @@ static cudaError_t launch_rect_staged(const RectParams& p, cudaStream_t st) {
   const uint64_t units = cpr * p.R1 * p.R2;
   const uint64_t blocks = units < (uint64_t)sms * ST_BPS ? units : (uint64_t)sms * ST_BPS;
   k_rect_staged<<<(unsigned)blocks, ST_THREADS, smem, st>>>(p, cpr, units);
-  count_launch();
+  count_launch("k_rect_staged");
   return cudaGetLastError();
 }
 
@@ -360,7 +360,10 @@ cudaError_t launch_rect(RectParams& p, int mode, cudaStream_t st) {
     case RECT_FILL: k_rect<RECT_FILL, U><<<grd, blk, 0, st>>>(p); break;
     default: k_rect<RECT_FILL_IMAGE, U><<<grd, blk, 0, st>>>(p); break;
   }
-  count_launch();
+  count_launch(mode == RECT_COPY_ALIGNED ? "k_rect<COPY_ALIGNED>"
+               : mode == RECT_COPY       ? "k_rect<COPY>"
+               : mode == RECT_FILL       ? "k_rect<FILL>"
+                                         : "k_rect<FILL_IMAGE>");
   return cudaGetLastError();
 }
 
@@ -382,7 +385,7 @@ __global__ void __launch_bounds__(256) k_write(const WriteParams p) {
 cudaError_t launch_write(const WriteParams& p, cudaStream_t st) {
   if (p.n == 0) return cudaSuccess;
   k_write<<<(unsigned)((p.n + 255) / 256), 256, 0, st>>>(p);
-  count_launch();
+  count_launch("k_write");
   return cudaGetLastError();
 }
 

@@ -813,7 +813,7 @@ static cudaError_t go_grid(const SampleParams& p, cudaStream_t st) {
   dim3 grd((p.ow + 31) / 32, (p.oh + 7) / 8, p.od);
   if (is_shard(p)) k_sample_grid<WithShard<C, true>, OUTC><<<grd, blk, 0, st>>>(p);
   else k_sample_grid<WithShard<C, false>, OUTC><<<grd, blk, 0, st>>>(p);
-  count_launch();
+  count_launch("k_sample_grid");
   return cudaGetLastError();
 }
 
@@ -827,7 +827,7 @@ static cudaError_t go_walk(const SampleParams& p, cudaStream_t st) {
     grd = dim3((p.ow + 32 * XPT - 1) / (32 * XPT), (p.oh + 4 * WALK - 1) / (4 * WALK), p.od);
   if (is_shard(p)) k_sample_grid_walk<WithShard<C, true>, OUTC, XPT, WALK><<<grd, blk, 0, st>>>(p);
   else k_sample_grid_walk<WithShard<C, false>, OUTC, XPT, WALK><<<grd, blk, 0, st>>>(p);
-  count_launch();
+  count_launch("k_sample_grid_walk");
   return cudaGetLastError();
 }
 
@@ -837,7 +837,7 @@ static cudaError_t go_walk4(const SampleParams& p, cudaStream_t st) {
   dim3 grd((p.ow + 511) / 512, p.oh, (p.od + WALK - 1) / WALK);
   if (is_shard(p)) k_sample_grid_walk4<WithShard<C, true>, WALK><<<grd, blk, 0, st>>>(p);
   else k_sample_grid_walk4<WithShard<C, false>, WALK><<<grd, blk, 0, st>>>(p);
-  count_launch();
+  count_launch("k_sample_grid_walk4");
   return cudaGetLastError();
 }
 
@@ -856,7 +856,7 @@ static cudaError_t go_tile(const SampleParams& p, cudaStream_t st) {
   dim3 grd((p.ow + 63) / 64, (p.oh + TH - 1) / TH, p.od);
   if (is_shard(p)) k_sample_grid_tile<WithShard<C, true>, 64, TH><<<grd, blk, 0, st>>>(p);
   else k_sample_grid_tile<WithShard<C, false>, 64, TH><<<grd, blk, 0, st>>>(p);
-  count_launch();
+  count_launch("k_sample_grid_tile");
   return cudaGetLastError();
 }
 
@@ -890,7 +890,7 @@ static bool go_fold(const SampleParams& p, cudaStream_t st, cudaError_t* err) {
   dim3 grd((fm.Px + 63) / 64, (fm.Py + 15) / 16, p.od);
   if (is_shard(p)) k_sample_grid_fold<WithShard<C, true>><<<grd, 128, 0, st>>>(p, fm);
   else k_sample_grid_fold<WithShard<C, false>><<<grd, 128, 0, st>>>(p, fm);
-  count_launch();
+  count_launch("k_sample_grid_fold");
   *err = cudaGetLastError();
   return true;
 }
@@ -901,7 +901,7 @@ static cudaError_t go_sep(const SampleParams& p, cudaStream_t st) {
   dim3 grd((p.ow + 32 * XPT - 1) / (32 * XPT), (p.oh + 4 * RPW - 1) / (4 * RPW), p.od);
   if (is_shard(p)) k_sample_grid_sep<WithShard<C, true>, OUTC, XPT, RPW><<<grd, blk, 0, st>>>(p);
   else k_sample_grid_sep<WithShard<C, false>, OUTC, XPT, RPW><<<grd, blk, 0, st>>>(p);
-  count_launch();
+  count_launch("k_sample_grid_sep");
   return cudaGetLastError();
 }
 
@@ -925,7 +925,7 @@ static cudaError_t go_list(const SampleParams& p, bool int_coord, cudaStream_t s
     if (sh) k_sample_list<Cs, false><<<(unsigned)blocks, 256, 0, st>>>(p);
     else k_sample_list<Cp, false><<<(unsigned)blocks, 256, 0, st>>>(p);
   }
-  count_launch();
+  count_launch("k_sample_list");
   return cudaGetLastError();
 }
 
@@ -998,6 +998,13 @@ cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st
         default: return go_sep<Generic<3>, RT, 2, 2>(p, st);
       }
     }
+    // any other affine map of a 2D RGBA32F image (rotations): the TMA-staged
+    // footprint box (sample_box.cu), else one thread per sample
+    if (fk == 0 && !is_shard(p)) {
+      bool used = false;
+      const cudaError_t e = launch_sample_box(p, st, &used);
+      if (used || e != cudaSuccess) return e;
+    }
     if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_REPEAT, F_LINEAR)) return go_grid<C2Repeat, 4>(p, st);
     if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_MIRROR, F_LINEAR)) return go_grid<C2Mirror, 4>(p, st);
     if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR)) {
@@ -1029,7 +1036,12 @@ cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st
 }
 
 static std::atomic<uint64_t> g_launches{0};
-void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+static thread_local const char* g_last_kernel = "";
+void count_launch(const char* kernel) {
+  g_launches.fetch_add(1, std::memory_order_relaxed);
+  g_last_kernel = kernel ? kernel : "";
+}
 uint64_t launch_count() { return g_launches.load(std::memory_order_relaxed); }
+const char* last_kernel() { return g_last_kernel; }
 
 }  // namespace b2cl

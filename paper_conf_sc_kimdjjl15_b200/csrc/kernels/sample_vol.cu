@@ -860,7 +860,7 @@ static cudaError_t go_vol(const SampleParams& p, cudaStream_t st, bool* used) {
                 &grid))
     return cudaSuccess;
   k_sample_grid_vol<C><<<grid, VOL_THREADS, smem, st>>>(p, tl, tm);
-  count_launch();
+  count_launch("k_sample_grid_vol");
   *used = true;
   return cudaGetLastError();
 }
@@ -903,7 +903,7 @@ static cudaError_t go_volr(const SampleParams& p, cudaStream_t st, bool* used) {
                 &grid))
     return cudaSuccess;
   k_sample_grid_volr<C><<<grid, VOLR_THREADS, smem, st>>>(p, tl, g, tm);
-  count_launch();
+  count_launch("k_sample_grid_volr");
   *used = true;
   return cudaGetLastError();
 }

@@ -2208,7 +2208,7 @@ extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uin
     e = cudaLaunchKernel(fn, dim3((unsigned)grid[0], (unsigned)grid[1], (unsigned)grid[2]),
                          dim3((unsigned)Lw[0], (unsigned)Lw[1], (unsigned)Lw[2]), argp.data(),
                          local_bytes, q->stream);
-    if (e == cudaSuccess) count_launch();
+    if (e == cudaSuccess) count_launch("user kernel (clEnqueueNDRangeKernel)");
   }
   cl_int st = enq_end(E, e);
   if (st == CL_SUCCESS)
@@ -2218,3 +2218,5 @@ extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uin
 }
 
 extern "C" cl_ulong b2clGetKernelLaunchCount(void) { return launch_count(); }
+
+extern "C" const char* b2clGetLastKernelName(void) { return last_kernel(); }

@@ -30,3 +30,18 @@ def sess():
     S = cl.Session(0)
     yield S
     S.close()
+
+
+def pytest_terminal_summary(terminalreporter):
+    """Worst LINEAR error per parity check, in fp32 ulps (reading A10)."""
+    try:
+        from tests.gpu_helpers import WORST
+    except Exception:
+        return
+    if not WORST:
+        return
+    items = sorted(WORST.items(), key=lambda kv: -kv[1])
+    terminalreporter.write_line(f"LINEAR parity: {len(items)} checks, worst {items[0][1]:.2f} ulp "
+                                f"({items[0][0]}); bound 4 ulp, 1e-6 abs below 2^-10")
+    for what, u in items[:10]:
+        terminalreporter.write_line(f"  {u:5.2f} ulp  {what}")

@@ -10,7 +10,7 @@ import pytest
 
 from paper_conf_sc_kimdjjl15_b200 import cl, synth
 
-from tests.gpu_helpers import (VALID_SAMPLERS, assert_parity, gpu_read_grid,
+from tests.gpu_helpers import (VALID_SAMPLERS, assert_parity, parity_read, gpu_read_grid,
                          gpu_read_samples, rtype_of)
 
 pytestmark = pytest.mark.gpu
@@ -63,8 +63,8 @@ def test_array_samples_all_samplers(sess, orc, dims, fmt):
         smp = sess.sampler(bool(norm), addr, filt)
         co = _coords(g, 700, dims, W, H or 1, L, norm, False)
         got = gpu_read_samples(sess, img, smp, rt, co)
-        exp = orc.read_samples(oimg, bool(norm), addr, filt, rt, co)
-        assert_parity(got, exp, lin, f"{dims}D array {fmt} {norm} {addr:#x} {filt:#x}")
+        rd = lambda im: orc.read_samples(im, bool(norm), addr, filt, rt, co)  # noqa: E731
+        parity_read(got, rd(oimg), lin, f"{dims}D array {fmt} {norm} {addr:#x} {filt:#x}", orc, oimg, rd)
         if not norm and not lin:  # integer coordinates (reading A30)
             ci = _coords(g, 300, dims, W, H or 1, L, norm, True)
             got = gpu_read_samples(sess, img, smp, rt, ci, int_coords=True)
@@ -89,8 +89,8 @@ def test_array_grid(sess, orc, dims):
             continue  # unnormalized keeps the map readable; normalized is covered by samples
         smp = sess.sampler(False, addr, filt)
         got = gpu_read_grid(sess, img, smp, cl.B2CL_RTYPE_FLOAT, A, out, 4)
-        exp = orc.read_grid(oimg, False, addr, filt, orc.RT_F, np.array(A, np.float32), out, 4)
-        assert_parity(got, exp, filt == cl.CL_FILTER_LINEAR, f"grid {dims}D array {addr:#x}")
+        rd = lambda im: orc.read_grid(im, False, addr, filt, orc.RT_F, np.array(A, np.float32), out, 4)  # noqa: E731
+        parity_read(got, rd(oimg), filt == cl.CL_FILTER_LINEAR, f"grid {dims}D array {addr:#x}", orc, oimg, rd)
         cl.lib().clReleaseSampler(smp)
     sess.release(img)
 

@@ -18,7 +18,7 @@ import numpy as np
 import pytest
 
 from paper_conf_sc_kimdjjl15_b200 import cl, synth
-from tests.gpu_helpers import assert_parity
+from tests.gpu_helpers import assert_parity, parity_read
 
 pytestmark = pytest.mark.gpu
 
@@ -76,12 +76,14 @@ def _dyadic(c):
 def _check_both(orc, got, cl_img, tex_img, mode, filt, rmode, norm, rt, co, nch, what):
     """got: (n, nch) as uint32 bits; co: the coordinates (tex order)."""
     linear = filt == 1
-    exp = orc.read_samples(cl_img, norm, CL_ADDR[mode], CL_FILT[filt], rt, co).view(np.uint32)[:, :nch]
     dt = np.float32 if rt == orc.RT_F else np.uint32
-    assert_parity(got.view(dt), np.ascontiguousarray(exp).view(dt), linear, what + " vs read_imageX")
-    cu = orc.tex_fetch(tex_img, [mode] * 3, filt, rmode, norm, co)[:, :nch]
+    rd = lambda im: np.ascontiguousarray(  # noqa: E731
+        orc.read_samples(im, norm, CL_ADDR[mode], CL_FILT[filt], rt, co).view(np.uint32)[:, :nch]).view(dt)
+    parity_read(got.view(dt), rd(cl_img), linear, what + " vs read_imageX", orc, cl_img, rd)
     keep = np.ones(co.shape[0], bool) if mode != 2 else _dyadic(co[:, :tex_img.dims])
-    assert_parity(got[keep].view(dt), np.ascontiguousarray(cu[keep]).view(dt), linear, what + " vs CUDA")
+    rt_ = lambda im: np.ascontiguousarray(  # noqa: E731
+        orc.tex_fetch(im, [mode] * 3, filt, rmode, norm, co)[:, :nch][keep]).view(dt)
+    parity_read(got[keep].view(dt), rt_(tex_img), linear, what + " vs CUDA", orc, tex_img, rt_)
 
 
 @pytest.mark.parametrize("mode", [0, 1, 2, 3])
