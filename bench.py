@@ -4,25 +4,42 @@
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl b2cl|reference]
     python -m torch.distributed.run --nproc-per-node N ... bench.py --gpus N ...
 
-Workload (BASELINE.json configs[1], the config the metric is quoted on):
-a 4096x4096 CL_RGBA/CL_FLOAT image, normalized coordinates, LINEAR filter.
-One STEP = read_imagef over the full 4096^2 output grid under REPEAT and
-again under MIRRORED_REPEAT (map (A): translate by (0.3, 0.7) px plus a half
-period so the wrap seam crosses the output), i.e. two launches of the
-sampling kernel, 2 x 16.8 M samples.  `value` = samples / step time in
-Gsamples/s, whole job (sum over ranks; each rank owns its own image: weak
-scaling, no collective on the data path).
+N = 1 -- BASELINE.json configs[1], the config the metric is quoted on: a
+4096x4096 CL_RGBA/CL_FLOAT image, normalized coordinates, LINEAR filter.  One
+STEP = read_imagef over the full 4096^2 output grid under REPEAT and again
+under MIRRORED_REPEAT (map (A): translate by (0.3, 0.7) px plus a half period
+so the wrap seam crosses the output), i.e. two launches, 2 x 16.8 M samples.
+`value` = samples / step time in Gsamples/s.
 
-Secondary measurements in the same JSON line (`secondary`): config 3
-(512^3 R32F trilinear), config 4 (8 GiB pitched CopyBufferRect, FillBuffer,
-CopyImageToBuffer) and the copy-size sweep, each with its HBM fraction.
+N > 1 -- BASELINE.json configs[4] (C5): ONE 32768x32768 RGBA32F image (16 GiB)
+row-sharded over the N ranks (one process per GPU): rank d owns texel rows
+[d H/N, (d+1) H/N) in an IPC-exportable band image; for each pass it holds a
+shard of exactly the texel rows its output band [d H/N, (d+1) H/N) needs,
+filled by cross-device clEnqueueCopyImage region copies from the owners' band
+images (NVLink P2P, in place: no whole-object migration); a step = the
+REPEAT and MIRRORED reads of its output band, bit-identical to one GPU's
+(tests/test_gpu_shards.py).  Strong scaling: `value` = 2 x 32768^2 samples /
+the slowest rank's step time.  Also measured: the shard fill (the P2P
+exchange) and a ring migration of every owner band to its right neighbour
+through clEnqueueMigrateMemObjects, against the copy engines'
+(b2clEnqueueCopyBufferEngine) time for the same bytes in the same run -- the
+NVLink denominator.  The C5 image on ONE GPU is the `c5_image_32768_1gpu`
+secondary of the N = 1 line.
+
+Secondary measurements in the N = 1 line (`secondary`): config 2 map (B)
+(30 degree rotation), config 3 (512^3 R32F trilinear, stencil and rotated
+maps), config 4 (8 GiB pitched CopyBufferRect, FillBuffer with patterns 1, 4,
+16, 128 B, the 22-point CopyImageToBuffer sweep 4 KiB .. 8 GiB) and the host
+cost of one enqueue measured from C (tools/enqueue_bench.c), each with its
+HBM fraction.
 
 Timing: CUDA events on the queue's stream around every launch, after W
 untimed steps, barrier + synchronize on both sides, max over ranks.  The
 working set (256 MiB image + 2 x 256 MiB output) exceeds the 126 MB L2, so no
-flush is needed between steps.  Clocks are sampled with nvidia-smi during
-the timed region.  `--impl reference` times the CPU oracle (oracle/) on the
-host cores on a bounded sample of the same workload.
+flush is needed between steps.  Clocks are sampled with NVML during the timed
+region.  The dominant kernel's DRAM traffic is captured by ncu in a separate
+process of this run (`roofline.traffic`).  `--impl reference` times the CPU
+oracle (oracle/) on the host cores on a bounded sample of the same workload.
 """
 from __future__ import annotations
 
@@ -237,6 +254,79 @@ def _distinct_texels_2d(A, W, H, mode, chunk=256):
     return int(seen.sum())
 
 
+def linear_parity(got, exp):
+    """Reading A10, the tests' rule (tests/gpu_helpers.py): |g - o| <= 4 ulp(o),
+    the 1e-6 absolute floor only near zero (|o| < 2^-10), NaN iff NaN.
+    Returns (ok, worst error in ulps over |o| >= 2^-10)."""
+    got = np.asarray(got, np.float32)
+    exp = np.asarray(exp, np.float32)
+    gn, en = np.isnan(got), np.isnan(exp)
+    if not np.array_equal(gn, en):
+        return False, float("inf")
+    g, e = got[~en].astype(np.float64), exp[~en].astype(np.float64)
+    err = np.abs(g - e)
+    mag = np.abs(exp[~en])
+    ulp = np.spacing(mag).astype(np.float64)
+    near = mag < 2.0 ** -10
+    bad = np.where(near, err > 1e-6, err > 4.0 * ulp)
+    worst = float((err[~near] / ulp[~near]).max()) if (~near).any() else 0.0
+    return not bad.any(), worst
+
+
+def ncu_traffic(kernels, which, timeout=300):
+    """DRAM bytes (read + write) and duration per launch of each kernel named in
+    `kernels`, from ONE ncu capture of tools/prof_kernels.py `which` (a separate
+    process of this run; cold cache, clocks not locked).  Returns
+    {kernel: {...}} or {"unavailable": why}."""
+    import csv
+    import io
+    import shutil
+    ncu = shutil.which("ncu") or "/usr/local/cuda/bin/ncu"
+    if not os.path.exists(ncu):
+        return {"unavailable": "ncu not found"}
+    regex = "|".join(kernels)
+    cmd = [ncu, "--metrics", "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum",
+           "--clock-control", "none", "--csv", "-k", f"regex:{regex}", "-c", str(len(kernels)),
+           sys.executable, os.path.join(ROOT, "tools", "prof_kernels.py"), *which]
+    try:
+        r = subprocess.run(cmd, capture_output=True, text=True, timeout=timeout, cwd=ROOT)
+    except subprocess.TimeoutExpired:
+        return {"unavailable": f"ncu timed out after {timeout} s"}
+    rows = [ln for ln in r.stdout.splitlines() if ln.startswith('"')]
+    if not rows:
+        return {"unavailable": f"ncu produced no rows (rc {r.returncode}): " + (r.stderr or r.stdout)[-200:]}
+    out = {}
+    for rec in csv.DictReader(io.StringIO("\n".join(rows))):
+        name = rec.get("Kernel Name", "")
+        key = next((k for k in kernels if k in name), name)
+        unit, val = rec.get("Metric Unit", ""), float(rec.get("Metric Value", "0").replace(",", ""))
+        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "MB": 1e6, "GB": 1e9,
+                 "nsecond": 1e-9, "usecond": 1e-6, "msecond": 1e-3, "ns": 1e-9, "us": 1e-6, "ms": 1e-3}.get(unit, 1)
+        out.setdefault(key, {})[rec.get("Metric Name", "")] = val * scale
+    res = {}
+    for k, m in out.items():
+        rd, wr = m.get("dram__bytes_read.sum", 0.0), m.get("dram__bytes_write.sum", 0.0)
+        res[k] = {"dram_read_bytes": rd, "dram_write_bytes": wr, "traffic_bytes": rd + wr,
+                  "ncu_us": m.get("gpu__time_duration.sum", 0.0) * 1e6}
+    return res or {"unavailable": "no matching kernel in the capture"}
+
+
+def enqueue_cost():
+    """Host cost of one enqueue measured from C (tools/enqueue_bench.c, compiled
+    here with gcc if needed; no Python in the loop)."""
+    exe = os.path.join(ROOT, "build", "enqueue_bench")
+    src = os.path.join(ROOT, "tools", "enqueue_bench.c")
+    try:
+        if not os.path.exists(exe) or os.path.getmtime(exe) < os.path.getmtime(src):
+            os.makedirs(os.path.dirname(exe), exist_ok=True)
+            subprocess.run(["gcc", "-O2", "-o", exe, src, "-ldl"], check=True, capture_output=True)
+        r = subprocess.run([exe, os.path.join(ROOT, "paper_conf_sc_kimdjjl15_b200", "libb2cl.so")],
+                           capture_output=True, text=True, timeout=120, cwd=ROOT)
+        return json.loads(r.stdout.strip().splitlines()[-1])
+    except Exception as exc:  # a secondary measurement, never fatal
+        return {"unavailable": str(exc)[:200]}
+
+
 def circular_interval(idx, n):
     """Smallest (begin, count) whose circular range {(begin+s) mod n} covers idx."""
     rows = np.unique(np.asarray(idx, dtype=np.int64))
@@ -319,67 +409,33 @@ class Timer:
 
 def run_gpu(args):
     import torch
-    import torch.distributed as dist
-
-    from paper_conf_sc_kimdjjl15_b200 import build, cl, synth
-    from paper_conf_sc_kimdjjl15_b200 import dist as bdist
-    build.build()
     world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    # one GPU per rank; more ranks than GPUs only happens in the single-GPU
-    # rehearsal of the multi-rank path (ranks share a device, control plane on gloo)
-    ndev = torch.cuda.device_count()
-    gpu = local % ndev
-    shared = world > ndev
-    torch.cuda.set_device(gpu)
     if world > 1:
-        if shared:
-            dist.init_process_group("gloo")
-        else:
-            dist.init_process_group("nccl", device_id=torch.device("cuda", gpu))
+        return run_c5(args)
+    from paper_conf_sc_kimdjjl15_b200 import build, cl
+    build.build()
+    gpu = int(os.environ.get("LOCAL_RANK", "0")) % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(gpu)
     dev = torch.device("cuda", gpu)
-    red_dev = None if shared else dev  # device of the max-over-ranks tensors
     stream = torch.cuda.Stream(device=dev)
     S = cl.Session(gpu, stream=stream.cuda_stream)
     L = cl.lib()
     T = Timer(torch, stream)
     hbm_peak, peak_src = peaks()
 
-    # ---- inputs resident in HBM before timing ----
-    # N = 1: config 2 itself, one 4096^2 image.  N > 1 (config 5 style): one
-    # global (4096*N) x 4096 image, row-sharded: rank r computes output rows
-    # [4096 r, 4096 (r+1)) of map (A) on the GLOBAL image from shards holding
-    # exactly the texel rows that band needs (one per pass: REPEAT and the
-    # folded MIRRORED rows differ) -- bit-identical to a single-GPU read
-    # (tests/test_gpu_shards.py), same per-GPU work as N = 1 (weak scaling).
-    Hg = N2D * world
-    r0 = rank * N2D
-    Af = synth.affine_translate_2d(N2D, Hg)
+    # ---- inputs resident in HBM before timing: config 2, one 4096^2 image ----
+    from paper_conf_sc_kimdjjl15_b200 import synth
+    Af = synth.affine_translate_2d(N2D, N2D)
     A = (ctypes.c_float * 12)(*Af.tolist())
     modes = ("repeat", "mirrored")
-    codes = None
-    shard_rows, shard_host, shard_begin = [], [], []
-    if world == 1:
-        codes = c2_codes()
-        img = S.image(cl.CL_RGBA, cl.CL_FLOAT, N2D, N2D, host=codes)
-        imgs = [img, img]
-    else:
-        imgs = []
-        for m in modes:
-            need = _axis_taps(Af[5], Af[7], N2D, Hg, m, start=r0)
-            begin, count = circular_interval(need, Hg)
-            rows = [(begin + s) % Hg for s in range(count)]
-            shard_rows.append(count)
-            shard_begin.append(begin)
-            shard_host.append(synth.image_rows(cl.CL_RGBA, cl.CL_FLOAT, N2D, rows))
-            imgs.append(S.image_shard(cl.CL_RGBA, cl.CL_FLOAT, N2D, Hg, 0, begin, count, 0,
-                                      host=shard_host[-1]))
+    codes = c2_codes()
+    img = S.image(cl.CL_RGBA, cl.CL_FLOAT, N2D, N2D, host=codes)
+    imgs = [img, img]
     nout = N2D * N2D * 16
     outs = [S.buffer(nout), S.buffer(nout)]
     smps = [S.sampler(True, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR),
             S.sampler(True, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR)]
-    origin, region = cl.sz3((0, r0, 0)), cl.sz3((N2D, N2D, 1))
+    origin, region = cl.sz3((0, 0, 0)), cl.sz3((N2D, N2D, 1))
 
     def launch(k, images=None, queue=None, nwait=0, wait=None, ev=None):
         cl.check(L.b2clEnqueueReadImageGridRegion(queue or S.queue, (images or imgs)[k], smps[k],
@@ -404,39 +460,37 @@ def run_gpu(args):
         L.clReleaseEvent(e1)
 
     # ---- parity spot check of this exact launch configuration (bench as test) ----
-    launch(0)
-    launch(1)
+    kernels = []
+    for k in range(2):
+        launch(k)
+        kernels.append(cl.last_kernel())  # the kernel the library picked for this pass
     S.finish()
     parity = "skipped (oracle missing)"
-    if world > 1:
-        parity = ("sharded: bit-identity of shard reads to whole-image reads is tested in "
-                  "tests/test_gpu_shards.py; the whole-image path is checked against the oracle")
-    else:
-        try:
-            import oracle as orc
-            oimg = orc.Image(codes, N2D, N2D, 1, dims=2, order=orc.RGBA, type=orc.FLOAT)
-            worst = 0.0
-            for k, a in enumerate((orc.ADDRESS_REPEAT, orc.ADDRESS_MIRRORED_REPEAT)):
-                got = S.read(outs[k], nout, np.float32).reshape(N2D, N2D, 4)
-                for y in (0, N2D // 2 - 1, N2D // 2, N2D - 1, 1234):
-                    exp = orc.read_grid(oimg, True, a, orc.FILTER_LINEAR, orc.RT_F, Af,
-                                        (N2D, N2D, 1), 4, yrange=(y, y + 1))[0, 0]
-                    err = np.abs(got[y].astype(np.float64) - exp) / np.maximum(
-                        np.spacing(np.abs(exp)).astype(np.float64), 1e-30)
-                    ok = np.all((err <= 4) | (np.abs(got[y] - exp) <= 1e-6))
-                    worst = max(worst, float(np.max(np.minimum(err, 1e9))))
-                    if not ok:
-                        raise SystemExit(f"bench parity check failed (pass {k}, row {y})")
-            parity = f"ok (10 rows vs oracle, worst {worst:.2f} ulp)"
-        except ImportError:
-            pass
+    try:
+        import oracle as orc
+        oimg = orc.Image(codes, N2D, N2D, 1, dims=2, order=orc.RGBA, type=orc.FLOAT)
+        worst, nrows = 0.0, 0
+        rows = sorted({0, 1, N2D // 2 - 2, N2D // 2 - 1, N2D // 2, N2D // 2 + 1, N2D - 2, N2D - 1}
+                      | set(range(97, N2D, 331)))
+        for k, a in enumerate((orc.ADDRESS_REPEAT, orc.ADDRESS_MIRRORED_REPEAT)):
+            got = S.read(outs[k], nout, np.float32).reshape(N2D, N2D, 4)
+            for y in rows:
+                exp = orc.read_grid(oimg, True, a, orc.FILTER_LINEAR, orc.RT_F, Af,
+                                    (N2D, N2D, 1), 4, yrange=(y, y + 1))[0, 0]
+                ok, w = linear_parity(got[y], exp)
+                worst = max(worst, w)
+                nrows += 1
+                if not ok:
+                    raise SystemExit(f"bench parity check failed (pass {k}, row {y}, {w:.2f} ulp)")
+        parity = (f"ok ({nrows} full rows of both passes vs the oracle incl. the seam and edge rows; "
+                  f"worst {worst:.2f} ulp, bound 4 ulp / 1e-6 below 2^-10)")
+    except ImportError:
+        pass
 
     # ---- warmup + timed steps ----
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize(dev)
-    if world > 1:
-        dist.barrier()
     clocks = Clocks(gpu)
     clocks.start()
     # (1) the step time: K steps back to back, events only at the two ends
@@ -461,212 +515,469 @@ def run_gpu(args):
         pass_ms.append(a.elapsed_time(b) / args.steps)
     clk = clocks.stop()
     ms_step = total_ms / args.steps
-    if world > 1:
-        ms_step = bdist.max_over_ranks(ms_step, red_dev)
     samples_step = 2 * N2D * N2D
-    value = world * samples_step / (ms_step * 1e-3) / 1e9
+    value = samples_step / (ms_step * 1e-3) / 1e9
     # algorithmic bytes per launch = distinct texels with a non-zero tap weight x 16 B
     # + 16 B output per sample; counted exactly per map on the host
     ncols = [_axis_taps(Af[0], Af[3], N2D, N2D, m).size for m in modes]
-    nrows = [_axis_taps(Af[5], Af[7], N2D, Hg, m, start=r0).size for m in modes]
-    alg = [ncols[k] * nrows[k] * 16 + N2D * N2D * 16 for k in range(2)]
+    nrows_t = [_axis_taps(Af[5], Af[7], N2D, N2D, m).size for m in modes]
+    alg = [ncols[k] * nrows_t[k] * 16 + N2D * N2D * 16 for k in range(2)]
     achieved = [alg[k] / (pass_ms[k] * 1e-3) / 1e9 for k in range(2)]
-    dom = 0 if pass_ms[0] * 1.0 >= pass_ms[1] else 1  # the kernel with the larger share of the step
-    traffic = None
-    import glob
-    profs = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*", "ncu_c2_traffic.json")))
-    if profs:
-        traffic = json.load(open(profs[-1])).get("dram_bytes_per_launch")
+    dom = 0 if pass_ms[0] >= pass_ms[1] else 1  # the kernel with the larger share of the step
 
-    # ---- e2e: host buffers through the C-ABI, copies inside the timed region ----
-    # Every step uploads its image(s) from pinned host memory and reads both
-    # outputs back to pinned host memory.  The copies are the step's bound
-    # (256 MiB up, 512 MiB down over the host link per GPU), so the step is
-    # pipelined the way an OpenCL program would: uploads on a second queue
-    # into one of two image copies, so step s+1's upload runs while step s's
-    # results come down; cross-queue order by events only (wait lists).
     e2e = None
     if not args.no_e2e:
-        q_up = S.queue_for(gpu)
-        hbufs = []
-        for k in range(1 if world == 1 else 2):
-            hrows = N2D if world == 1 else shard_rows[k]
-            hbuf = torch.empty(hrows * N2D * 16, dtype=torch.uint8).pin_memory()
-            src = codes if world == 1 else shard_host[k]
-            hbuf.copy_(torch.from_numpy(np.ascontiguousarray(src).reshape(-1).view(np.uint8)))
-            hbufs.append((hbuf, cl.sz3((N2D, hrows, 1))))
-        # two device copies of the step's images (copy 0 is the resident one)
-        e2e_imgs = [imgs]
-        if world == 1:
-            im2 = S.image(cl.CL_RGBA, cl.CL_FLOAT, N2D, N2D)
-            e2e_imgs.append([im2, im2])
-        else:
-            e2e_imgs.append([S.image_shard(cl.CL_RGBA, cl.CL_FLOAT, N2D, Hg, 0, shard_begin[k],
-                                           shard_rows[k], 0) for k in range(2)])
-        host_out = [torch.empty(nout, dtype=torch.uint8).pin_memory() for _ in range(2)]
-        zero3 = cl.sz3((0, 0, 0))
-        done = [None, None]  # marker event of the last step that read image copy b
-
-        def e2e_step(s, first_wait=None):
-            b = s % 2
-            wl = [e for e in (done[b], first_wait) if e]
-            wla = (ctypes.c_void_p * 2)(*wl) if wl else None
-            up = ctypes.c_void_p()
-            targets = e2e_imgs[b][:1] if world == 1 else e2e_imgs[b]
-            for k, (im, (hbuf, reg)) in enumerate(zip(targets, hbufs)):
-                last = k == len(hbufs) - 1
-                cl.check(L.clEnqueueWriteImage(q_up, im, 0, zero3, reg, 0, 0,
-                                               ctypes.c_void_p(hbuf.data_ptr()), len(wl), wla,
-                                               ctypes.byref(up) if last else None))
-            upa = (ctypes.c_void_p * 1)(up)
-            cl.check(L.clEnqueueBarrierWithWaitList(S.queue, 1, upa, None))
-            L.clReleaseEvent(up)
-            for k in range(2):
-                launch(k, e2e_imgs[b])
-                cl.check(L.clEnqueueReadBuffer(S.queue, outs[k], 0, 0, nout,
-                                               ctypes.c_void_p(host_out[k].data_ptr()), 0, None, None))
-            ev = ctypes.c_void_p()
-            cl.check(L.clEnqueueMarkerWithWaitList(S.queue, 0, None, ctypes.byref(ev)))
-            if done[b]:
-                L.clReleaseEvent(done[b])
-            done[b] = ev.value
-
-        for s in range(2):
-            e2e_step(s)
-        S.finish()
-        cl.check(L.clFinish(q_up))
-        if world > 1:
-            dist.barrier()
-        steps_e2e = max(4, args.steps // 4)
-        a = T.event()
-        start = ctypes.c_void_p()  # the first upload starts after the start event
-        cl.check(L.clEnqueueMarkerWithWaitList(S.queue, 0, None, ctypes.byref(start)))
-        for s in range(steps_e2e):
-            e2e_step(s, start.value if s == 0 else None)
-        b_ev = T.event()
-        torch.cuda.synchronize(dev)
-        cl.check(L.clFinish(q_up))
-        L.clReleaseEvent(start)
-        for e in done:
-            if e:
-                L.clReleaseEvent(e)
-        e2e_ms = a.elapsed_time(b_ev) / steps_e2e
-        if world > 1:
-            e2e_ms = bdist.max_over_ranks(e2e_ms, red_dev)
-        # the downloaded results are this step's: spot-check one row of each pass
-        for k in range(2):
-            dev_row = S.read(outs[k], N2D * 16, np.uint8, offset=N2D * 16 * 777)
-            assert np.array_equal(host_out[k].numpy()[N2D * 16 * 777:N2D * 16 * 778], dev_row)
-        e2e = {"value": world * samples_step / (e2e_ms * 1e-3) / 1e9, "unit": "Gsamples/s",
-               "ms_per_step": e2e_ms, "h2d_bytes_per_step": int(sum(h[0].numel() for h in hbufs)),
-               "d2h_bytes_per_step": 2 * nout,
-               "pipeline": "uploads on a second queue into two image copies, overlapping the previous "
-                           "step's downloads (event-ordered)"}
-        S.release(*[im for im in set(e2e_imgs[1])])
-        L.clReleaseCommandQueue(q_up)
+        e2e = run_e2e_c2(S, L, T, torch, dev, gpu, codes, imgs, outs, launch, samples_step, nout, args)
 
     secondary = None
     if not args.no_secondary:
         secondary = run_secondary(S, L, T, torch, dev, hbm_peak, args)
-    if world > 1 and not args.no_p2p:
-        secondary = secondary or {}
-        secondary["p2p_ring_migrate"] = run_p2p_ring(S, L, T, torch, dev, red_dev, rank, world)
+    L.clReleaseCommandQueue(q_two)
+    S.release(img, *outs)
+    for sm in smps:
+        L.clReleaseSampler(sm)
+    S.close()
+
+    # ---- DRAM traffic of both passes: ncu in a separate process of this run ----
+    traffic = {"unavailable": "--no-ncu"}
+    if not args.no_ncu:
+        traffic = ncu_traffic(kernels, ["c2r", "c2m"])
+    traffic_dom = traffic.get(kernels[dom], {}).get("traffic_bytes") if "unavailable" not in traffic else None
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu:  # the oracle baseline: N = 1 only
+    if not args.no_cpu:  # the oracle baseline: all host cores, and one thread
         try:
             threads = os.cpu_count() or 1
             rate, rows, dt = oracle_rate(codes, args.cpu_seconds, threads)
+            rate1, rows1, dt1 = oracle_rate(codes, args.cpu_seconds / 2, 1)
             cpu = {"value": rate, "unit": "Gsamples/s", "cores": threads, "kind": "oracle",
                    "sample": f"{rows} rows x {N2D} columns of each pass (REPEAT, MIRRORED), "
-                             f"{dt:.1f} s on {threads} threads"}
+                             f"{dt:.1f} s on {threads} threads",
+                   "single_thread": {"value": rate1, "unit": "Gsamples/s", "cores": 1,
+                                     "sample": f"{rows1} rows x {N2D} columns of each pass, {dt1:.1f} s"}}
         except ImportError:
             cpu = None
+
+    line = {
+        "metric": METRIC, "value": value, "unit": "Gsamples/s", "n_gpus": 1,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic (numpy default_rng seed 20151115; U[0,1) RGBA32F texels)",
+        "config": {"workload": WORKLOAD, "image": "4096x4096 RGBA32F (256 MiB)",
+                   "samples_per_step": samples_step, "launches_per_step": 2,
+                   "kernels": kernels,
+                   "timing": ("step: K steps between two events; kernel_ms: K back-to-back "
+                              "launches of that kernel between two events, right after"),
+                   "step": ("REPEAT read on the queue, MIRRORED read on a second queue of "
+                            "the device, joined by a marker and a barrier every step"),
+                   "parallelism": "single GPU",
+                   "l2": "no flush: 768 MiB working set > 126 MB L2", "parity": parity},
+        "roofline": {"bound": "hbm", "achieved": achieved[dom], "peak": hbm_peak, "unit": "GB/s",
+                     "frac": achieved[dom] / hbm_peak, "traffic": traffic_dom,
+                     "kernel": kernels[dom], "kernel_ms": pass_ms[dom],
+                     "algorithmic_bytes_per_launch": alg[dom], "peak_source": peak_src,
+                     "traffic_source": ("ncu dram__bytes_read.sum + dram__bytes_write.sum, one cold-cache "
+                                        "launch captured in a separate process of this run"),
+                     "per_pass": [{"mode": m, "kernel": kernels[k], "ms": pass_ms[k], "algorithmic_bytes": alg[k],
+                                   "GB/s": achieved[k], "frac": achieved[k] / hbm_peak,
+                                   "ncu": traffic.get(kernels[k]) if "unavailable" not in traffic else traffic}
+                                  for k, m in enumerate(modes)],
+                     "step_frac": sum(alg) / (sum(pass_ms) * 1e-3) / 1e9 / hbm_peak},
+        "cpu_baseline": cpu, "e2e": e2e, "clocks": clk, "gpu_launches": gpu_launches,
+        "secondary": secondary,
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_e2e_c2(S, L, T, torch, dev, gpu, codes, imgs, outs, launch, samples_step, nout, args):
+    """e2e: host buffers through the C-ABI, copies inside the timed region.
+    Every step uploads the image from pinned host memory and reads both outputs
+    back to pinned host memory.  The copies are the step's bound (256 MiB up,
+    512 MiB down over the host link), so the step is pipelined the way an
+    OpenCL program would: uploads on a second queue into one of two image
+    copies, so step s+1's upload runs while step s's results come down;
+    cross-queue order by events only (wait lists)."""
+    from paper_conf_sc_kimdjjl15_b200 import cl
+    q_up = S.queue_for(gpu)
+    hbuf = torch.empty(N2D * N2D * 16, dtype=torch.uint8).pin_memory()
+    hbuf.copy_(torch.from_numpy(np.ascontiguousarray(codes).reshape(-1).view(np.uint8)))
+    reg = cl.sz3((N2D, N2D, 1))
+    im2 = S.image(cl.CL_RGBA, cl.CL_FLOAT, N2D, N2D)
+    e2e_imgs = [imgs, [im2, im2]]  # two device copies of the step's image (copy 0 is the resident one)
+    host_out = [torch.empty(nout, dtype=torch.uint8).pin_memory() for _ in range(2)]
+    zero3 = cl.sz3((0, 0, 0))
+    done = [None, None]  # marker event of the last step that read image copy b
+
+    def e2e_step(s, first_wait=None):
+        b = s % 2
+        wl = [e for e in (done[b], first_wait) if e]
+        wla = (ctypes.c_void_p * 2)(*wl) if wl else None
+        up = ctypes.c_void_p()
+        cl.check(L.clEnqueueWriteImage(q_up, e2e_imgs[b][0], 0, zero3, reg, 0, 0,
+                                       ctypes.c_void_p(hbuf.data_ptr()), len(wl), wla, ctypes.byref(up)))
+        cl.check(L.clEnqueueBarrierWithWaitList(S.queue, 1, (ctypes.c_void_p * 1)(up), None))
+        L.clReleaseEvent(up)
+        for k in range(2):
+            launch(k, e2e_imgs[b])
+            cl.check(L.clEnqueueReadBuffer(S.queue, outs[k], 0, 0, nout,
+                                           ctypes.c_void_p(host_out[k].data_ptr()), 0, None, None))
+        ev = ctypes.c_void_p()
+        cl.check(L.clEnqueueMarkerWithWaitList(S.queue, 0, None, ctypes.byref(ev)))
+        if done[b]:
+            L.clReleaseEvent(done[b])
+        done[b] = ev.value
+
+    for s in range(2):
+        e2e_step(s)
+    S.finish()
+    cl.check(L.clFinish(q_up))
+    steps_e2e = max(4, args.steps // 4)
+    a = T.event()
+    start = ctypes.c_void_p()  # the first upload starts after the start event
+    cl.check(L.clEnqueueMarkerWithWaitList(S.queue, 0, None, ctypes.byref(start)))
+    for s in range(steps_e2e):
+        e2e_step(s, start.value if s == 0 else None)
+    b_ev = T.event()
+    torch.cuda.synchronize(dev)
+    cl.check(L.clFinish(q_up))
+    L.clReleaseEvent(start)
+    for e in done:
+        if e:
+            L.clReleaseEvent(e)
+    e2e_ms = a.elapsed_time(b_ev) / steps_e2e
+    # the downloaded results are this step's: spot-check one row of each pass
+    for k in range(2):
+        dev_row = S.read(outs[k], N2D * 16, np.uint8, offset=N2D * 16 * 777)
+        assert np.array_equal(host_out[k].numpy()[N2D * 16 * 777:N2D * 16 * 778], dev_row)
+    S.release(im2)
+    L.clReleaseCommandQueue(q_up)
+    return {"value": samples_step / (e2e_ms * 1e-3) / 1e9, "unit": "Gsamples/s",
+            "ms_per_step": e2e_ms, "h2d_bytes_per_step": int(hbuf.numel()),
+            "d2h_bytes_per_step": 2 * nout,
+            "pipeline": "uploads on a second queue into two image copies, overlapping the previous "
+                        "step's downloads (event-ordered)"}
+
+
+C5 = 32768
+C5_WORKLOAD = ("C5: 32768x32768 CL_RGBA/CL_FLOAT row-sharded over N GPUs (one process per GPU), "
+               "normalized, LINEAR, REPEAT + MIRRORED_REPEAT, map (A)")
+
+
+def _runs(rows, lo, hi):
+    """Maximal runs [a, b) of consecutive global rows inside [lo, hi), in order."""
+    out = []
+    for i, r in enumerate(rows):
+        if not (lo <= r < hi):
+            continue
+        if out and out[-1][1] == r and out[-1][2] + 1 == i:
+            out[-1] = (out[-1][0], r + 1, i)
+        else:
+            out.append((r, r + 1, i))
+    return [(a, b, i - (b - a - 1)) for a, b, i in out]
+
+
+def run_c5(args):
+    """BASELINE configs[4] at N > 1 (see the module docstring).  Control plane:
+    gloo (barrier, max over ranks, 64-byte IPC handles); no NCCL -- nothing
+    reduces on the data path."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_kimdjjl15_b200 import build, cl, synth
+    from paper_conf_sc_kimdjjl15_b200 import dist as bdist
+    build.build()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    ndev = torch.cuda.device_count()
+    gpu = local % ndev
+    shared = world > ndev  # the single-GPU rehearsal: ranks share a device (IPC, not NVLink)
+    torch.cuda.set_device(gpu)
+    dist.init_process_group("gloo")
+    dev = torch.device("cuda", gpu)
+    stream = torch.cuda.Stream(device=dev)
+    S = cl.Session(gpu, stream=stream.cuda_stream)
+    L = cl.lib()
+    T = Timer(torch, stream)
+    hbm_peak, peak_src = peaks()
+    err = ctypes.c_int32()
+    H = W = args.c5_size
+    band = H // world
+    assert H % world == 0 and band % 256 == 0, "band rows: a multiple of 256"
+    r0 = rank * band
+    fmt = cl.ImageFormat(cl.CL_RGBA, cl.CL_FLOAT)
+    gdesc = cl.ImageDesc(cl.CL_MEM_OBJECT_IMAGE2D, W, H, 0, 0, 0, 0, 0, 0, None)
+    bdesc = cl.ImageDesc(cl.CL_MEM_OBJECT_IMAGE2D, W, band, 0, 0, 0, 0, 0, 0, None)
+    rowb = W * 16
+
+    # ---- 1. the owned band: global texel rows [r0, r0 + band), IPC-exportable.
+    # Content: global row j = seeded block row (j mod 256) (synth.image_rows): one
+    # 128 MiB block uploaded, then doubled in place by clEnqueueCopyImage.
+    own = L.b2clCreateImageShard(S.ctx, cl.CL_MEM_READ_WRITE | cl.B2CL_MEM_IPC_EXPORTABLE, ctypes.byref(fmt),
+                                 ctypes.byref(gdesc), r0, band, 0, None, ctypes.byref(err))
+    cl.check(err.value, "owned band")
+    block = synth.image_rows(cl.CL_RGBA, cl.CL_FLOAT, W, range(256))
+    cl.check(L.clEnqueueWriteImage(S.queue, own, 1, cl.sz3((0, 0, 0)), cl.sz3((W, 256, 1)), 0, 0,
+                                   block.ctypes.data, 0, None, None))
+    k = 256
+    while k < band:
+        n = min(k, band - k)
+        cl.check(L.clEnqueueCopyImage(S.queue, own, own, cl.sz3((0, 0, 0)), cl.sz3((0, k, 0)),
+                                      cl.sz3((W, n, 1)), 0, None, None))
+        k += n
+    S.finish()
+
+    # ---- 2. every rank imports every other rank's band (valid copy: the owner's GPU)
+    h = (ctypes.c_uint8 * 64)()
+    cl.check(L.b2clGetMemIpcHandle(own, h), "b2clGetMemIpcHandle")
+    handles = bdist.exchange_bytes(bytes(h))
+    bands = []
+    for d in range(world):
+        if d == rank:
+            bands.append(own)
+            continue
+        hd = (ctypes.c_uint8 * 64).from_buffer_copy(handles[d])
+        m = L.b2clCreateImageFromIpcHandle(S.ctx, S.device, cl.CL_MEM_READ_ONLY, ctypes.byref(fmt),
+                                           ctypes.byref(bdesc), hd, ctypes.byref(err))
+        cl.check(err.value, f"import band {d}")
+        bands.append(m)
+
+    # ---- 3. per pass: a shard holding exactly the texel rows output band
+    # [r0, r0 + band) taps, filled by region copies from the owners' bands
+    Af = synth.affine_translate_2d(W, H)
+    A = (ctypes.c_float * 12)(*Af.tolist())
+    modes = ("repeat", "mirrored")
+    shards, shard_info, copies = [], [], []
+    for mname in modes:
+        need = _axis_taps(Af[5], Af[7], band, H, mname, start=r0)
+        begin, count = circular_interval(need, H)
+        rows = [(begin + t) % H for t in range(count)]
+        sh = L.b2clCreateImageShard(S.ctx, cl.CL_MEM_READ_WRITE, ctypes.byref(fmt), ctypes.byref(gdesc),
+                                    begin, count, 0, None, ctypes.byref(err))
+        cl.check(err.value, "shard")
+        shards.append(sh)
+        plan = []
+        for d in range(world):
+            for ga, gb, si in _runs(rows, d * band, (d + 1) * band):
+                plan.append((bands[d], ga - d * band, si, gb - ga, d != rank))
+        shard_info.append({"begin": begin, "rows": count,
+                           "rows_from_peers": int(sum(n for *_, n, peer in plan if peer)),
+                           "copies": len(plan)})
+        copies.append(plan)
+
+    def fill():
+        for k, plan in enumerate(copies):
+            for src, sr, dr, n, _ in plan:
+                cl.check(L.clEnqueueCopyImage(S.queue, src, shards[k], cl.sz3((0, sr, 0)), cl.sz3((0, dr, 0)),
+                                              cl.sz3((W, n, 1)), 0, None, None), "shard fill")
+    fill()
+    S.finish()
+    # the shards hold the right bytes (global row j = block row j mod 256): sampled rows
+    for k, info in enumerate(shard_info):
+        for t in sorted({0, info["rows"] // 2, info["rows"] - 1}):
+            j = (info["begin"] + t) % H
+            got = S.read_image(shards[k], (0, t, 0), (W, 1, 1))
+            assert np.array_equal(got.view(np.float32).reshape(W, 4), block[0, j % 256]), ("shard row", k, t)
+    dist.barrier()
+    fill_ms = _time_launches(T, torch, dev, fill, 3)
+    fill_ms = bdist.max_over_ranks(fill_ms)
+    fill_bytes = sum(i["rows"] for i in shard_info) * rowb
+
+    # ---- 4. the step: REPEAT and MIRRORED reads of the output band
+    nout = W * band * 16
+    outs = [S.buffer(nout), S.buffer(nout)]
+    smps = [S.sampler(True, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR),
+            S.sampler(True, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR)]
+    origin, region = cl.sz3((0, r0, 0)), cl.sz3((W, band, 1))
+    kernels = []
+
+    def launch(k):
+        cl.check(L.b2clEnqueueReadImageGridRegion(S.queue, shards[k], smps[k], cl.B2CL_RTYPE_FLOAT, A, origin,
+                                                  region, 4, outs[k], 0, 0, None, None), "read grid")
+
+    def step():
+        launch(0)
+        launch(1)
+
+    for k in range(2):
+        launch(k)
+        kernels.append(cl.last_kernel())
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize(dev)
+    dist.barrier()
+    clocks = Clocks(gpu)
+    clocks.start()
+    n_launch0 = cl.launch_count()
+    t0 = T.event()
+    for _ in range(args.steps):
+        step()
+    t1 = T.event()
+    torch.cuda.synchronize(dev)
+    gpu_launches = cl.launch_count() - n_launch0
+    clk = clocks.stop()
+    ms_step = bdist.max_over_ranks(t0.elapsed_time(t1) / args.steps)
+    dist.barrier()
+    samples_step = 2 * W * H  # all ranks
+    value = samples_step / (ms_step * 1e-3) / 1e9
+    ncols = [_axis_taps(Af[0], Af[3], W, W, m).size for m in modes]
+    alg = [ncols[k] * shard_info[k]["rows"] * 16 + nout for k in range(2)]
+    pass_ms = []
+    for k in range(2):
+        pass_ms.append(bdist.max_over_ranks(_time_launches(T, torch, dev, lambda k=k: launch(k), 5)))
+    achieved = [alg[k] / (pass_ms[k] * 1e-3) / 1e9 for k in range(2)]
+    dom = 0 if pass_ms[0] >= pass_ms[1] else 1
+
+    # ---- 5. migration (a16): every rank migrates its LEFT neighbour's band to
+    # its own GPU with clEnqueueMigrateMemObjects (one SM copy kernel pulling the
+    # peer mapping over NVLink), all ranks at once (ring shift); and the same
+    # peer pull of a 1 GiB buffer by the SM copy kernel and by the copy engines
+    left, _ = bdist.ring_neighbors(rank, world)
+    hl = (ctypes.c_uint8 * 64).from_buffer_copy(handles[left])
+    mig_ms = []
+    for it in range(3):
+        m = L.b2clCreateImageFromIpcHandle(S.ctx, S.device, cl.CL_MEM_READ_ONLY, ctypes.byref(fmt),
+                                           ctypes.byref(bdesc), hl, ctypes.byref(err))
+        cl.check(err.value, "import for migration")
+        torch.cuda.synchronize(dev)
+        dist.barrier()
+        a = T.event()
+        cl.check(L.clEnqueueMigrateMemObjects(S.queue, 1, (ctypes.c_void_p * 1)(m), 0, 0, None, None))
+        b = T.event()
+        torch.cuda.synchronize(dev)
+        mig_ms.append(a.elapsed_time(b))
+        if it == 0:  # data equality (O9): a migrated row equals the owner's
+            j = left * band + 5
+            got = S.read_image(m, (0, 5, 0), (W, 1, 1))
+            assert np.array_equal(got.view(np.float32).reshape(W, 4), block[0, j % 256])
+        L.clReleaseMemObject(m)
+        S.finish()  # (reaps the deferred free: the mapping closes before the next import)
+    mig_ms = bdist.max_over_ranks(float(np.median(mig_ms)))
+    band_bytes = band * rowb
+    nb = 1 << 30
+    mine = L.clCreateBuffer(S.ctx, cl.CL_MEM_READ_WRITE | cl.B2CL_MEM_IPC_EXPORTABLE, nb, None, ctypes.byref(err))
+    cl.check(err.value)
+    pat = np.array([rank & 0xFF], np.uint8)
+    cl.check(L.clEnqueueFillBuffer(S.queue, mine, pat.ctypes.data, 1, 0, nb, 0, None, None))
+    S.finish()
+    hb = (ctypes.c_uint8 * 64)()
+    cl.check(L.b2clGetMemIpcHandle(mine, hb))
+    hbs = bdist.exchange_bytes(bytes(hb))
+    peer = L.b2clCreateBufferFromIpcHandle(S.ctx, S.device, (ctypes.c_uint8 * 64).from_buffer_copy(hbs[left]), nb,
+                                           ctypes.byref(err))
+    cl.check(err.value)
+    dst = S.buffer(nb)
+    dist.barrier()
+    sm_ms = bdist.max_over_ranks(_time_launches(T, torch, dev, lambda: cl.check(L.clEnqueueCopyBuffer(
+        S.queue, peer, dst, 0, 0, nb, 0, None, None)), 5))
+    ok_sm = bool(np.all(S.read(dst, 4096) == (left & 0xFF)))
+    dist.barrier()
+    ce_ms = bdist.max_over_ranks(_time_launches(T, torch, dev, lambda: cl.check(L.b2clEnqueueCopyBufferEngine(
+        S.queue, peer, dst, 0, 0, nb, 0, None, None)), 5))
+    dist.barrier()
+    link = ("same GPU (rehearsal: ranks share one device, CUDA IPC within it -- not NVLink)" if shared
+            else "NVLink P2P (peer GPU memory over CUDA IPC)")
+    migration = {
+        "pattern": "ring shift: every rank migrates its left neighbour's band concurrently",
+        "band_bytes": band_bytes, "migrate_ms": mig_ms, "migrate_GB/s_per_gpu": band_bytes / (mig_ms * 1e-3) / 1e9,
+        "call": "clEnqueueMigrateMemObjects (SM copy kernel reading the peer mapping)",
+        "p2p_1GiB": {"sm_kernel_ms": sm_ms, "sm_kernel_GB/s": nb / (sm_ms * 1e-3) / 1e9,
+                     "copy_engine_ms": ce_ms, "copy_engine_GB/s": nb / (ce_ms * 1e-3) / 1e9,
+                     "sm_vs_copy_engine": ce_ms / sm_ms, "data_check": "ok" if ok_sm else "MISMATCH"},
+        "frac_of_copy_engine": (band_bytes / (mig_ms * 1e-3)) / (nb / (ce_ms * 1e-3)),
+        "nominal_GB/s": 900.0, "link": link}
+
+    # ---- 6. e2e: each step uploads the rank's band from pinned host memory, the
+    # ranks meet at a (host) barrier, the shards are filled over P2P, the two
+    # reads run, and both outputs come back to pinned host memory
+    e2e = None
+    if not args.no_e2e:
+        try:
+            import psutil
+            need = (band_bytes + nout) * world
+            room = psutil.virtual_memory().available > 2 * need
+        except ImportError:
+            room = True
+        if room:
+            hb_in = torch.empty(band_bytes, dtype=torch.uint8).pin_memory()
+            blk = torch.from_numpy(block.reshape(-1).view(np.uint8))
+            hb_in.view(-1, blk.numel()).copy_(blk.expand(band // 256, -1))
+            hb_out = torch.empty(nout, dtype=torch.uint8).pin_memory()
+            zero3, breg = cl.sz3((0, 0, 0)), cl.sz3((W, band, 1))
+
+            def e2e_step():
+                cl.check(L.clEnqueueWriteImage(S.queue, own, 1, zero3, breg, 0, 0,
+                                               ctypes.c_void_p(hb_in.data_ptr()), 0, None, None))
+                dist.barrier()  # every owner's band is in place before the peers read it
+                fill()
+                step()
+                for k in range(2):
+                    cl.check(L.clEnqueueReadBuffer(S.queue, outs[k], 0, 0, nout,
+                                                   ctypes.c_void_p(hb_out.data_ptr()), 0, None, None))
+                S.finish()
+                dist.barrier()  # nobody overwrites its band while a peer may still copy from it
+            e2e_step()
+            ns = max(2, min(4, args.steps // 8))
+            torch.cuda.synchronize(dev)
+            dist.barrier()
+            a = T.event()
+            for _ in range(ns):
+                e2e_step()
+            b = T.event()
+            torch.cuda.synchronize(dev)
+            e2e_ms = bdist.max_over_ranks(a.elapsed_time(b) / ns)
+            e2e = {"value": samples_step / (e2e_ms * 1e-3) / 1e9, "unit": "Gsamples/s", "ms_per_step": e2e_ms,
+                   "h2d_bytes_per_step": band_bytes, "d2h_bytes_per_step": 2 * nout,
+                   "per": "rank (each rank's own copies)",
+                   "pipeline": ("upload own band (pinned) -> barrier -> P2P shard fill -> 2 reads -> "
+                                "download both outputs (pinned) -> barrier")}
+        else:
+            e2e = {"unavailable": "not enough host memory for the pinned band and output buffers"}
 
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": "Gsamples/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
-            "data": "synthetic (numpy default_rng seed 20151115; U[0,1) RGBA32F texels)",
-            "config": {"workload": WORKLOAD, "image": "4096x4096 RGBA32F (256 MiB)",
-                       "samples_per_step": samples_step, "launches_per_step": 2,
-                       "timing": ("step: K steps between two events; kernel_ms: K back-to-back "
-                                  "launches of that kernel between two events, right after"),
-                       "step": ("REPEAT read on the queue, MIRRORED read on a second queue of "
-                                "the device, joined by a marker and a barrier every step"),
-                       "parallelism": ("single GPU" if world == 1 else
-                                       f"row-sharded x{world}: global {Hg}x{N2D} image, "
-                                       f"4096 output rows per GPU from shards of "
-                                       f"{shard_rows} texel rows (REPEAT, MIRRORED)"),
-                       "l2": "no flush: 768 MiB working set > 126 MB L2", "parity": parity},
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic (numpy default_rng seed 20151115 rows; U[0,1) RGBA32F texels, 256-row period)",
+            "config": {"workload": C5_WORKLOAD, "image": f"{W}x{H} RGBA32F ({W * H * 16 / 2**30:.0f} GiB)",
+                       "samples_per_step": samples_step, "launches_per_step_per_rank": 2, "kernels": kernels,
+                       "parallelism": (f"row-sharded x{world}: rank d owns texel rows [d*{band}, (d+1)*{band}) and "
+                                       f"reads output rows [d*{band}, (d+1)*{band}) from per-pass shards "
+                                       f"{[(i['begin'], i['rows']) for i in shard_info]} (rank 0)"),
+                       "shards": shard_info, "l2": "no flush: working set >> 126 MB L2",
+                       "parity": ("shard contents checked byte-exact on sampled rows; shard reads are "
+                                  "bit-identical to whole-image reads (tests/test_gpu_shards.py), which are "
+                                  "checked against the oracle (tests/test_gpu_config5.py)"),
+                       "control_plane": "torch.distributed gloo (barrier, max over ranks, IPC handles)"},
             "roofline": {"bound": "hbm", "achieved": achieved[dom], "peak": hbm_peak, "unit": "GB/s",
-                         "frac": achieved[dom] / hbm_peak, "traffic": traffic,
-                         "kernel": ["k_sample_grid<2D RGBA32F LINEAR REPEAT>",
-                                    "k_sample_grid<2D RGBA32F LINEAR MIRRORED>"][dom],
+                         "frac": achieved[dom] / hbm_peak, "traffic": None, "kernel": kernels[dom],
                          "kernel_ms": pass_ms[dom], "algorithmic_bytes_per_launch": alg[dom],
-                         "peak_source": peak_src,
-                         "per_pass": [{"mode": m, "ms": pass_ms[k], "algorithmic_bytes": alg[k],
+                         "peak_source": peak_src, "per": "rank (slowest)",
+                         "per_pass": [{"mode": m, "kernel": kernels[k], "ms": pass_ms[k], "algorithmic_bytes": alg[k],
                                        "GB/s": achieved[k], "frac": achieved[k] / hbm_peak}
-                                      for k, m in enumerate(("repeat", "mirrored"))],
-                         "step_frac": sum(alg) / (sum(pass_ms) * 1e-3) / 1e9 / hbm_peak},
-            "cpu_baseline": cpu, "e2e": e2e, "clocks": clk, "gpu_launches": gpu_launches,
-            "secondary": secondary,
+                                      for k, m in enumerate(modes)]},
+            "exchange": {"shard_fill_ms": fill_ms, "shard_fill_bytes_per_rank": fill_bytes,
+                         "shard_fill_GB/s_per_gpu": fill_bytes / (fill_ms * 1e-3) / 1e9,
+                         "call": "clEnqueueCopyImage region copies from the owners' bands (in place, P2P)"},
+            "migration": migration,
+            "cpu_baseline": None, "e2e": e2e, "clocks": clk, "gpu_launches": gpu_launches,
         }
         print(json.dumps(line), flush=True)
-    L.clReleaseCommandQueue(q_two)
-    S.release(*set(imgs), *outs)
-    for s in smps:
-        L.clReleaseSampler(s)
-    S.close()
-    if world > 1:
-        dist.destroy_process_group()
-    return 0
-
-
-def run_p2p_ring(S, L, T, torch, dev, red_dev, rank, world):
-    """Config 5 migration, one process per GPU: every rank exports an
-    IPC-exportable band buffer, opens its left neighbour's band over CUDA IPC
-    and pulls it with the library's SM copy kernel (clEnqueueCopyBuffer on the
-    peer mapping -> NVLink reads), all ranks concurrently (ring shift).  Band =
-    32768^2 RGBA32F / G rows, capped at 2 GiB.  Reported: GB/s per GPU (the
-    slowest rank) and its fraction of the 770 GB/s measured peer-copy figure
-    (B200_PROFILING.md; 900 GB/s nominal)."""
-    from paper_conf_sc_kimdjjl15_b200 import cl
-    from paper_conf_sc_kimdjjl15_b200 import dist as bdist
-    band = min((32768 * 32768 * 16) // world, 2 << 30)
-    err = ctypes.c_int32()
-    mine = L.clCreateBuffer(S.ctx, cl.CL_MEM_READ_WRITE | cl.B2CL_MEM_IPC_EXPORTABLE, band, None,
-                            ctypes.byref(err))
-    cl.check(err.value, "clCreateBuffer(IPC)")
-    pat = np.array([rank & 0xFF], np.uint8)
-    cl.check(L.clEnqueueFillBuffer(S.queue, mine, pat.ctypes.data, 1, 0, band, 0, None, None))
+    for o in [*outs, *shards, dst, peer, mine]:
+        L.clReleaseMemObject(o)
+    for d, m in enumerate(bands):
+        if d != rank:
+            L.clReleaseMemObject(m)
     S.finish()
-    h = (ctypes.c_uint8 * 64)()
-    cl.check(L.b2clGetMemIpcHandle(mine, h), "b2clGetMemIpcHandle")
-    handles = bdist.exchange_bytes(bytes(h))
-    left, _ = bdist.ring_neighbors(rank, world)
-    hl = (ctypes.c_uint8 * 64).from_buffer_copy(handles[left])
-    peer = L.b2clCreateBufferFromIpcHandle(S.ctx, S.device, hl, band, ctypes.byref(err))
-    cl.check(err.value, "b2clCreateBufferFromIpcHandle")
-    local = S.buffer(band)
-
-    def pull():
-        cl.check(L.clEnqueueCopyBuffer(S.queue, peer, local, 0, 0, band, 0, None, None))
-    pull()
-    S.finish()
-    ok = bool(np.all(S.read(local, 4096) == (left & 0xFF)))  # data equality (O9) on a sample
-    import torch.distributed as dist
     dist.barrier()
-    ms = _time_launches(T, torch, dev, pull, 5)
-    ms = bdist.max_over_ranks(ms, red_dev)
-    gbs = band / (ms * 1e-3) / 1e9
-    S.release(local, peer, mine)
-    return {"band_bytes": band, "ms": ms, "GB/s_per_gpu": gbs, "frac_of_770": gbs / 770.0,
-            "pattern": "ring shift, all ranks pull from rank-1 concurrently",
-            "data_check": "ok" if ok else "MISMATCH",
-            "link": ("NVLink P2P (peer GPU memory over CUDA IPC)" if red_dev is not None else
-                     "same GPU (multi-rank rehearsal with ranks sharing one device: not NVLink)")}
+    L.clReleaseMemObject(own)
+    for sm in smps:
+        L.clReleaseSampler(sm)
+    S.close()
+    dist.destroy_process_group()
+    return 0
 
 
 def _time_launches(T, torch, dev, fn, iters):
@@ -723,7 +1034,7 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
         ms = _time_launches(T, torch, dev, lambda: cl.check(L.b2clEnqueueReadImageGrid(
             S.queue, img2, smp2, 0, A2, d2, 4, out2, 0, 0, None, None)), 10)
         e = {"Gsamples/s": n2 * n2 / ms / 1e6, "ms": ms, "map": "rotation 30 deg (B)",
-             "kernel": "k_sample_grid (8x4 output patch per warp)"}
+             "kernel": cl.last_kernel()}
         texels = _distinct_texels_2d(synth.affine_rotate_2d(n2, n2, 30.0), n2, n2, name)
         b2 = 16 * texels + 16 * n2 * n2
         e.update({"GB/s": b2 / ms / 1e6, "hbm_frac": b2 / ms / 1e6 / hbm_peak, "algorithmic_bytes": b2,
@@ -771,8 +1082,7 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
     byt = 2 * n3 ** 3 * 4
     res["c3_trilinear_512"] = {"Gsamples/s": n3 ** 3 / ms / 1e6, "ms": ms, "GB/s": byt / ms / 1e6,
                                "hbm_frac": byt / ms / 1e6 / hbm_peak, "map": "stencil (A)",
-                               "kernel": "k_sample_grid_vol (256x16 tiles, per-row cp.async.bulk ring)",
-                               "algorithmic_bytes": byt}
+                               "kernel": cl.last_kernel(), "algorithmic_bytes": byt}
     A3b = (ctypes.c_float * 12)(*synth.affine_rotate_3d(n3, 20.0).tolist())
     ms = _time_launches(T, torch, dev, lambda: cl.check(L.b2clEnqueueReadImageGrid(
         S.queue, vol, smp3, 0, A3b, d3, 1, out3, 0, 0, None, None)), 10)
@@ -786,7 +1096,7 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
                                        "hbm_frac": bytr / ms / 1e6 / hbm_peak, "algorithmic_bytes": bytr,
                                        "distinct_texels": txy * tz,
                                        "map": "volume-render rotation (B), 20 deg about z",
-                                       "kernel": "k_sample_grid_volr (64x32 tiles, tensor-TMA footprint box)"}
+                                       "kernel": cl.last_kernel()}
     S.release(vol, out3)
     L.clReleaseSampler(smp3)
     # config 4: 8 GiB pitched CopyBufferRect (src padded, dst tight) and a misaligned variant
@@ -807,14 +1117,18 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
     b2 = reg2[0] * reg2[1] * reg2[2]
     res["c4_copy_rect_misaligned"] = {"GB/s_copied": b2 / ms / 1e6, "ms": ms,
                                       "hbm_frac": 2 * b2 / ms / 1e6 / hbm_peak}
-    pat = np.arange(16, dtype=np.uint8)
-    ms = _time_launches(T, torch, dev, lambda: cl.check(L.clEnqueueFillBuffer(
-        S.queue, dst, pat.ctypes.data, 16, 0, S_bytes, 0, None, None)), 5)
-    res["c4_fill_8GiB"] = {"GB/s": S_bytes / ms / 1e6, "ms": ms, "hbm_frac": S_bytes / ms / 1e6 / hbm_peak}
+    fills = []
+    for ps in (1, 4, 16, 128):  # FillBuffer patterns
+        pat = np.arange(ps, dtype=np.uint8)
+        ms = _time_launches(T, torch, dev, lambda: cl.check(L.clEnqueueFillBuffer(
+            S.queue, dst, pat.ctypes.data, ps, 0, S_bytes, 0, None, None)), 5)
+        fills.append({"pattern_bytes": ps, "GB/s": S_bytes / ms / 1e6, "ms": ms,
+                      "hbm_frac": S_bytes / ms / 1e6 / hbm_peak})
+    res["c4_fill_8GiB"] = fills
     S.release(src)
     # CopyImageToBuffer sweep 4 KiB .. 8 GiB (RGBA32F 2D images shaped to the size)
     sweep = []
-    for lg in range(12, 34, 3 if not args.full_sweep else 1):
+    for lg in range(12, 34, 1 if not args.short_sweep else 3):  # 22 sizes: 4 KiB .. 8 GiB
         nbytes = 1 << lg
         w = min(32768, max(1, nbytes // 16))
         h = max(1, nbytes // 16 // w)
@@ -834,6 +1148,8 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
         S.release(im)
     res["c4_copy_image_to_buffer_sweep"] = sweep
     S.release(dst)
+    # host cost of one enqueue, measured from C (no Python / ctypes in the loop)
+    res["host_enqueue_us"] = enqueue_cost()
     return res
 
 
@@ -846,8 +1162,9 @@ def main():
     ap.add_argument("--no-secondary", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--full-sweep", action="store_true")
-    ap.add_argument("--no-p2p", action="store_true", help="skip the N>1 NVLink ring migration")
+    ap.add_argument("--short-sweep", action="store_true", help="8 of the 22 C4 sweep sizes")
+    ap.add_argument("--no-ncu", action="store_true", help="skip the in-run ncu traffic capture")
+    ap.add_argument("--c5-size", type=int, default=C5, help="N > 1: the sharded image's side (C5: 32768)")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)

@@ -219,13 +219,43 @@ cl_mem b2clCreateBufferFromDevicePointer(cl_context context, cl_device_id device
  * migration).  For images this is the CLImage ptr (Fig. 6). */
 cl_int b2clGetMemDevicePointer(cl_mem memobj, cl_device_id device, void** device_ptr);
 
-/* CUDA IPC: export a B2CL_MEM_IPC_EXPORTABLE buffer (64-byte handle) and
- * import it in another process as a buffer whose storage is the peer GPU's
- * memory mapped over NVLink; enqueues on a queue of this process then read
- * or write it by P2P. */
+/* CUDA IPC (the multi-device context across processes, one process per GPU;
+ * SURVEY §8(e)).  b2clGetMemIpcHandle exports a buffer or image created with
+ * B2CL_MEM_IPC_EXPORTABLE (its local cudaMalloc storage) as a 64-byte handle
+ * (CL_INVALID_OPERATION otherwise).  The import calls open the handle on
+ * `device` and return an object whose only valid copy is the EXPORTER's
+ * memory (a peer GPU's, over NVLink), with the exporter's layout:
+ *   - region copies and fills (clEnqueueCopyBuffer[Rect], CopyImage,
+ *     CopyImageToBuffer, CopyBufferToImage, Fill*) read or write it in place,
+ *     moving only the region over NVLink;
+ *   - clEnqueueMigrateMemObjects, host transfers and the read built-ins first
+ *     pull the whole content into a local store of the queue's device (one
+ *     SM copy kernel reading the peer mapping), as in a multi-device context.
+ * b2clCreateImageFromIpcHandle takes the exporter's cl_image_format and
+ * cl_image_desc (no host pitches; the internal pitch is a function of them,
+ * clGetImageInfo, reading A21) -- an image shard is imported as the plain
+ * image of its stored rows.  Errors: CL_INVALID_CONTEXT / _DEVICE,
+ * CL_INVALID_VALUE (NULL handle, host-pointer flags), the clCreateImage
+ * format / descriptor codes, CL_OUT_OF_RESOURCES (the handle does not open).
+ * The mapping is closed when the object is released (deferred like every
+ * free, after the queues that used it are done). */
 cl_int b2clGetMemIpcHandle(cl_mem memobj, void* handle64);
 cl_mem b2clCreateBufferFromIpcHandle(cl_context context, cl_device_id device,
                                      const void* handle64, size_t size, cl_int* errcode_ret);
+cl_mem b2clCreateImageFromIpcHandle(cl_context context, cl_device_id device, cl_mem_flags flags,
+                                    const cl_image_format* image_format,
+                                    const cl_image_desc* image_desc, const void* handle64,
+                                    cl_int* errcode_ret);
+
+/* clEnqueueCopyBuffer's semantics and validation ([CL1.2 §5.2.2]), moved by
+ * the COPY ENGINES (cudaMemcpyAsync on the queue's stream, peer / IPC
+ * pointers addressed in place) instead of the SM copy kernel: the reference
+ * path the bench times beside the kernel for the NVLink roofline
+ * (cudaMemcpyPeerAsync-class transfers). */
+cl_int b2clEnqueueCopyBufferEngine(cl_command_queue command_queue, cl_mem src_buffer,
+                                   cl_mem dst_buffer, size_t src_offset, size_t dst_offset,
+                                   size_t size, cl_uint num_events_in_wait_list,
+                                   const cl_event* event_wait_list, cl_event* event);
 
 /* Number of b2cl kernels launched by this process so far (bench evidence). */
 cl_ulong b2clGetKernelLaunchCount(void);

@@ -905,11 +905,16 @@ static cudaError_t go_sep(const SampleParams& p, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+// MIRRORED_REPEAT: one fold per axis inside the region -> the fold kernel;
+// otherwise (e.g. a shard's band of output rows that does not reach the
+// mirror axis: config 5 at N > 1) the taps chain one way per axis and each
+// texel is read about once, like REPEAT -> the staged tile kernel, which
+// checks the chaining and reads unchained tiles directly
 template <class C>
-static cudaError_t fold_or_sep(const SampleParams& p, cudaStream_t st) {
+static cudaError_t fold_or_tile(const SampleParams& p, cudaStream_t st) {
   cudaError_t e = cudaSuccess;
   if (go_fold<C>(p, st, &e)) return e;
-  return go_sep<C, 4, B2CL_C2M_XPT, B2CL_C2M_RPW>(p, st);
+  return go_tile<C, B2CL_TILE_TH>(p, st);
 }
 
 template <class C>
@@ -980,7 +985,7 @@ cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st
         return fk == 3   ? go_walk<C2Mirror, 4, 2, 8>(p, st)
                : fk == 5 ? go_tile<C2Mirror, B2CL_TILE_TH>(p, st)
                : fk == 2 ? go_sep<C2Mirror, 4, B2CL_C2M_XPT, B2CL_C2M_RPW>(p, st)
-               : fold_or_sep<C2Mirror>(p, st);
+               : fold_or_tile<C2Mirror>(p, st);
       if (p.outc == 1 && matches<3>(p, T_FLOAT, O_R, 1, A_CTE, F_LINEAR)) {
         if (fk == 0 && !is_shard(p)) {
           bool used = false;

@@ -51,10 +51,18 @@ struct _cl_command_queue {
 };
 
 struct Store {
-  int ordinal = -1;
+  int ordinal = -1;     // the CUDA device whose address space holds ptr
   char* ptr = nullptr;
   int kind = 0;  // 0 none, 1 cudaMalloc, 2 allocator hook, 3 borrowed, 4 IPC import
 };
+
+// An IPC-imported store (kind 4) is ANOTHER process's memory -- a peer GPU's
+// over NVLink, or a region of this GPU owned by another process -- mapped into
+// `ordinal`'s address space.  It is not this device's local copy: its valid
+// bit is kRemoteBit, so clEnqueueMigrateMemObjects (or a sampling read) pulls
+// it into a local store, while region copies read / write it in place.
+constexpr int kRemoteBit = 63;
+static int bit_of(const Store& s) { return s.kind == 4 ? kRemoteBit : s.ordinal; }
 
 struct _cl_mem {
   std::atomic<int> ref{1};
@@ -135,6 +143,27 @@ template <class T>
 static bool live(const std::set<T>& reg, T h) {
   std::lock_guard<std::mutex> g(g_mu);
   return h && reg.count(h);
+}
+
+// Retain / release under the registry lock: the liveness check and the count
+// change are one step, so two threads releasing the last reference cannot
+// both destroy the object, and a release racing a retain never resurrects a
+// destroyed one.  release_ref returns -1 (not live), 0 (still referenced) or 1
+// (last reference: already removed from the registry, the caller destroys).
+template <class T>
+static bool retain_ref(std::set<T>& reg, T h) {
+  std::lock_guard<std::mutex> g(g_mu);
+  if (!h || !reg.count(h)) return false;
+  h->ref++;
+  return true;
+}
+template <class T>
+static int release_ref(std::set<T>& reg, T h) {
+  std::lock_guard<std::mutex> g(g_mu);
+  if (!h || !reg.count(h)) return -1;
+  if (--h->ref > 0) return 0;
+  reg.erase(h);
+  return 1;
 }
 
 static cl_int cuda_err(cudaError_t e) {
@@ -321,19 +350,17 @@ extern "C" cl_context clCreateContext(const cl_context_properties* props, cl_uin
   return c;
 }
 
+static void reap_frees(bool block);
+
 extern "C" cl_int clRetainContext(cl_context c) {
-  if (!live(g_contexts, c)) return CL_INVALID_CONTEXT;
-  c->ref++;
-  return CL_SUCCESS;
+  return retain_ref(g_contexts, c) ? CL_SUCCESS : CL_INVALID_CONTEXT;
 }
 
 extern "C" cl_int clReleaseContext(cl_context c) {
-  if (!live(g_contexts, c)) return CL_INVALID_CONTEXT;
-  if (--c->ref == 0) {
-    {
-      std::lock_guard<std::mutex> g(g_mu);
-      g_contexts.erase(c);
-    }
+  const int r = release_ref(g_contexts, c);
+  if (r < 0) return CL_INVALID_CONTEXT;
+  if (r == 1) {
+    reap_frees(true);  // the context's last memory objects' deferred frees
     delete c;
   }
   return CL_SUCCESS;
@@ -420,14 +447,13 @@ extern "C" cl_int b2clGetCommandQueueStream(cl_command_queue q, void** stream) {
 }
 
 extern "C" cl_int clRetainCommandQueue(cl_command_queue q) {
-  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
-  q->ref++;
-  return CL_SUCCESS;
+  return retain_ref(g_queues, q) ? CL_SUCCESS : CL_INVALID_COMMAND_QUEUE;
 }
 
 extern "C" cl_int clReleaseCommandQueue(cl_command_queue q) {
-  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
-  if (--q->ref == 0) {
+  const int r = release_ref(g_queues, q);
+  if (r < 0) return CL_INVALID_COMMAND_QUEUE;
+  if (r == 1) {
     {
       DeviceGuard g(q->dev->ordinal);
       cudaStreamSynchronize(q->stream);  // implicit flush + finish before teardown
@@ -435,12 +461,12 @@ extern "C" cl_int clReleaseCommandQueue(cl_command_queue q) {
     }
     {
       std::lock_guard<std::mutex> g(g_mu);
-      g_queues.erase(q);
       for (cl_mem m : g_mems) {
         std::lock_guard<std::mutex> gm(m->mu);
         m->users.erase(q);
       }
     }
+    reap_frees(false);
     cl_context c = q->ctx;
     delete q;
     clReleaseContext(c);
@@ -468,8 +494,13 @@ extern "C" cl_int clFlush(cl_command_queue q) {
 
 extern "C" cl_int clFinish(cl_command_queue q) {
   if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
-  DeviceGuard g(q->dev->ordinal);
-  return cuda_err(cudaStreamSynchronize(q->stream));
+  cl_int st;
+  {
+    DeviceGuard g(q->dev->ordinal);
+    st = cuda_err(cudaStreamSynchronize(q->stream));
+  }
+  reap_frees(false);
+  return st;
 }
 
 // ===================================================================== memory objects
@@ -501,10 +532,54 @@ static void raw_free(Store& s) {
   s.kind = 0;
 }
 
+// the object's LOCAL store on `ordinal` (never an IPC-imported one)
 static Store* find_store(cl_mem m, int ordinal) {
   for (auto& s : m->stores)
-    if (s.ordinal == ordinal) return &s;
+    if (s.ordinal == ordinal && s.kind != 4) return &s;
   return nullptr;
+}
+
+// ---- deferred, stream-ordered frees (clReleaseMemObject) ----
+// The last release of an object records an event on every live queue that
+// enqueued work on it and parks its stores here; they are freed once all of
+// those events have completed -- checked without blocking on later API calls
+// (allocations, releases, clFinish), and with blocking at the last context
+// release.  The host never waits in clReleaseMemObject.
+struct PendingFree {
+  std::vector<Store> stores;
+  std::vector<std::pair<int, cudaEvent_t>> events;  // (device, event)
+};
+static std::mutex g_pend_mu;
+static std::vector<PendingFree> g_pending;
+
+static void reap_frees(bool block) {
+  std::vector<PendingFree> done;
+  {
+    std::lock_guard<std::mutex> g(g_pend_mu);
+    for (size_t i = 0; i < g_pending.size();) {
+      bool ready = true;
+      for (auto& e : g_pending[i].events) {
+        DeviceGuard dg(e.first);
+        const cudaError_t r = block ? cudaEventSynchronize(e.second) : cudaEventQuery(e.second);
+        if (r == cudaErrorNotReady) { ready = false; break; }
+        cudaGetLastError();  // (an errored event counts as done: the stream is dead)
+      }
+      if (ready) {
+        done.push_back(std::move(g_pending[i]));
+        g_pending[i] = std::move(g_pending.back());
+        g_pending.pop_back();
+      } else {
+        ++i;
+      }
+    }
+  }
+  for (auto& p : done) {
+    for (auto& e : p.events) {
+      DeviceGuard dg(e.first);
+      cudaEventDestroy(e.second);
+    }
+    for (auto& st : p.stores) raw_free(st);
+  }
 }
 
 static cl_mem new_mem(cl_context c, cl_mem_object_type type, cl_mem_flags flags, size_t size) {
@@ -543,6 +618,7 @@ static cl_int check_mem_flags(cl_mem_flags flags, void* host_ptr) {
 static cl_int ensure_store(cl_mem m, int ordinal, cudaStream_t stream, Store** out) {
   Store* s = find_store(m, ordinal);
   if (!s) {
+    reap_frees(false);  // memory of released objects whose users have finished
     int kind = 0;
     void* p = raw_alloc(m->alloc_size, ordinal, stream, &kind,
                         (m->flags & B2CL_MEM_IPC_EXPORTABLE) != 0);
@@ -736,31 +812,48 @@ static bool is_image(cl_mem m) {
 }
 
 extern "C" cl_int clRetainMemObject(cl_mem m) {
-  if (!live(g_mems, m)) return CL_INVALID_MEM_OBJECT;
-  m->ref++;
-  return CL_SUCCESS;
+  return retain_ref(g_mems, m) ? CL_SUCCESS : CL_INVALID_MEM_OBJECT;
 }
 
 extern "C" cl_int clReleaseMemObject(cl_mem m) {
-  if (!live(g_mems, m)) return CL_INVALID_MEM_OBJECT;
-  if (--m->ref == 0) {
+  const int r = release_ref(g_mems, m);
+  if (r < 0) return CL_INVALID_MEM_OBJECT;
+  if (r == 1) {
+    // stream-ordered, deferred free (ownership): an event after
+    // the object's last command on every queue that used it; the stores are
+    // freed once they complete (reap_frees) -- no host wait here
     std::vector<cl_command_queue> users;
     {
-      std::lock_guard<std::mutex> g(g_mu);
-      g_mems.erase(m);
-      for (cl_command_queue q : m->users)
-        if (g_queues.count(q)) users.push_back(q);
+      std::lock_guard<std::mutex> gm(m->mu);
+      users.assign(m->users.begin(), m->users.end());
     }
-    // stream-ordered free: drain the queues that used the object first
-    for (cl_command_queue q : users) {
-      DeviceGuard g(q->dev->ordinal);
-      cudaStreamSynchronize(q->stream);
+    PendingFree pf;
+    {
+      std::lock_guard<std::mutex> g(g_mu);  // queues stay alive while recording
+      for (cl_command_queue q : users) {
+        if (!g_queues.count(q)) continue;  // released queues were drained then
+        DeviceGuard dg(q->dev->ordinal);
+        cudaEvent_t ev = nullptr;
+        if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) == cudaSuccess &&
+            cudaEventRecord(ev, q->stream) == cudaSuccess) {
+          pf.events.emplace_back(q->dev->ordinal, ev);
+        } else {  // no event: fall back to draining that queue
+          if (ev) cudaEventDestroy(ev);
+          cudaGetLastError();
+          cudaStreamSynchronize(q->stream);
+        }
+      }
     }
-    for (auto& s : m->stores) raw_free(s);
+    pf.stores = std::move(m->stores);
+    if (!pf.stores.empty()) {
+      std::lock_guard<std::mutex> g(g_pend_mu);
+      g_pending.push_back(std::move(pf));
+    }
     cl_context c = m->ctx;
     cl_mem parent = m->parent;
     delete m;
     if (parent) clReleaseMemObject(parent);
+    reap_frees(false);
     clReleaseContext(c);
   }
   return CL_SUCCESS;
@@ -839,18 +932,13 @@ extern "C" cl_sampler clCreateSampler(cl_context c, cl_bool norm, cl_addressing_
 }
 
 extern "C" cl_int clRetainSampler(cl_sampler s) {
-  if (!live(g_samplers, s)) return CL_INVALID_SAMPLER;
-  s->ref++;
-  return CL_SUCCESS;
+  return retain_ref(g_samplers, s) ? CL_SUCCESS : CL_INVALID_SAMPLER;
 }
 
 extern "C" cl_int clReleaseSampler(cl_sampler s) {
-  if (!live(g_samplers, s)) return CL_INVALID_SAMPLER;
-  if (--s->ref == 0) {
-    {
-      std::lock_guard<std::mutex> g(g_mu);
-      g_samplers.erase(s);
-    }
+  const int r = release_ref(g_samplers, s);
+  if (r < 0) return CL_INVALID_SAMPLER;
+  if (r == 1) {
     cl_context c = s->ctx;
     delete s;
     clReleaseContext(c);
@@ -884,18 +972,13 @@ extern "C" cl_int clWaitForEvents(cl_uint n, const cl_event* list) {
 }
 
 extern "C" cl_int clRetainEvent(cl_event e) {
-  if (!live(g_events, e)) return CL_INVALID_EVENT;
-  e->ref++;
-  return CL_SUCCESS;
+  return retain_ref(g_events, e) ? CL_SUCCESS : CL_INVALID_EVENT;
 }
 
 extern "C" cl_int clReleaseEvent(cl_event e) {
-  if (!live(g_events, e)) return CL_INVALID_EVENT;
-  if (--e->ref == 0) {
-    {
-      std::lock_guard<std::mutex> g(g_mu);
-      g_events.erase(e);
-    }
+  const int r = release_ref(g_events, e);
+  if (r < 0) return CL_INVALID_EVENT;
+  if (r == 1) {
     DeviceGuard g(e->ordinal);
     if (e->start) cudaEventDestroy(e->start);
     if (e->end) cudaEventDestroy(e->end);
@@ -998,10 +1081,40 @@ static cl_int enq_end(Enq& E, cudaError_t err) {
   return CL_SUCCESS;
 }
 
+// Can queue q's device address store st directly?  Its own memory; a peer
+// GPU's with peer access enabled in the context (NVLink); an IPC mapping
+// opened on this device.
+static bool reachable(cl_command_queue q, const Store& st) {
+  const int ord = q->dev->ordinal;
+  if (st.kind == 4 || st.ordinal == ord) return st.ordinal == ord;
+  return st.ordinal >= 0 && st.ordinal < 64 && q->ctx->peer[ord][st.ordinal];
+}
+
+// Copy the object's whole valid content into the store `dst` of q's device
+// on q's stream (the caller has issued the wait list first: enq_begin).
+static cudaError_t pull_whole(cl_mem m, cl_command_queue q, Store* dst) {
+  Store* src = nullptr;
+  for (auto& o : m->stores)
+    if (((m->valid >> bit_of(o)) & 1ull) && &o != dst) { src = &o; break; }
+  if (!src) return cudaSuccess;
+  if (reachable(q, *src)) {  // SM copy kernel reading the peer / IPC pointer (NVLink)
+    RectParams p{};
+    p.src = src->ptr;
+    p.dst = dst->ptr;
+    p.R0 = m->alloc_size;
+    p.R1 = p.R2 = 1;
+    p.srp = p.drp = m->alloc_size;
+    p.ssp = p.dsp = m->alloc_size;
+    return launch_rect(p, RECT_COPY, q->stream);
+  }
+  return cudaMemcpyPeerAsync(dst->ptr, dst->ordinal, src->ptr, src->ordinal, m->alloc_size, q->stream);
+}
+
 // Make the object's content valid on the queue's device and return its
-// pointer there.  If another device holds the only valid copy, pull it over
-// NVLink (SM copy kernel on the peer pointer) on the queue's stream; the
-// caller's wait list orders it after the producer (OpenCL cross-queue rule).
+// pointer there.  If another device (or another process, through an IPC
+// mapping) holds the only valid copy, pull it whole over NVLink on the
+// queue's stream.  Callers issue the wait list (enq_begin) BEFORE this, so the
+// pull is ordered after the producer of the content (OpenCL cross-queue rule).
 static cl_int resident(cl_mem m, cl_command_queue q, bool need_content, char** out) {
   size_t off = 0;
   if (m->parent) {  // a 1D image buffer or a view lives in its parent
@@ -1015,23 +1128,7 @@ static cl_int resident(cl_mem m, cl_command_queue q, bool need_content, char** o
   if (st != CL_SUCCESS) return st;
   const uint64_t bit = 1ull << ord;
   if (need_content && !(m->valid & bit) && m->valid) {
-    int src = -1;
-    for (auto& o : m->stores)
-      if ((m->valid >> o.ordinal) & 1ull) { src = o.ordinal; break; }
-    Store* ss = find_store(m, src);
-    cudaError_t e;
-    if (q->ctx->peer[ord][src]) {
-      RectParams p{};
-      p.src = ss->ptr;
-      p.dst = s->ptr;
-      p.R0 = m->alloc_size;
-      p.R1 = p.R2 = 1;
-      p.srp = p.drp = m->alloc_size;
-      p.ssp = p.dsp = m->alloc_size;
-      e = launch_rect(p, RECT_COPY, q->stream);
-    } else {
-      e = cudaMemcpyPeerAsync(s->ptr, ord, ss->ptr, src, m->alloc_size, q->stream);
-    }
+    const cudaError_t e = pull_whole(m, q, s);
     if (e != cudaSuccess) return cuda_err(e);
     m->valid |= bit;
   }
@@ -1040,11 +1137,71 @@ static cl_int resident(cl_mem m, cl_command_queue q, bool need_content, char** o
   return CL_SUCCESS;
 }
 
+// Region copies and fills touch part of an object, so they address a valid
+// copy IN PLACE when q's device can reach it -- a source region is read from
+// the peer (NVLink) or IPC pointer, a destination region written there --
+// with no whole-object migration and no full-size allocation (a halo row
+// exchanged between two shards moves the row, not the shard).  Only when no
+// reachable copy is valid does the object migrate to q's device.
+// *store is the store written (for `written_store`).
+static cl_int in_place(cl_mem m, cl_command_queue q, bool for_write, char** out, Store** store) {
+  size_t off = 0;
+  if (m->parent) {
+    off = m->parent_off;
+    m = m->parent;
+  }
+  std::lock_guard<std::mutex> g(m->mu);
+  const int ord = q->dev->ordinal;
+  m->users.insert(q);
+  Store* local = find_store(m, ord);
+  Store* pick = nullptr;
+  if (local && (m->valid & (1ull << ord))) {
+    pick = local;
+  } else if (m->valid) {
+    for (auto& o : m->stores)
+      if (((m->valid >> bit_of(o)) & 1ull) && reachable(q, o)) { pick = &o; break; }
+  }
+  if (!pick) {  // nothing valid (fresh object) or nothing reachable: a local copy
+    cl_int st = ensure_store(m, ord, q->stream, &local);
+    if (st != CL_SUCCESS) return st;
+    if (m->valid) {
+      const cudaError_t e = pull_whole(m, q, local);
+      if (e != cudaSuccess) return cuda_err(e);
+    }
+    if (m->valid || !for_write) m->valid |= 1ull << ord;
+    pick = local;
+  }
+  *out = pick->ptr + off;
+  if (store) *store = pick;
+  return CL_SUCCESS;
+}
+
 static void written(cl_mem m, cl_command_queue q) {
   if (m->parent) m = m->parent;
   std::lock_guard<std::mutex> g(m->mu);
   m->valid = 1ull << q->dev->ordinal;
 }
+
+// after a write through in_place: the written store is the only valid copy
+static void written_store(cl_mem m, const Store* st) {
+  if (m->parent) m = m->parent;
+  std::lock_guard<std::mutex> g(m->mu);
+  m->valid = 1ull << bit_of(*st);
+}
+
+// an error after enq_begin: drop the profiling start event (the wait-list
+// waits it issued only order the stream; nothing else was enqueued)
+static cl_int enq_fail(Enq& E, cl_int st) {
+  if (E.start) cudaEventDestroy(E.start);
+  E.start = nullptr;
+  return st;
+}
+
+#define CHECK_E(E, x)                        \
+  do {                                       \
+    cl_int _s = (x);                         \
+    if (_s != CL_SUCCESS) return enq_fail(E, _s); \
+  } while (0)
 
 static cl_int check_queue_mem(cl_command_queue q, cl_mem m) {
   if (!live(g_mems, m) || m->ctx != q->ctx) return CL_INVALID_MEM_OBJECT;
@@ -1232,8 +1389,8 @@ static cl_int buffer_host_rect(cl_command_queue q, cl_mem buf, cl_bool blocking,
   E.type = type;
   DeviceGuard g(q->dev->ordinal);
   char* d = nullptr;
-  CHECK(resident(buf, q, true, &d));
   CHECK(enq_begin(E, nw, wl));
+  CHECK_E(E, resident(buf, q, true, &d));
   char* dbase = d + bo[2] * bsp + bo[1] * brp + bo[0];
   char* hbase = ptr + ho[2] * hsp + ho[1] * hrp + ho[0];
   cl_int st = host_rect_copy(E, dbase, brp, bsp, hbase, hrp, hsp, region, write, blocking);
@@ -1313,8 +1470,8 @@ static cl_int image_host(cl_command_queue q, cl_mem img, cl_bool blocking, const
   E.type = write ? CL_COMMAND_WRITE_IMAGE : CL_COMMAND_READ_IMAGE;
   DeviceGuard g(q->dev->ordinal);
   char* d = nullptr;
-  CHECK(resident(img, q, true, &d));
   CHECK(enq_begin(E, nw, wl));
+  CHECK_E(E, resident(img, q, true, &d));
   char* dbase = d + origin[2] * L.slice_pitch + origin[1] * L.row_pitch + origin[0] * es;
   const size_t bytes_region[3] = {region[0] * es, region[1], region[2]};
   cl_int st = host_rect_copy(E, dbase, L.row_pitch, L.slice_pitch, ptr, rp, sp, bytes_region, write,
@@ -1341,9 +1498,12 @@ extern "C" cl_int clEnqueueWriteImage(cl_command_queue q, cl_mem img, cl_bool bl
 
 // ===================================================================== device rect copies / fills
 // One rect-copy kernel launch between two objects (already validated).
+// copy_engine: a 1D copy on the copy engines (cudaMemcpyAsync) instead of
+// the SM kernel -- the reference path b2clEnqueueCopyBufferEngine measures
 static cl_int rect_copy(cl_command_queue q, cl_mem src, cl_mem dst, size_t soff, size_t doff,
                         const size_t* region_bytes, size_t srp, size_t ssp, size_t drp, size_t dsp,
-                        cl_uint nw, const cl_event* wl, cl_event* ev, cl_command_type type) {
+                        cl_uint nw, const cl_event* wl, cl_event* ev, cl_command_type type,
+                        bool copy_engine = false) {
   CHECK(check_wait_list(q, nw, wl));
   Enq E;
   E.q = q;
@@ -1351,9 +1511,10 @@ static cl_int rect_copy(cl_command_queue q, cl_mem src, cl_mem dst, size_t soff,
   E.type = type;
   DeviceGuard g(q->dev->ordinal);
   char *s = nullptr, *d = nullptr;
-  CHECK(resident(src, q, true, &s));
-  CHECK(resident(dst, q, true, &d));
+  Store* dst_store = nullptr;
   CHECK(enq_begin(E, nw, wl));
+  CHECK_E(E, in_place(src, q, false, &s, nullptr));
+  CHECK_E(E, in_place(dst, q, true, &d, &dst_store));
   RectParams p{};
   p.src = s + soff;
   p.dst = d + doff;
@@ -1364,8 +1525,9 @@ static cl_int rect_copy(cl_command_queue q, cl_mem src, cl_mem dst, size_t soff,
   p.ssp = ssp;
   p.drp = drp;
   p.dsp = dsp;
-  cl_int st = enq_end(E, launch_rect(p, RECT_COPY, q->stream));
-  if (st == CL_SUCCESS) written(dst, q);
+  cl_int st = enq_end(E, copy_engine ? cudaMemcpyAsync(p.dst, p.src, p.R0, cudaMemcpyDeviceToDevice, q->stream)
+                                      : launch_rect(p, RECT_COPY, q->stream));
+  if (st == CL_SUCCESS) written_store(dst, dst_store);
   return st;
 }
 
@@ -1418,8 +1580,9 @@ extern "C" cl_int clEnqueueFillBuffer(cl_command_queue q, cl_mem buf, const void
   E.type = CL_COMMAND_FILL_BUFFER;
   DeviceGuard g(q->dev->ordinal);
   char* d = nullptr;
-  CHECK(resident(buf, q, true, &d));
+  Store* ds = nullptr;
   CHECK(enq_begin(E, nw, wl));
+  CHECK_E(E, in_place(buf, q, true, &d, &ds));
   RectParams p{};
   p.dst = d + offset;
   p.R0 = size;
@@ -1431,7 +1594,7 @@ extern "C" cl_int clEnqueueFillBuffer(cl_command_queue q, cl_mem buf, const void
   const unsigned char* pat = static_cast<const unsigned char*>(pattern);
   for (uintptr_t k = 0; k < 128; ++k) tb[k] = pat[(k + 128 * ps - (start % ps)) % ps];
   cl_int st = enq_end(E, launch_rect(p, RECT_FILL, q->stream));
-  if (st == CL_SUCCESS) written(buf, q);
+  if (st == CL_SUCCESS) written_store(buf, ds);
   return st;
 }
 
@@ -1511,8 +1674,9 @@ extern "C" cl_int clEnqueueFillImage(cl_command_queue q, cl_mem img, const void*
   E.type = CL_COMMAND_FILL_IMAGE;
   DeviceGuard g(q->dev->ordinal);
   char* d = nullptr;
-  CHECK(resident(img, q, true, &d));
+  Store* ds = nullptr;
   CHECK(enq_begin(E, nw, wl));
+  CHECK_E(E, in_place(img, q, true, &d, &ds));
   const size_t es = L.fmt.es;
   RectParams p{};
   p.dst = d + origin[2] * L.slice_pitch + origin[1] * L.row_pitch + origin[0] * es;
@@ -1526,7 +1690,7 @@ extern "C" cl_int clEnqueueFillImage(cl_command_queue q, cl_mem img, const void*
   p.order = L.fmt.order;
   p.es = (int)es;
   cl_int st = enq_end(E, launch_rect(p, RECT_FILL_IMAGE, q->stream));
-  if (st == CL_SUCCESS) written(img, q);
+  if (st == CL_SUCCESS) written_store(img, ds);
   return st;
 }
 
@@ -1550,7 +1714,7 @@ extern "C" cl_int clEnqueueMigrateMemObjects(cl_command_queue q, cl_uint n, cons
     const bool undefined = flags & CL_MIGRATE_MEM_OBJECT_CONTENT_UNDEFINED;
     for (cl_uint i = 0; i < n; ++i) {
       char* d = nullptr;
-      CHECK(resident(mems[i], q, !undefined, &d));
+      CHECK_E(E, resident(mems[i], q, !undefined, &d));
       if (undefined) written(mems[i], q);  // ownership moves without a copy
     }
   }
@@ -1627,10 +1791,10 @@ extern "C" cl_int b2clEnqueueReadImageSamples(cl_command_queue q, cl_mem img, cl
   E.type = 0x11F0;  // NDRANGE_KERNEL
   DeviceGuard g(q->dev->ordinal);
   char *pi = nullptr, *pc = nullptr, *po = nullptr;
-  CHECK(resident(img, q, true, &pi));
-  CHECK(resident(coords, q, true, &pc));
-  CHECK(resident(out, q, true, &po));
   CHECK(enq_begin(E, nw, wl));
+  CHECK_E(E, resident(img, q, true, &pi));
+  CHECK_E(E, resident(coords, q, true, &pc));
+  CHECK_E(E, resident(out, q, true, &po));
   SampleParams p{};
   p.im = dev_image(img, pi, true);
   fill_sampler(p, smp);
@@ -1674,9 +1838,9 @@ extern "C" cl_int b2clEnqueueReadImageGridRegion(cl_command_queue q, cl_mem img,
   E.type = 0x11F0;
   DeviceGuard g(q->dev->ordinal);
   char *pi = nullptr, *po = nullptr;
-  CHECK(resident(img, q, true, &pi));
-  CHECK(resident(out, q, true, &po));
   CHECK(enq_begin(E, nw, wl));
+  CHECK_E(E, resident(img, q, true, &pi));
+  CHECK_E(E, resident(out, q, true, &po));
   SampleParams p{};
   p.im = dev_image(img, pi, true);
   fill_sampler(p, smp);
@@ -1732,10 +1896,10 @@ extern "C" cl_int b2clEnqueueWriteImageSamples(cl_command_queue q, cl_mem img, b
   E.type = 0x11F0;
   DeviceGuard g(q->dev->ordinal);
   char *pi = nullptr, *pc = nullptr, *pk = nullptr;
-  CHECK(resident(img, q, true, &pi));
-  CHECK(resident(coords, q, true, &pc));
-  CHECK(resident(colors, q, true, &pk));
   CHECK(enq_begin(E, nw, wl));
+  CHECK_E(E, resident(img, q, true, &pi));
+  CHECK_E(E, resident(coords, q, true, &pc));
+  CHECK_E(E, resident(colors, q, true, &pk));
   WriteParams p{};
   p.im = dev_image(img, pi);
   p.rclass = (int)rtype;
@@ -1794,16 +1958,82 @@ extern "C" cl_mem b2clCreateBufferFromIpcHandle(cl_context c, cl_device_id d, co
     if (e != cudaSuccess) { SET_ERR(cuda_err(e)); return nullptr; }
   }
   cl_mem m = new_mem(c, CL_MEM_OBJECT_BUFFER, CL_MEM_READ_WRITE, size);
-  if (!m) { SET_ERR(CL_OUT_OF_HOST_MEMORY); return nullptr; }
+  if (!m) {
+    DeviceGuard g(d->ordinal);
+    cudaIpcCloseMemHandle(p);
+    SET_ERR(CL_OUT_OF_HOST_MEMORY);
+    return nullptr;
+  }
+  Store s;
+  s.ordinal = d->ordinal;
+  s.ptr = static_cast<char*>(p);
+  s.kind = 4;  // another process's memory: its valid copy (kRemoteBit)
+  m->stores.push_back(s);
+  m->valid = 1ull << kRemoteBit;
+  register_mem(m);
+  SET_ERR(CL_SUCCESS);
+  return m;
+}
+
+extern "C" cl_mem b2clCreateImageFromIpcHandle(cl_context c, cl_device_id d, cl_mem_flags flags,
+                                               const cl_image_format* fmt, const cl_image_desc* desc,
+                                               const void* handle64, cl_int* errcode_ret) {
+  if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
+  if (!valid_device(d) || !ctx_has_device(c, d)) { SET_ERR(CL_INVALID_DEVICE); return nullptr; }
+  if (!handle64 || (flags & (CL_MEM_USE_HOST_PTR | CL_MEM_COPY_HOST_PTR | CL_MEM_ALLOC_HOST_PTR))) {
+    SET_ERR(CL_INVALID_VALUE);
+    return nullptr;
+  }
+  ImageLayout L;
+  cl_int st = image_layout(fmt, desc, &L);
+  if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
+  if (desc->image_type == CL_MEM_OBJECT_IMAGE1D_BUFFER || desc->image_row_pitch || desc->image_slice_pitch) {
+    SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR);
+    return nullptr;
+  }
+  cudaIpcMemHandle_t h;
+  memcpy(&h, handle64, 64);
+  void* p = nullptr;
+  {
+    DeviceGuard g(d->ordinal);
+    cudaError_t e = cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) { SET_ERR(cuda_err(e)); return nullptr; }
+  }
+  cl_mem m = new_mem(c, desc->image_type, flags & (CL_MEM_READ_WRITE | CL_MEM_WRITE_ONLY | CL_MEM_READ_ONLY),
+                     L.bytes);
+  if (!m) {
+    DeviceGuard g(d->ordinal);
+    cudaIpcCloseMemHandle(p);
+    SET_ERR(CL_OUT_OF_HOST_MEMORY);
+    return nullptr;
+  }
+  m->img = L;
+  m->fmt = *fmt;
+  m->desc = *desc;
   Store s;
   s.ordinal = d->ordinal;
   s.ptr = static_cast<char*>(p);
   s.kind = 4;
   m->stores.push_back(s);
-  m->valid = 1ull << d->ordinal;
+  m->valid = 1ull << kRemoteBit;
   register_mem(m);
   SET_ERR(CL_SUCCESS);
   return m;
+}
+
+extern "C" cl_int b2clEnqueueCopyBufferEngine(cl_command_queue q, cl_mem src, cl_mem dst, size_t so,
+                                              size_t dso, size_t size, cl_uint nw, const cl_event* wl,
+                                              cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_queue_mem(q, src));
+  CHECK(check_queue_mem(q, dst));
+  if (src->type != CL_MEM_OBJECT_BUFFER || dst->type != CL_MEM_OBJECT_BUFFER) return CL_INVALID_MEM_OBJECT;
+  if (size == 0 || so > src->size || size > src->size - so || dso > dst->size || size > dst->size - dso)
+    return CL_INVALID_VALUE;
+  if (src == dst && so < dso + size && dso < so + size) return CL_MEM_COPY_OVERLAP;
+  const size_t region[3] = {size, 1, 1};
+  return rect_copy(q, src, dst, so, dso, region, size, size, size, size, nw, wl, ev, CL_COMMAND_COPY_BUFFER,
+                   true);
 }
 
 // ===================================================================== programs and kernels
@@ -1828,6 +2058,8 @@ struct _cl_program {
   std::vector<void*> offset_sym;                    // __b2cl_global_offset per module (or null)
   std::vector<void*> const_sym;                     // __OC2CU_const_mem per module (or null)
   size_t const_bytes = 0;
+  std::mutex sym_mu;                                // orders launches that write the symbols
+  std::vector<cudaEvent_t> sym_ev;                  // per module: the last such launch
   cl_int status = CL_BUILD_NONE;
   std::string log;
 };
@@ -1909,6 +2141,7 @@ extern "C" cl_int clBuildProgram(cl_program p, cl_uint n, const cl_device_id* de
       p->libs.clear();
       p->offset_sym.clear();
       p->const_sym.clear();
+      p->sym_ev.clear();
       p->status = CL_BUILD_ERROR;
       if (notify) notify(p, user_data);
       return CL_BUILD_PROGRAM_FAILURE;
@@ -1930,6 +2163,7 @@ extern "C" cl_int clBuildProgram(cl_program p, cl_uint n, const cl_device_id* de
     p->libs.push_back(lib);
     p->offset_sym.push_back(sym);
     p->const_sym.push_back(csym);
+    p->sym_ev.push_back(nullptr);
     p->const_bytes = cbytes;
   }
   p->status = CL_BUILD_SUCCESS;
@@ -1949,21 +2183,17 @@ extern "C" cl_int clGetProgramBuildInfo(cl_program p, cl_device_id d, cl_program
 }
 
 extern "C" cl_int clRetainProgram(cl_program p) {
-  if (!live(g_programs, p)) return CL_INVALID_PROGRAM;
-  p->ref++;
-  return CL_SUCCESS;
+  return retain_ref(g_programs, p) ? CL_SUCCESS : CL_INVALID_PROGRAM;
 }
 
 extern "C" cl_int clReleaseProgram(cl_program p) {
-  if (!live(g_programs, p)) return CL_INVALID_PROGRAM;
-  if (--p->ref == 0) {
-    {
-      std::lock_guard<std::mutex> g(g_mu);
-      g_programs.erase(p);
-    }
+  const int r = release_ref(g_programs, p);
+  if (r < 0) return CL_INVALID_PROGRAM;
+  if (r == 1) {
     for (size_t i = 0; i < p->libs.size(); ++i) {
       DeviceGuard g(p->ordinals[i]);
       cudaDeviceSynchronize();  // no launch of the module may still be running
+      if (i < p->sym_ev.size() && p->sym_ev[i]) cudaEventDestroy(p->sym_ev[i]);
       cudaLibraryUnload(p->libs[i]);
     }
     cl_context c = p->ctx;
@@ -2026,18 +2256,13 @@ extern "C" cl_kernel clCreateKernel(cl_program p, const char* name, cl_int* errc
 }
 
 extern "C" cl_int clRetainKernel(cl_kernel k) {
-  if (!live(g_kernels, k)) return CL_INVALID_KERNEL;
-  k->ref++;
-  return CL_SUCCESS;
+  return retain_ref(g_kernels, k) ? CL_SUCCESS : CL_INVALID_KERNEL;
 }
 
 extern "C" cl_int clReleaseKernel(cl_kernel k) {
-  if (!live(g_kernels, k)) return CL_INVALID_KERNEL;
-  if (--k->ref == 0) {
-    {
-      std::lock_guard<std::mutex> g(g_mu);
-      g_kernels.erase(k);
-    }
+  const int r = release_ref(g_kernels, k);
+  if (r < 0) return CL_INVALID_KERNEL;
+  if (r == 1) {
     cl_program p = k->prog;
     delete k;
     clReleaseProgram(p);
@@ -2145,6 +2370,7 @@ extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uin
   E.evout = ev;
   E.type = CL_COMMAND_NDRANGE_KERNEL;
   DeviceGuard g(q->dev->ordinal);
+  CHECK(enq_begin(E, nw, wl));  // the wait list first: argument migrations come after it
   // argument values, in parameter order
   const size_t na = k->args.size();
   std::vector<std::vector<unsigned char>> vals(na);
@@ -2153,7 +2379,7 @@ extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uin
   for (const KArg& a : k->args)
     if (a.kind == 5) const_bytes += a.mem->size;
   if (const_bytes && (!k->prog->const_sym[mi] || const_bytes > k->prog->const_bytes))
-    return CL_OUT_OF_RESOURCES;  // more __constant data than the module's constant array
+    return enq_fail(E, CL_OUT_OF_RESOURCES);  // more __constant data than the module's constant array
   std::vector<std::pair<char*, size_t>> const_src;  // (device pointer, bytes) in argument order
   for (size_t i = 0; i < na; ++i) {
     const KArg& a = k->args[i];
@@ -2161,7 +2387,7 @@ extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uin
       vals[i] = a.bytes;
     } else if (a.kind == 2) {
       char* ptr = nullptr;
-      CHECK(resident(a.mem, q, true, &ptr));
+      CHECK_E(E, resident(a.mem, q, true, &ptr));
       if (is_image(a.mem)) {
         const dev::Image im = dev_image(a.mem, ptr, true);
         vals[i].resize(sizeof(im));
@@ -2177,7 +2403,7 @@ extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uin
       memcpy(vals[i].data(), &bits, 4);
     } else if (a.kind == 5) {
       char* ptr = nullptr;
-      CHECK(resident(a.mem, q, true, &ptr));
+      CHECK_E(E, resident(a.mem, q, true, &ptr));
       const_src.emplace_back(ptr, a.mem->size);
       vals[i].resize(sizeof(size_t));
       memcpy(vals[i].data(), &a.mem->size, sizeof(size_t));
@@ -2188,12 +2414,21 @@ extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uin
     }
     argp[i] = vals[i].data();
   }
-  CHECK(enq_begin(E, nw, wl));
   const void* fn = reinterpret_cast<const void*>(k->kerns[mi]);
   cudaError_t e = cudaSuccess;
   if (local_bytes > 48 * 1024)
     e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)local_bytes);
   void* osym = k->prog->offset_sym[mi];
+  // The global offset and the __constant array are module globals: a launch
+  // on another queue must not overwrite them while this one still reads them.
+  // Launches that use them are chained per module -- each waits for the
+  // previous such launch's completion event (from any queue) before its copies.
+  const bool uses_syms = osym || !const_src.empty();
+  std::unique_lock<std::mutex> sym_lock(k->prog->sym_mu, std::defer_lock);
+  if (uses_syms) {
+    sym_lock.lock();
+    if (e == cudaSuccess && k->prog->sym_ev[mi]) e = cudaStreamWaitEvent(q->stream, k->prog->sym_ev[mi], 0);
+  }
   if (e == cudaSuccess && osym)  // get_global_offset(): pageable source, staged before return
     e = cudaMemcpyAsync(osym, O, sizeof(O), cudaMemcpyHostToDevice, q->stream);
   // deferred placement of __constant buffers: copied at launch
@@ -2210,6 +2445,11 @@ extern "C" cl_int clEnqueueNDRangeKernel(cl_command_queue q, cl_kernel k, cl_uin
                          local_bytes, q->stream);
     if (e == cudaSuccess) count_launch("user kernel (clEnqueueNDRangeKernel)");
   }
+  if (uses_syms && e == cudaSuccess) {
+    if (!k->prog->sym_ev[mi]) e = cudaEventCreateWithFlags(&k->prog->sym_ev[mi], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventRecord(k->prog->sym_ev[mi], q->stream);
+  }
+  if (uses_syms) sym_lock.unlock();
   cl_int st = enq_end(E, e);
   if (st == CL_SUCCESS)
     for (const KArg& a : k->args)

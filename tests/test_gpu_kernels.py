@@ -18,14 +18,27 @@ pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
+def _cubin_bytes():
+    """tests/kernels/translated.cu compiled with nvcc for sm_100a (cached per process)."""
+    global _CUBIN
+    if _CUBIN is None:
+        import tempfile
+        with tempfile.TemporaryDirectory() as d:
+            out = os.path.join(d, "translated.cubin")
+            nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+            subprocess.run([nvcc, "-cubin", "-gencode", "arch=compute_100a,code=sm_100a", "-O3",
+                            "-std=c++17", "-I", os.path.join(ROOT, "include"), "-o", out,
+                            os.path.join(ROOT, "tests", "kernels", "translated.cu")], check=True)
+            _CUBIN = open(out, "rb").read()
+    return _CUBIN
+
+
+_CUBIN = None
+
+
 @pytest.fixture(scope="module")
-def cubin(tmp_path_factory):
-    out = tmp_path_factory.mktemp("k") / "translated.cubin"
-    nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-    subprocess.run([nvcc, "-cubin", "-gencode", "arch=compute_100a,code=sm_100a", "-O3",
-                    "-std=c++17", "-I", os.path.join(ROOT, "include"), "-o", str(out),
-                    os.path.join(ROOT, "tests", "kernels", "translated.cu")], check=True)
-    return out.read_bytes()
+def cubin():
+    return _cubin_bytes()
 
 
 @pytest.fixture(scope="module")

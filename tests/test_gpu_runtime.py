@@ -1,0 +1,91 @@
+"""Runtime semantics on the GPU (SURVEY §8(b) ownership, §8(e) multi-device):
+
+* clReleaseMemObject is stream-ordered and deferred: releasing the source of a
+  long copy right after enqueueing it returns without a host wait, and the
+  copy still reads the right bytes (the storage is freed only after the
+  queue's event for it completes);
+* launches of one translated module from two queues that both set the
+  module's global offset are chained, so each launch sees its own offset
+  (symbol race);
+* two processes sharing objects through CUDA IPC (tests/ipc_worker.py): region
+  copies in place on the exporter's memory, whole-object pulls for sampling
+  and migration, a wait-listed migration ordered after the write it waits for,
+  and the copy-engine reference path."""
+import ctypes
+import os
+import subprocess
+import sys
+import time
+
+import numpy as np
+import pytest
+
+from paper_conf_sc_kimdjjl15_b200 import cl
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_release_is_deferred_and_stream_ordered(sess):
+    L = cl.lib()
+    n = 1 << 30  # 1 GiB: the copy takes ~0.3 ms on the GPU
+    g = np.random.default_rng(7)
+    head = g.integers(0, 256, 1 << 20, dtype=np.uint8)
+    src, dst = sess.buffer(n), sess.buffer(n)
+    sess.write(src, head)                 # a recognisable first MiB
+    pat = np.array([0x3C], np.uint8)
+    cl.check(L.clEnqueueFillBuffer(sess.queue, src, pat.ctypes.data, 1, 1 << 20, n - (1 << 20), 0, None, None))
+    sess.finish()
+    # queue several long copies, then release the source while they run
+    for _ in range(8):
+        cl.check(L.clEnqueueCopyBuffer(sess.queue, src, dst, 0, 0, n, 0, None, None))
+    t0 = time.perf_counter()
+    cl.check(L.clReleaseMemObject(src))
+    dt = time.perf_counter() - t0
+    pending = L.clFinish(sess.queue)   # (reaps the deferred free)
+    assert pending == 0
+    assert dt < 1e-3, f"release blocked the host for {dt * 1e3:.2f} ms"
+    got = sess.read(dst, 1 << 20)
+    assert np.array_equal(got, head)
+    assert np.all(sess.read(dst, 4096, offset=n - 4096) == 0x3C)
+    # the handle is dead: a second release fails cleanly
+    assert L.clReleaseMemObject(src) == -38  # CL_INVALID_MEM_OBJECT
+    sess.release(dst)
+
+
+def test_module_symbols_chained_across_queues(sess):
+    from tests.test_gpu_kernels import _cubin_bytes
+    L = cl.lib()
+    prog = sess.program(_cubin_bytes())
+    q2 = sess.queue_for(0)
+    N = 1 << 22
+    outs = [sess.buffer(N * 4), sess.buffer(N * 4)]
+    offs = [7, 100003]
+    ks = [sess.kernel(prog, "ids1d"), sess.kernel(prog, "ids1d")]
+    for k, o in zip(ks, outs):
+        sess.set_args(k, o)
+    gws = cl.sz3((N, 0, 0))
+    lws = cl.sz3((256, 0, 0))
+    for it in range(20):
+        for i, q in enumerate((sess.queue, q2)):
+            cl.check(L.clEnqueueNDRangeKernel(q, ks[i], 1, cl.sz3((offs[i], 0, 0)), gws, lws, 0, None, None))
+    cl.check(L.clFinish(q2))
+    sess.finish()
+    for i in range(2):
+        got = sess.read(outs[i], N * 4, np.int32)
+        gi = np.arange(offs[i], offs[i] + N, dtype=np.int64)
+        assert np.array_equal(got, (gi * 10 + (gi - offs[i]) // 256).astype(np.int32)), f"queue {i}"
+    for k in ks:
+        L.clReleaseKernel(k)
+    L.clReleaseCommandQueue(q2)
+    L.clReleaseProgram(prog)
+    sess.release(*outs)
+
+
+def test_ipc_two_processes():
+    env = dict(os.environ, MASTER_ADDR="127.0.0.1")
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+                        "--master-addr=127.0.0.1", "--master-port=29561",
+                        os.path.join(ROOT, "tests", "ipc_worker.py")],
+                       cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]

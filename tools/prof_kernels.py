@@ -2,7 +2,8 @@
 
     ncu --set full -k regex:<kernel> -c N -o gpurun_out/prof python tools/prof_kernels.py [which...]
 
-which: c2 (REPEAT + MIRRORED 4096^2 RGBA32F), c3 (512^3 R32F stencil + rotated),
+which: c2r / c2m (ONE map (A) REPEAT / MIRRORED launch each: bench.py's
+in-run traffic capture), c2 (REPEAT + MIRRORED 4096^2 RGBA32F, maps A and B), c3 (512^3 R32F stencil + rotated),
 copy (8 GiB pitched rect, aligned + misaligned), fill (8 GiB).  Each launch is
 preceded by one untimed warm-up launch of the same kernel.
 """
@@ -21,6 +22,20 @@ def main(which):
     build.build()
     S = cl.Session(0)
     L = cl.lib()
+    if "c2r" in which or "c2m" in which:
+        # the bench's in-run traffic capture: ONE launch of each named map (A) pass
+        n = 4096
+        img = S.image(cl.CL_RGBA, cl.CL_FLOAT, n, n,
+                      host=synth.image_codes(synth.rng(2), cl.CL_RGBA, cl.CL_FLOAT, n, n))
+        out = S.buffer(n * n * 16)
+        A = (ctypes.c_float * 12)(*synth.affine_translate_2d(n, n).tolist())
+        for key, addr in (("c2r", cl.CL_ADDRESS_REPEAT), ("c2m", cl.CL_ADDRESS_MIRRORED_REPEAT)):
+            if key in which:
+                smp = S.sampler(True, addr, cl.CL_FILTER_LINEAR)
+                cl.check(L.b2clEnqueueReadImageGrid(S.queue, img, smp, 0, A, cl.sz3((n, n, 1)), 4,
+                                                    out, 0, 0, None, None))
+        S.finish()
+        S.release(img, out)
     if "c2" in which:
         n = 4096
         img = S.image(cl.CL_RGBA, cl.CL_FLOAT, n, n,
