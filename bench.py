@@ -313,18 +313,29 @@ def ncu_traffic(kernels, which, timeout=300):
 
 def enqueue_cost():
     """Host cost of one enqueue measured from C (tools/enqueue_bench.c, compiled
-    here with gcc if needed; no Python in the loop)."""
-    exe = os.path.join(ROOT, "build", "enqueue_bench")
-    src = os.path.join(ROOT, "tools", "enqueue_bench.c")
+    here with gcc; no Python in the loop), beside the CUDA runtime's own cost of
+    launching an empty kernel on this host (tools/launch_floor.cu, nvcc): the
+    difference is the library's overhead per call."""
+    out = {}
     try:
-        if not os.path.exists(exe) or os.path.getmtime(exe) < os.path.getmtime(src):
-            os.makedirs(os.path.dirname(exe), exist_ok=True)
-            subprocess.run(["gcc", "-O2", "-o", exe, src, "-ldl"], check=True, capture_output=True)
+        exe = os.path.join(ROOT, "build", "enqueue_bench")
+        os.makedirs(os.path.dirname(exe), exist_ok=True)
+        subprocess.run(["gcc", "-O2", "-o", exe, os.path.join(ROOT, "tools", "enqueue_bench.c"), "-ldl"],
+                       check=True, capture_output=True)
         r = subprocess.run([exe, os.path.join(ROOT, "paper_conf_sc_kimdjjl15_b200", "libb2cl.so")],
                            capture_output=True, text=True, timeout=120, cwd=ROOT)
-        return json.loads(r.stdout.strip().splitlines()[-1])
+        out.update(json.loads(r.stdout.strip().splitlines()[-1]))
+        fl = os.path.join(ROOT, "build", "launch_floor")
+        subprocess.run([os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc"), "-O2", "-gencode",
+                        "arch=compute_100a,code=sm_100a", "-o", fl, os.path.join(ROOT, "tools", "launch_floor.cu")],
+                       check=True, capture_output=True, timeout=300)
+        r = subprocess.run([fl], capture_output=True, text=True, timeout=120)
+        floor = json.loads(r.stdout.strip().splitlines()[-1])
+        out["cuda_launch_floor"] = floor
+        out["library_overhead_us"] = out["copy_image_to_buffer_4KiB_us"] - floor["launch_us_256B"]
     except Exception as exc:  # a secondary measurement, never fatal
-        return {"unavailable": str(exc)[:200]}
+        out["unavailable"] = str(exc)[:200]
+    return out
 
 
 def circular_interval(idx, n):
@@ -665,16 +676,28 @@ C5_WORKLOAD = ("C5: 32768x32768 CL_RGBA/CL_FLOAT row-sharded over N GPUs (one pr
 
 
 def _runs(rows, lo, hi):
-    """Maximal runs [a, b) of consecutive global rows inside [lo, hi), in order."""
+    """Maximal runs of consecutive global rows inside [lo, hi), in order:
+    (first row, end row, index in `rows` of the first row)."""
     out = []
     for i, r in enumerate(rows):
         if not (lo <= r < hi):
             continue
-        if out and out[-1][1] == r and out[-1][2] + 1 == i:
-            out[-1] = (out[-1][0], r + 1, i)
+        if out and out[-1][1] == r and out[-1][2] + (out[-1][1] - out[-1][0]) == i:
+            out[-1] = (out[-1][0], r + 1, out[-1][2])
         else:
             out.append((r, r + 1, i))
-    return [(a, b, i - (b - a - 1)) for a, b, i in out]
+    return out
+
+
+def shard_copy_plan(rows, band, world):
+    """Region copies that fill a shard holding global texel rows `rows` (shard
+    row t = rows[t]) from the owners' bands (rank d owns [d*band, (d+1)*band)):
+    [(owner d, first row in d's band, first shard row, row count)]."""
+    plan = []
+    for d in range(world):
+        for ga, gb, si in _runs(rows, d * band, (d + 1) * band):
+            plan.append((d, ga - d * band, si, gb - ga))
+    return plan
 
 
 def run_c5(args):
@@ -757,10 +780,7 @@ def run_c5(args):
                                     begin, count, 0, None, ctypes.byref(err))
         cl.check(err.value, "shard")
         shards.append(sh)
-        plan = []
-        for d in range(world):
-            for ga, gb, si in _runs(rows, d * band, (d + 1) * band):
-                plan.append((bands[d], ga - d * band, si, gb - ga, d != rank))
+        plan = [(bands[d], sr, dr, n, d != rank) for d, sr, dr, n in shard_copy_plan(rows, band, world)]
         shard_info.append({"begin": begin, "rows": count,
                            "rows_from_peers": int(sum(n for *_, n, peer in plan if peer)),
                            "copies": len(plan)})

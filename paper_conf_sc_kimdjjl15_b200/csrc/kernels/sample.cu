@@ -26,6 +26,7 @@
 
 #include "../device/read.cuh"
 #include "launch.h"
+#include "tma.h"
 
 namespace b2cl {
 using namespace dev;
@@ -607,8 +608,12 @@ __device__ __forceinline__ int fold_prim(int pi, int M, int A) { return pi < A ?
 #ifndef B2CL_FOLD_MINB
 #define B2CL_FOLD_MINB 1
 #endif
+#ifndef B2CL_FOLD_TMA
+#define B2CL_FOLD_TMA 0  // 1: stage the union box with one cp.async.bulk.tensor.3d (measured 61.5 vs 58.2 us for the 16-B cp.async)
+#endif
 template <class C>
-__global__ void __launch_bounds__(128, B2CL_FOLD_MINB) k_sample_grid_fold(const SampleParams p, const FoldMap fm) {
+__global__ void __launch_bounds__(128, B2CL_FOLD_MINB)
+    k_sample_grid_fold(const SampleParams p, const FoldMap fm, const __grid_constant__ CUtensorMap tmap) {
   static_assert(C::type == T_FLOAT && C::order == O_RGBA && C::dims == 2, "2D RGBA32F");
   static_assert(C::addr == A_REPEAT || C::addr == A_MIRROR, "taps always in range");
 #ifndef B2CL_FOLD_PAD
@@ -616,11 +621,12 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB) k_sample_grid_fold(const 
 #endif
   // the staged box: the tile's taps plus room for the mirror images' offsets
   constexpr int TW = 64, TH = 16, BW = TW + B2CL_FOLD_PAD, BH = TH + B2CL_FOLD_PAD;
-  __shared__ __align__(16) float4 box[BH][BW];
+  __shared__ __align__(128) float4 box[BH][BW];
   __shared__ int cI0[2][TW], cI1[2][TW], cX[2][TW], rY[2][TH];
   __shared__ float cA[2][TW], cOma[2][TW];
   __shared__ float4 rT[2][TH];  // per row: {b, 1 - b, j0 bits, j1 bits}
   __shared__ int bb[4];         // column min, max, row min, max of the staged box
+  __shared__ uint64_t fbar;     // the TMA box's completion
   const Image& im = p.im;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int xp0 = blockIdx.x * TW, yp0 = blockIdx.y * TH;
@@ -667,7 +673,16 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB) k_sample_grid_fold(const 
   const bool staged = bb[1] >= c0 && bb[1] - c0 < BW && bb[3] >= r0 && bb[3] - r0 < BH;
   const uint64_t zoff = (uint64_t)blockIdx.z * p.oh;
   float4* out = reinterpret_cast<float4*>(p.out) + zoff * p.ow;
-  if (staged) {  // the union box: warp w copies box rows w, w + 4, ...; 16-byte async copies
+  constexpr bool kTma = B2CL_FOLD_TMA && !C::shard;  // (shard rows may wrap in storage)
+  if (staged && kTma) {  // the union box: ONE tensor copy (TMA) of BH rows x BW texels
+    if (tid == 0) {
+      mbar_init(&fbar, 1);
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      mbar_expect_tx(&fbar, (uint32_t)(BW * BH * 16));
+      tma_load_3d(&box[0][0], &tmap, 0, c0, r0, &fbar);
+    }
+  } else if (staged) {  // warp w copies box rows w, w + 4, ...; 16-byte async copies
     const int nc = bb[1] - c0 + 1, nr = bb[3] - r0 + 1;
     for (int rr = warp; rr < nr; rr += 4) {
       const char* src = row_ptr<C>(im, r0 + rr, 0) + (uint64_t)(unsigned)c0 * 16u;
@@ -679,6 +694,7 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB) k_sample_grid_fold(const 
     asm volatile("cp.async.wait_all;" ::: "memory");
   }
   __syncthreads();
+  if (staged && kTma) mbar_wait(&fbar, 0);
   // warp w: columns (w & 1)*32 + lane, rows (w >> 1)*8 .. +8, for each of the
   // four (column set, row set) combinations
   const int c = (warp & 1) * 32 + lane, rb = (warp >> 1) * (TH / 2);
@@ -888,8 +904,25 @@ static bool go_fold(const SampleParams& p, cudaStream_t st, cudaError_t* err) {
   if (!fold_axis((double)p.A[0], (double)p.A[3], p.ox, p.ow, &fm.Mx, &fm.Ax, &fm.Px)) return false;
   if (!fold_axis((double)p.A[5], (double)p.A[7], p.oy, p.oh, &fm.My, &fm.Ay, &fm.Py)) return false;
   dim3 grd((fm.Px + 63) / 64, (fm.Py + 15) / 16, p.od);
-  if (is_shard(p)) k_sample_grid_fold<WithShard<C, true>><<<grd, 128, 0, st>>>(p, fm);
-  else k_sample_grid_fold<WithShard<C, false>><<<grd, 128, 0, st>>>(p, fm);
+  // the image as a (4 channels, width, height) fp32 tensor for the box copy
+  // (a 70-texel row is 280 floats: over one dimension's 256-element box limit)
+  CUtensorMap tm;
+  memset(&tm, 0, sizeof(tm));
+  bool tma = B2CL_FOLD_TMA && !is_shard(p);
+  if (tma) {
+    auto enc = tma_encode_fn();
+    const cuuint64_t dims[3] = {4, (cuuint64_t)p.im.w, (cuuint64_t)p.im.h};
+    const cuuint64_t strides[2] = {16, p.im.rp};
+    const cuuint32_t box[3] = {4, (cuuint32_t)(64 + B2CL_FOLD_PAD), (cuuint32_t)(16 + B2CL_FOLD_PAD)};
+    const cuuint32_t es[3] = {1, 1, 1};
+    tma = enc && !(reinterpret_cast<uintptr_t>(p.im.ptr) & 15) && !(p.im.rp & 15) &&
+          enc(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, p.im.ptr, dims, strides, box, es,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+  }
+  if (!tma && B2CL_FOLD_TMA && !is_shard(p)) return false;  // (no encoder: the separable path)
+  if (is_shard(p)) k_sample_grid_fold<WithShard<C, true>><<<grd, 128, 0, st>>>(p, fm, tm);
+  else k_sample_grid_fold<WithShard<C, false>><<<grd, 128, 0, st>>>(p, fm, tm);
   count_launch("k_sample_grid_fold");
   *err = cudaGetLastError();
   return true;

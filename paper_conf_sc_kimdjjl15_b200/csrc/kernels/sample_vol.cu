@@ -527,6 +527,9 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
 #ifndef B2CL_VOLR_S
 #define B2CL_VOLR_S 8
 #endif
+#ifndef B2CL_VOLR_LEAN
+#define B2CL_VOLR_LEAN 0  // 1: the interior-tile slice with precomputed offsets and paired blends (measured 247.9 vs 240.9 us)
+#endif
 constexpr int VOLR_S = B2CL_VOLR_S;           // samples (rows) per consumer thread
 constexpr int RT_W = 64, RT_H = 4 * VOLR_S;   // output tile (256 consumer threads: 64 columns x 4 row groups)
 constexpr int RB_MAXW = 128, RB_MAXH = 128;   // largest staged box (texels)
@@ -690,17 +693,56 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
       }
       continue;
     }
-    auto slice = [&](float V[VOLR_S]) {
-      vol_wait(&full[s], ph);
-      const float* buf = reinterpret_cast<const float*>(volr_buf + s * g.stride);
+    // Interior tiles (every tap pair unclamped: i1 = i0 + 1, j1 = j0 + 1 --
+    // all but the tiles at the image's edges) take the lean slice: byte
+    // offsets precomputed, the 4 taps at fixed deltas, the x-blend of rows
+    // j0 and j1 as one paired FMUL2 + FFMA2 (each lane lerp1's fma / mul).
+#if B2CL_VOLR_LEAN
+    int interior = 1;
+#pragma unroll
+    for (int r = 0; r < VOLR_S; ++r) interior &= (off[r] >> 16) == 3 || !(x < p.ow && y0 + r < p.oh);
+    asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, 256, P; selp.s32 %0, 1, 0, Q; }"
+                 : "=r"(interior) : "r"(interior) : "memory");
+    float oma[VOLR_S], omb[VOLR_S];
+    if (interior) {
 #pragma unroll
       for (int r = 0; r < VOLR_S; ++r) {
-        const float* t0 = buf + (off[r] & 0xffff);
-        const int dx = off[r] >> 16 & 1, dy = (off[r] >> 17) * g.bw;
-        const float oma = __fsub_rn(1.0f, wa[r]), omb = __fsub_rn(1.0f, wb[r]);
-        const float h0 = lerp1(wa[r], oma, t0[0], t0[dx]);
-        const float h1 = lerp1(wa[r], oma, t0[dy], t0[dy + dx]);
-        V[r] = lerp1(wb[r], omb, h0, h1);
+        off[r] = (off[r] & 0xffff) * 4;
+        oma[r] = __fsub_rn(1.0f, wa[r]);
+        omb[r] = __fsub_rn(1.0f, wb[r]);
+      }
+    }
+    const uint32_t rowb = (uint32_t)g.bw * 4u;
+#else
+    const int interior = 0;
+    float oma[1], omb[1];
+    const uint32_t rowb = 0;
+#endif
+    auto slice = [&](float V[VOLR_S]) {
+      vol_wait(&full[s], ph);
+      if (interior) {
+        const char* buf = reinterpret_cast<const char*>(volr_buf + s * g.stride);
+#pragma unroll
+        for (int r = 0; r < VOLR_S && B2CL_VOLR_LEAN; ++r) {
+          const char* t = buf + (uint32_t)off[r];
+          const char* t2 = t + rowb;
+          const float2 lo = make_float2(*reinterpret_cast<const float*>(t), *reinterpret_cast<const float*>(t2));
+          const float2 hi =
+              make_float2(*reinterpret_cast<const float*>(t + 4), *reinterpret_cast<const float*>(t2 + 4));
+          const float2 h = __ffma2_rn(make_float2(wa[r], wa[r]), hi, __fmul2_rn(make_float2(oma[r], oma[r]), lo));
+          V[r] = lerp1(wb[r], omb[r], h.x, h.y);
+        }
+      } else {
+        const float* buf = reinterpret_cast<const float*>(volr_buf + s * g.stride);
+#pragma unroll
+        for (int r = 0; r < VOLR_S; ++r) {
+          const float* t0 = buf + (off[r] & 0xffff);
+          const int dx = off[r] >> 16 & 1, dy = (off[r] >> 17) * g.bw;
+          const float oma1 = __fsub_rn(1.0f, wa[r]), omb1 = __fsub_rn(1.0f, wb[r]);
+          const float h0 = lerp1(wa[r], oma1, t0[0], t0[dx]);
+          const float h1 = lerp1(wa[r], oma1, t0[dy], t0[dy + dx]);
+          V[r] = lerp1(wb[r], omb1, h0, h1);
+        }
       }
       __syncwarp();
       if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(vol_smem(&empty[s])) : "memory");
