@@ -55,6 +55,9 @@ constexpr int BX_W = 32, BX_H = B2CL_BOX_TH;  // output tile
 #ifndef B2CL_BOX_STAGE
 #define B2CL_BOX_STAGE 0  // 0: tensor TMA box, 1: bulk copy per row, 2: 16-B cp.async by all threads
 #endif
+#ifndef B2CL_BOX_PF
+#define B2CL_BOX_PF 592  // L2 prefetch distance in tiles (0: none): 148 SMs x 4 (measured 148 / 296 / 444 / 592 / 888 / 1776: 96.6 / 92.6 / 90.9 / 90.5 / 91.8 / 114.1 us, none 100.2)
+#endif
 #ifndef B2CL_BOX_L2PROMO
 #define B2CL_BOX_L2PROMO 3  // CU_TENSOR_MAP_L2_PROMOTION_L2_256B
 #endif
@@ -260,6 +263,25 @@ __global__ void __launch_bounds__(BX_THREADS, B2CL_BOX_MINB)
       mbar_expect_tx(&full, (uint32_t)(g.bw * g.bh * 16));
       tma_load_2d(box_buf, &tmap, 4 * xlo, ylo, &full);
     }
+#if B2CL_BOX_PF
+    // warm L2 with the box of the tile B2CL_BOX_PF launch positions ahead (the
+    // one that starts about when this wave of CTAs retires): its first-touch
+    // texels come from DRAM now, so that tile's own copy hits L2
+    {
+      const long long nx = gridDim.x, ny = gridDim.y;
+      const long long t = blockIdx.x + nx * (blockIdx.y + ny * (long long)blockIdx.z) + B2CL_BOX_PF;
+      if (t < nx * ny * (long long)gridDim.z) {
+        const int fz = (int)(t / (nx * ny)), fy = (int)((t / nx) % ny), fx = (int)(t % nx);
+        int pxl, pyl;
+        const bool pok = tile_box<C>(p, g, fx * BX_W, fy * BX_H, fz, lane, pxl, pyl);
+        if (lane == 0 && pok)
+          asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];" ::"l"(
+                           reinterpret_cast<uint64_t>(&tmap)),
+                       "r"(4 * pxl), "r"(pyl)
+                       : "memory");
+      }
+    }
+#endif
 #elif B2CL_BOX_STAGE == 1  // one plain bulk copy per box row, rows spread over the lanes
     if (ok) {
       // the taps of REPEAT / MIRRORED_REPEAT / CLAMP_TO_EDGE never leave the

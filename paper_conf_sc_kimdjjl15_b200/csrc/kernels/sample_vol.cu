@@ -44,6 +44,12 @@
 namespace b2cl {
 using namespace dev;
 
+#ifndef B2CL_VOL_PF
+#define B2CL_VOL_PF 0  // L2 prefetch distance in slices of the stencil row copies (0: none; 2 / 4 / 8 measured 210 / 211 / 216 vs 184 us)
+#endif
+#ifndef B2CL_VOLR_PF
+#define B2CL_VOLR_PF 0  // L2 prefetch distance in slices of the rotated boxes (0: none; 2 / 4 / 8 measured 242.6 / 243.7 / 244.7 vs 240.9 us)
+#endif
 #ifndef B2CL_VOL_BULK
 #define B2CL_VOL_BULK 1
 #endif
@@ -249,6 +255,15 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
                     vol_smem(vol_buf + s * VB_STRIDE + lane * VB_W * 4)),
                 "l"(im.ptr + (uint64_t)k * im.sp + (uint64_t)(yb + lane) * im.rp + (uint64_t)xb * 4u), "r"(rb), "r"(fb)
                 : "memory");
+#if B2CL_VOL_PF
+          // warm L2 with the same rows B2CL_VOL_PF slices ahead
+          if (lane < nrow && k + B2CL_VOL_PF < im.d)
+            asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(
+                             im.ptr + (uint64_t)(k + B2CL_VOL_PF) * im.sp + (uint64_t)(yb + lane) * im.rp +
+                             (uint64_t)xb * 4u),
+                         "r"(rb)
+                         : "memory");
+#endif
 #else
           vol_wait(&empty[s], ph ^ 1u);
           asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(VB_BYTES)
@@ -616,6 +631,15 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
               " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(vol_smem(volr_buf + s * g.stride)),
               "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(bx.xb), "r"(bx.yb), "r"(k), "r"(fb)
               : "memory");
+#if B2CL_VOLR_PF
+          // warm L2 with the same box B2CL_VOLR_PF slices ahead: its first-touch
+          // texels come from DRAM while this slice is blended
+          if (k + B2CL_VOLR_PF < im.d)
+            asm volatile("cp.async.bulk.prefetch.tensor.3d.L2.global.tile [%0, {%1, %2, %3}];" ::"l"(
+                             reinterpret_cast<uint64_t>(&tmap)),
+                         "r"(bx.xb), "r"(bx.yb), "r"(k + B2CL_VOLR_PF)
+                         : "memory");
+#endif
           if (++s == VOLR_NS) { s = 0; ph ^= 1u; }
         }
         kA = az.i0;
