@@ -82,10 +82,17 @@ def test_module_symbols_chained_across_queues(sess):
     sess.release(*outs)
 
 
+def _free_port():
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        return so.getsockname()[1]
+
+
 def test_ipc_two_processes():
     env = dict(os.environ, MASTER_ADDR="127.0.0.1")
     r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
-                        "--master-addr=127.0.0.1", "--master-port=29561",
+                        "--master-addr=127.0.0.1", f"--master-port={_free_port()}",
                         os.path.join(ROOT, "tests", "ipc_worker.py")],
                        cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
