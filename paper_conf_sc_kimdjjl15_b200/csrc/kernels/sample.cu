@@ -601,12 +601,16 @@ constexpr int kFoldWalkUnroll = B2CL_FOLD_WALK_UNROLL;  // rows of the walk unro
 struct FoldMap {
   int Mx, Ax, Px;  // columns
   int My, Ay, Py;  // rows
+  int gx, gy, gz;  // tiles along x, y, z
 };
 
 __device__ __forceinline__ int fold_prim(int pi, int M, int A) { return pi < A ? pi : M + 1 + (pi - A); }
 
 #ifndef B2CL_FOLD_MINB
 #define B2CL_FOLD_MINB 1
+#endif
+#ifndef B2CL_FOLD_CTAS
+#define B2CL_FOLD_CTAS 0  // persistent CTAs per SM for the fold kernel (0: one CTA per tile)
 #endif
 #ifndef B2CL_FOLD_PF
 #define B2CL_FOLD_PF 0  // L2 prefetch distance in tiles of the fold kernel (0: none; 148 / 444 / 740 measured 61.5 / 61.9 / 61.8 vs 57.7 us)
@@ -633,7 +637,14 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB)
   __shared__ uint64_t fbar;     // the TMA box's completion
   const Image& im = p.im;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int xp0 = blockIdx.x * TW, yp0 = blockIdx.y * TH;
+  // tiles (x fastest): one per CTA, or a grid-stride loop when the launch is
+  // persistent (B2CL_FOLD_CTAS: a fixed number of CTAs per SM that run beside
+  // the concurrent REPEAT read of the step)
+  const long long ntiles = (long long)fm.gx * fm.gy * fm.gz;
+  for (long long tile = blockIdx.x + (long long)gridDim.x * (blockIdx.y + (long long)gridDim.y * blockIdx.z);
+       tile < ntiles; tile += (long long)gridDim.x * gridDim.y * gridDim.z) {
+  const int BX = (int)(tile % fm.gx), BY = (int)((tile / fm.gx) % fm.gy), BZ = (int)(tile / ((long long)fm.gx * fm.gy));
+  const int xp0 = BX * TW, yp0 = BY * TH;
   if (tid == 0) { bb[0] = 0x7fffffff; bb[1] = -1; bb[2] = 0x7fffffff; bb[3] = -1; }
   __syncthreads();
   // tables: [0] primary, [1] partner; x / y = -1 marks an absent output
@@ -693,10 +704,9 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB)
   // columns and rows and of the primary segments' ends (a prefetch only; the
   // tile's own box is computed exactly when it runs)
   if (warp == 3 && !C::shard) {
-    const long long t = blockIdx.x + (long long)gridDim.x * (blockIdx.y + (long long)gridDim.y * blockIdx.z) +
-                        B2CL_FOLD_PF;
-    if (t < (long long)gridDim.x * gridDim.y * gridDim.z) {
-      const int fx = (int)(t % gridDim.x), fy = (int)((t / gridDim.x) % gridDim.y);
+    const long long t = tile + B2CL_FOLD_PF;
+    if (t < ntiles) {
+      const int fx = (int)(t % fm.gx), fy = (int)((t / fm.gx) % fm.gy);
       const bool rowax = lane >= 4;
       const int k = lane & 3;
       const int base = rowax ? fy * TH : fx * TW, len = rowax ? TH : TW, P = rowax ? fm.Py : fm.Px;
@@ -731,7 +741,7 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB)
   __syncthreads();
   const int c0 = bb[0], r0 = bb[2];
   const bool staged = bb[1] >= c0 && bb[1] - c0 < BW && bb[3] >= r0 && bb[3] - r0 < BH;
-  const uint64_t zoff = (uint64_t)blockIdx.z * p.oh;
+  const uint64_t zoff = (uint64_t)BZ * p.oh;
   float4* out = reinterpret_cast<float4*>(p.out) + zoff * p.ow;
   constexpr bool kTma = B2CL_FOLD_TMA && !C::shard;  // (shard rows may wrap in storage)
   if (staged && kTma) {  // the union box: ONE tensor copy (TMA) of BH rows x BW texels
@@ -836,6 +846,8 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB)
         emit(y, ry, n0, n1);
       }
     }
+  }
+  __syncthreads();  // (the next tile of a persistent CTA reuses the tables and the box)
   }
 }
 
@@ -955,7 +967,19 @@ static bool go_fold(const SampleParams& p, cudaStream_t st, cudaError_t* err) {
   if (!p.smp.norm) return false;
   if (!fold_axis((double)p.A[0], (double)p.A[3], p.ox, p.ow, &fm.Mx, &fm.Ax, &fm.Px)) return false;
   if (!fold_axis((double)p.A[5], (double)p.A[7], p.oy, p.oh, &fm.My, &fm.Ay, &fm.Py)) return false;
-  dim3 grd((fm.Px + 63) / 64, (fm.Py + 15) / 16, p.od);
+  fm.gx = (fm.Px + 63) / 64;
+  fm.gy = (fm.Py + 15) / 16;
+  fm.gz = p.od;
+  dim3 grd(fm.gx, fm.gy, fm.gz);
+  static const char* ctas_env = getenv("B2CL_FOLD_CTAS");  // A/B: persistent CTAs per SM (0: one per tile)
+  const int ctas = ctas_env ? atoi(ctas_env) : B2CL_FOLD_CTAS;
+  if (ctas > 0) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const long long nt = (long long)fm.gx * fm.gy * fm.gz;
+    grd = dim3((unsigned)std::min<long long>(nt, (long long)sms * ctas), 1, 1);
+  }
   // the image as a (4 channels, width, height) fp32 tensor for the box copy
   // (a 70-texel row is 280 floats: over one dimension's 256-element box limit)
   CUtensorMap tm;
