@@ -9,6 +9,9 @@
 // (3) waits for the wait-list events, (4) launches ONE kernel (or a copy
 // engine transfer for host memory), (5) returns an event if asked.
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
+#include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -1033,6 +1036,7 @@ struct Enq {
   cl_event* evout = nullptr;
   cl_command_type type = 0;
   cudaEvent_t start = nullptr;
+  uint64_t launches0 = 0;  // library launch count at enq_begin (tracing)
 };
 
 static cl_int check_wait_list(cl_command_queue q, cl_uint n, const cl_event* list) {
@@ -1044,6 +1048,7 @@ static cl_int check_wait_list(cl_command_queue q, cl_uint n, const cl_event* lis
 
 // after validation: make the stream wait for the wait list; start event
 static cl_int enq_begin(Enq& E, cl_uint n, const cl_event* list) {
+  E.launches0 = launch_count();
   for (cl_uint i = 0; i < n; ++i) cudaStreamWaitEvent(E.q->stream, list[i]->end, 0);
   if (E.evout && (E.q->props & CL_QUEUE_PROFILING_ENABLE)) {
     if (cudaEventCreate(&E.start) != cudaSuccess) return CL_OUT_OF_RESOURCES;
@@ -1052,7 +1057,46 @@ static cl_int enq_begin(Enq& E, cl_uint n, const cl_event* list) {
   return CL_SUCCESS;
 }
 
+// ---- tracing: B2CL_LOG=1 prints one line per enqueued command
+// to stderr (command, queue, device, the kernel the library picked, status);
+// B2CL_NVTX=1 drops an NVTX mark with the same text (nsys / ncu --nvtx).
+static const char* command_name(cl_command_type t) {
+  switch (t) {
+    case CL_COMMAND_NDRANGE_KERNEL: return "NDRANGE_KERNEL";
+    case CL_COMMAND_READ_BUFFER: return "READ_BUFFER";
+    case CL_COMMAND_WRITE_BUFFER: return "WRITE_BUFFER";
+    case CL_COMMAND_COPY_BUFFER: return "COPY_BUFFER";
+    case CL_COMMAND_READ_IMAGE: return "READ_IMAGE";
+    case CL_COMMAND_WRITE_IMAGE: return "WRITE_IMAGE";
+    case CL_COMMAND_COPY_IMAGE: return "COPY_IMAGE";
+    case CL_COMMAND_COPY_IMAGE_TO_BUFFER: return "COPY_IMAGE_TO_BUFFER";
+    case CL_COMMAND_COPY_BUFFER_TO_IMAGE: return "COPY_BUFFER_TO_IMAGE";
+    case CL_COMMAND_MARKER: return "MARKER";
+    case CL_COMMAND_READ_BUFFER_RECT: return "READ_BUFFER_RECT";
+    case CL_COMMAND_WRITE_BUFFER_RECT: return "WRITE_BUFFER_RECT";
+    case CL_COMMAND_COPY_BUFFER_RECT: return "COPY_BUFFER_RECT";
+    case CL_COMMAND_BARRIER: return "BARRIER";
+    case CL_COMMAND_MIGRATE_MEM_OBJECTS: return "MIGRATE_MEM_OBJECTS";
+    case CL_COMMAND_FILL_BUFFER: return "FILL_BUFFER";
+    case CL_COMMAND_FILL_IMAGE: return "FILL_IMAGE";
+    default: return "COMMAND";
+  }
+}
+
+static void trace_command(const Enq& E, cl_int status) {
+  static const int log = getenv("B2CL_LOG") ? atoi(getenv("B2CL_LOG")) : 0;
+  static const int nvtx = getenv("B2CL_NVTX") ? atoi(getenv("B2CL_NVTX")) : 0;
+  if (!log && !nvtx) return;
+  char buf[160];
+  snprintf(buf, sizeof(buf), "b2cl %s queue=%p dev=%d kernel=%s status=%d", command_name(E.type),
+           static_cast<void*>(E.q), E.q->dev->ordinal, launch_count() > E.launches0 ? last_kernel() : "-",
+           status);
+  if (log) fprintf(stderr, "[%s]\n", buf);
+  if (nvtx) nvtxMarkA(buf);
+}
+
 static cl_int enq_end(Enq& E, cudaError_t err) {
+  trace_command(E, err == cudaSuccess ? CL_SUCCESS : cuda_err(err));
   if (err != cudaSuccess) {
     if (E.start) cudaEventDestroy(E.start);
     return cuda_err(err);

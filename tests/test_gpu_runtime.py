@@ -96,3 +96,18 @@ def test_ipc_two_processes():
                         os.path.join(ROOT, "tests", "ipc_worker.py")],
                        cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
+
+
+def test_trace_log_names_command_and_kernel():
+    """B2CL_LOG=1: one stderr line per enqueued command with the kernel used."""
+    code = ("import numpy as np\n"
+            "from paper_conf_sc_kimdjjl15_b200 import cl\n"
+            "S = cl.Session(0)\n"
+            "b = S.buffer(4096)\n"
+            "p = np.arange(4, dtype=np.uint8)\n"
+            "cl.check(cl.lib().clEnqueueFillBuffer(S.queue, b, p.ctypes.data, 4, 0, 4096, 0, None, None))\n"
+            "S.finish()\n")
+    r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, env=dict(os.environ, B2CL_LOG="1"),
+                       capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+    assert "[b2cl FILL_BUFFER" in r.stderr and "kernel=k_rect<FILL>" in r.stderr, r.stderr[-2000:]
