@@ -1130,8 +1130,13 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
     zero = cl.sz3((0, 0, 0))
     ms = _time_launches(T, torch, dev, lambda: cl.check(L.clEnqueueCopyBufferRect(
         S.queue, src, dst, zero, zero, cl.sz3(region), srp, ssp, 0, 0, 0, None, None)), 5)
+    ms_ce = _time_launches(T, torch, dev, lambda: cl.check(L.b2clEnqueueCopyBufferRectEngine(
+        S.queue, src, dst, zero, zero, cl.sz3(region), srp, ssp, 0, 0, 0, None, None)), 5)
     res["c4_copy_rect_8GiB"] = {"GB/s_copied": S_bytes / ms / 1e6, "ms": ms,
-                                "hbm_frac": 2 * S_bytes / ms / 1e6 / hbm_peak}
+                                "hbm_frac": 2 * S_bytes / ms / 1e6 / hbm_peak, "kernel": cl.last_kernel(),
+                                "copy_engine_reference": {"call": "b2clEnqueueCopyBufferRectEngine (cudaMemcpy3DAsync)",
+                                                          "ms": ms_ce, "GB/s_copied": S_bytes / ms_ce / 1e6,
+                                                          "kernel_vs_engine": ms_ce / ms}}
     reg2 = (16384, 2048, 255)
     ms = _time_launches(T, torch, dev, lambda: cl.check(L.clEnqueueCopyBufferRect(
         S.queue, src, dst, cl.sz3((3, 0, 0)), zero, cl.sz3(reg2), 16387, 16387 * 2056, 0, 0, 0, None,
@@ -1146,6 +1151,11 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
             S.queue, dst, pat.ctypes.data, ps, 0, S_bytes, 0, None, None)), 5)
         fills.append({"pattern_bytes": ps, "GB/s": S_bytes / ms / 1e6, "ms": ms,
                       "hbm_frac": S_bytes / ms / 1e6 / hbm_peak})
+    pat4 = np.arange(4, dtype=np.uint8)
+    ms_ce = _time_launches(T, torch, dev, lambda: cl.check(L.b2clEnqueueFillBufferEngine(
+        S.queue, dst, pat4.ctypes.data, 4, 0, S_bytes, 0, None, None)), 5)
+    fills.append({"pattern_bytes": 4, "reference": "b2clEnqueueFillBufferEngine (cuMemsetD32Async)",
+                  "GB/s": S_bytes / ms_ce / 1e6, "ms": ms_ce, "hbm_frac": S_bytes / ms_ce / 1e6 / hbm_peak})
     res["c4_fill_8GiB"] = fills
     S.release(src)
     # CopyImageToBuffer sweep 4 KiB .. 8 GiB (RGBA32F 2D images shaped to the size)

@@ -256,6 +256,23 @@ cl_int b2clEnqueueCopyBufferEngine(cl_command_queue command_queue, cl_mem src_bu
                                    cl_mem dst_buffer, size_t src_offset, size_t dst_offset,
                                    size_t size, cl_uint num_events_in_wait_list,
                                    const cl_event* event_wait_list, cl_event* event);
+/* clEnqueueCopyBufferRect's semantics and validation ([CL1.2 §5.2.2]) on the
+ * copy engines (cudaMemcpy3DAsync when both slice pitches are whole rows,
+ * else cudaMemcpy2DAsync per slice): the SURVEY §8(d) config-4 reference. */
+cl_int b2clEnqueueCopyBufferRectEngine(cl_command_queue command_queue, cl_mem src_buffer,
+                                       cl_mem dst_buffer, const size_t* src_origin,
+                                       const size_t* dst_origin, const size_t* region,
+                                       size_t src_row_pitch, size_t src_slice_pitch,
+                                       size_t dst_row_pitch, size_t dst_slice_pitch,
+                                       cl_uint num_events_in_wait_list,
+                                       const cl_event* event_wait_list, cl_event* event);
+/* clEnqueueFillBuffer ([CL1.2 §5.2.3]) for pattern sizes 1, 2, 4 through
+ * cuMemsetD8/D16/D32Async (the config-4 fill reference); other pattern sizes
+ * -> CL_INVALID_VALUE. */
+cl_int b2clEnqueueFillBufferEngine(cl_command_queue command_queue, cl_mem buffer, const void* pattern,
+                                   size_t pattern_size, size_t offset, size_t size,
+                                   cl_uint num_events_in_wait_list, const cl_event* event_wait_list,
+                                   cl_event* event);
 
 /* Number of b2cl kernels launched by this process so far (bench evidence). */
 cl_ulong b2clGetKernelLaunchCount(void);

@@ -143,6 +143,9 @@ PROTOTYPES = {
     "b2clCreateBufferFromIpcHandle": (_H, [_H, _H, _P, _S, _PI]),
     "b2clCreateImageFromIpcHandle": (_H, [_H, _H, _L, _P, _P, _P, _PI]),
     "b2clEnqueueCopyBufferEngine": (_I, [_H, _H, _H, _S, _S, _S, _U, POINTER(_H), POINTER(_H)]),
+    "b2clEnqueueCopyBufferRectEngine": (_I, [_H, _H, _H, _SZ3, _SZ3, _SZ3, _S, _S, _S, _S, _U,
+                                             POINTER(_H), POINTER(_H)]),
+    "b2clEnqueueFillBufferEngine": (_I, [_H, _H, _P, _S, _S, _S, _U, POINTER(_H), POINTER(_H)]),
     "b2clGetKernelLaunchCount": (_L, []),
     "b2clGetLastKernelName": (ctypes.c_char_p, []),
     "b2clValidateCopyBufferRect": (_I, [_S, _S, _I, _SZ3, _SZ3, _SZ3, _S, _S, _S, _S]),

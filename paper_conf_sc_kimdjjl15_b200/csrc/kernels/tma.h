@@ -33,15 +33,26 @@ __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
 }
 
+#ifndef B2CL_MBAR_HINT
+#define B2CL_MBAR_HINT 0  // try_wait suspend-time hint in ns (0: the hardware default)
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   const uint32_t b = smem_u32(bar);
   uint32_t done;
   do {
+#if B2CL_MBAR_HINT
+    asm volatile(
+        "{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2, %3; selp.u32 %0, 1, 0, P; }"
+        : "=r"(done)
+        : "r"(b), "r"(parity), "r"(B2CL_MBAR_HINT)
+        : "memory");
+#else
     asm volatile(
         "{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2; selp.u32 %0, 1, 0, P; }"
         : "=r"(done)
         : "r"(b), "r"(parity)
         : "memory");
+#endif
   } while (!done);
 }
 

@@ -8,6 +8,7 @@
 // (2) makes the touched objects resident on the queue's device,
 // (3) waits for the wait-list events, (4) launches ONE kernel (or a copy
 // engine transfer for host memory), (5) returns an event if asked.
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <nvtx3/nvToolsExt.h>
 #include <stdio.h>
@@ -1542,8 +1543,29 @@ extern "C" cl_int clEnqueueWriteImage(cl_command_queue q, cl_mem img, cl_bool bl
 
 // ===================================================================== device rect copies / fills
 // One rect-copy kernel launch between two objects (already validated).
-// copy_engine: a 1D copy on the copy engines (cudaMemcpyAsync) instead of
-// the SM kernel -- the reference path b2clEnqueueCopyBufferEngine measures
+// The same box on the copy engines (the reference path of the
+// b2clEnqueue*Engine extensions): cudaMemcpyAsync for one row,
+// cudaMemcpy3DAsync when both slice pitches are whole rows, else one
+// cudaMemcpy2DAsync per slice.
+static cudaError_t engine_copy(const RectParams& p, cudaStream_t st) {
+  if (p.R1 == 1 && p.R2 == 1) return cudaMemcpyAsync(p.dst, p.src, p.R0, cudaMemcpyDeviceToDevice, st);
+  if (p.R2 == 1 || (p.ssp % p.srp == 0 && p.dsp % p.drp == 0)) {
+    cudaMemcpy3DParms m{};
+    m.srcPtr = make_cudaPitchedPtr(const_cast<char*>(p.src), p.srp, p.R0, p.R2 == 1 ? p.R1 : p.ssp / p.srp);
+    m.dstPtr = make_cudaPitchedPtr(p.dst, p.drp, p.R0, p.R2 == 1 ? p.R1 : p.dsp / p.drp);
+    m.extent = make_cudaExtent(p.R0, p.R1, p.R2);
+    m.kind = cudaMemcpyDeviceToDevice;
+    return cudaMemcpy3DAsync(&m, st);
+  }
+  cudaError_t e = cudaSuccess;
+  for (uint32_t z = 0; z < p.R2 && e == cudaSuccess; ++z)
+    e = cudaMemcpy2DAsync(p.dst + z * p.dsp, p.drp, p.src + z * p.ssp, p.srp, p.R0, p.R1, cudaMemcpyDeviceToDevice,
+                          st);
+  return e;
+}
+
+// copy_engine: the copy on the copy engines (engine_copy) instead of the SM
+// kernel -- the reference path b2clEnqueueCopyBuffer{,Rect}Engine measure
 static cl_int rect_copy(cl_command_queue q, cl_mem src, cl_mem dst, size_t soff, size_t doff,
                         const size_t* region_bytes, size_t srp, size_t ssp, size_t drp, size_t dsp,
                         cl_uint nw, const cl_event* wl, cl_event* ev, cl_command_type type,
@@ -1569,8 +1591,7 @@ static cl_int rect_copy(cl_command_queue q, cl_mem src, cl_mem dst, size_t soff,
   p.ssp = ssp;
   p.drp = drp;
   p.dsp = dsp;
-  cl_int st = enq_end(E, copy_engine ? cudaMemcpyAsync(p.dst, p.src, p.R0, cudaMemcpyDeviceToDevice, q->stream)
-                                      : launch_rect(p, RECT_COPY, q->stream));
+  cl_int st = enq_end(E, copy_engine ? engine_copy(p, q->stream) : launch_rect(p, RECT_COPY, q->stream));
   if (st == CL_SUCCESS) written_store(dst, dst_store);
   return st;
 }
@@ -2078,6 +2099,64 @@ extern "C" cl_int b2clEnqueueCopyBufferEngine(cl_command_queue q, cl_mem src, cl
   const size_t region[3] = {size, 1, 1};
   return rect_copy(q, src, dst, so, dso, region, size, size, size, size, nw, wl, ev, CL_COMMAND_COPY_BUFFER,
                    true);
+}
+
+extern "C" cl_int b2clEnqueueCopyBufferRectEngine(cl_command_queue q, cl_mem src, cl_mem dst, const size_t* so,
+                                                  const size_t* dso, const size_t* region, size_t srp, size_t ssp,
+                                                  size_t drp, size_t dsp, cl_uint nw, const cl_event* wl,
+                                                  cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_queue_mem(q, src));
+  CHECK(check_queue_mem(q, dst));
+  if (src->type != CL_MEM_OBJECT_BUFFER || dst->type != CL_MEM_OBJECT_BUFFER) return CL_INVALID_MEM_OBJECT;
+  CHECK(validate_copy_rect(src->size, dst->size, src == dst, so, dso, region, srp, ssp, drp, dsp));
+  if (region[1] > 0xffffffffull || region[2] > 0xffffffffull) return CL_INVALID_VALUE;
+  const size_t soff = so[2] * ssp + so[1] * srp + so[0];
+  const size_t doff = dso[2] * dsp + dso[1] * drp + dso[0];
+  return rect_copy(q, src, dst, soff, doff, region, srp, ssp, drp, dsp, nw, wl, ev, CL_COMMAND_COPY_BUFFER_RECT,
+                   true);
+}
+
+extern "C" cl_int b2clEnqueueFillBufferEngine(cl_command_queue q, cl_mem buf, const void* pattern, size_t ps,
+                                              size_t offset, size_t size, cl_uint nw, const cl_event* wl,
+                                              cl_event* ev) {
+  if (!live(g_queues, q)) return CL_INVALID_COMMAND_QUEUE;
+  CHECK(check_queue_mem(q, buf));
+  if (buf->type != CL_MEM_OBJECT_BUFFER) return CL_INVALID_MEM_OBJECT;
+  if (!pattern || (ps != 1 && ps != 2 && ps != 4)) return CL_INVALID_VALUE;  // cuMemsetD8/16/32
+  CHECK(validate_fill_buffer(buf->size, ps, offset, size));
+  CHECK(check_wait_list(q, nw, wl));
+  using memset_fn = CUresult (*)(CUdeviceptr, unsigned int, size_t, CUstream);
+  static memset_fn fns[3] = {nullptr, nullptr, nullptr};
+  static std::once_flag once;
+  std::call_once(once, [] {
+    const char* names[3] = {"cuMemsetD8Async", "cuMemsetD16Async", "cuMemsetD32Async"};
+    for (int i = 0; i < 3; ++i) {
+      void* f = nullptr;
+      cudaDriverEntryPointQueryResult r;
+      if (cudaGetDriverEntryPoint(names[i], &f, cudaEnableDefault, &r) == cudaSuccess &&
+          r == cudaDriverEntryPointSuccess)
+        fns[i] = reinterpret_cast<memset_fn>(f);
+    }
+  });
+  const int which = ps == 1 ? 0 : (ps == 2 ? 1 : 2);
+  if (!fns[which]) return CL_OUT_OF_RESOURCES;
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = CL_COMMAND_FILL_BUFFER;
+  DeviceGuard g(q->dev->ordinal);
+  char* d = nullptr;
+  Store* ds = nullptr;
+  CHECK(enq_begin(E, nw, wl));
+  CHECK_E(E, in_place(buf, q, true, &d, &ds));
+  unsigned int v = 0;
+  memcpy(&v, pattern, ps);
+  const CUresult r = fns[which](reinterpret_cast<CUdeviceptr>(d + offset), v, size / ps,
+                                reinterpret_cast<CUstream>(q->stream));
+  cl_int st = enq_end(E, r == CUDA_SUCCESS ? cudaSuccess : cudaErrorUnknown);
+  if (st == CL_SUCCESS) written_store(buf, ds);
+  return st;
 }
 
 // ===================================================================== programs and kernels

@@ -363,3 +363,31 @@ def test_config4_full_size_sampled(sess, orc):
         orc.fill_buffer(exp, pat.tobytes(), 0, 8192)
         assert np.array_equal(sess.read(dst, 8192, offset=off), exp), off
     sess.release(src, dst)
+
+
+def test_engine_reference_paths(sess, orc):
+    """b2clEnqueueCopyBufferRectEngine / FillBufferEngine (the copy-engine
+    references of config 4) give the oracle's bytes, like the SM kernels."""
+    L = cl.lib()
+    g = synth.rng(321)
+    for so, do, region, srp, ssp, drp, dsp in [synth.random_rect(g) for _ in range(6)] + [
+            ((0, 0, 0), (0, 0, 0), (64, 8, 3), 80, 80 * 9, 64, 64 * 8)]:
+        src = g.integers(0, 256, ssp * (so[2] + region[2]) + 64, dtype=np.uint8)
+        dst = g.integers(0, 256, dsp * (do[2] + region[2]) + 64, dtype=np.uint8)
+        sb, db = sess.buffer(src.nbytes, src), sess.buffer(dst.nbytes, dst)
+        cl.check(L.b2clEnqueueCopyBufferRectEngine(sess.queue, sb, db, cl.sz3(so), cl.sz3(do), cl.sz3(region),
+                                                   srp, ssp, drp, dsp, 0, None, None))
+        exp = dst.copy()
+        orc.copy_rect(src, exp, so, do, region, srp, ssp, drp, dsp)
+        assert np.array_equal(sess.read(db, dst.nbytes), exp)
+        sess.release(sb, db)
+    buf = np.zeros(4096, np.uint8)
+    b = sess.buffer(buf.nbytes, buf)
+    for ps in (1, 2, 4):
+        pat = g.integers(0, 256, ps, dtype=np.uint8)
+        cl.check(L.b2clEnqueueFillBufferEngine(sess.queue, b, pat.ctypes.data, ps, 8 * ps, 1000 * ps, 0, None, None))
+        orc.fill_buffer(buf, pat.tobytes(), 8 * ps, 1000 * ps)
+        assert np.array_equal(sess.read(b, buf.nbytes), buf)
+    pat = np.arange(8, dtype=np.uint8)
+    assert L.b2clEnqueueFillBufferEngine(sess.queue, b, pat.ctypes.data, 8, 0, 64, 0, None, None) == -30
+    sess.release(b)
