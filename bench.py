@@ -1063,6 +1063,21 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
                   "distinct_texels": texels})
         res[f"c2_map_b_{name}"] = e
         L.clReleaseSampler(smp2)
+    # the same rotated read from TILED storage (B2CL_MEM_TILED_IMAGE, 8 x 8-texel
+    # 1 KiB tiles; the one-thread-per-sample kernel), against that kernel on the
+    # pitched image: does block-linear storage help the rotated gathers?
+    imgt = S.image(cl.CL_RGBA, cl.CL_FLOAT, n2, n2, host=synth.image_codes(synth.rng(2), cl.CL_RGBA, cl.CL_FLOAT, n2, n2),
+                   flags=cl.CL_MEM_READ_WRITE | cl.B2CL_MEM_TILED_IMAGE)
+    smp2 = S.sampler(True, cl.CL_ADDRESS_REPEAT, cl.CL_FILTER_LINEAR)
+    ms_t = _time_launches(T, torch, dev, lambda: cl.check(L.b2clEnqueueReadImageGrid(
+        S.queue, imgt, smp2, 0, A2, d2, 4, out2, 0, 0, None, None)), 10)
+    kt = cl.last_kernel()
+    b2 = res["c2_map_b_repeat"]["algorithmic_bytes"]
+    res["c2_map_b_repeat_tiled_storage"] = {"Gsamples/s": n2 * n2 / ms_t / 1e6, "ms": ms_t, "kernel": kt,
+                                            "hbm_frac": b2 / ms_t / 1e6 / hbm_peak,
+                                            "storage": "B2CL_MEM_TILED_IMAGE (1 KiB tiles of 8 x 8 texels)"}
+    S.release(imgt)
+    L.clReleaseSampler(smp2)
     # config 5's image on one GPU (the N = 1 point of its row-sharded scaling):
     # 32768^2 RGBA32F, 16 GiB, map (A), both samplers.  Its rows are the
     # 4096-row seeded band above copied 8 times (device copies; the texel

@@ -36,6 +36,18 @@ typedef cl_uint b2cl_ctype;
  * b2clGetMemIpcHandle can export the object to another process. */
 #define B2CL_MEM_IPC_EXPORTABLE ((cl_mem_flags)1 << 40)
 
+/* custom cl_mem_flags bit for clCreateImage: TILED (block-linear) storage of a
+ * CL_MEM_OBJECT_IMAGE2D -- 1 KiB tiles of 8 rows x 128 bytes (128 / elem_size
+ * texels), tiles row-major (the north_star's "pitched and tiled image
+ * storage").  The layout is internal and invisible through the API: every
+ * pixel-box operation (Read/WriteImage, CopyImage with linear or tiled
+ * partners, CopyImageToBuffer / BufferToImage, FillImage), the read / write
+ * built-ins and translated kernels give the same texels as a pitched image;
+ * clGetImageInfo reports CL_IMAGE_ROW_PITCH = width * elem_size (reading A46).
+ * Any other image type, image shards, texture views and IPC import of a tiled
+ * image -> CL_INVALID_VALUE. */
+#define B2CL_MEM_TILED_IMAGE ((cl_mem_flags)1 << 41)
+
 /* read_image{f,i,ui}(image, sampler, coord) for n coordinates
  * ([CL1.2 §6.12.14.2, §8.1-8.3]; steps a3-a7).
  *  coords:  buffer holding n coordinates starting at coords_offset, packed

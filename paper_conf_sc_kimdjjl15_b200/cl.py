@@ -26,6 +26,7 @@ CL_QUEUE_PROFILING_ENABLE = 1 << 1
 CL_MEM_READ_WRITE, CL_MEM_WRITE_ONLY, CL_MEM_READ_ONLY = 1, 2, 4
 CL_MEM_USE_HOST_PTR, CL_MEM_ALLOC_HOST_PTR, CL_MEM_COPY_HOST_PTR = 8, 16, 32
 B2CL_MEM_IPC_EXPORTABLE = 1 << 40
+B2CL_MEM_TILED_IMAGE = 1 << 41
 CL_MEM_OBJECT_BUFFER, CL_MEM_OBJECT_IMAGE2D, CL_MEM_OBJECT_IMAGE3D = 0x10F0, 0x10F1, 0x10F2
 CL_MEM_OBJECT_IMAGE2D_ARRAY, CL_MEM_OBJECT_IMAGE1D = 0x10F3, 0x10F4
 CL_MEM_OBJECT_IMAGE1D_ARRAY, CL_MEM_OBJECT_IMAGE1D_BUFFER = 0x10F5, 0x10F6

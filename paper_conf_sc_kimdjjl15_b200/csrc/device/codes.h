@@ -39,6 +39,11 @@ struct Image {            // the CLImage of Fig. 6, device view
   // image has ob = 0 and os = its extent; a shard (b2clCreateImageShard)
   // stores its band plus halo rows of a larger global image.
   int ob, os;
+  // Tiled storage (B2CL_MEM_TILED_IMAGE, 2D images): 1 KiB tiles of 8 rows x
+  // 128 bytes (2^tshift texels); rp is then the bytes of one band of 8 rows
+  // (tiles_x KiB), and texel (i, j) lives at
+  //   ptr + (j >> 3) * rp + (i >> tshift) * 1024 + (j & 7) * 128 + (i & (2^tshift - 1)) * es.
+  int tiled, tshift;
 };
 
 struct Sampler {

@@ -201,8 +201,20 @@ __device__ __forceinline__ void map_order(int order, const uint32_t m[4], uint32
   }
 }
 
-// texel address (Fig. 6: ptr + k*slice_pitch + j*row_pitch + i*elem_size)
+// byte offset of column i inside a tiled row (see Image::tiled)
+__device__ __forceinline__ uint64_t tiled_col(const Image& im, int i) {
+  return ((uint64_t)((unsigned)i >> im.tshift) << 10) +
+         (uint64_t)((unsigned)i & ((1u << im.tshift) - 1u)) * (unsigned)im.es;
+}
+// start of texel row j of a tiled image (its 128-byte row inside the band)
+__device__ __forceinline__ const char* tiled_row(const Image& im, int j) {
+  return im.ptr + (uint64_t)((unsigned)j >> 3) * im.rp + (uint64_t)((unsigned)j & 7u) * 128u;
+}
+
+// texel address (Fig. 6: ptr + k*slice_pitch + j*row_pitch + i*elem_size;
+// tiled storage: the tile's address, see Image::tiled)
 __device__ __forceinline__ const char* texel_ptr(const Image& im, int i, int j, int k) {
+  if (im.tiled) return tiled_row(im, j) + tiled_col(im, i);
   return im.ptr + (uint64_t)(unsigned)k * im.sp + (uint64_t)(unsigned)j * im.rp +
          (uint64_t)(unsigned)i * (unsigned)im.es;
 }

@@ -19,6 +19,13 @@ struct Cfg {
   static constexpr int nch = ORDER == RT ? RT : order_channels(ORDER);
   static constexpr bool arr = false;   // image array (see Layered)
   static constexpr int cdims = DIMS;   // coordinates per sample
+  static constexpr bool tiled = false; // compile-time tiled storage (see TiledStore)
+};
+
+// C reading a TILED image (B2CL_MEM_TILED_IMAGE) with its format compiled in
+template <class C>
+struct TiledStore : C {
+  static constexpr bool tiled = true;
 };
 
 // C with the image-shard row mapping compiled in (SH) or out (plain images)
@@ -103,8 +110,20 @@ __device__ __forceinline__ int storage_row(const Image& im, int o, int extent) {
   return min(max(l, 0), im.os - 1);
 }
 
+// Tiled images (Image::tiled) reach only the run-time-format instances
+// (C::type == RT: the library's dispatch routes them there, and the device
+// header's built-ins are all run-time); the compile-time hot instances keep
+// the plain pitched addressing with no extra test.
+template <class C>
+__device__ __forceinline__ bool tiled_of(const Image& im) {
+  if constexpr (C::tiled) return true;
+  else if constexpr (C::type == RT) return im.tiled != 0;
+  else return false;
+}
+
 template <class C>
 __device__ __forceinline__ const char* row_ptr(const Image& im, int j, int k) {
+  if (tiled_of<C>(im)) return tiled_row(im, j);  // (2D only: k = 0)
   if constexpr (C::shard) {
     if (C::dims == 3) k = storage_row(im, k, im.d);
     else if (C::dims == 2) j = storage_row(im, j, im.h);
@@ -144,7 +163,7 @@ __device__ __forceinline__ void fetch(const Image& im, const char* row, int i, b
   const int es = elem_size<C>(im);
   m[0] = m[1] = m[2] = m[3] = 0u;
   if (!ok) return;
-  Raw r = load_raw(row + (uint64_t)(unsigned)i * (unsigned)es, es);
+  Raw r = load_raw(row + (tiled_of<C>(im) ? tiled_col(im, i) : (uint64_t)(unsigned)i * (unsigned)es), es);
   if (is_packed(type)) {  // normalized only (read_imagef)
     unpack_rgb(r.w[0], type, m);
     // CL_RGBx: the in-range alpha 1 is carried as a channel, so that a border

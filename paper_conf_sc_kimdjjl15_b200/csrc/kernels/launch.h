@@ -49,6 +49,28 @@ struct WriteParams {
 
 enum RectMode : int { RECT_COPY = 0, RECT_FILL = 1, RECT_FILL_IMAGE = 2, RECT_COPY_ALIGNED = 3 };
 
+// Texel-addressed box copy / fill for TILED images (B2CL_MEM_TILED_IMAGE):
+// each side is pitched-linear or tiled (dev::Image::tiled); one thread per
+// texel moves es bytes (or writes the fill colour converted with the
+// write_image rules).  Used for every pixel-box operation that touches a
+// tiled image: Copy{Image,ImageToBuffer,BufferToImage}, FillImage, the
+// host transfers (through a linear staging buffer) and the upload at creation.
+struct TexSide {
+  char* ptr;        // texel (0,0,0) of the box (linear) or the image base (tiled)
+  uint64_t rp, sp;  // linear: row / slice pitch; tiled: rp = bytes of a band of 8 rows
+  int tiled, tshift;
+  int ox, oy;       // tiled: the box origin (texels, rows)
+};
+struct TexCopyParams {
+  TexSide src, dst;
+  uint32_t w, h, d;     // box (texels)
+  int es;               // element size
+  int fill;             // 1: write the colour below instead of copying
+  uint32_t color[4];
+  int type, order;      // fill: the format (dev::TypeCode, OrderCode)
+};
+cudaError_t launch_texcopy(const TexCopyParams& p, cudaStream_t stream);
+
 // Each launcher enqueues exactly one kernel (or none for empty work) on
 // `stream` and returns the launch status.
 cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t stream);

@@ -17,6 +17,7 @@
 // (bulk-async staging through shared memory, below).  Sources are always
 // local to the launching device except for migration, whose source and
 // destination offsets are both 0 (the aligned instance).
+#include <algorithm>
 #include <atomic>
 
 #include "../device/image.cuh"
@@ -364,6 +365,41 @@ cudaError_t launch_rect(RectParams& p, int mode, cudaStream_t st) {
                : mode == RECT_COPY       ? "k_rect<COPY>"
                : mode == RECT_FILL       ? "k_rect<FILL>"
                                          : "k_rect<FILL_IMAGE>");
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------- tiled images
+__device__ __forceinline__ char* tex_addr(const TexSide& s, uint32_t x, uint32_t y, uint32_t z, int es) {
+  if (s.tiled) {
+    const uint32_t i = (uint32_t)s.ox + x, j = (uint32_t)s.oy + y;
+    return s.ptr + (uint64_t)(j >> 3) * s.rp + ((uint64_t)(i >> s.tshift) << 10) + (uint64_t)(j & 7u) * 128u +
+           (uint64_t)(i & ((1u << s.tshift) - 1u)) * (unsigned)es;
+  }
+  return s.ptr + (uint64_t)z * s.sp + (uint64_t)y * s.rp + (uint64_t)x * (unsigned)es;
+}
+
+__global__ void __launch_bounds__(256) k_texcopy(const TexCopyParams p) {
+  const uint64_t n = (uint64_t)p.w * p.h * p.d;
+  Raw fill;
+  if (p.fill) fill = encode_texel(p.color, p.type, p.order);  // (A23: converted once per thread)
+  for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < n; t += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t x = (uint32_t)(t % p.w), y = (uint32_t)((t / p.w) % p.h), z = (uint32_t)(t / ((uint64_t)p.w * p.h));
+    char* d = tex_addr(p.dst, x, y, z, p.es);
+    if (p.fill) {
+      store_raw(d, p.es, fill);
+    } else {
+      const char* s = tex_addr(p.src, x, y, z, p.es);
+      store_raw(d, p.es, load_raw(s, p.es));
+    }
+  }
+}
+
+cudaError_t launch_texcopy(const TexCopyParams& p, cudaStream_t st) {
+  const uint64_t n = (uint64_t)p.w * p.h * p.d;
+  if (n == 0) return cudaSuccess;
+  const uint64_t blocks = std::min<uint64_t>((n + 255) / 256, 148ull * 16);
+  k_texcopy<<<(unsigned)blocks, 256, 0, st>>>(p);
+  count_launch(p.fill ? "k_texcopy<FILL>" : "k_texcopy");
   return cudaGetLastError();
 }
 

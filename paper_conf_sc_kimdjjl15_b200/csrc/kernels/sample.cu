@@ -1077,6 +1077,17 @@ static bool separable(const SampleParams& p) {
 }
 
 cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st) {
+  if (p.im.tiled) {  // tiled storage (2D): the one-thread-per-sample kernels with tiled addressing
+    if (coord_mode == COORD_GRID) {
+      if ((uint64_t)p.ow * p.oh * p.od == 0) return cudaSuccess;
+      if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_REPEAT, F_LINEAR))
+        return go_grid<TiledStore<C2Repeat>, 4>(p, st);
+      if (p.outc == 4 && matches<2>(p, T_FLOAT, O_RGBA, 1, A_MIRROR, F_LINEAR))
+        return go_grid<TiledStore<C2Mirror>, 4>(p, st);
+      return go_grid<Generic<2>, RT>(p, st);
+    }
+    return p.n == 0 ? cudaSuccess : go_list<Generic<2>>(p, coord_mode == COORD_LIST_I, st);
+  }
   if (coord_mode == COORD_GRID) {
     if ((uint64_t)p.ow * p.oh * p.od == 0) return cudaSuccess;
     // B2CL_GRID_KERNEL=general|sep|walk|4|tile forces a kernel family (A/B runs under ncu);

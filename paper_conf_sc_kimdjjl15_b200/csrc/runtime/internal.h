@@ -33,7 +33,13 @@ struct ImageLayout {
   int arrayed;  // 1 for CL_MEM_OBJECT_IMAGE1D_ARRAY / IMAGE2D_ARRAY
   size_t w, h, d;
   size_t row_pitch, slice_pitch, bytes;
+  // tiled storage (B2CL_MEM_TILED_IMAGE): 1 KiB tiles of 8 rows x 128 B;
+  // row_pitch is then the bytes of one band of 8 rows, slice_pitch the total
+  int tiled = 0, tshift = 0;
 };
+
+// turn a 2D image layout into the tiled one (false: not a tileable image)
+bool tile_layout(ImageLayout* L);
 
 int type_code(cl_channel_type t);
 int order_code(cl_channel_order o);

@@ -17,6 +17,7 @@
 
 #include <algorithm>
 #include <atomic>
+#include <functional>
 #include <mutex>
 #include <new>
 #include <set>
@@ -610,7 +611,7 @@ static cl_int check_mem_flags(cl_mem_flags flags, void* host_ptr) {
   const cl_mem_flags known = CL_MEM_READ_WRITE | CL_MEM_WRITE_ONLY | CL_MEM_READ_ONLY |
                              CL_MEM_USE_HOST_PTR | CL_MEM_ALLOC_HOST_PTR | CL_MEM_COPY_HOST_PTR |
                              CL_MEM_HOST_WRITE_ONLY | CL_MEM_HOST_READ_ONLY |
-                             CL_MEM_HOST_NO_ACCESS | B2CL_MEM_IPC_EXPORTABLE;
+                             CL_MEM_HOST_NO_ACCESS | B2CL_MEM_IPC_EXPORTABLE | B2CL_MEM_TILED_IMAGE;
   if (flags & ~known) return CL_INVALID_VALUE;
   if (flags & CL_MEM_USE_HOST_PTR) return CL_INVALID_VALUE;  // reading A33
   const bool copy = flags & CL_MEM_COPY_HOST_PTR;
@@ -643,6 +644,7 @@ extern "C" cl_mem clCreateBuffer(cl_context c, cl_mem_flags flags, size_t size, 
   if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
   cl_int st = check_mem_flags(flags, host_ptr);
   if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
+  if (flags & B2CL_MEM_TILED_IMAGE) { SET_ERR(CL_INVALID_VALUE); return nullptr; }  // images only
   if (size == 0) { SET_ERR(CL_INVALID_BUFFER_SIZE); return nullptr; }
   cl_mem m = new_mem(c, CL_MEM_OBJECT_BUFFER, flags, size);
   if (!m) { SET_ERR(CL_OUT_OF_HOST_MEMORY); return nullptr; }
@@ -716,9 +718,12 @@ extern "C" cl_mem clCreateImage(cl_context c, cl_mem_flags flags, const cl_image
   ImageLayout L;
   cl_int st = image_layout(fmt, desc, &L);
   if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
+  if (flags & B2CL_MEM_TILED_IMAGE) {  // tiled storage: 2D images only
+    if (desc->image_type != CL_MEM_OBJECT_IMAGE2D || !tile_layout(&L)) { SET_ERR(CL_INVALID_VALUE); return nullptr; }
+  }
   if (desc->image_type == CL_MEM_OBJECT_IMAGE1D_BUFFER)
     return image_from_buffer(c, flags, fmt, desc, L, host_ptr, errcode_ret);
-  st = check_mem_flags(flags & ~B2CL_MEM_IPC_EXPORTABLE, host_ptr);
+  st = check_mem_flags(flags & ~(B2CL_MEM_IPC_EXPORTABLE | B2CL_MEM_TILED_IMAGE), host_ptr);
   if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
   // host pitches ([CL1.2 §5.3.1]): nonzero only with a host pointer, >= tight,
   // multiple of the element size.  Slice pitch: 3D images and 2D arrays
@@ -747,7 +752,31 @@ extern "C" cl_mem clCreateImage(cl_context c, cl_mem_flags flags, const cl_image
   Store* s = nullptr;
   st = ensure_store(m, ord, nullptr, &s);
   if (st != CL_SUCCESS) { delete m; SET_ERR(st); return nullptr; }
-  if (host_ptr) {  // clCreateImage uploads the contents
+  if (host_ptr && L.tiled) {  // through a linear staging copy, then tiled on the device
+    DeviceGuard g(ord);
+    void* stg = nullptr;
+    cudaError_t e = cudaMalloc(&stg, L.w * L.fmt.es * L.h);
+    if (e == cudaSuccess)
+      e = cudaMemcpy2D(stg, L.w * L.fmt.es, host_ptr, hrp, L.w * L.fmt.es, L.h, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) {
+      TexCopyParams tp{};
+      tp.src.ptr = static_cast<char*>(stg);
+      tp.src.rp = L.w * L.fmt.es;
+      tp.src.sp = tp.src.rp * L.h;
+      tp.dst.ptr = s->ptr;
+      tp.dst.rp = L.row_pitch;
+      tp.dst.tiled = 1;
+      tp.dst.tshift = L.tshift;
+      tp.w = (uint32_t)L.w;
+      tp.h = (uint32_t)L.h;
+      tp.d = 1;
+      tp.es = (int)L.fmt.es;
+      e = launch_texcopy(tp, nullptr);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(nullptr);
+    }
+    if (stg) cudaFree(stg);
+    if (e != cudaSuccess) { raw_free(*s); delete m; SET_ERR(cuda_err(e)); return nullptr; }
+  } else if (host_ptr) {  // clCreateImage uploads the contents
     DeviceGuard g(ord);
     for (size_t k = 0; k < L.d; ++k) {
       cudaError_t e = cudaMemcpy2D(s->ptr + k * L.slice_pitch, L.row_pitch,
@@ -768,6 +797,7 @@ extern "C" cl_mem b2clCreateImageShard(cl_context c, cl_mem_flags flags, const c
                                        cl_int* errcode_ret) {
   if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
   if (!global_desc) { SET_ERR(CL_INVALID_IMAGE_DESCRIPTOR); return nullptr; }
+  if (flags & B2CL_MEM_TILED_IMAGE) { SET_ERR(CL_INVALID_VALUE); return nullptr; }  // shards are pitched
   ImageLayout G;
   cl_int st = image_layout(fmt, global_desc, &G);
   if (st != CL_SUCCESS) { SET_ERR(st); return nullptr; }
@@ -887,7 +917,8 @@ extern "C" cl_int clGetImageInfo(cl_mem m, cl_image_info name, size_t size, void
   switch (name) {
     case CL_IMAGE_FORMAT: return get_info<cl_image_format>(m->fmt, size, value, size_ret);
     case CL_IMAGE_ELEMENT_SIZE: return get_info<size_t>(L.fmt.es, size, value, size_ret);
-    case CL_IMAGE_ROW_PITCH: return get_info<size_t>(L.row_pitch, size, value, size_ret);
+    case CL_IMAGE_ROW_PITCH:  // (tiled storage: the pitch of its linear view, reading A46)
+      return get_info<size_t>(L.tiled ? L.w * L.fmt.es : L.row_pitch, size, value, size_ret);
     case CL_IMAGE_SLICE_PITCH: {
       // 3D: bytes per slice; arrays: bytes per layer; 1D, 1D buffer and 2D: 0
       const size_t sp = (L.dims == 3) ? L.slice_pitch : (L.arrayed ? L.row_pitch : 0);
@@ -1296,7 +1327,7 @@ extern "C" cl_int b2clCreateTextureObject(cl_context c, const b2cl_resource_desc
   cl_mem_object_type vtype = 0;
   cl_uint sdims = 1;  // sampled axes
   if (rd->res_type == B2CL_RESOURCE_ARRAY) {
-    if (!is_image(src) || src->shard || src->type == CL_MEM_OBJECT_IMAGE1D_BUFFER)
+    if (!is_image(src) || src->shard || src->type == CL_MEM_OBJECT_IMAGE1D_BUFFER || src->img.tiled)
       return CL_INVALID_MEM_OBJECT;
     stored = src->fmt;
     L = src->img;
@@ -1391,12 +1422,116 @@ static dev::Image dev_image(cl_mem m, char* ptr, bool sampling = false) {
   im.sp = L.slice_pitch;
   im.ob = 0;
   im.os = L.dims == 3 ? im.d : im.h;
+  im.tiled = L.tiled;
+  im.tshift = L.tshift;
   if (sampling && m->shard) {
     im.ob = (int)m->shard_ob;
     if (L.dims == 3) im.d = (int)m->shard_extent;
     else im.h = (int)m->shard_extent;
   }
   return im;
+}
+
+// ===================================================================== tiled images
+// A pixel box of an image as one side of k_texcopy (the box origin `o`, texels).
+static TexSide image_side(cl_mem m, char* base, const size_t* o) {
+  const ImageLayout& L = m->img;
+  TexSide t{};
+  t.rp = L.row_pitch;
+  t.sp = L.slice_pitch;
+  if (L.tiled) {
+    t.ptr = base;
+    t.tiled = 1;
+    t.tshift = L.tshift;
+    t.ox = (int)o[0];
+    t.oy = (int)o[1];
+  } else {
+    t.ptr = base + o[2] * L.slice_pitch + o[1] * L.row_pitch + o[0] * L.fmt.es;
+  }
+  return t;
+}
+
+static TexSide linear_side(char* p, size_t rp, size_t sp) {
+  TexSide t{};
+  t.ptr = p;
+  t.rp = rp;
+  t.sp = sp;
+  return t;
+}
+
+// One k_texcopy between memory objects (at least one a tiled image): the
+// wait list, then the objects addressed in place (A44), then the kernel.
+// `build` fills the parameters from the resolved base pointers.
+static cl_int tex_enqueue(cl_command_queue q, cl_mem src, cl_mem dst,
+                          const std::function<void(char*, char*, TexCopyParams&)>& build, cl_uint nw,
+                          const cl_event* wl, cl_event* ev, cl_command_type type) {
+  CHECK(check_wait_list(q, nw, wl));
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = type;
+  DeviceGuard g(q->dev->ordinal);
+  char *s = nullptr, *d = nullptr;
+  Store* ds = nullptr;
+  CHECK(enq_begin(E, nw, wl));
+  if (src) CHECK_E(E, in_place(src, q, false, &s, nullptr));
+  CHECK_E(E, in_place(dst, q, true, &d, &ds));
+  TexCopyParams p{};
+  build(s, d, p);
+  const cl_int st = enq_end(E, launch_texcopy(p, q->stream));
+  if (st == CL_SUCCESS) written_store(dst, ds);
+  return st;
+}
+
+// Read/WriteImage of a tiled image: the host rows go through a linear
+// staging buffer on the queue's stream (stream-ordered allocation), tiled or
+// untiled on the device by k_texcopy.
+static cl_int tiled_image_host(cl_command_queue q, cl_mem img, cl_bool blocking, const size_t* origin,
+                               const size_t* region, size_t hrp, size_t hsp, char* ptr, bool write, cl_uint nw,
+                               const cl_event* wl, cl_event* ev) {
+  CHECK(check_wait_list(q, nw, wl));
+  const ImageLayout& L = img->img;
+  const size_t es = L.fmt.es, row = region[0] * es, bytes = row * region[1] * region[2];
+  Enq E;
+  E.q = q;
+  E.evout = ev;
+  E.type = write ? CL_COMMAND_WRITE_IMAGE : CL_COMMAND_READ_IMAGE;
+  DeviceGuard g(q->dev->ordinal);
+  CHECK(enq_begin(E, nw, wl));
+  char* d = nullptr;
+  Store* ds = nullptr;
+  CHECK_E(E, write ? in_place(img, q, true, &d, &ds) : resident(img, q, true, &d));
+  void* stg = nullptr;
+  cudaError_t e = cudaMallocAsync(&stg, bytes, q->stream);
+  if (e != cudaSuccess) return enq_fail(E, cuda_err(e));
+  TexCopyParams p{};
+  p.w = (uint32_t)region[0];
+  p.h = (uint32_t)region[1];
+  p.d = (uint32_t)region[2];
+  p.es = (int)es;
+  const TexSide lin = linear_side(static_cast<char*>(stg), row, row * region[1]);
+  const TexSide im = image_side(img, d, origin);
+  if (write) {
+    for (size_t k = 0; k < region[2] && e == cudaSuccess; ++k)
+      e = cudaMemcpy2DAsync(static_cast<char*>(stg) + k * row * region[1], row, ptr + k * hsp, hrp, row, region[1],
+                            cudaMemcpyHostToDevice, q->stream);
+    p.src = lin;
+    p.dst = im;
+    if (e == cudaSuccess) e = launch_texcopy(p, q->stream);
+  } else {
+    p.src = im;
+    p.dst = lin;
+    e = launch_texcopy(p, q->stream);
+    for (size_t k = 0; k < region[2] && e == cudaSuccess; ++k)
+      e = cudaMemcpy2DAsync(ptr + k * hsp, hrp, static_cast<char*>(stg) + k * row * region[1], row, row, region[1],
+                            cudaMemcpyDeviceToHost, q->stream);
+  }
+  cudaFreeAsync(stg, q->stream);
+  cl_int st = enq_end(E, e);
+  if (st != CL_SUCCESS) return st;
+  if (write) written_store(img, ds);
+  if (blocking) return cuda_err(cudaStreamSynchronize(q->stream));
+  return CL_SUCCESS;
 }
 
 // ===================================================================== host <-> device transfers
@@ -1508,6 +1643,7 @@ static cl_int image_host(cl_command_queue q, cl_mem img, cl_bool blocking, const
     if (sp == 0) sp = rp * region[1];
     else if (sp < rp * region[1]) return CL_INVALID_VALUE;
   }
+  if (L.tiled) return tiled_image_host(q, img, blocking, origin, region, rp, sp, ptr, write, nw, wl, ev);
   CHECK(check_wait_list(q, nw, wl));
   Enq E;
   E.q = q;
@@ -1680,6 +1816,14 @@ extern "C" cl_int clEnqueueCopyImage(cl_command_queue q, cl_mem src, cl_mem dst,
   CHECK(validate_image_box(A.dims, A.w, A.h, A.d, so, region));
   CHECK(validate_image_box(B.dims, B.w, B.h, B.d, dso, region));
   if (src == dst && image_boxes_overlap(so, dso, region)) return CL_MEM_COPY_OVERLAP;
+  if (A.tiled || B.tiled) {
+    return tex_enqueue(q, src, dst, [&](char* s, char* d, TexCopyParams& p) {
+      p.src = image_side(src, s, so);
+      p.dst = image_side(dst, d, dso);
+      p.w = (uint32_t)region[0]; p.h = (uint32_t)region[1]; p.d = (uint32_t)region[2];
+      p.es = (int)A.fmt.es;
+    }, nw, wl, ev, CL_COMMAND_COPY_IMAGE);
+  }
   const size_t es = A.fmt.es;
   const size_t soff = so[2] * A.slice_pitch + so[1] * A.row_pitch + so[0] * es;
   const size_t doff = dso[2] * B.slice_pitch + dso[1] * B.row_pitch + dso[0] * es;
@@ -1700,6 +1844,14 @@ extern "C" cl_int clEnqueueCopyImageToBuffer(cl_command_queue q, cl_mem src, cl_
   const size_t es = A.fmt.es, row = region[0] * es;
   const size_t bytes = row * region[1] * region[2];
   if (doff > dst->size || bytes > dst->size - doff) return CL_INVALID_VALUE;
+  if (A.tiled) {
+    return tex_enqueue(q, src, dst, [&](char* s, char* d, TexCopyParams& p) {
+      p.src = image_side(src, s, so);
+      p.dst = linear_side(d + doff, row, row * region[1]);
+      p.w = (uint32_t)region[0]; p.h = (uint32_t)region[1]; p.d = (uint32_t)region[2];
+      p.es = (int)es;
+    }, nw, wl, ev, CL_COMMAND_COPY_IMAGE_TO_BUFFER);
+  }
   const size_t soff = so[2] * A.slice_pitch + so[1] * A.row_pitch + so[0] * es;
   const size_t rb[3] = {row, region[1], region[2]};
   return rect_copy(q, src, dst, soff, doff, rb, A.row_pitch, A.slice_pitch, row, row * region[1],
@@ -1718,6 +1870,14 @@ extern "C" cl_int clEnqueueCopyBufferToImage(cl_command_queue q, cl_mem src, cl_
   const size_t es = B.fmt.es, row = region[0] * es;
   const size_t bytes = row * region[1] * region[2];
   if (soff > src->size || bytes > src->size - soff) return CL_INVALID_VALUE;
+  if (B.tiled) {
+    return tex_enqueue(q, src, dst, [&](char* s, char* d, TexCopyParams& p) {
+      p.src = linear_side(s + soff, row, row * region[1]);
+      p.dst = image_side(dst, d, dso);
+      p.w = (uint32_t)region[0]; p.h = (uint32_t)region[1]; p.d = (uint32_t)region[2];
+      p.es = (int)es;
+    }, nw, wl, ev, CL_COMMAND_COPY_BUFFER_TO_IMAGE);
+  }
   const size_t doff = dso[2] * B.slice_pitch + dso[1] * B.row_pitch + dso[0] * es;
   const size_t rb[3] = {row, region[1], region[2]};
   return rect_copy(q, src, dst, soff, doff, rb, row, row * region[1], B.row_pitch, B.slice_pitch,
@@ -1732,6 +1892,17 @@ extern "C" cl_int clEnqueueFillImage(cl_command_queue q, cl_mem img, const void*
   if (!color) return CL_INVALID_VALUE;
   const ImageLayout& L = img->img;
   CHECK(validate_image_box(L.dims, L.w, L.h, L.d, origin, region));
+  if (L.tiled) {
+    return tex_enqueue(q, nullptr, img, [&](char*, char* d, TexCopyParams& p) {
+      p.dst = image_side(img, d, origin);
+      p.w = (uint32_t)region[0]; p.h = (uint32_t)region[1]; p.d = (uint32_t)region[2];
+      p.es = (int)L.fmt.es;
+      p.fill = 1;
+      memcpy(p.color, color, 16);
+      p.type = L.fmt.type;
+      p.order = L.fmt.order;
+    }, nw, wl, ev, CL_COMMAND_FILL_IMAGE);
+  }
   CHECK(check_wait_list(q, nw, wl));
   Enq E;
   E.q = q;
@@ -2045,7 +2216,7 @@ extern "C" cl_mem b2clCreateImageFromIpcHandle(cl_context c, cl_device_id d, cl_
                                                const void* handle64, cl_int* errcode_ret) {
   if (!live(g_contexts, c)) { SET_ERR(CL_INVALID_CONTEXT); return nullptr; }
   if (!valid_device(d) || !ctx_has_device(c, d)) { SET_ERR(CL_INVALID_DEVICE); return nullptr; }
-  if (!handle64 || (flags & (CL_MEM_USE_HOST_PTR | CL_MEM_COPY_HOST_PTR | CL_MEM_ALLOC_HOST_PTR))) {
+  if (!handle64 || (flags & (CL_MEM_USE_HOST_PTR | CL_MEM_COPY_HOST_PTR | CL_MEM_ALLOC_HOST_PTR | B2CL_MEM_TILED_IMAGE))) {
     SET_ERR(CL_INVALID_VALUE);
     return nullptr;
   }

@@ -141,6 +141,19 @@ cl_int image_layout(const cl_image_format* fmt, const cl_image_desc* desc, Image
   return CL_SUCCESS;
 }
 
+bool tile_layout(ImageLayout* L) {
+  if (L->dims != 2 || L->arrayed || L->fmt.es == 0 || L->fmt.es > 128 || (L->fmt.es & (L->fmt.es - 1))) return false;
+  int sh = 0;
+  while ((size_t)(1u << sh) * L->fmt.es < 128) ++sh;  // 2^sh texels per 128-byte tile row
+  const size_t tiles_x = (L->w + (1u << sh) - 1) >> sh, bands = (L->h + 7) / 8;
+  L->tiled = 1;
+  L->tshift = sh;
+  L->row_pitch = tiles_x * 1024;  // one band of 8 rows
+  L->slice_pitch = L->row_pitch * bands;
+  L->bytes = L->slice_pitch;
+  return true;
+}
+
 // ---- rect copies ----
 static bool rect_pitches(const size_t* region, size_t& rp, size_t& sp) {
   // pitch 0 -> defaults; a given pitch must be >= the default and the slice

@@ -32,8 +32,10 @@ def main():
     S = cl.Session(0, stream=st.cuda_stream)
     L = cl.lib()
     n = 4096
+    tiled = "--tiled" in sys.argv  # B2CL_MEM_TILED_IMAGE storage
     img = S.image(cl.CL_RGBA, cl.CL_FLOAT, n, n,
-                  host=synth.image_codes(synth.rng(2), cl.CL_RGBA, cl.CL_FLOAT, n, n))
+                  host=synth.image_codes(synth.rng(2), cl.CL_RGBA, cl.CL_FLOAT, n, n),
+                  flags=cl.CL_MEM_READ_WRITE | (cl.B2CL_MEM_TILED_IMAGE if tiled else 0))
     out = S.buffer(n * n * 16)
     A = (ctypes.c_float * 12)(*synth.affine_rotate_2d(n, n, 30.0).tolist())
     d = cl.sz3((n, n, 1))
@@ -43,7 +45,7 @@ def main():
         res.append(timed(st, lambda: cl.check(L.b2clEnqueueReadImageGrid(S.queue, img, smp, 0, A, d, 4, out, 0, 0,
                                                                            None, None))))
     S.release(img, out)
-    print(f"{os.path.basename(os.environ.get('B2CL_LIB', 'libb2cl.so'))} "
+    print(f"{os.path.basename(os.environ.get('B2CL_LIB', 'libb2cl.so'))}{' tiled' if tiled else ''} "
           f"[{os.environ.get('B2CL_GRID_KERNEL', 'default')}]: C2 map B REPEAT {res[0]:.1f} us, "
           f"MIRRORED {res[1]:.1f} us ({n * n / res[0] / 1e3:.0f} / {n * n / res[1] / 1e3:.0f} Gsamples/s)")
 
