@@ -363,10 +363,70 @@ def c2_codes():
     return synth.image_codes(g, cl.CL_RGBA, cl.CL_FLOAT, N2D, N2D, 1)
 
 
+def run_reference_c5(args, world):
+    """The reference arm at N > 1: the oracle on a bounded sample of output rows
+    of the GPU arm's workload, C5 (a 32768^2 RGBA32F image, map (A), REPEAT +
+    MIRRORED).  The oracle image is a lazily zero-filled 16 GiB array in which
+    only the texel rows the sampled output rows tap are written (row j = the
+    seeded block row j mod 256, as on the GPU), so host memory holds only those."""
+    import oracle as orc
+    from paper_conf_sc_kimdjjl15_b200 import synth
+    threads = os.cpu_count() or 1
+    H = W = args.c5_size
+    data = np.zeros((H, W, 4), np.float32)  # calloc'd: untouched pages stay unmapped
+    block = synth.image_rows(0x10B5, 0x10DE, W, range(256))[0]
+    img = orc.Image(data, W, H, 1, dims=2, order=orc.RGBA, type=orc.FLOAT)
+    A = synth.affine_translate_2d(W, H)
+    filled = set()
+
+    def rows_for(y0, n):
+        for mname in ("repeat", "mirrored"):
+            for j in _axis_taps(A[5], A[7], n, H, mname, start=y0):
+                if int(j) not in filled:
+                    data[int(j)] = block[int(j) % 256]
+                    filled.add(int(j))
+
+    def run(y0, n):
+        rows_for(y0, n)
+        for a in (orc.ADDRESS_REPEAT, orc.ADDRESS_MIRRORED_REPEAT):
+            orc.read_grid(img, True, a, orc.FILTER_LINEAR, orc.RT_F, A, (W, H, 1), 4, yrange=(y0, y0 + n),
+                          nthreads=threads)
+    t0 = time.perf_counter()
+    run(0, 2)
+    per_row = (time.perf_counter() - t0) / 2
+    budget = 60.0 / max(1, args.steps + args.warmup)
+    rows = int(max(1, min(H // 2, budget / max(per_row, 1e-6))))
+
+    def step(i):
+        run((i * 4099) % (H - rows), rows)
+    for i in range(args.warmup):
+        step(i)
+    t0 = time.perf_counter()
+    for i in range(args.steps):
+        step(args.warmup + i)
+    dt = (time.perf_counter() - t0) / args.steps
+    value = 2 * rows * W / dt / 1e9
+    sample = (f"{rows} output rows x {W} columns of each pass (REPEAT, MIRRORED) per step, from the {W}x{H} "
+              f"image (only the tapped texel rows materialised)")
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "Gsamples/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": dt * 1e3, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic (seed 20151115 rows, 256-row period)",
+            "config": {"workload": C5_WORKLOAD, "sample": sample},
+            "cpu_baseline": {"value": value, "unit": "Gsamples/s", "cores": threads, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": value, "unit": "Gsamples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world > 1:  # the GPU arm's N > 1 workload is config 5
+        return run_reference_c5(args, world)
     threads = os.cpu_count() or 1
     codes = c2_codes()
     total_budget = 60.0
