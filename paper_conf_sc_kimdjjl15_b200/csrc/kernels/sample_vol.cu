@@ -546,7 +546,13 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
 #define B2CL_VOLR_LEAN 0  // 1: the interior-tile slice with precomputed offsets and paired blends (measured 247.9 vs 240.9 us)
 #endif
 constexpr int VOLR_S = B2CL_VOLR_S;           // samples (rows) per consumer thread
-constexpr int RT_W = 64, RT_H = 4 * VOLR_S;   // output tile (256 consumer threads: 64 columns x 4 row groups)
+#ifndef B2CL_VOLR_TW
+#define B2CL_VOLR_TW 64
+#endif
+#ifndef B2CL_VOLR_BW32
+#define B2CL_VOLR_BW32 0  // 1: round the box row up to a multiple of 32 texels (bank group = column)
+#endif
+constexpr int RT_W = B2CL_VOLR_TW, RT_H = (256 / RT_W) * VOLR_S;  // output tile (256 consumer threads)
 constexpr int RB_MAXW = 128, RB_MAXH = 128;   // largest staged box (texels)
 constexpr int VOLR_NS = B2CL_VOLR_NS;
 constexpr int VOLR_THREADS = 288;             // 8 consumer warps + 1 producer warp
@@ -585,6 +591,64 @@ __device__ __forceinline__ VolrBox volr_box(const SampleParams& p, const VolrGeo
   return b;
 }
 
+#ifndef B2CL_VOLR_ROWS
+#define B2CL_VOLR_ROWS 0  // 1: stage only each box row's tapped segment (one cp.async.bulk per row: 41 % fewer bytes, but ~190-byte copies: 849.5 vs 236.5 us); 0: the whole box (TMA)
+#endif
+
+// Columns [c0, c1) (box coordinates, multiples of 4 texels) of the taps in
+// box row r (texel row yb + r) of a tile: the taps of a texel row j come from
+// the samples with floor(t_v) in {j-1, j}, i.e. t_v in [j-1, j+1); the tile's
+// sample coordinates (t = u - 1/2, texel units) lie in the parallelogram of
+// its four corners' coordinates, so the row's taps lie between the x-extremes
+// of that parallelogram clipped to the slab, widened by 2 texels each side
+// (floor, the i0 + 1 tap, fp rounding).  Every operation is an explicitly
+// rounded intrinsic (never contracted), so the producer warp and the consumer
+// warps compute identical ranges; the consumers still check every tap against
+// them, so the ranges only decide speed, never results.
+__device__ __forceinline__ int volr_row_seg(const float cu[4], const float cv[4], int row, int xb, int bw, int nw) {
+  const float lo = __int2float_rn(row - 1), hi = __int2float_rn(row + 1);
+  float xmin = 3.0e38f, xmax = -3.0e38f;
+  const int ea[4] = {0, 1, 3, 2}, eb[4] = {1, 3, 2, 0};  // the parallelogram's edges
+#pragma unroll
+  for (int e = 0; e < 4; ++e) {
+    const float xa = cu[ea[e]], va = cv[ea[e]], xe = cu[eb[e]], ve = cv[eb[e]];
+    float t0 = 0.f, t1 = 1.f;
+    const float dv = __fsub_rn(ve, va);
+    if (dv == 0.f) {
+      if (!(va >= lo && va <= hi)) continue;
+    } else {
+      float ta = __fdiv_rn(__fsub_rn(lo, va), dv), tb = __fdiv_rn(__fsub_rn(hi, va), dv);
+      if (ta > tb) { const float t = ta; ta = tb; tb = t; }
+      t0 = fmaxf(t0, ta);
+      t1 = fminf(t1, tb);
+      if (!(t0 <= t1)) continue;
+    }
+    const float dx = __fsub_rn(xe, xa);
+    const float x0 = __fadd_rn(xa, __fmul_rn(t0, dx)), x1 = __fadd_rn(xa, __fmul_rn(t1, dx));
+    xmin = fminf(xmin, fminf(x0, x1));
+    xmax = fmaxf(xmax, fmaxf(x0, x1));
+  }
+  if (!(xmin <= xmax)) return 0;  // no tap in this row
+  int c0 = max(__float2int_rd(xmin) - 2, 0) - xb, c1 = min(__float2int_rd(xmax) + 3, nw) - xb;
+  c0 = max(c0, 0) & ~3;
+  c1 = min((c1 + 3) & ~3, bw);
+  return c1 > c0 ? (c0 | c1 << 16) : 0;
+}
+
+// the tile's corner coordinates in texel units (t = u - 1/2; normalized maps scaled by the extent)
+template <class C>
+__device__ __forceinline__ void volr_corners(const SampleParams& p, int x0, int y0, int z, float cu[4], float cv[4]) {
+  const int x1 = min(x0 + RT_W, p.ow) - 1, y1 = min(y0 + RT_H, p.oh) - 1;
+  const float fw = p.smp.norm ? __int2float_rn(p.im.w) : 1.0f, fh = p.smp.norm ? __int2float_rn(p.im.h) : 1.0f;
+  const float zf = __int2float_rn(p.oz + z);
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    const float xf = __int2float_rn(p.ox + ((c & 1) ? x1 : x0)), yf = __int2float_rn(p.oy + ((c & 2) ? y1 : y0));
+    cu[c] = __fsub_rn(__fmul_rn(affine_coord(p.A, xf, yf, zf), fw), 0.5f);
+    cv[c] = __fsub_rn(__fmul_rn(affine_coord(p.A + 4, xf, yf, zf), fh), 0.5f);
+  }
+}
+
 template <class C>
 __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
     k_sample_grid_volr(const SampleParams p, const VolTiles tl, const VolrGeom g,
@@ -592,6 +656,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
   static_assert(C::dims == 3 && C::nch == 1 && C::type == T_FLOAT && C::addr == A_CTE, "R32F, CLAMP_TO_EDGE");
   extern __shared__ __align__(128) unsigned char volr_buf[];
   __shared__ uint64_t full[VOLR_NS], empty[VOLR_NS];
+  __shared__ int segtab[RB_MAXH];  // the consumers' copy of the current tile's row segments
   const Image& im = p.im;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -612,7 +677,26 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
       const VolSeg q = vol_seg(p, tl, t);
       const VolrBox bx = volr_box<C>(p, g, q.tx * RT_W, q.ty * RT_H, q.w0, lane);
-      if (!bx.ok || lane != 0) continue;  // (not ok: the consumers read this tile directly)
+      if (!bx.ok) continue;  // (not ok: the consumers read this tile directly)
+#if B2CL_VOLR_ROWS
+      // this lane's box rows (lane, lane + 32, ...: at most 4) and their segments
+      int seg[RB_MAXH / 32];
+      uint32_t txb = 0;
+      {
+        float cu[4], cv[4];
+        volr_corners<C>(p, q.tx * RT_W, q.ty * RT_H, q.w0, cu, cv);
+#pragma unroll
+        for (int m = 0; m < RB_MAXH / 32; ++m) {
+          const int r = lane + 32 * m;
+          seg[m] = (r < g.bh && bx.yb + r < im.h) ? volr_row_seg(cu, cv, bx.yb + r, bx.xb, g.bw, im.w) : 0;
+          txb += (uint32_t)((seg[m] >> 16) - (seg[m] & 0xffff)) * 4u;
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) txb += __shfl_xor_sync(0xffffffffu, txb, o);
+      }
+#else
+      if (lane != 0) continue;
+#endif
       int kA = NONE, kB = NONE;
       for (int w = 0; w < q.nst; ++w) {
         const AxL az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
@@ -623,6 +707,24 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
           if (!(h ? need1 : need0)) continue;
           const int k = h ? az.i1 : az.i0;
           const uint32_t fb = vol_smem(&full[s]);
+#if B2CL_VOLR_ROWS
+          if (lane == 0) {
+            vol_wait(&empty[s], ph ^ 1u);
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(txb) : "memory");
+          }
+          __syncwarp();
+#pragma unroll
+          for (int m = 0; m < RB_MAXH / 32; ++m) {
+            const int c0 = seg[m] & 0xffff, c1 = seg[m] >> 16, r = lane + 32 * m;
+            if (c1 > c0)
+              asm volatile(
+                  "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                      vol_smem(volr_buf + s * g.stride + ((uint32_t)r * g.bw + c0) * 4u)),
+                  "l"(im.ptr + (uint64_t)k * im.sp + (uint64_t)(bx.yb + r) * im.rp + (uint64_t)(bx.xb + c0) * 4u),
+                  "r"((uint32_t)(c1 - c0) * 4u), "r"(fb)
+                  : "memory");
+          }
+#else
           vol_wait(&empty[s], ph ^ 1u);
           asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(g.bw * g.bh * 4)
                        : "memory");
@@ -631,6 +733,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
               " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(vol_smem(volr_buf + s * g.stride)),
               "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(bx.xb), "r"(bx.yb), "r"(k), "r"(fb)
               : "memory");
+#endif
 #if B2CL_VOLR_PF
           // warm L2 with the same box B2CL_VOLR_PF slices ahead: its first-touch
           // texels come from DRAM while this slice is blended
@@ -663,14 +766,30 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
     int in = bx.ok;
     const float xf = __int2float_rn(p.ox + x), zf = __int2float_rn(p.oz + q.w0);
 #pragma unroll
+#if B2CL_VOLR_ROWS
+    // the staged columns of each box row (computed as the producer does)
+    if (bx.ok) {
+      float cu[4], cv[4];
+      volr_corners<C>(p, q.tx * RT_W, q.ty * RT_H, q.w0, cu, cv);
+      for (int r = threadIdx.x; r < g.bh; r += 256)
+        segtab[r] = bx.yb + r < im.h ? volr_row_seg(cu, cv, bx.yb + r, bx.xb, g.bw, im.w) : 0;
+    }
+    asm volatile("bar.sync 1, 256;" ::: "memory");
+#endif
     for (int r = 0; r < VOLR_S; ++r) {
       const float yf = __int2float_rn(p.oy + y0 + r);
       const AxL ax = axis_l<C>(p.smp, affine_coord(p.A, xf, yf, zf), im.w);
       const AxL ay = axis_l<C>(p.smp, affine_coord(p.A + 4, xf, yf, zf), im.h);
       const int sx0 = ax.i0 - bx.xb, sx1 = ax.i1 - bx.xb, sy0 = ay.i0 - bx.yb, sy1 = ay.i1 - bx.yb;
       const bool v = x < p.ow && y0 + r < p.oh;
-      const bool ok = sx0 >= 0 && sx1 >= sx0 && sx1 - sx0 <= 1 && sx1 < g.bw && sy0 >= 0 && sy1 >= sy0 &&
-                      sy1 - sy0 <= 1 && sy1 < g.bh;
+      bool ok = sx0 >= 0 && sx1 >= sx0 && sx1 - sx0 <= 1 && sx1 < g.bw && sy0 >= 0 && sy1 >= sy0 &&
+                sy1 - sy0 <= 1 && sy1 < g.bh;
+#if B2CL_VOLR_ROWS
+      if (ok) {  // both tap columns inside the staged segment of both tap rows
+        const int s0 = segtab[sy0], s1 = segtab[sy1];
+        ok = sx0 >= (s0 & 0xffff) && sx1 < (s0 >> 16) && sx0 >= (s1 & 0xffff) && sx1 < (s1 >> 16);
+      }
+#endif
       in = in && (ok || !v);
       off[r] = ok ? (sy0 * g.bw + sx0) | (sx1 - sx0) << 16 | (sy1 - sy0) << 17 : 0;
       wa[r] = ax.a;
@@ -945,6 +1064,7 @@ static cudaError_t go_volr(const SampleParams& p, cudaStream_t st, bool* used) {
   if (!(fw < RB_MAXW && fh < RB_MAXH)) return cudaSuccess;
   VolrGeom g;
   g.bw = std::min(RB_MAXW, ((int)std::ceil(fw) + 1 + 2 + 3 + 3) & ~3);
+  if (B2CL_VOLR_BW32) g.bw = std::min(RB_MAXW, (g.bw + 31) & ~31);
   g.bh = std::min(RB_MAXH, (int)std::ceil(fh) + 1 + 2);
   g.stride = (g.bw * g.bh * 4 + 127) & ~127;
   auto enc = encode_fn();
