@@ -1090,10 +1090,15 @@ cudaError_t launch_sample(const SampleParams& p, int coord_mode, cudaStream_t st
   }
   if (coord_mode == COORD_GRID) {
     if ((uint64_t)p.ow * p.oh * p.od == 0) return cudaSuccess;
-    // B2CL_GRID_KERNEL=general|sep|walk|4|tile forces a kernel family (A/B runs under ncu);
+    // B2CL_GRID_KERNEL=general|sep|walk|4|tile|box forces a kernel family (A/B runs under ncu);
     // the default picks the variant measured fastest on B200 for each hot config
     static const char* force = getenv("B2CL_GRID_KERNEL");
-    const int fk = !force ? 0 : (force[0] == 'g' ? 1 : (force[0] == 's' ? 2 : (force[0] == 'w' ? 3 : (force[0] == '4' ? 4 : (force[0] == 't' ? 5 : 0)))));
+    const int fk = !force ? 0 : (force[0] == 'g' ? 1 : (force[0] == 's' ? 2 : (force[0] == 'w' ? 3 : (force[0] == '4' ? 4 : (force[0] == 't' ? 5 : (force[0] == 'b' ? 6 : 0))))));
+    if (fk == 6 && !is_shard(p)) {  // b: the footprint-box kernel for any map it accepts
+      bool used = false;
+      const cudaError_t e = launch_sample_box(p, st, &used);
+      if (used || e != cudaSuccess) return e;
+    }
     if (p.arr)  // image arrays: the general kernel, fully run-time format and sampler
       return p.dims == 1 ? go_grid<Layered<Generic<1>>, RT>(p, st) : go_grid<Layered<Generic<2>>, RT>(p, st);
     if (separable(p) && fk != 1) {
