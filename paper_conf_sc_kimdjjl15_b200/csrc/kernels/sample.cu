@@ -609,6 +609,9 @@ __device__ __forceinline__ int fold_prim(int pi, int M, int A) { return pi < A ?
 #ifndef B2CL_FOLD_MINB
 #define B2CL_FOLD_MINB 1
 #endif
+#ifndef B2CL_FOLD_PAIRED
+#define B2CL_FOLD_PAIRED 0  // 1: the blends on channel pairs (FFMA2 / FMUL2): measured 70.6 vs 62.0 us
+#endif
 #ifndef B2CL_FOLD_CTAS
 #define B2CL_FOLD_CTAS 0  // persistent CTAs per SM for the fold kernel (0: one CTA per tile)
 #endif
@@ -796,6 +799,25 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB)
     // columns read slot 0 and store nothing)
     const uint32_t o0 = x >= 0 ? (uint32_t)(i0 - c0) * 16u : 0u, o1 = x >= 0 ? (uint32_t)(i1 - c0) * 16u : 0u;
     const char* bbase = reinterpret_cast<const char*>(&box[0][0]);
+#if B2CL_FOLD_PAIRED
+    // lerp1 on channel pairs (x, y) and (z, w): FMUL2 + FFMA2, each lane the
+    // same IEEE mul / fma as lerp1 (a mul feeding an fma's addend: nothing fuses)
+    const float2 a2 = make_float2(a, a), oma2 = make_float2(oma, oma);
+    auto xblend = [&](int j, float4& h) {
+      const char* row = bbase + (uint32_t)(j - r0) * (BW * 16);
+      const float4 t0 = *reinterpret_cast<const float4*>(row + o0);
+      const float4 t1 = *reinterpret_cast<const float4*>(row + o1);
+      const float2 lo = __ffma2_rn(a2, make_float2(t1.x, t1.y), __fmul2_rn(oma2, make_float2(t0.x, t0.y)));
+      const float2 hi = __ffma2_rn(a2, make_float2(t1.z, t1.w), __fmul2_rn(oma2, make_float2(t0.z, t0.w)));
+      h = make_float4(lo.x, lo.y, hi.x, hi.y);
+    };
+    auto emit = [&](int y, const float4& ry, const float4& n0, const float4& n1) {
+      const float2 b2 = make_float2(ry.x, ry.x), omb2 = make_float2(ry.y, ry.y);
+      const float2 lo = __ffma2_rn(b2, make_float2(n1.x, n1.y), __fmul2_rn(omb2, make_float2(n0.x, n0.y)));
+      const float2 hi = __ffma2_rn(b2, make_float2(n1.z, n1.w), __fmul2_rn(omb2, make_float2(n0.z, n0.w)));
+      if (x >= 0) __stcs(out + ((uint64_t)y * p.ow + x), make_float4(lo.x, lo.y, hi.x, hi.y));
+    };
+#else
     auto xblend = [&](int j, float4& h) {
       const char* row = bbase + (uint32_t)(j - r0) * (BW * 16);
       const float4 t0 = *reinterpret_cast<const float4*>(row + o0);
@@ -808,6 +830,7 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB)
         __stcs(out + ((uint64_t)y * p.ow + x), make_float4(lerp1(ry.x, ry.y, n0.x, n1.x), lerp1(ry.x, ry.y, n0.y, n1.y),
                                                            lerp1(ry.x, ry.y, n0.z, n1.z), lerp1(ry.x, ry.y, n0.w, n1.w)));
     };
+#endif
     // the warp's 8 rows of this row set: all present and chained one way
     // (j1 of a row = j0 of the next: UP; j0 = j1 of the next: DOWN), so each
     // texel row is x-blended once; otherwise both taps per row
