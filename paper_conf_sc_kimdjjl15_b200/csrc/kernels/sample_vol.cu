@@ -56,6 +56,9 @@ using namespace dev;
 #ifndef B2CL_VOL_NS
 #define B2CL_VOL_NS 3
 #endif
+#ifndef B2CL_VOL_SETUP
+#define B2CL_VOL_SETUP 0.0  // the stencil kernel's chunk cost for vol_plan (0: balanced rounds)
+#endif
 #ifndef B2CL_VOL_MIN_STEPS
 #define B2CL_VOL_MIN_STEPS 8
 #endif
@@ -536,6 +539,9 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
 #ifndef B2CL_VOLR_NS
 #define B2CL_VOLR_NS 4
 #endif
+#ifndef B2CL_VOLR_SETUP
+#define B2CL_VOLR_SETUP 2.0  // a z chunk's fixed cost in steps (vol_plan; fitted: walks of 14 / 16 / 32 at 236.9 / 231.7 / 219.2 us)
+#endif
 #ifndef B2CL_VOLR_MINB
 #define B2CL_VOLR_MINB 2
 #endif
@@ -726,6 +732,9 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
           }
 #else
           vol_wait(&empty[s], ph ^ 1u);
+#ifdef B2CL_VOLR_NOTMA  // A/B experiment only (wrong results): the ring without the box copies
+          asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(fb) : "memory");
+#else
           asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(g.bw * g.bh * 4)
                        : "memory");
           asm volatile(
@@ -733,6 +742,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
               " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(vol_smem(volr_buf + s * g.stride)),
               "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(bx.xb), "r"(bx.yb), "r"(k), "r"(fb)
               : "memory");
+#endif
 #endif
 #if B2CL_VOLR_PF
           // warm L2 with the same box B2CL_VOLR_PF slices ahead: its first-touch
@@ -991,10 +1001,13 @@ static bool vol_tensor_map(const Image& im, CUtensorMap* m) {
 }
 
 // Persistent-grid plan shared by the staged kernels: one CTA per resident
-// slot; z chunks: a multiple of G / gcd(G, tiles per plane) so the tiles
-// split evenly over the CTAs, each chunk at least VOL_MIN_STEPS slices long.
+// slot.  setup == 0: z chunks a multiple of G / gcd(G, tiles per plane) so the
+// tiles split evenly over the CTAs, each chunk at least VOL_MIN_STEPS slices
+// long.  setup > 0: the chunk count minimising (rounds of G tiles) x (walk +
+// setup), setup = a chunk's fixed cost (its per-tile coordinates and first
+// slice) in units of one step -- longer walks at a small imbalance.
 static bool vol_plan(const SampleParams& p, int tw, int th, const void* fn, int threads, size_t smem, int* occ,
-                     VolTiles* tl, int* grid) {
+                     VolTiles* tl, int* grid, double setup = 0.0) {
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 64) return false;
@@ -1018,6 +1031,15 @@ static bool vol_plan(const SampleParams& p, int tw, int th, const void* fn, int 
   long long nzc = unit;
   while (nzc * 2 <= p.od / VOL_MIN_STEPS && nzc * 2 <= 4 * unit) nzc *= 2;
   if ((p.od + nzc - 1) / nzc < VOL_MIN_STEPS) nzc = std::max<long long>(1, p.od / VOL_MIN_STEPS);
+  if (setup > 0.0) {
+    double best = 1e300;
+    for (long long walk = 1; walk <= p.od; ++walk) {
+      const long long n = (p.od + walk - 1) / walk;
+      if ((p.od + n - 1) / n != walk) continue;  // (each n once, with its shortest walk)
+      const double cost = (double)((plane * n + G - 1) / G) * ((double)walk + setup);
+      if (cost < best) { best = cost; nzc = n; }
+    }
+  }
   tl->walk = (int)((p.od + nzc - 1) / nzc);
   tl->nzc = (p.od + tl->walk - 1) / tl->walk;
   *grid = (int)std::max<long long>(1, std::min<long long>(G, plane * tl->nzc));
@@ -1042,7 +1064,7 @@ static cudaError_t go_vol(const SampleParams& p, cudaStream_t st, bool* used) {
   VolTiles tl;
   int grid = 0;
   if (!vol_plan(p, VT_W, VT_H, reinterpret_cast<const void*>(k_sample_grid_vol<C>), VOL_THREADS, smem, occ, &tl,
-                &grid))
+                &grid, B2CL_VOL_SETUP))
     return cudaSuccess;
   k_sample_grid_vol<C><<<grid, VOL_THREADS, smem, st>>>(p, tl, tm);
   count_launch("k_sample_grid_vol");
@@ -1086,7 +1108,7 @@ static cudaError_t go_volr(const SampleParams& p, cudaStream_t st, bool* used) {
   VolTiles tl;
   int grid = 0;
   if (!vol_plan(p, RT_W, RT_H, reinterpret_cast<const void*>(k_sample_grid_volr<C>), VOLR_THREADS, smem, occ, &tl,
-                &grid))
+                &grid, B2CL_VOLR_SETUP))
     return cudaSuccess;
   k_sample_grid_volr<C><<<grid, VOLR_THREADS, smem, st>>>(p, tl, g, tm);
   count_launch("k_sample_grid_volr");
