@@ -289,6 +289,97 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
   // --------------------------------------------------------------- consumers
   int s = 0;
   uint32_t ph = 0;
+#if B2CL_VOLR_INWARP
+  // Warp 0 also stages the slices: a cursor over the producer's copy order
+  // above (the same tiles, steps and need rules), advanced before each of
+  // warp 0's own waits -- blocking until the slice it waits for is issued,
+  // then as far as NS slices ahead while their ring stages are free.
+  int ct = blockIdx.x, cw = 0, chh = 0, ckA = NONE, ckB = NONE, cw0 = 0, cnst = 0, cxb = 0, cyb = 0, cok = 0;
+  int ci0 = 0, ci1 = 0, cazw = -1;  // the z taps of step cw (cached)
+  int cs = 0, cn = 0, consumed = 0;
+  uint32_t cph = 0;
+  auto cur_tile = [&]() {
+    const VolSeg q = vol_seg(p, tl, ct);
+    const VolrBox bx = volr_box<C>(p, g, q.tx * RT_W, q.ty * RT_H, q.w0, lane);
+    cw = 0;
+    chh = 0;
+    ckA = ckB = NONE;
+    cw0 = q.w0;
+    cnst = q.nst;
+    cxb = bx.xb;
+    cyb = bx.yb;
+    cok = bx.ok;
+    cazw = -1;
+  };
+  if (warp == 0 && ct < ntiles) cur_tile();
+  auto cur_next = [&](int& k) -> bool {
+    for (;;) {
+      if (ct >= ntiles) return false;
+      if (!cok || cw >= cnst) {
+        ct += gridDim.x;
+        if (ct < ntiles) cur_tile();
+        continue;
+      }
+      if (cazw != cw) {
+        const AxL az = vol_axis<C>(p, 10, p.oz, cw0 + cw, im.d);
+        ci0 = az.i0;
+        ci1 = az.i1;
+        cazw = cw;
+      }
+      const bool need0 = !(ci0 == ckA || ci0 == ckB);
+      if (chh == 0) {
+        chh = 1;
+        if (need0) { k = ci0; return true; }
+      }
+      const bool need1 = !(ci1 == ci0 || (!need0 && ci1 == ckB));
+      chh = 0;
+      ckA = ci0;
+      ckB = ci1;
+      ++cw;
+      if (need1) { k = ci1; return true; }
+    }
+  };
+  auto cur_issue = [&](bool block) -> bool {
+    if (!block) {
+      uint32_t ready = 0;
+      if (lane == 0)
+        asm volatile(
+            "{ .reg .pred P; mbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2; selp.u32 %0, 1, 0, P; }"
+            : "=r"(ready)
+            : "r"(vol_smem(&empty[cs])), "r"(cph ^ 1u)
+            : "memory");
+      if (!__shfl_sync(0xffffffffu, ready, 0)) return false;
+    }
+    int k = 0;
+    if (!cur_next(k)) return false;
+    if (lane == 0) {
+      if (block) vol_wait(&empty[cs], cph ^ 1u);
+      const uint32_t fb = vol_smem(&full[cs]);
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(g.bw * g.bh * 4)
+                   : "memory");
+      asm volatile(
+          "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+          " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(vol_smem(volr_buf + cs * g.stride)),
+          "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(cxb), "r"(cyb), "r"(k), "r"(fb)
+          : "memory");
+    }
+    if (++cs == VOLR_NS) { cs = 0; cph ^= 1u; }
+    ++cn;
+    return true;
+  };
+  auto acquire = [&]() {
+    if (warp == 0) {
+      while (cn <= consumed && cur_issue(true)) {
+      }
+      while (cn < consumed + VOLR_NS && cur_issue(false)) {
+      }
+      ++consumed;
+    }
+    vol_wait(&full[s], ph);
+  };
+#else
+  auto acquire = [&]() { vol_wait(&full[s], ph); };
+#endif
   for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
     const VolSeg q = vol_seg(p, tl, t);
     const int xt = q.tx * VT_W, yt = q.ty * VT_H;
@@ -548,6 +639,15 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
 #ifndef B2CL_VOLR_S
 #define B2CL_VOLR_S 8
 #endif
+#ifndef B2CL_VOLR_NOHOIST
+#define B2CL_VOLR_NOHOIST 1  // 1: 1 - w recomputed per slice, not held in 16 registers (fewer spills: 200.5 vs 215.5 us)
+#endif
+#ifndef B2CL_VOLR_FUSED
+#define B2CL_VOLR_FUSED 1  // 1: runs of common steps hold one slice (fused blend + store)
+#endif
+#ifndef B2CL_VOLR_EIDX
+#define B2CL_VOLR_EIDX 0  // 1: the output address recomputed per step from z (no 64-bit row pointer and stride held)
+#endif
 #ifndef B2CL_VOLR_LEAN
 #define B2CL_VOLR_LEAN 0  // 1: the interior-tile slice with precomputed offsets and paired blends (measured 247.9 vs 240.9 us)
 #endif
@@ -561,7 +661,10 @@ constexpr int VOLR_S = B2CL_VOLR_S;           // samples (rows) per consumer thr
 constexpr int RT_W = B2CL_VOLR_TW, RT_H = (256 / RT_W) * VOLR_S;  // output tile (256 consumer threads)
 constexpr int RB_MAXW = 128, RB_MAXH = 128;   // largest staged box (texels)
 constexpr int VOLR_NS = B2CL_VOLR_NS;
-constexpr int VOLR_THREADS = 288;             // 8 consumer warps + 1 producer warp
+#ifndef B2CL_VOLR_INWARP
+#define B2CL_VOLR_INWARP 0  // 1: consumer warp 0 also issues the copies (256 threads: 128 registers, no spill; measured 255.4 vs 216.4 us: warp 0 becomes the straggler); 0: a 9th producer warp (96 registers, a small spill)
+#endif
+constexpr int VOLR_THREADS = B2CL_VOLR_INWARP ? 256 : 288;  // 8 consumer warps (+ 1 producer warp)
 
 struct VolrBox {
   int xb, yb;    // first staged texel column (16-B aligned) and row
@@ -677,7 +780,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
   const int ntiles = tl.ntx * tl.nty * tl.nzc;
   constexpr int NONE = -2147483647 - 1;
 
-  if (warp == 8) {  // ------------------------------------------------ producer
+  if (!B2CL_VOLR_INWARP && warp == 8) {  // --------------------------- producer
     int s = 0;
     uint32_t ph = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
@@ -765,6 +868,97 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
   // --------------------------------------------------------------- consumers
   int s = 0;
   uint32_t ph = 0;
+#if B2CL_VOLR_INWARP
+  // Warp 0 also stages the slices: a cursor over the producer's copy order
+  // above (the same tiles, steps and need rules), advanced before each of
+  // warp 0's own waits -- blocking until the slice it waits for is issued,
+  // then as far as NS slices ahead while their ring stages are free.
+  int ct = blockIdx.x, cw = 0, chh = 0, ckA = NONE, ckB = NONE, cw0 = 0, cnst = 0, cxb = 0, cyb = 0, cok = 0;
+  int ci0 = 0, ci1 = 0, cazw = -1;  // the z taps of step cw (cached)
+  int cs = 0, cn = 0, consumed = 0;
+  uint32_t cph = 0;
+  auto cur_tile = [&]() {
+    const VolSeg q = vol_seg(p, tl, ct);
+    const VolrBox bx = volr_box<C>(p, g, q.tx * RT_W, q.ty * RT_H, q.w0, lane);
+    cw = 0;
+    chh = 0;
+    ckA = ckB = NONE;
+    cw0 = q.w0;
+    cnst = q.nst;
+    cxb = bx.xb;
+    cyb = bx.yb;
+    cok = bx.ok;
+    cazw = -1;
+  };
+  if (warp == 0 && ct < ntiles) cur_tile();
+  auto cur_next = [&](int& k) -> bool {
+    for (;;) {
+      if (ct >= ntiles) return false;
+      if (!cok || cw >= cnst) {
+        ct += gridDim.x;
+        if (ct < ntiles) cur_tile();
+        continue;
+      }
+      if (cazw != cw) {
+        const AxL az = vol_axis<C>(p, 10, p.oz, cw0 + cw, im.d);
+        ci0 = az.i0;
+        ci1 = az.i1;
+        cazw = cw;
+      }
+      const bool need0 = !(ci0 == ckA || ci0 == ckB);
+      if (chh == 0) {
+        chh = 1;
+        if (need0) { k = ci0; return true; }
+      }
+      const bool need1 = !(ci1 == ci0 || (!need0 && ci1 == ckB));
+      chh = 0;
+      ckA = ci0;
+      ckB = ci1;
+      ++cw;
+      if (need1) { k = ci1; return true; }
+    }
+  };
+  auto cur_issue = [&](bool block) -> bool {
+    if (!block) {
+      uint32_t ready = 0;
+      if (lane == 0)
+        asm volatile(
+            "{ .reg .pred P; mbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2; selp.u32 %0, 1, 0, P; }"
+            : "=r"(ready)
+            : "r"(vol_smem(&empty[cs])), "r"(cph ^ 1u)
+            : "memory");
+      if (!__shfl_sync(0xffffffffu, ready, 0)) return false;
+    }
+    int k = 0;
+    if (!cur_next(k)) return false;
+    if (lane == 0) {
+      if (block) vol_wait(&empty[cs], cph ^ 1u);
+      const uint32_t fb = vol_smem(&full[cs]);
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(g.bw * g.bh * 4)
+                   : "memory");
+      asm volatile(
+          "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+          " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(vol_smem(volr_buf + cs * g.stride)),
+          "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(cxb), "r"(cyb), "r"(k), "r"(fb)
+          : "memory");
+    }
+    if (++cs == VOLR_NS) { cs = 0; cph ^= 1u; }
+    ++cn;
+    return true;
+  };
+  auto acquire = [&]() {
+    if (warp == 0) {
+      while (cn <= consumed && cur_issue(true)) {
+      }
+      while (cn < consumed + VOLR_NS && cur_issue(false)) {
+      }
+      ++consumed;
+    }
+    vol_wait(&full[s], ph);
+  };
+#else
+  auto acquire = [&]() { vol_wait(&full[s], ph); };
+#endif
   const int col = threadIdx.x & (RT_W - 1), rg = threadIdx.x / RT_W;  // column, row group of VOLR_S
   for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
     const VolSeg q = vol_seg(p, tl, t);
@@ -820,7 +1014,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
           const bool need0 = !(az.i0 == kA || az.i0 == kB);
           const bool need1 = !(az.i1 == az.i0 || (!need0 && az.i1 == kB));
           for (int h = 0; h < (int)need0 + (int)need1; ++h) {
-            vol_wait(&full[s], ph);
+            acquire();
             __syncwarp();
             if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(vol_smem(&empty[s])) : "memory");
             if (++s == VOLR_NS) { s = 0; ph ^= 1u; }
@@ -871,8 +1065,29 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
     float oma[1], omb[1];
     const uint32_t rowb = 0;
 #endif
+    // sample r's (x, y)-blend of one staged slice
+    auto tap_blend = [&](const float* buf, int r) -> float {
+      const float* t0 = buf + (off[r] & 0xffff);
+      const int dx = off[r] >> 16 & 1, dy = (off[r] >> 17) * g.bw;
+#if B2CL_VOLR_NOHOIST
+      // 1 - w recomputed per slice (volatile: not hoisted into 16 live registers)
+      float oma1, omb1;
+      asm volatile("sub.rn.f32 %0, 0f3F800000, %1;" : "=f"(oma1) : "f"(wa[r]));
+      asm volatile("sub.rn.f32 %0, 0f3F800000, %1;" : "=f"(omb1) : "f"(wb[r]));
+#else
+      const float oma1 = __fsub_rn(1.0f, wa[r]), omb1 = __fsub_rn(1.0f, wb[r]);
+#endif
+      const float h0 = lerp1(wa[r], oma1, t0[0], t0[dx]);
+      const float h1 = lerp1(wa[r], oma1, t0[dy], t0[dy + dx]);
+      return lerp1(wb[r], omb1, h0, h1);
+    };
+    auto release = [&]() {
+      __syncwarp();
+      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(vol_smem(&empty[s])) : "memory");
+      if (++s == VOLR_NS) { s = 0; ph ^= 1u; }
+    };
     auto slice = [&](float V[VOLR_S]) {
-      vol_wait(&full[s], ph);
+      acquire();
       if (interior) {
         const char* buf = reinterpret_cast<const char*>(volr_buf + s * g.stride);
 #pragma unroll
@@ -888,25 +1103,25 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
       } else {
         const float* buf = reinterpret_cast<const float*>(volr_buf + s * g.stride);
 #pragma unroll
-        for (int r = 0; r < VOLR_S; ++r) {
-          const float* t0 = buf + (off[r] & 0xffff);
-          const int dx = off[r] >> 16 & 1, dy = (off[r] >> 17) * g.bw;
-          const float oma1 = __fsub_rn(1.0f, wa[r]), omb1 = __fsub_rn(1.0f, wb[r]);
-          const float h0 = lerp1(wa[r], oma1, t0[0], t0[dx]);
-          const float h1 = lerp1(wa[r], oma1, t0[dy], t0[dy + dx]);
-          V[r] = lerp1(wb[r], omb1, h0, h1);
-        }
+        for (int r = 0; r < VOLR_S; ++r) V[r] = tap_blend(buf, r);
       }
-      __syncwarp();
-      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(vol_smem(&empty[s])) : "memory");
-      if (++s == VOLR_NS) { s = 0; ph ^= 1u; }
+      release();
     };
+#if B2CL_VOLR_EIDX
+    const uint32_t po = (uint32_t)y0 * (uint32_t)p.ow + (uint32_t)x;  // (y0, x) in the output plane
+    int oz = q.w0;
+#else
     float* orow = reinterpret_cast<float*>(p.out) + ((uint64_t)q.w0 * p.oh + y0) * p.ow + x;
     const uint64_t zstride = (uint64_t)p.oh * p.ow;
+#endif
     int nrow = x < p.ow ? min(VOLR_S, p.oh - y0) : 0;
     const int ow = p.ow;
     auto emit = [&](const AxL& az, const float L[VOLR_S], const float H[VOLR_S]) {
+#if B2CL_VOLR_EIDX
+      float* o = reinterpret_cast<float*>(p.out) + ((uint64_t)(uint32_t)oz * ((uint64_t)p.oh * p.ow) + po);
+#else
       float* o = orow;
+#endif
       if (nrow == VOLR_S) {
 #pragma unroll
         for (int r = 0; r < VOLR_S; ++r, o += ow) __stcs(o, lerp1(az.a, az.oma, L[r], H[r]));
@@ -915,12 +1130,47 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
         for (int r = 0; r < VOLR_S; ++r, o += ow)
           if (r < nrow) __stcs(o, lerp1(az.a, az.oma, L[r], H[r]));
       }
+#if B2CL_VOLR_EIDX
+      ++oz;
+#else
       orow += zstride;
+#endif
     };
     auto copy = [](float D[VOLR_S], const float S[VOLR_S]) {
 #pragma unroll
       for (int r = 0; r < VOLR_S; ++r) D[r] = S[r];
     };
+#if B2CL_VOLR_FUSED
+    // one common step with a single held slice: each sample's new (x, y)-blend
+    // is z-blended with the held value, stored, and replaces it
+    auto fused = [&](const AxL& az, float V[VOLR_S]) {
+      acquire();
+      const float* buf = reinterpret_cast<const float*>(volr_buf + s * g.stride);
+#if B2CL_VOLR_EIDX
+      float* o = reinterpret_cast<float*>(p.out) + ((uint64_t)(uint32_t)oz * ((uint64_t)p.oh * p.ow) + po);
+      ++oz;
+#else
+      float* o = orow;
+      orow += zstride;
+#endif
+      if (nrow == VOLR_S) {
+#pragma unroll
+        for (int r = 0; r < VOLR_S; ++r, o += ow) {
+          const float h = tap_blend(buf, r);
+          __stcs(o, lerp1(az.a, az.oma, V[r], h));
+          V[r] = h;
+        }
+      } else {
+#pragma unroll
+        for (int r = 0; r < VOLR_S; ++r, o += ow) {
+          const float h = tap_blend(buf, r);
+          if (r < nrow) __stcs(o, lerp1(az.a, az.oma, V[r], h));
+          V[r] = h;
+        }
+      }
+      release();
+    };
+#endif
     // the z walk of k_sample_grid_vol (same roles, same staging order)
     float VA[VOLR_S], VB[VOLR_S];
     int kA = NONE, kB = NONE;
@@ -928,6 +1178,37 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
 #pragma unroll 1
     while (w < q.nst) {
       AxL az = vol_axis<C>(p, 10, p.oz, q.w0 + w, im.d);
+#if B2CL_VOLR_FUSED
+      // A run of common steps (lo = the previous hi, one new hi) whose next
+      // step does not reuse this step's lo holds ONE slice in registers (the
+      // fused step); VA / VB are rebuilt from it when the run ends.  The held
+      // pair is then (hi, hi): kA = kB = hi, which decides the next step's
+      // staging exactly as the producer's (lo, hi) does, because that step's
+      // lo differs from this one's (checked before each fused step).
+      if (az.i0 == kB && az.i1 != az.i0) {
+        AxL nz = az;
+        const bool rep = w + 1 < q.nst && (nz = vol_axis<C>(p, 10, p.oz, q.w0 + w + 1, im.d)).i0 == az.i0;
+        if (!rep) {
+          float V[VOLR_S];
+          copy(V, VB);
+#pragma unroll 1
+          for (;;) {
+            fused(az, V);
+            kA = kB = az.i1;
+            if (++w >= q.nst) break;
+            az = nz;
+            if (!(az.i0 == kB && az.i1 != az.i0)) break;
+            if (w + 1 < q.nst) {
+              nz = vol_axis<C>(p, 10, p.oz, q.w0 + w + 1, im.d);
+              if (nz.i0 == az.i0) break;
+            }
+          }
+          copy(VA, V);
+          copy(VB, V);
+          continue;
+        }
+      }
+#endif
       if (az.i0 == kB && az.i1 != az.i0) {
         slice(VA);
         emit(az, VB, VA);
@@ -1087,6 +1368,9 @@ static cudaError_t go_volr(const SampleParams& p, cudaStream_t st, bool* used) {
   VolrGeom g;
   g.bw = std::min(RB_MAXW, ((int)std::ceil(fw) + 1 + 2 + 3 + 3) & ~3);
   if (B2CL_VOLR_BW32) g.bw = std::min(RB_MAXW, (g.bw + 31) & ~31);
+#ifdef B2CL_VOLR_BWPAD  // A/B experiment: a wider box (row pitch) than the footprint needs
+  g.bw = std::min(RB_MAXW, g.bw + B2CL_VOLR_BWPAD);
+#endif
   g.bh = std::min(RB_MAXH, (int)std::ceil(fh) + 1 + 2);
   g.stride = (g.bw * g.bh * 4 + 127) & ~127;
   auto enc = encode_fn();

@@ -210,6 +210,9 @@ GRID_CASES = [
     (3, R, F32, (90, 90, 21), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d", (100, 70, 25), 1),
     (3, R, F32, (90, 90, 21), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d-min", (70, 66, 9), 1),
     (3, R, F32, (90, 90, 21), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d-zhalf", (130, 33, 30), 1),
+    # several tiles and z chunks per CTA (the staging cursor crosses tiles)
+    (3, R, F32, (200, 160, 300), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d", (256, 200, 300), 1),
+    (3, R, F32, (120, 100, 200), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d-zhalf", (150, 120, 300), 1),
 ]
 
 
