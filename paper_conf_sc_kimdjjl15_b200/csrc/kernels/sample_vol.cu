@@ -289,97 +289,6 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
   // --------------------------------------------------------------- consumers
   int s = 0;
   uint32_t ph = 0;
-#if B2CL_VOLR_INWARP
-  // Warp 0 also stages the slices: a cursor over the producer's copy order
-  // above (the same tiles, steps and need rules), advanced before each of
-  // warp 0's own waits -- blocking until the slice it waits for is issued,
-  // then as far as NS slices ahead while their ring stages are free.
-  int ct = blockIdx.x, cw = 0, chh = 0, ckA = NONE, ckB = NONE, cw0 = 0, cnst = 0, cxb = 0, cyb = 0, cok = 0;
-  int ci0 = 0, ci1 = 0, cazw = -1;  // the z taps of step cw (cached)
-  int cs = 0, cn = 0, consumed = 0;
-  uint32_t cph = 0;
-  auto cur_tile = [&]() {
-    const VolSeg q = vol_seg(p, tl, ct);
-    const VolrBox bx = volr_box<C>(p, g, q.tx * RT_W, q.ty * RT_H, q.w0, lane);
-    cw = 0;
-    chh = 0;
-    ckA = ckB = NONE;
-    cw0 = q.w0;
-    cnst = q.nst;
-    cxb = bx.xb;
-    cyb = bx.yb;
-    cok = bx.ok;
-    cazw = -1;
-  };
-  if (warp == 0 && ct < ntiles) cur_tile();
-  auto cur_next = [&](int& k) -> bool {
-    for (;;) {
-      if (ct >= ntiles) return false;
-      if (!cok || cw >= cnst) {
-        ct += gridDim.x;
-        if (ct < ntiles) cur_tile();
-        continue;
-      }
-      if (cazw != cw) {
-        const AxL az = vol_axis<C>(p, 10, p.oz, cw0 + cw, im.d);
-        ci0 = az.i0;
-        ci1 = az.i1;
-        cazw = cw;
-      }
-      const bool need0 = !(ci0 == ckA || ci0 == ckB);
-      if (chh == 0) {
-        chh = 1;
-        if (need0) { k = ci0; return true; }
-      }
-      const bool need1 = !(ci1 == ci0 || (!need0 && ci1 == ckB));
-      chh = 0;
-      ckA = ci0;
-      ckB = ci1;
-      ++cw;
-      if (need1) { k = ci1; return true; }
-    }
-  };
-  auto cur_issue = [&](bool block) -> bool {
-    if (!block) {
-      uint32_t ready = 0;
-      if (lane == 0)
-        asm volatile(
-            "{ .reg .pred P; mbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2; selp.u32 %0, 1, 0, P; }"
-            : "=r"(ready)
-            : "r"(vol_smem(&empty[cs])), "r"(cph ^ 1u)
-            : "memory");
-      if (!__shfl_sync(0xffffffffu, ready, 0)) return false;
-    }
-    int k = 0;
-    if (!cur_next(k)) return false;
-    if (lane == 0) {
-      if (block) vol_wait(&empty[cs], cph ^ 1u);
-      const uint32_t fb = vol_smem(&full[cs]);
-      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(g.bw * g.bh * 4)
-                   : "memory");
-      asm volatile(
-          "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
-          " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(vol_smem(volr_buf + cs * g.stride)),
-          "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(cxb), "r"(cyb), "r"(k), "r"(fb)
-          : "memory");
-    }
-    if (++cs == VOLR_NS) { cs = 0; cph ^= 1u; }
-    ++cn;
-    return true;
-  };
-  auto acquire = [&]() {
-    if (warp == 0) {
-      while (cn <= consumed && cur_issue(true)) {
-      }
-      while (cn < consumed + VOLR_NS && cur_issue(false)) {
-      }
-      ++consumed;
-    }
-    vol_wait(&full[s], ph);
-  };
-#else
-  auto acquire = [&]() { vol_wait(&full[s], ph); };
-#endif
   for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
     const VolSeg q = vol_seg(p, tl, t);
     const int xt = q.tx * VT_W, yt = q.ty * VT_H;
@@ -628,28 +537,31 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
 // sample keeps its own tap offsets and weights (8 samples per thread, one
 // column and 8 rows), the blend order is linear_at's: bit-identical results.
 #ifndef B2CL_VOLR_NS
-#define B2CL_VOLR_NS 4
+#define B2CL_VOLR_NS 8  // most ring stages (fewer when the box is large)
 #endif
 #ifndef B2CL_VOLR_SETUP
 #define B2CL_VOLR_SETUP 2.0  // a z chunk's fixed cost in steps (vol_plan; fitted: walks of 14 / 16 / 32 at 236.9 / 231.7 / 219.2 us)
 #endif
 #ifndef B2CL_VOLR_MINB
-#define B2CL_VOLR_MINB 2
+#define B2CL_VOLR_MINB 1
 #endif
 #ifndef B2CL_VOLR_S
 #define B2CL_VOLR_S 8
 #endif
 #ifndef B2CL_VOLR_NOHOIST
-#define B2CL_VOLR_NOHOIST 1  // 1: 1 - w recomputed per slice, not held in 16 registers (fewer spills: 200.5 vs 215.5 us)
+#define B2CL_VOLR_NOHOIST 0  // 1: 1 - w recomputed per slice, not held in 16 registers (with 8 consumer warps and 96 registers: 200.5 vs 215.5 us)
 #endif
 #ifndef B2CL_VOLR_FUSED
 #define B2CL_VOLR_FUSED 1  // 1: runs of common steps hold one slice (fused blend + store)
+#endif
+#ifndef B2CL_VOLR_ONEPATH
+#define B2CL_VOLR_ONEPATH 0  // 1: one fused-step body with predicated stores (no full-tile copy)
 #endif
 #ifndef B2CL_VOLR_EIDX
 #define B2CL_VOLR_EIDX 0  // 1: the output address recomputed per step from z (no 64-bit row pointer and stride held)
 #endif
 #ifndef B2CL_VOLR_LEAN
-#define B2CL_VOLR_LEAN 0  // 1: the interior-tile slice with precomputed offsets and paired blends (measured 247.9 vs 240.9 us)
+#define B2CL_VOLR_LEAN 0  // 1: interior tiles read the 4 taps at fixed byte deltas (209.4 vs 195.4 us: more spills)
 #endif
 constexpr int VOLR_S = B2CL_VOLR_S;           // samples (rows) per consumer thread
 #ifndef B2CL_VOLR_TW
@@ -658,13 +570,17 @@ constexpr int VOLR_S = B2CL_VOLR_S;           // samples (rows) per consumer thr
 #ifndef B2CL_VOLR_BW32
 #define B2CL_VOLR_BW32 0  // 1: round the box row up to a multiple of 32 texels (bank group = column)
 #endif
-constexpr int RT_W = B2CL_VOLR_TW, RT_H = (256 / RT_W) * VOLR_S;  // output tile (256 consumer threads)
+#ifndef B2CL_VOLR_CW
+#define B2CL_VOLR_CW 12  // consumer warps per CTA (13 warps, one CTA per SM: 128 registers, no spill)
+#endif
+constexpr int VOLR_CW = B2CL_VOLR_CW, VOLR_CT = 32 * VOLR_CW;
+constexpr int RT_W = B2CL_VOLR_TW, RT_H = (VOLR_CT / RT_W) * VOLR_S;  // output tile (one sample column of VOLR_S rows per consumer thread)
 constexpr int RB_MAXW = 128, RB_MAXH = 128;   // largest staged box (texels)
 constexpr int VOLR_NS = B2CL_VOLR_NS;
 #ifndef B2CL_VOLR_INWARP
 #define B2CL_VOLR_INWARP 0  // 1: consumer warp 0 also issues the copies (256 threads: 128 registers, no spill; measured 255.4 vs 216.4 us: warp 0 becomes the straggler); 0: a 9th producer warp (96 registers, a small spill)
 #endif
-constexpr int VOLR_THREADS = B2CL_VOLR_INWARP ? 256 : 288;  // 8 consumer warps (+ 1 producer warp)
+constexpr int VOLR_THREADS = B2CL_VOLR_INWARP ? VOLR_CT : VOLR_CT + 32;  // consumer warps (+ 1 producer warp)
 
 struct VolrBox {
   int xb, yb;    // first staged texel column (16-B aligned) and row
@@ -674,6 +590,7 @@ struct VolrBox {
 struct VolrGeom {
   int bw, bh;    // staged box (texels), chosen per launch from the map's footprint
   int stride;    // bytes per ring stage (128-B multiple)
+  int ns;        // ring stages (<= VOLR_NS, as many as 200 KB hold)
 };
 
 // the tile's staged box from its corners' taps (identical in every warp)
@@ -769,9 +686,9 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
   const Image& im = p.im;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
-    for (int s = 0; s < VOLR_NS; ++s) {
+    for (int s = 0; s < g.ns; ++s) {
       asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(vol_smem(&full[s])) : "memory");
-      asm volatile("mbarrier.init.shared::cta.b64 [%0], 8;" ::"r"(vol_smem(&empty[s])) : "memory");
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(vol_smem(&empty[s])), "n"(VOLR_CW) : "memory");
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -780,7 +697,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
   const int ntiles = tl.ntx * tl.nty * tl.nzc;
   constexpr int NONE = -2147483647 - 1;
 
-  if (!B2CL_VOLR_INWARP && warp == 8) {  // --------------------------- producer
+  if (!B2CL_VOLR_INWARP && warp == VOLR_CW) {  // -------------------- producer
     int s = 0;
     uint32_t ph = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
@@ -856,7 +773,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
                          "r"(bx.xb), "r"(bx.yb), "r"(k + B2CL_VOLR_PF)
                          : "memory");
 #endif
-          if (++s == VOLR_NS) { s = 0; ph ^= 1u; }
+          if (++s == g.ns) { s = 0; ph ^= 1u; }
         }
         kA = az.i0;
         kB = az.i1;
@@ -942,7 +859,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
           "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(cxb), "r"(cyb), "r"(k), "r"(fb)
           : "memory");
     }
-    if (++cs == VOLR_NS) { cs = 0; cph ^= 1u; }
+    if (++cs == g.ns) { cs = 0; cph ^= 1u; }
     ++cn;
     return true;
   };
@@ -950,7 +867,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
     if (warp == 0) {
       while (cn <= consumed && cur_issue(true)) {
       }
-      while (cn < consumed + VOLR_NS && cur_issue(false)) {
+      while (cn < consumed + g.ns && cur_issue(false)) {
       }
       ++consumed;
     }
@@ -975,10 +892,10 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
     if (bx.ok) {
       float cu[4], cv[4];
       volr_corners<C>(p, q.tx * RT_W, q.ty * RT_H, q.w0, cu, cv);
-      for (int r = threadIdx.x; r < g.bh; r += 256)
+      for (int r = threadIdx.x; r < g.bh; r += VOLR_CT)
         segtab[r] = bx.yb + r < im.h ? volr_row_seg(cu, cv, bx.yb + r, bx.xb, g.bw, im.w) : 0;
     }
-    asm volatile("bar.sync 1, 256;" ::: "memory");
+    asm volatile("bar.sync 1, %0;" ::"n"(VOLR_CT) : "memory");
 #endif
     for (int r = 0; r < VOLR_S; ++r) {
       const float yf = __int2float_rn(p.oy + y0 + r);
@@ -1000,8 +917,8 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
       wb[r] = ay.a;
     }
     int fast;
-    asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, 256, P; selp.s32 %0, 1, 0, Q; }"
-                 : "=r"(fast) : "r"(in) : "memory");
+    asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, %2, P; selp.s32 %0, 1, 0, Q; }"
+                 : "=r"(fast) : "r"(in), "n"(VOLR_CT) : "memory");
     if (!fast) {  // the taps directly (read_image, the general kernel's coordinates)
       // (CLAMP_TO_EDGE indices are monotone in x and y, so every tap of a tile
       // whose corner box fits lies in it and this does not happen; should it,
@@ -1017,7 +934,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
             acquire();
             __syncwarp();
             if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(vol_smem(&empty[s])) : "memory");
-            if (++s == VOLR_NS) { s = 0; ph ^= 1u; }
+            if (++s == g.ns) { s = 0; ph ^= 1u; }
           }
           kA = az.i0;
           kB = az.i1;
@@ -1045,65 +962,65 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
     // offsets precomputed, the 4 taps at fixed deltas, the x-blend of rows
     // j0 and j1 as one paired FMUL2 + FFMA2 (each lane lerp1's fma / mul).
 #if B2CL_VOLR_LEAN
+    // Interior tiles (every tap pair unclamped: i1 = i0 + 1, j1 = j0 + 1 --
+    // all but the tiles at the image's edges): byte offsets, the 4 taps at
+    // fixed deltas (+4, +row, +row+4)
     int interior = 1;
 #pragma unroll
     for (int r = 0; r < VOLR_S; ++r) interior &= (off[r] >> 16) == 3 || !(x < p.ow && y0 + r < p.oh);
-    asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, 256, P; selp.s32 %0, 1, 0, Q; }"
-                 : "=r"(interior) : "r"(interior) : "memory");
-    float oma[VOLR_S], omb[VOLR_S];
+    asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, %2, P; selp.s32 %0, 1, 0, Q; }"
+                 : "=r"(interior) : "r"(interior), "n"(VOLR_CT) : "memory");
     if (interior) {
 #pragma unroll
-      for (int r = 0; r < VOLR_S; ++r) {
-        off[r] = (off[r] & 0xffff) * 4;
-        oma[r] = __fsub_rn(1.0f, wa[r]);
-        omb[r] = __fsub_rn(1.0f, wb[r]);
-      }
+      for (int r = 0; r < VOLR_S; ++r) off[r] = (off[r] & 0xffff) * 4;
     }
     const uint32_t rowb = (uint32_t)g.bw * 4u;
 #else
     const int interior = 0;
-    float oma[1], omb[1];
     const uint32_t rowb = 0;
 #endif
-    // sample r's (x, y)-blend of one staged slice
-    auto tap_blend = [&](const float* buf, int r) -> float {
-      const float* t0 = buf + (off[r] & 0xffff);
-      const int dx = off[r] >> 16 & 1, dy = (off[r] >> 17) * g.bw;
+    auto one_minus = [](float w) -> float {
 #if B2CL_VOLR_NOHOIST
-      // 1 - w recomputed per slice (volatile: not hoisted into 16 live registers)
-      float oma1, omb1;
-      asm volatile("sub.rn.f32 %0, 0f3F800000, %1;" : "=f"(oma1) : "f"(wa[r]));
-      asm volatile("sub.rn.f32 %0, 0f3F800000, %1;" : "=f"(omb1) : "f"(wb[r]));
+      // recomputed per slice (volatile: not hoisted into 16 live registers)
+      float o;
+      asm volatile("sub.rn.f32 %0, 0f3F800000, %1;" : "=f"(o) : "f"(w));
+      return o;
 #else
-      const float oma1 = __fsub_rn(1.0f, wa[r]), omb1 = __fsub_rn(1.0f, wb[r]);
+      return __fsub_rn(1.0f, w);
 #endif
+    };
+    // sample r's (x, y)-blend of one staged slice (buf: the stage)
+    auto tap_gen = [&](const char* buf, int r) -> float {
+      const float* t0 = reinterpret_cast<const float*>(buf) + (off[r] & 0xffff);
+      const int dx = off[r] >> 16 & 1, dy = (off[r] >> 17) * g.bw;
+      const float oma1 = one_minus(wa[r]), omb1 = one_minus(wb[r]);
       const float h0 = lerp1(wa[r], oma1, t0[0], t0[dx]);
       const float h1 = lerp1(wa[r], oma1, t0[dy], t0[dy + dx]);
+      return lerp1(wb[r], omb1, h0, h1);
+    };
+    auto tap_lean = [&](const char* buf, int r) -> float {
+      const char* t = buf + (uint32_t)off[r];
+      const char* t2 = t + rowb;
+      const float oma1 = one_minus(wa[r]), omb1 = one_minus(wb[r]);
+      const float h0 = lerp1(wa[r], oma1, *reinterpret_cast<const float*>(t), *reinterpret_cast<const float*>(t + 4));
+      const float h1 =
+          lerp1(wa[r], oma1, *reinterpret_cast<const float*>(t2), *reinterpret_cast<const float*>(t2 + 4));
       return lerp1(wb[r], omb1, h0, h1);
     };
     auto release = [&]() {
       __syncwarp();
       if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(vol_smem(&empty[s])) : "memory");
-      if (++s == VOLR_NS) { s = 0; ph ^= 1u; }
+      if (++s == g.ns) { s = 0; ph ^= 1u; }
     };
     auto slice = [&](float V[VOLR_S]) {
       acquire();
+      const char* buf = reinterpret_cast<const char*>(volr_buf + s * g.stride);
       if (interior) {
-        const char* buf = reinterpret_cast<const char*>(volr_buf + s * g.stride);
 #pragma unroll
-        for (int r = 0; r < VOLR_S && B2CL_VOLR_LEAN; ++r) {
-          const char* t = buf + (uint32_t)off[r];
-          const char* t2 = t + rowb;
-          const float2 lo = make_float2(*reinterpret_cast<const float*>(t), *reinterpret_cast<const float*>(t2));
-          const float2 hi =
-              make_float2(*reinterpret_cast<const float*>(t + 4), *reinterpret_cast<const float*>(t2 + 4));
-          const float2 h = __ffma2_rn(make_float2(wa[r], wa[r]), hi, __fmul2_rn(make_float2(oma[r], oma[r]), lo));
-          V[r] = lerp1(wb[r], omb[r], h.x, h.y);
-        }
+        for (int r = 0; r < VOLR_S; ++r) V[r] = tap_lean(buf, r);
       } else {
-        const float* buf = reinterpret_cast<const float*>(volr_buf + s * g.stride);
 #pragma unroll
-        for (int r = 0; r < VOLR_S; ++r) V[r] = tap_blend(buf, r);
+        for (int r = 0; r < VOLR_S; ++r) V[r] = tap_gen(buf, r);
       }
       release();
     };
@@ -1145,7 +1062,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
     // is z-blended with the held value, stored, and replaces it
     auto fused = [&](const AxL& az, float V[VOLR_S]) {
       acquire();
-      const float* buf = reinterpret_cast<const float*>(volr_buf + s * g.stride);
+      const char* buf = reinterpret_cast<const char*>(volr_buf + s * g.stride);
 #if B2CL_VOLR_EIDX
       float* o = reinterpret_cast<float*>(p.out) + ((uint64_t)(uint32_t)oz * ((uint64_t)p.oh * p.ow) + po);
       ++oz;
@@ -1153,21 +1070,36 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
       float* o = orow;
       orow += zstride;
 #endif
-      if (nrow == VOLR_S) {
+      auto body = [&](auto tap) {
+#if B2CL_VOLR_ONEPATH
 #pragma unroll
         for (int r = 0; r < VOLR_S; ++r, o += ow) {
-          const float h = tap_blend(buf, r);
-          __stcs(o, lerp1(az.a, az.oma, V[r], h));
-          V[r] = h;
-        }
-      } else {
-#pragma unroll
-        for (int r = 0; r < VOLR_S; ++r, o += ow) {
-          const float h = tap_blend(buf, r);
+          const float h = tap(buf, r);
           if (r < nrow) __stcs(o, lerp1(az.a, az.oma, V[r], h));
           V[r] = h;
         }
-      }
+#else
+        if (nrow == VOLR_S) {
+#pragma unroll
+          for (int r = 0; r < VOLR_S; ++r, o += ow) {
+            const float h = tap(buf, r);
+            __stcs(o, lerp1(az.a, az.oma, V[r], h));
+            V[r] = h;
+          }
+        } else {
+#pragma unroll
+          for (int r = 0; r < VOLR_S; ++r, o += ow) {
+            const float h = tap(buf, r);
+            if (r < nrow) __stcs(o, lerp1(az.a, az.oma, V[r], h));
+            V[r] = h;
+          }
+        }
+#endif
+      };
+      if (interior)
+        body(tap_lean);
+      else
+        body(tap_gen);
       release();
     };
 #endif
@@ -1387,8 +1319,9 @@ static cudaError_t go_volr(const SampleParams& p, cudaStream_t st, bool* used) {
           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
     return cudaSuccess;
   int occ[64] = {0};  // (occupancy depends on this launch's box)
-  const size_t smem = (size_t)VOLR_NS * g.stride;
-  if (smem > 200 * 1024) return cudaSuccess;
+  g.ns = std::min(VOLR_NS, (200 * 1024) / g.stride);
+  if (g.ns < 2) return cudaSuccess;
+  const size_t smem = (size_t)g.ns * g.stride;
   VolTiles tl;
   int grid = 0;
   if (!vol_plan(p, RT_W, RT_H, reinterpret_cast<const void*>(k_sample_grid_volr<C>), VOLR_THREADS, smem, occ, &tl,

@@ -210,6 +210,7 @@ GRID_CASES = [
     (3, R, F32, (90, 90, 21), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d", (100, 70, 25), 1),
     (3, R, F32, (90, 90, 21), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d-min", (70, 66, 9), 1),
     (3, R, F32, (90, 90, 21), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d-zhalf", (130, 33, 30), 1),
+    (3, R, F32, (150, 150, 20), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d-wide", (160, 120, 24), 1),
     # several tiles and z chunks per CTA (the staging cursor crosses tiles)
     (3, R, F32, (200, 160, 300), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d", (256, 200, 300), 1),
     (3, R, F32, (120, 100, 200), (1, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR), "rotate3d-zhalf", (150, 120, 300), 1),
@@ -242,6 +243,10 @@ def _affine(kind, size, out):
         A = synth.affine_stencil_3d(W)
         A[5], A[7] = 1.0 / H, (0.5 + 0.6) / H
         A[10], A[11] = -1.0 / D, (D - 0.5 + 0.2) / D
+        return A
+    if kind == "rotate3d-wide":  # 45 degrees at 1.5x minification: a box near the kernel's largest (fewer ring stages)
+        A = synth.affine_rotate_3d(W, 45.0)
+        A[[0, 1, 4, 5]] *= 1.5
         return A
     if kind.startswith("rotate3d-"):
         A = synth.affine_rotate_3d(W, 20.0)
