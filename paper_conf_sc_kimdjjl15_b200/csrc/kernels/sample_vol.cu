@@ -530,12 +530,15 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
 // are any affine function of the output (x, y) and the z coordinate depends
 // on the output z alone (A[2] = A[6] = A[8] = A[9] = 0).  The z axis is then
 // walked exactly as above -- (x,y)-blended slices held in registers, one new
-// slice per common step -- while the (x,y) footprint of a 64 x 32 output tile
+// slice per common step -- while the (x,y) footprint of a 64 x 48 output tile
 // is the bounding box of the taps of its four corners (the fp32 coordinate is
 // monotone in x and in y separately, and so are the axis indices): at most
-// RB_W x RB_H texels, staged per slice by one cp.async.bulk per box row.  Each
-// sample keeps its own tap offsets and weights (8 samples per thread, one
-// column and 8 rows), the blend order is linear_at's: bit-identical results.
+// RB_MAXW x RB_MAXH texels, staged per slice by one cp.async.bulk.tensor.3d
+// into a ring of up to 8 stages.  One CTA per SM: 12 consumer warps (128
+// registers each: every per-sample value stays in registers) and a producer
+// warp.  Each sample keeps its own tap offsets and weights (8 samples per
+// thread, one column and 8 rows); the blend order is linear_at's:
+// bit-identical results.
 #ifndef B2CL_VOLR_NS
 #define B2CL_VOLR_NS 8  // most ring stages (fewer when the box is large)
 #endif
@@ -549,26 +552,14 @@ __global__ void __launch_bounds__(VOL_THREADS, B2CL_VOL_MINB)
 #define B2CL_VOLR_S 8
 #endif
 #ifndef B2CL_VOLR_NOHOIST
-#define B2CL_VOLR_NOHOIST 0  // 1: 1 - w recomputed per slice, not held in 16 registers (with 8 consumer warps and 96 registers: 200.5 vs 215.5 us)
+#define B2CL_VOLR_NOHOIST 0  // 1: 1 - w recomputed per slice, not held in 16 registers (helped with 8 consumer warps at 96 registers: 200.5 vs 215.5 us; 12 warps at 128: 188 held vs 195 recomputed)
 #endif
 #ifndef B2CL_VOLR_FUSED
 #define B2CL_VOLR_FUSED 1  // 1: runs of common steps hold one slice (fused blend + store)
 #endif
-#ifndef B2CL_VOLR_ONEPATH
-#define B2CL_VOLR_ONEPATH 0  // 1: one fused-step body with predicated stores (no full-tile copy)
-#endif
-#ifndef B2CL_VOLR_EIDX
-#define B2CL_VOLR_EIDX 0  // 1: the output address recomputed per step from z (no 64-bit row pointer and stride held)
-#endif
-#ifndef B2CL_VOLR_LEAN
-#define B2CL_VOLR_LEAN 0  // 1: interior tiles read the 4 taps at fixed byte deltas (209.4 vs 195.4 us: more spills)
-#endif
 constexpr int VOLR_S = B2CL_VOLR_S;           // samples (rows) per consumer thread
 #ifndef B2CL_VOLR_TW
 #define B2CL_VOLR_TW 64
-#endif
-#ifndef B2CL_VOLR_BW32
-#define B2CL_VOLR_BW32 0  // 1: round the box row up to a multiple of 32 texels (bank group = column)
 #endif
 #ifndef B2CL_VOLR_CW
 #define B2CL_VOLR_CW 12  // consumer warps per CTA (13 warps, one CTA per SM: 128 registers, no spill)
@@ -577,10 +568,7 @@ constexpr int VOLR_CW = B2CL_VOLR_CW, VOLR_CT = 32 * VOLR_CW;
 constexpr int RT_W = B2CL_VOLR_TW, RT_H = (VOLR_CT / RT_W) * VOLR_S;  // output tile (one sample column of VOLR_S rows per consumer thread)
 constexpr int RB_MAXW = 128, RB_MAXH = 128;   // largest staged box (texels)
 constexpr int VOLR_NS = B2CL_VOLR_NS;
-#ifndef B2CL_VOLR_INWARP
-#define B2CL_VOLR_INWARP 0  // 1: consumer warp 0 also issues the copies (256 threads: 128 registers, no spill; measured 255.4 vs 216.4 us: warp 0 becomes the straggler); 0: a 9th producer warp (96 registers, a small spill)
-#endif
-constexpr int VOLR_THREADS = B2CL_VOLR_INWARP ? VOLR_CT : VOLR_CT + 32;  // consumer warps (+ 1 producer warp)
+constexpr int VOLR_THREADS = VOLR_CT + 32;  // consumer warps + 1 producer warp
 
 struct VolrBox {
   int xb, yb;    // first staged texel column (16-B aligned) and row
@@ -697,7 +685,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
   const int ntiles = tl.ntx * tl.nty * tl.nzc;
   constexpr int NONE = -2147483647 - 1;
 
-  if (!B2CL_VOLR_INWARP && warp == VOLR_CW) {  // -------------------- producer
+  if (warp == VOLR_CW) {  // ---------------------------------------- producer
     int s = 0;
     uint32_t ph = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
@@ -785,97 +773,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
   // --------------------------------------------------------------- consumers
   int s = 0;
   uint32_t ph = 0;
-#if B2CL_VOLR_INWARP
-  // Warp 0 also stages the slices: a cursor over the producer's copy order
-  // above (the same tiles, steps and need rules), advanced before each of
-  // warp 0's own waits -- blocking until the slice it waits for is issued,
-  // then as far as NS slices ahead while their ring stages are free.
-  int ct = blockIdx.x, cw = 0, chh = 0, ckA = NONE, ckB = NONE, cw0 = 0, cnst = 0, cxb = 0, cyb = 0, cok = 0;
-  int ci0 = 0, ci1 = 0, cazw = -1;  // the z taps of step cw (cached)
-  int cs = 0, cn = 0, consumed = 0;
-  uint32_t cph = 0;
-  auto cur_tile = [&]() {
-    const VolSeg q = vol_seg(p, tl, ct);
-    const VolrBox bx = volr_box<C>(p, g, q.tx * RT_W, q.ty * RT_H, q.w0, lane);
-    cw = 0;
-    chh = 0;
-    ckA = ckB = NONE;
-    cw0 = q.w0;
-    cnst = q.nst;
-    cxb = bx.xb;
-    cyb = bx.yb;
-    cok = bx.ok;
-    cazw = -1;
-  };
-  if (warp == 0 && ct < ntiles) cur_tile();
-  auto cur_next = [&](int& k) -> bool {
-    for (;;) {
-      if (ct >= ntiles) return false;
-      if (!cok || cw >= cnst) {
-        ct += gridDim.x;
-        if (ct < ntiles) cur_tile();
-        continue;
-      }
-      if (cazw != cw) {
-        const AxL az = vol_axis<C>(p, 10, p.oz, cw0 + cw, im.d);
-        ci0 = az.i0;
-        ci1 = az.i1;
-        cazw = cw;
-      }
-      const bool need0 = !(ci0 == ckA || ci0 == ckB);
-      if (chh == 0) {
-        chh = 1;
-        if (need0) { k = ci0; return true; }
-      }
-      const bool need1 = !(ci1 == ci0 || (!need0 && ci1 == ckB));
-      chh = 0;
-      ckA = ci0;
-      ckB = ci1;
-      ++cw;
-      if (need1) { k = ci1; return true; }
-    }
-  };
-  auto cur_issue = [&](bool block) -> bool {
-    if (!block) {
-      uint32_t ready = 0;
-      if (lane == 0)
-        asm volatile(
-            "{ .reg .pred P; mbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2; selp.u32 %0, 1, 0, P; }"
-            : "=r"(ready)
-            : "r"(vol_smem(&empty[cs])), "r"(cph ^ 1u)
-            : "memory");
-      if (!__shfl_sync(0xffffffffu, ready, 0)) return false;
-    }
-    int k = 0;
-    if (!cur_next(k)) return false;
-    if (lane == 0) {
-      if (block) vol_wait(&empty[cs], cph ^ 1u);
-      const uint32_t fb = vol_smem(&full[cs]);
-      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(g.bw * g.bh * 4)
-                   : "memory");
-      asm volatile(
-          "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
-          " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(vol_smem(volr_buf + cs * g.stride)),
-          "l"(reinterpret_cast<uint64_t>(&tmap)), "r"(cxb), "r"(cyb), "r"(k), "r"(fb)
-          : "memory");
-    }
-    if (++cs == g.ns) { cs = 0; cph ^= 1u; }
-    ++cn;
-    return true;
-  };
-  auto acquire = [&]() {
-    if (warp == 0) {
-      while (cn <= consumed && cur_issue(true)) {
-      }
-      while (cn < consumed + g.ns && cur_issue(false)) {
-      }
-      ++consumed;
-    }
-    vol_wait(&full[s], ph);
-  };
-#else
   auto acquire = [&]() { vol_wait(&full[s], ph); };
-#endif
   const int col = threadIdx.x & (RT_W - 1), rg = threadIdx.x / RT_W;  // column, row group of VOLR_S
   for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
     const VolSeg q = vol_seg(p, tl, t);
@@ -961,24 +859,6 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
     // all but the tiles at the image's edges) take the lean slice: byte
     // offsets precomputed, the 4 taps at fixed deltas, the x-blend of rows
     // j0 and j1 as one paired FMUL2 + FFMA2 (each lane lerp1's fma / mul).
-#if B2CL_VOLR_LEAN
-    // Interior tiles (every tap pair unclamped: i1 = i0 + 1, j1 = j0 + 1 --
-    // all but the tiles at the image's edges): byte offsets, the 4 taps at
-    // fixed deltas (+4, +row, +row+4)
-    int interior = 1;
-#pragma unroll
-    for (int r = 0; r < VOLR_S; ++r) interior &= (off[r] >> 16) == 3 || !(x < p.ow && y0 + r < p.oh);
-    asm volatile("{ .reg .pred P, Q; setp.ne.s32 P, %1, 0; bar.red.and.pred Q, 1, %2, P; selp.s32 %0, 1, 0, Q; }"
-                 : "=r"(interior) : "r"(interior), "n"(VOLR_CT) : "memory");
-    if (interior) {
-#pragma unroll
-      for (int r = 0; r < VOLR_S; ++r) off[r] = (off[r] & 0xffff) * 4;
-    }
-    const uint32_t rowb = (uint32_t)g.bw * 4u;
-#else
-    const int interior = 0;
-    const uint32_t rowb = 0;
-#endif
     auto one_minus = [](float w) -> float {
 #if B2CL_VOLR_NOHOIST
       // recomputed per slice (volatile: not hoisted into 16 live registers)
@@ -990,21 +870,12 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
 #endif
     };
     // sample r's (x, y)-blend of one staged slice (buf: the stage)
-    auto tap_gen = [&](const char* buf, int r) -> float {
+    auto tap_blend = [&](const char* buf, int r) -> float {
       const float* t0 = reinterpret_cast<const float*>(buf) + (off[r] & 0xffff);
       const int dx = off[r] >> 16 & 1, dy = (off[r] >> 17) * g.bw;
       const float oma1 = one_minus(wa[r]), omb1 = one_minus(wb[r]);
       const float h0 = lerp1(wa[r], oma1, t0[0], t0[dx]);
       const float h1 = lerp1(wa[r], oma1, t0[dy], t0[dy + dx]);
-      return lerp1(wb[r], omb1, h0, h1);
-    };
-    auto tap_lean = [&](const char* buf, int r) -> float {
-      const char* t = buf + (uint32_t)off[r];
-      const char* t2 = t + rowb;
-      const float oma1 = one_minus(wa[r]), omb1 = one_minus(wb[r]);
-      const float h0 = lerp1(wa[r], oma1, *reinterpret_cast<const float*>(t), *reinterpret_cast<const float*>(t + 4));
-      const float h1 =
-          lerp1(wa[r], oma1, *reinterpret_cast<const float*>(t2), *reinterpret_cast<const float*>(t2 + 4));
       return lerp1(wb[r], omb1, h0, h1);
     };
     auto release = [&]() {
@@ -1015,30 +886,16 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
     auto slice = [&](float V[VOLR_S]) {
       acquire();
       const char* buf = reinterpret_cast<const char*>(volr_buf + s * g.stride);
-      if (interior) {
 #pragma unroll
-        for (int r = 0; r < VOLR_S; ++r) V[r] = tap_lean(buf, r);
-      } else {
-#pragma unroll
-        for (int r = 0; r < VOLR_S; ++r) V[r] = tap_gen(buf, r);
-      }
+      for (int r = 0; r < VOLR_S; ++r) V[r] = tap_blend(buf, r);
       release();
     };
-#if B2CL_VOLR_EIDX
-    const uint32_t po = (uint32_t)y0 * (uint32_t)p.ow + (uint32_t)x;  // (y0, x) in the output plane
-    int oz = q.w0;
-#else
     float* orow = reinterpret_cast<float*>(p.out) + ((uint64_t)q.w0 * p.oh + y0) * p.ow + x;
     const uint64_t zstride = (uint64_t)p.oh * p.ow;
-#endif
     int nrow = x < p.ow ? min(VOLR_S, p.oh - y0) : 0;
     const int ow = p.ow;
     auto emit = [&](const AxL& az, const float L[VOLR_S], const float H[VOLR_S]) {
-#if B2CL_VOLR_EIDX
-      float* o = reinterpret_cast<float*>(p.out) + ((uint64_t)(uint32_t)oz * ((uint64_t)p.oh * p.ow) + po);
-#else
       float* o = orow;
-#endif
       if (nrow == VOLR_S) {
 #pragma unroll
         for (int r = 0; r < VOLR_S; ++r, o += ow) __stcs(o, lerp1(az.a, az.oma, L[r], H[r]));
@@ -1047,11 +904,7 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
         for (int r = 0; r < VOLR_S; ++r, o += ow)
           if (r < nrow) __stcs(o, lerp1(az.a, az.oma, L[r], H[r]));
       }
-#if B2CL_VOLR_EIDX
-      ++oz;
-#else
       orow += zstride;
-#endif
     };
     auto copy = [](float D[VOLR_S], const float S[VOLR_S]) {
 #pragma unroll
@@ -1060,46 +913,26 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
 #if B2CL_VOLR_FUSED
     // one common step with a single held slice: each sample's new (x, y)-blend
     // is z-blended with the held value, stored, and replaces it
-    auto fused = [&](const AxL& az, float V[VOLR_S]) {
+    auto fused = [&](const AxL& az, const float L[VOLR_S], float H[VOLR_S]) {
       acquire();
       const char* buf = reinterpret_cast<const char*>(volr_buf + s * g.stride);
-#if B2CL_VOLR_EIDX
-      float* o = reinterpret_cast<float*>(p.out) + ((uint64_t)(uint32_t)oz * ((uint64_t)p.oh * p.ow) + po);
-      ++oz;
-#else
       float* o = orow;
       orow += zstride;
-#endif
-      auto body = [&](auto tap) {
-#if B2CL_VOLR_ONEPATH
+      if (nrow == VOLR_S) {
 #pragma unroll
         for (int r = 0; r < VOLR_S; ++r, o += ow) {
-          const float h = tap(buf, r);
-          if (r < nrow) __stcs(o, lerp1(az.a, az.oma, V[r], h));
-          V[r] = h;
+          const float h = tap_blend(buf, r);
+          __stcs(o, lerp1(az.a, az.oma, L[r], h));
+          H[r] = h;
         }
-#else
-        if (nrow == VOLR_S) {
+      } else {
 #pragma unroll
-          for (int r = 0; r < VOLR_S; ++r, o += ow) {
-            const float h = tap(buf, r);
-            __stcs(o, lerp1(az.a, az.oma, V[r], h));
-            V[r] = h;
-          }
-        } else {
-#pragma unroll
-          for (int r = 0; r < VOLR_S; ++r, o += ow) {
-            const float h = tap(buf, r);
-            if (r < nrow) __stcs(o, lerp1(az.a, az.oma, V[r], h));
-            V[r] = h;
-          }
+        for (int r = 0; r < VOLR_S; ++r, o += ow) {
+          const float h = tap_blend(buf, r);
+          if (r < nrow) __stcs(o, lerp1(az.a, az.oma, L[r], h));
+          H[r] = h;
         }
-#endif
-      };
-      if (interior)
-        body(tap_lean);
-      else
-        body(tap_gen);
+      }
       release();
     };
 #endif
@@ -1121,22 +954,36 @@ __global__ void __launch_bounds__(VOLR_THREADS, B2CL_VOLR_MINB)
         AxL nz = az;
         const bool rep = w + 1 < q.nst && (nz = vol_axis<C>(p, 10, p.oz, q.w0 + w + 1, im.d)).i0 == az.i0;
         if (!rep) {
-          float V[VOLR_S];
-          copy(V, VB);
-#pragma unroll 1
-          for (;;) {
-            fused(az, V);
+          // after a fused step: the next step's indices; false ends the run
+          auto more = [&]() -> bool {
             kA = kB = az.i1;
-            if (++w >= q.nst) break;
+            if (++w >= q.nst) return false;
             az = nz;
-            if (!(az.i0 == kB && az.i1 != az.i0)) break;
+            if (!(az.i0 == kB && az.i1 != az.i0)) return false;
             if (w + 1 < q.nst) {
               nz = vol_axis<C>(p, 10, p.oz, q.w0 + w + 1, im.d);
-              if (nz.i0 == az.i0) break;
+              if (nz.i0 == az.i0) return false;
+            }
+            return true;
+          };
+          // the held slice alternates between P and Q (no register copies)
+          float P[VOLR_S], Q[VOLR_S];
+          copy(P, VB);
+#pragma unroll 1
+          for (;;) {
+            fused(az, P, Q);
+            if (!more()) {
+              copy(VA, Q);
+              copy(VB, Q);
+              break;
+            }
+            fused(az, Q, P);
+            if (!more()) {
+              copy(VA, P);
+              copy(VB, P);
+              break;
             }
           }
-          copy(VA, V);
-          copy(VB, V);
           continue;
         }
       }
@@ -1299,10 +1146,6 @@ static cudaError_t go_volr(const SampleParams& p, cudaStream_t st, bool* used) {
   if (!(fw < RB_MAXW && fh < RB_MAXH)) return cudaSuccess;
   VolrGeom g;
   g.bw = std::min(RB_MAXW, ((int)std::ceil(fw) + 1 + 2 + 3 + 3) & ~3);
-  if (B2CL_VOLR_BW32) g.bw = std::min(RB_MAXW, (g.bw + 31) & ~31);
-#ifdef B2CL_VOLR_BWPAD  // A/B experiment: a wider box (row pitch) than the footprint needs
-  g.bw = std::min(RB_MAXW, g.bw + B2CL_VOLR_BWPAD);
-#endif
   g.bh = std::min(RB_MAXH, (int)std::ceil(fh) + 1 + 2);
   g.stride = (g.bw * g.bh * 4 + 127) & ~127;
   auto enc = encode_fn();
