@@ -2,12 +2,13 @@
 // images under separable maps (config 3: 512^3 R32F, CLAMP_TO_EDGE, LINEAR).
 //
 // Steps a3-a7 of the read built-in ([CL1.2 §8.1-8.2]) for every output of a
-// 256 x 16 x walk box, with the texel fetches (a5: through the CLImage
+// 512 x 12 x walk box, with the texel fetches (a5: through the CLImage
 // pointer) moved by the TMA engine:
-//   * a persistent grid of CTAs strides over output tiles; each CTA has one
-//     PRODUCER warp and eight CONSUMER warps (2 across x, 4 down y);
+//   * a persistent grid of CTAs (one per SM) strides over output tiles; each
+//     CTA has one PRODUCER warp and twelve CONSUMER warps (4 across x, 3 down
+//     y; 123 registers each, no spill);
 //   * per output slice the producer stages the tile's texel footprint in that
-//     slice -- a (260 x 17)-texel box starting at the tile's first tap (i0 of
+//     slice -- a (516 x 13)-texel box starting at the tile's first tap (i0 of
 //     its first column rounded down to 16 bytes, and of its first row) -- in a
 //     shared-memory ring: one cp.async.bulk per box row (one per lane),
 //     completing on a `full` mbarrier.  (B2CL_VOL_BULK=0 B2CL_VOL_XW=1
@@ -17,7 +18,7 @@
 //   * consumers x-blend each staged texel row once, y-blend neighbouring rows,
 //     keep the (x,y)-blended slice in registers and z-blend it with the next
 //     one, then release the stage on an `empty` mbarrier.
-// Bytes in flight are the ring (STAGES x 17.7 KB per CTA), independent of
+// Bytes in flight are the ring (STAGES x 26.8 KB per CTA), independent of
 // registers -- the limit of the register-pipelined walk kernels.
 //
 // Exactness.  Every output is computed with the operations and operands of
@@ -54,7 +55,7 @@ using namespace dev;
 #define B2CL_VOL_BULK 1
 #endif
 #ifndef B2CL_VOL_NS
-#define B2CL_VOL_NS 3
+#define B2CL_VOL_NS 6  // (5 - 8 within 0.5 us with one CTA per SM; 3 was best at two CTAs per SM)
 #endif
 #ifndef B2CL_VOL_SETUP
 #define B2CL_VOL_SETUP 0.0  // the stencil kernel's chunk cost for vol_plan (0: balanced rounds)
@@ -63,16 +64,16 @@ using namespace dev;
 #define B2CL_VOL_MIN_STEPS 8
 #endif
 #ifndef B2CL_VOL_MINB
-#define B2CL_VOL_MINB 2
+#define B2CL_VOL_MINB 1  // one CTA of 13 warps per SM: 123 registers, no spill (two 9-warp CTAs: 96 and a spill, 183.7 vs 176.7 us)
 #endif
 #ifndef B2CL_VOL_XW
-#define B2CL_VOL_XW 2
+#define B2CL_VOL_XW 4
 #endif
 constexpr int VOL_XW = B2CL_VOL_XW;       // consumer warps across x (1: TMA boxes; 4: row copies)
 static_assert(VOL_XW == 1 || B2CL_VOL_BULK, "a TMA box is at most 256 texels wide");
 constexpr int VT_W = 128 * VOL_XW;        // output columns per tile (32 lanes x 4 per warp)
 #ifndef B2CL_VOL_YW
-#define B2CL_VOL_YW 4
+#define B2CL_VOL_YW 3
 #endif
 constexpr int VOL_YW = B2CL_VOL_YW;       // consumer warps down y
 constexpr int VOL_CW = VOL_XW * VOL_YW;   // consumer warps
@@ -168,7 +169,7 @@ __device__ __forceinline__ bool vol_in_window(const SampleParams& p, int xc, int
   return ok;
 }
 
-// Work split.  Tiles are (tx, ty, zc): 128 x 16 output columns/rows and a
+// Work split.  Tiles are (tx, ty, zc): VT_W x VT_H output columns/rows and a
 // chunk of `walk` output slices, ordered tx fastest, then ty, then zc, and
 // dealt round-robin to a persistent grid, so the CTAs resident at any time
 // read neighbouring boxes of the same slices (DRAM pages and the shared halo
