@@ -589,6 +589,9 @@ __global__ void __launch_bounds__(128) k_sample_grid_tile(const SampleParams p) 
 //   Primary columns: xp in [0, Px) maps to x = xp for xp < Ax, else
 //   Mx + 1 + (xp - Ax) (the columns whose mirror image is outside the
 //   output); column x's partner Mx - x is used when inside [0, ow) and != x.
+// Once the box origin is known, each row's two texel rows are turned into
+// shared-memory addresses and its output row into a global row pointer, so
+// the blend loop addresses a tap with one add and a store with one 64-bit add.
 #ifndef B2CL_FOLD_UNROLL
 #define B2CL_FOLD_UNROLL 1
 #endif
@@ -607,10 +610,7 @@ struct FoldMap {
 __device__ __forceinline__ int fold_prim(int pi, int M, int A) { return pi < A ? pi : M + 1 + (pi - A); }
 
 #ifndef B2CL_FOLD_MINB
-#define B2CL_FOLD_MINB 1
-#endif
-#ifndef B2CL_FOLD_PAIRED
-#define B2CL_FOLD_PAIRED 0  // 1: the blends on channel pairs (FFMA2 / FMUL2): measured 70.6 vs 62.0 us
+#define B2CL_FOLD_MINB 5  // 5 CTAs of 4 warps per SM: at most 96 registers (1: 104 registers, 4 CTAs; 6 / 7: 80 / 72 -- 59.6 / 58.6 / 59.2 vs 57.8 us)
 #endif
 #ifndef B2CL_FOLD_CTAS
 #define B2CL_FOLD_CTAS 0  // persistent CTAs per SM for the fold kernel (0: one CTA per tile)
@@ -621,21 +621,222 @@ __device__ __forceinline__ int fold_prim(int pi, int M, int A) { return pi < A ?
 #ifndef B2CL_FOLD_TMA
 #define B2CL_FOLD_TMA 0  // 1: stage the union box with one cp.async.bulk.tensor.3d (measured 61.5 vs 58.2 us for the 16-B cp.async)
 #endif
+#ifndef B2CL_FOLD_PAD
+#define B2CL_FOLD_PAD 6
+#endif
+// the staged box: the tile's taps plus room for the mirror images' offsets
+constexpr int FOLD_TW = 64, FOLD_TH = 16, FOLD_BW = FOLD_TW + B2CL_FOLD_PAD, FOLD_BH = FOLD_TH + B2CL_FOLD_PAD;
+
+// one tile's tables: [0] primary, [1] partner; x / y = -1 marks an absent output
+struct FoldTables {
+  float4 rT[2][FOLD_TH];  // per row: {b, 1 - b, j0, j1} -- j as int bits, or (staged tiles, after
+                          // fold_rows_addr) the shared addresses of box rows j0, j1
+  uint64_t rO[2][FOLD_TH];  // per row (staged tiles): the output row's address
+  int cI0[2][FOLD_TW], cI1[2][FOLD_TW], cX[2][FOLD_TW];
+  float cA[2][FOLD_TW], cOma[2][FOLD_TW];
+  int rY[2][FOLD_TH];
+  int rflag[2][2];  // per row set and 8-row block: 1 chained up, 2 down, 0 neither / absent rows
+};
+
+// column c of table h of the tile whose primary columns start at xp0; the
+// tap range joins [lo, hi]
+template <class C>
+__device__ __forceinline__ void fold_col(const SampleParams& p, const FoldMap& fm, FoldTables& T, int h, int c,
+                                         int xp0, int& lo, int& hi) {
+  const int xp = xp0 + c;
+  int x = xp < fm.Px ? fold_prim(xp, fm.Mx, fm.Ax) : -1;
+  if (h == 1 && x >= 0) {
+    const int xm = fm.Mx - x;
+    x = (xm >= 0 && xm < p.ow && xm != x) ? xm : -1;
+  }
+  T.cX[h][c] = x;
+  if (x >= 0) {
+    const AxL ax = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(p.ox + x)), p.A[3]), p.im.w);
+    T.cI0[h][c] = ax.i0; T.cI1[h][c] = ax.i1; T.cA[h][c] = ax.a; T.cOma[h][c] = ax.oma;
+    lo = min(lo, min(ax.i0, ax.i1));
+    hi = max(hi, max(ax.i0, ax.i1));
+  } else {
+    T.cI0[h][c] = T.cI1[h][c] = 0x3fffffff;  // (never staged, never stored)
+    T.cA[h][c] = 0.f; T.cOma[h][c] = 1.f;
+  }
+}
+
+// the rows of the tile whose primary rows start at yp0: called by one full
+// warp, lane = hr * 16 + r computes row r of table hr and (warp ballots) the
+// walk direction of each 8-row block of each row set -- all rows present and
+// chained UP (j1 of a row = j0 of the next) or DOWN (j0 = j1 of the next)
+template <class C>
+__device__ __forceinline__ void fold_rows(const SampleParams& p, const FoldMap& fm, FoldTables& T, int lane,
+                                          int yp0, int& lo, int& hi) {
+  const int hr = lane / FOLD_TH, r = lane % FOLD_TH;
+  const int yp = yp0 + r;
+  int y = yp < fm.Py ? fold_prim(yp, fm.My, fm.Ay) : -1;
+  if (hr == 1 && y >= 0) {
+    const int ym = fm.My - y;
+    y = (ym >= 0 && ym < p.oh && ym != y) ? ym : -1;
+  }
+  T.rY[hr][r] = y;
+  int j0 = 0, j1 = 0;
+  if (y >= 0) {
+    const AxL ay = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(p.oy + y)), p.A[7]), p.im.h);
+    T.rT[hr][r] = make_float4(ay.a, ay.oma, __int_as_float(ay.i0), __int_as_float(ay.i1));
+    lo = min(lo, min(ay.i0, ay.i1));
+    hi = max(hi, max(ay.i0, ay.i1));
+    j0 = ay.i0;
+    j1 = ay.i1;
+  }
+  const int nj0 = __shfl_down_sync(0xffffffffu, j0, 1), nj1 = __shfl_down_sync(0xffffffffu, j1, 1);
+  const bool last = (r & 7) == 7;
+  const unsigned pres = __ballot_sync(0xffffffffu, y >= 0);
+  const unsigned upm = __ballot_sync(0xffffffffu, last || j1 == nj0);
+  const unsigned dnm = __ballot_sync(0xffffffffu, last || j0 == nj1);
+  if ((r & 7) == 0) {
+    const unsigned m = 0xffu << lane;
+    T.rflag[hr][r >> 3] = ((pres & m) == m) ? (((upm & m) == m) ? 1 : (((dnm & m) == m) ? 2 : 0)) : 0;
+  }
+}
+
+// a staged tile's rows (same lanes as fold_rows, after the box origin r0 is
+// known): texel rows j0, j1 -> shared addresses of box rows j - r0; output
+// row y -> its address in the output slice `out`
+__device__ __forceinline__ void fold_rows_addr(const SampleParams& p, FoldTables& T, int lane, uint32_t box_s,
+                                               int r0, const float4* out) {
+  const int hr = lane / FOLD_TH, r = lane % FOLD_TH;
+  const int y = T.rY[hr][r];
+  if (y < 0) return;
+  const float4 t = T.rT[hr][r];
+  const uint32_t a0 = box_s + (uint32_t)(__float_as_int(t.z) - r0) * (FOLD_BW * 16u);
+  const uint32_t a1 = box_s + (uint32_t)(__float_as_int(t.w) - r0) * (FOLD_BW * 16u);
+  T.rT[hr][r] = make_float4(t.x, t.y, __uint_as_float(a0), __uint_as_float(a1));
+  T.rO[hr][r] = reinterpret_cast<uint64_t>(out + (uint64_t)y * p.ow);
+}
+
+__device__ __forceinline__ float4 lds_f4(uint32_t a) {
+  float4 v;
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(a));
+  return v;
+}
+
+// one warp's unit of a tile: column c (this lane) of column set hc, rows rb ..
+// rb + 7 of row set hr; from the box (origin column c0) when staged, else
+// the taps directly.  out = the output slice of the tile.
+template <class C>
+__device__ __forceinline__ void fold_unit(const SampleParams& p, const FoldTables& T, int c0, bool staged,
+                                          float4* out, int c, int rb, int hc, int hr) {
+  const Image& im = p.im;
+  const int x = T.cX[hc][c];
+  if (x < 0) return;  // (an absent column: nothing to store)
+  const int i0 = T.cI0[hc][c], i1 = T.cI1[hc][c];
+  const float a = T.cA[hc][c], oma = T.cOma[hc][c];
+  if (!staged) {  // the taps directly
+    const AxL ax{i0, i1, a, oma, true, true};
+#pragma unroll 1
+    for (int r = rb; r < rb + FOLD_TH / 2; ++r) {
+      const int y = T.rY[hr][r];
+      if (y < 0) continue;
+      const float4 ry = T.rT[hr][r];
+      const char* rows[4] = {row_ptr<C>(im, __float_as_int(ry.z), 0), row_ptr<C>(im, __float_as_int(ry.w), 0),
+                             nullptr, nullptr};
+      const bool rok[4] = {true, true, false, false};
+      uint32_t res[4];
+      linear_at<C>(p, rows, rok, ax, ry.x, ry.y, 0.f, 1.f, res, 4);
+      __stcs(out + ((uint64_t)y * p.ow + x), make_float4(__uint_as_float(res[0]), __uint_as_float(res[1]),
+                                                           __uint_as_float(res[2]), __uint_as_float(res[3])));
+    }
+    return;
+  }
+  // byte offsets of this column's two taps within a staged row, and of its
+  // output within an output row
+  const uint32_t o0 = (uint32_t)(i0 - c0) * 16u, o1 = (uint32_t)(i1 - c0) * 16u;
+  const uint64_t xo = (uint64_t)(unsigned)x * 16u;
+  auto xblend = [&](float rowaddr, float4& h) {
+    const uint32_t ra = __float_as_uint(rowaddr);
+    const float4 t0 = lds_f4(ra + o0);
+    const float4 t1 = lds_f4(ra + o1);
+    h = make_float4(lerp1(a, oma, t0.x, t1.x), lerp1(a, oma, t0.y, t1.y), lerp1(a, oma, t0.z, t1.z),
+                    lerp1(a, oma, t0.w, t1.w));
+  };
+  auto emit = [&](int r, const float4& ry, const float4& n0, const float4& n1) {
+    __stcs(reinterpret_cast<float4*>(T.rO[hr][r] + xo),
+           make_float4(lerp1(ry.x, ry.y, n0.x, n1.x), lerp1(ry.x, ry.y, n0.y, n1.y), lerp1(ry.x, ry.y, n0.z, n1.z),
+                       lerp1(ry.x, ry.y, n0.w, n1.w)));
+  };
+  // the unit's 8 rows: all present and chained one way, so each texel row is
+  // x-blended once; otherwise both taps per row
+  const int flag = T.rflag[hr][rb >> 3];
+  auto walk = [&](auto upc) {
+    constexpr bool UP = decltype(upc)::value;
+    float4 hp;  // x-blend of the texel row shared with the previous output row
+    {
+      const float4 ry = T.rT[hr][rb];
+      xblend(UP ? ry.z : ry.w, hp);
+    }
+#pragma unroll kFoldWalkUnroll
+    for (int r = rb; r < rb + FOLD_TH / 2; ++r) {
+      const float4 ry = T.rT[hr][r];
+      float4 hn;
+      xblend(UP ? ry.w : ry.z, hn);
+      if (UP) emit(r, ry, hp, hn);
+      else emit(r, ry, hn, hp);
+      hp = hn;
+    }
+  };
+  if (flag == 1) {
+    walk(std::true_type{});
+  } else if (flag == 2) {
+    walk(std::false_type{});
+  } else {
+#pragma unroll 1
+    for (int r = rb; r < rb + FOLD_TH / 2; ++r) {
+      if (T.rY[hr][r] < 0) continue;  // (warp-uniform)
+      const float4 ry = T.rT[hr][r];
+      float4 n0, n1;
+      xblend(ry.z, n0);
+      xblend(ry.w, n1);
+      emit(r, ry, n0, n1);
+    }
+  }
+}
+
+// an estimate of the union box of tile (fx, fy) from the taps of the ends of
+// its primary column / row segments, widened by one texel (for the L2
+// prefetch of a later tile): called by a full warp, lanes 0-3 columns and 4-7
+// rows; {c_lo, c_hi, r_lo, r_hi} clipped to the image, in every lane
+template <class C>
+__device__ __forceinline__ int4 fold_predict_box(const SampleParams& p, const FoldMap& fm, int fx, int fy, int lane) {
+  const bool rowax = lane >= 4;
+  const int k = lane & 3;
+  const int base = rowax ? fy * FOLD_TH : fx * FOLD_TW, len = rowax ? FOLD_TH : FOLD_TW, P = rowax ? fm.Py : fm.Px;
+  const int Aseg = rowax ? fm.Ay : fm.Ax, M = rowax ? fm.My : fm.Mx;
+  int pi = k == 0 ? base : (k == 1 ? base + len - 1 : (k == 2 ? Aseg - 1 : Aseg));
+  pi = min(max(pi, base), min(base + len, P) - 1);
+  int lo = 0x7fffffff, hi = -1;
+  if (lane < 8 && pi >= 0) {
+    const int o = fold_prim(pi, M, Aseg);
+    const float cc = rowax ? __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(p.oy + o)), p.A[7])
+                           : __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(p.ox + o)), p.A[3]);
+    const AxL a = axis_l<C>(p.smp, cc, rowax ? p.im.h : p.im.w);
+    lo = min(a.i0, a.i1);
+    hi = max(a.i0, a.i1);
+  }
+#pragma unroll
+  for (int o = 1; o < 4; o <<= 1) {
+    lo = min(lo, __shfl_xor_sync(0xffffffffu, lo, o));
+    hi = max(hi, __shfl_xor_sync(0xffffffffu, hi, o));
+  }
+  const int clo = __shfl_sync(0xffffffffu, lo, 0) - 1, chi = __shfl_sync(0xffffffffu, hi, 0) + 1;
+  const int rlo = __shfl_sync(0xffffffffu, lo, 4) - 1, rhi = __shfl_sync(0xffffffffu, hi, 4) + 1;
+  return make_int4(max(clo, 0), min(chi, p.im.w - 1), max(rlo, 0), min(rhi, p.im.h - 1));
+}
+
 template <class C>
 __global__ void __launch_bounds__(128, B2CL_FOLD_MINB)
     k_sample_grid_fold(const SampleParams p, const FoldMap fm, const __grid_constant__ CUtensorMap tmap) {
   static_assert(C::type == T_FLOAT && C::order == O_RGBA && C::dims == 2, "2D RGBA32F");
   static_assert(C::addr == A_REPEAT || C::addr == A_MIRROR, "taps always in range");
-#ifndef B2CL_FOLD_PAD
-#define B2CL_FOLD_PAD 6
-#endif
-  // the staged box: the tile's taps plus room for the mirror images' offsets
-  constexpr int TW = 64, TH = 16, BW = TW + B2CL_FOLD_PAD, BH = TH + B2CL_FOLD_PAD;
+  constexpr int TW = FOLD_TW, TH = FOLD_TH, BW = FOLD_BW, BH = FOLD_BH;
   __shared__ __align__(128) float4 box[BH][BW];
-  __shared__ int cI0[2][TW], cI1[2][TW], cX[2][TW], rY[2][TH];
-  __shared__ float cA[2][TW], cOma[2][TW];
-  __shared__ float4 rT[2][TH];  // per row: {b, 1 - b, j0 bits, j1 bits}
-  __shared__ int rflag[2][2];   // per row set and 8-row block: 1 chained up, 2 down, 0 neither / absent rows
+  __shared__ FoldTables T;
   __shared__ int bb[4];         // column min, max, row min, max of the staged box
   __shared__ uint64_t fbar;     // the TMA box's completion
   const Image& im = p.im;
@@ -650,93 +851,35 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB)
   const int xp0 = BX * TW, yp0 = BY * TH;
   if (tid == 0) { bb[0] = 0x7fffffff; bb[1] = -1; bb[2] = 0x7fffffff; bb[3] = -1; }
   __syncthreads();
-  // tables: [0] primary, [1] partner; x / y = -1 marks an absent output
   {
-    const int h = tid >> 6, c = tid & 63;  // 128 threads: 64 columns x {primary, partner}
-    const int xp = xp0 + c;
-    int x = xp < fm.Px ? fold_prim(xp, fm.Mx, fm.Ax) : -1;
-    if (h == 1 && x >= 0) {
-      const int xm = fm.Mx - x;
-      x = (xm >= 0 && xm < p.ow && xm != x) ? xm : -1;
+    // 128 threads: 64 columns x {primary, partner}; warp 0 also the rows
+    int lo = 0x7fffffff, hi = -1;
+    fold_col<C>(p, fm, T, tid >> 6, tid & 63, xp0, lo, hi);
+    if (hi >= 0) {
+      atomicMin(&bb[0], lo);
+      atomicMax(&bb[1], hi);
     }
-    cX[h][c] = x;
-    if (x >= 0) {
-      const AxL ax = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(p.ox + x)), p.A[3]), im.w);
-      cI0[h][c] = ax.i0; cI1[h][c] = ax.i1; cA[h][c] = ax.a; cOma[h][c] = ax.oma;
-      atomicMin(&bb[0], min(ax.i0, ax.i1));
-      atomicMax(&bb[1], max(ax.i0, ax.i1));
-    } else {
-      cI0[h][c] = cI1[h][c] = 0x3fffffff;  // (never staged, never stored)
-      cA[h][c] = 0.f; cOma[h][c] = 1.f;
-    }
-    if (tid < 2 * TH) {
-      const int hr = tid / TH, r = tid % TH;
-      const int yp = yp0 + r;
-      int y = yp < fm.Py ? fold_prim(yp, fm.My, fm.Ay) : -1;
-      if (hr == 1 && y >= 0) {
-        const int ym = fm.My - y;
-        y = (ym >= 0 && ym < p.oh && ym != y) ? ym : -1;
-      }
-      rY[hr][r] = y;
-      int j0 = 0, j1 = 0;
-      if (y >= 0) {
-        const AxL ay = axis_l<C>(p.smp, __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(p.oy + y)), p.A[7]), im.h);
-        rT[hr][r] = make_float4(ay.a, ay.oma, __int_as_float(ay.i0), __int_as_float(ay.i1));
-        atomicMin(&bb[2], min(ay.i0, ay.i1));
-        atomicMax(&bb[3], max(ay.i0, ay.i1));
-        j0 = ay.i0;
-        j1 = ay.i1;
-      }
-      // the walk direction of each 8-row block of each row set, once per CTA
-      // (warp 0 = these 32 threads: lane = hr * 16 + r): all rows present and
-      // chained UP (j1 of a row = j0 of the next) or DOWN (j0 = j1 of the next)
-      const int nj0 = __shfl_down_sync(0xffffffffu, j0, 1), nj1 = __shfl_down_sync(0xffffffffu, j1, 1);
-      const bool last = (r & 7) == 7;
-      const unsigned pres = __ballot_sync(0xffffffffu, y >= 0);
-      const unsigned upm = __ballot_sync(0xffffffffu, last || j1 == nj0);
-      const unsigned dnm = __ballot_sync(0xffffffffu, last || j0 == nj1);
-      if ((r & 7) == 0) {
-        const unsigned m = 0xffu << tid;
-        rflag[hr][r >> 3] = ((pres & m) == m) ? (((upm & m) == m) ? 1 : (((dnm & m) == m) ? 2 : 0)) : 0;
+    if (warp == 0) {
+      int rlo = 0x7fffffff, rhi = -1;
+      fold_rows<C>(p, fm, T, lane, yp0, rlo, rhi);
+      if (rhi >= 0) {
+        atomicMin(&bb[2], rlo);
+        atomicMax(&bb[3], rhi);
       }
     }
   }
 #if B2CL_FOLD_PF
-  // warm L2 with the box of the tile B2CL_FOLD_PF launch positions ahead:
-  // warp 3 estimates it from the taps of that tile's first / last primary
-  // columns and rows and of the primary segments' ends (a prefetch only; the
-  // tile's own box is computed exactly when it runs)
+  // warm L2 with the box of the tile B2CL_FOLD_PF launch positions ahead
+  // (an estimate: a prefetch only; the tile's own box is computed exactly
+  // when it runs)
   if (warp == 3 && !C::shard) {
     const long long t = tile + B2CL_FOLD_PF;
     if (t < ntiles) {
-      const int fx = (int)(t % fm.gx), fy = (int)((t / fm.gx) % fm.gy);
-      const bool rowax = lane >= 4;
-      const int k = lane & 3;
-      const int base = rowax ? fy * TH : fx * TW, len = rowax ? TH : TW, P = rowax ? fm.Py : fm.Px;
-      const int Aseg = rowax ? fm.Ay : fm.Ax, M = rowax ? fm.My : fm.Mx;
-      int pi = k == 0 ? base : (k == 1 ? base + len - 1 : (k == 2 ? Aseg - 1 : Aseg));
-      pi = min(max(pi, base), min(base + len, P) - 1);
-      int lo = 0x7fffffff, hi = -1;
-      if (lane < 8 && pi >= 0) {
-        const int o = fold_prim(pi, M, Aseg);
-        const float cc = rowax ? __fadd_rn(__fmul_rn(p.A[5], __int2float_rn(p.oy + o)), p.A[7])
-                               : __fadd_rn(__fmul_rn(p.A[0], __int2float_rn(p.ox + o)), p.A[3]);
-        const AxL a = axis_l<C>(p.smp, cc, rowax ? im.h : im.w);
-        lo = min(a.i0, a.i1);
-        hi = max(a.i0, a.i1);
-      }
-#pragma unroll
-      for (int o = 1; o < 4; o <<= 1) {
-        lo = min(lo, __shfl_xor_sync(0xffffffffu, lo, o));
-        hi = max(hi, __shfl_xor_sync(0xffffffffu, hi, o));
-      }
-      const int clo = __shfl_sync(0xffffffffu, lo, 0) - 1, chi = __shfl_sync(0xffffffffu, hi, 0) + 1;
-      const int rlo = __shfl_sync(0xffffffffu, lo, 4) - 1, rhi = __shfl_sync(0xffffffffu, hi, 4) + 1;
-      const int ca = max(clo, 0), cb = min(chi, im.w - 1), ra = max(rlo, 0), rbb = min(rhi, im.h - 1);
-      if (cb >= ca && rbb >= ra && cb - ca < BW + 8 && rbb - ra < BH + 8 && ra + lane <= rbb)
+      const int4 e = fold_predict_box<C>(p, fm, (int)(t % fm.gx), (int)((t / fm.gx) % fm.gy), lane);
+      if (e.y >= e.x && e.w >= e.z && e.y - e.x < BW + 8 && e.w - e.z < BH + 8 && e.z + lane <= e.w)
         asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(
-                         row_ptr<C>(im, ra + lane, 0) + (uint64_t)(unsigned)ca * 16u),
-                     "r"((uint32_t)(cb - ca + 1) * 16u)
+                         row_ptr<C>(im, e.z + lane, 0) + (uint64_t)(unsigned)e.x * 16u),
+                     "r"((uint32_t)(e.y - e.x + 1) * 16u)
                      : "memory");
     }
   }
@@ -759,117 +902,22 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB)
     const int nc = bb[1] - c0 + 1, nr = bb[3] - r0 + 1;
     for (int rr = warp; rr < nr; rr += 4) {
       const char* src = row_ptr<C>(im, r0 + rr, 0) + (uint64_t)(unsigned)c0 * 16u;
-      const uint32_t dst = static_cast<uint32_t>(__cvta_generic_to_shared(&box[rr][0]));
+      const uint32_t dst = smem_u32(&box[rr][0]);
       for (int cc = lane; cc < nc; cc += 32)
         asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst + cc * 16), "l"(src + cc * 16)
                      : "memory");
     }
-    asm volatile("cp.async.wait_all;" ::: "memory");
   }
+  if (staged && warp == 0) fold_rows_addr(p, T, lane, smem_u32(&box[0][0]), r0, out);
+  if (staged && !kTma) asm volatile("cp.async.wait_all;" ::: "memory");
   __syncthreads();
   if (staged && kTma) mbar_wait(&fbar, 0);
   // warp w: columns (w & 1)*32 + lane, rows (w >> 1)*8 .. +8, for each of the
   // four (column set, row set) combinations
   const int c = (warp & 1) * 32 + lane, rb = (warp >> 1) * (TH / 2);
 #pragma unroll kFoldUnroll
-  for (int combo = 0; combo < 4; ++combo) {
-    const int hc = combo & 1, hr = combo >> 1;
-    const int x = cX[hc][c];
-    const int i0 = cI0[hc][c], i1 = cI1[hc][c];
-    const float a = cA[hc][c], oma = cOma[hc][c];
-    if (!staged) {  // the taps directly
-      if (x < 0) continue;
-      const AxL ax{i0, i1, a, oma, true, true};
-#pragma unroll 1
-      for (int r = rb; r < rb + TH / 2; ++r) {
-        const int y = rY[hr][r];
-        if (y < 0) continue;
-        const float4 ry = rT[hr][r];
-        const char* rows[4] = {row_ptr<C>(im, __float_as_int(ry.z), 0), row_ptr<C>(im, __float_as_int(ry.w), 0),
-                               nullptr, nullptr};
-        const bool rok[4] = {true, true, false, false};
-        uint32_t res[4];
-        linear_at<C>(p, rows, rok, ax, ry.x, ry.y, 0.f, 1.f, res, 4);
-        __stcs(out + ((uint64_t)y * p.ow + x), make_float4(__uint_as_float(res[0]), __uint_as_float(res[1]),
-                                                             __uint_as_float(res[2]), __uint_as_float(res[3])));
-      }
-      continue;
-    }
-    // byte offsets of this column's two taps within a staged row (absent
-    // columns read slot 0 and store nothing)
-    const uint32_t o0 = x >= 0 ? (uint32_t)(i0 - c0) * 16u : 0u, o1 = x >= 0 ? (uint32_t)(i1 - c0) * 16u : 0u;
-    const char* bbase = reinterpret_cast<const char*>(&box[0][0]);
-#if B2CL_FOLD_PAIRED
-    // lerp1 on channel pairs (x, y) and (z, w): FMUL2 + FFMA2, each lane the
-    // same IEEE mul / fma as lerp1 (a mul feeding an fma's addend: nothing fuses)
-    const float2 a2 = make_float2(a, a), oma2 = make_float2(oma, oma);
-    auto xblend = [&](int j, float4& h) {
-      const char* row = bbase + (uint32_t)(j - r0) * (BW * 16);
-      const float4 t0 = *reinterpret_cast<const float4*>(row + o0);
-      const float4 t1 = *reinterpret_cast<const float4*>(row + o1);
-      const float2 lo = __ffma2_rn(a2, make_float2(t1.x, t1.y), __fmul2_rn(oma2, make_float2(t0.x, t0.y)));
-      const float2 hi = __ffma2_rn(a2, make_float2(t1.z, t1.w), __fmul2_rn(oma2, make_float2(t0.z, t0.w)));
-      h = make_float4(lo.x, lo.y, hi.x, hi.y);
-    };
-    auto emit = [&](int y, const float4& ry, const float4& n0, const float4& n1) {
-      const float2 b2 = make_float2(ry.x, ry.x), omb2 = make_float2(ry.y, ry.y);
-      const float2 lo = __ffma2_rn(b2, make_float2(n1.x, n1.y), __fmul2_rn(omb2, make_float2(n0.x, n0.y)));
-      const float2 hi = __ffma2_rn(b2, make_float2(n1.z, n1.w), __fmul2_rn(omb2, make_float2(n0.z, n0.w)));
-      if (x >= 0) __stcs(out + ((uint64_t)y * p.ow + x), make_float4(lo.x, lo.y, hi.x, hi.y));
-    };
-#else
-    auto xblend = [&](int j, float4& h) {
-      const char* row = bbase + (uint32_t)(j - r0) * (BW * 16);
-      const float4 t0 = *reinterpret_cast<const float4*>(row + o0);
-      const float4 t1 = *reinterpret_cast<const float4*>(row + o1);
-      h = make_float4(lerp1(a, oma, t0.x, t1.x), lerp1(a, oma, t0.y, t1.y), lerp1(a, oma, t0.z, t1.z),
-                      lerp1(a, oma, t0.w, t1.w));
-    };
-    auto emit = [&](int y, const float4& ry, const float4& n0, const float4& n1) {
-      if (x >= 0)
-        __stcs(out + ((uint64_t)y * p.ow + x), make_float4(lerp1(ry.x, ry.y, n0.x, n1.x), lerp1(ry.x, ry.y, n0.y, n1.y),
-                                                           lerp1(ry.x, ry.y, n0.z, n1.z), lerp1(ry.x, ry.y, n0.w, n1.w)));
-    };
-#endif
-    // the warp's 8 rows of this row set: all present and chained one way
-    // (j1 of a row = j0 of the next: UP; j0 = j1 of the next: DOWN), so each
-    // texel row is x-blended once; otherwise both taps per row
-    const int flag = rflag[hr][rb >> 3];  // (computed with the row tables)
-    const bool all = flag != 0, up = flag == 1, dn = flag == 2;
-    auto walk = [&](auto upc) {
-      constexpr bool UP = decltype(upc)::value;
-      float4 hp;  // x-blend of the texel row shared with the previous output row
-      {
-        const float4 ry = rT[hr][rb];
-        xblend(__float_as_int(UP ? ry.z : ry.w), hp);
-      }
-#pragma unroll kFoldWalkUnroll
-      for (int r = rb; r < rb + TH / 2; ++r) {
-        const float4 ry = rT[hr][r];
-        float4 hn;
-        xblend(__float_as_int(UP ? ry.w : ry.z), hn);
-        if (UP) emit(rY[hr][r], ry, hp, hn);
-        else emit(rY[hr][r], ry, hn, hp);
-        hp = hn;
-      }
-    };
-    if (all && up) {
-      walk(std::true_type{});
-    } else if (all && dn) {
-      walk(std::false_type{});
-    } else {
-#pragma unroll 1
-      for (int r = rb; r < rb + TH / 2; ++r) {
-        const int y = rY[hr][r];
-        if (y < 0) continue;  // (warp-uniform)
-        const float4 ry = rT[hr][r];
-        float4 n0, n1;
-        xblend(__float_as_int(ry.z), n0);
-        xblend(__float_as_int(ry.w), n1);
-        emit(y, ry, n0, n1);
-      }
-    }
-  }
+  for (int combo = 0; combo < 4; ++combo)
+    fold_unit<C>(p, T, c0, staged, out, c, rb, combo & 1, combo >> 1);
   __syncthreads();  // (the next tile of a persistent CTA reuses the tables and the box)
   }
 }

@@ -204,6 +204,9 @@ GRID_CASES = [
     (2, RGBA, F32, (257, 129, 1), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "fold-exact", (257, 129, 1), 4),
     (2, RGBA, F32, (200, 150, 1), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "fold-edge", (200, 150, 1), 4),
     (2, RGBA, F32, (160, 96, 1), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "translate", (160, 96, 3), 4),
+    # 1024 fold tiles (several waves of CTAs, tables turned into box / output
+    # addresses per tile)
+    (2, RGBA, F32, (2048, 2048, 1), (1, cl.CL_ADDRESS_MIRRORED_REPEAT, cl.CL_FILTER_LINEAR), "translate", (2048, 2048, 1), 4),
     # rotated-map staged kernel (k_sample_grid_volr): ragged tiles, the corners
     # clamped to the edges; 3x minification (footprint larger than the box:
     # direct tiles); z at half scale (repeated slice pairs)
