@@ -622,10 +622,13 @@ __device__ __forceinline__ int fold_prim(int pi, int M, int A) { return pi < A ?
 #define B2CL_FOLD_TMA 0  // 1: stage the union box with one cp.async.bulk.tensor.3d (measured 61.5 vs 58.2 us for the 16-B cp.async)
 #endif
 #ifndef B2CL_FOLD_PAD
-#define B2CL_FOLD_PAD 6
+#define B2CL_FOLD_PAD 6  // (4 / 5 / 8 within 0.3 us)
 #endif
 // the staged box: the tile's taps plus room for the mirror images' offsets
-constexpr int FOLD_TW = 64, FOLD_TH = 16, FOLD_BW = FOLD_TW + B2CL_FOLD_PAD, FOLD_BH = FOLD_TH + B2CL_FOLD_PAD;
+#ifndef B2CL_FOLD_TH
+#define B2CL_FOLD_TH 16  // primary rows per tile (16 or 32; 32 measured 58.4-60.2 vs 57.7 us)
+#endif
+constexpr int FOLD_TW = 64, FOLD_TH = B2CL_FOLD_TH, FOLD_BW = FOLD_TW + B2CL_FOLD_PAD, FOLD_BH = FOLD_TH + B2CL_FOLD_PAD;
 
 // one tile's tables: [0] primary, [1] partner; x / y = -1 marks an absent output
 struct FoldTables {
@@ -635,7 +638,7 @@ struct FoldTables {
   int cI0[2][FOLD_TW], cI1[2][FOLD_TW], cX[2][FOLD_TW];
   float cA[2][FOLD_TW], cOma[2][FOLD_TW];
   int rY[2][FOLD_TH];
-  int rflag[2][2];  // per row set and 8-row block: 1 chained up, 2 down, 0 neither / absent rows
+  int rflag[2][FOLD_TH / 8];  // per row set and 8-row block: 1 chained up, 2 down, 0 neither / absent rows
 };
 
 // column c of table h of the tile whose primary columns start at xp0; the
@@ -661,14 +664,14 @@ __device__ __forceinline__ void fold_col(const SampleParams& p, const FoldMap& f
   }
 }
 
-// the rows of the tile whose primary rows start at yp0: called by one full
-// warp, lane = hr * 16 + r computes row r of table hr and (warp ballots) the
+// the rows of the tile whose primary rows start at yp0: called by 2 * FOLD_TH
+// threads (full warps), idx = hr * FOLD_TH + r computes row r of table hr and (warp ballots) the
 // walk direction of each 8-row block of each row set -- all rows present and
 // chained UP (j1 of a row = j0 of the next) or DOWN (j0 = j1 of the next)
 template <class C>
-__device__ __forceinline__ void fold_rows(const SampleParams& p, const FoldMap& fm, FoldTables& T, int lane,
+__device__ __forceinline__ void fold_rows(const SampleParams& p, const FoldMap& fm, FoldTables& T, int idx,
                                           int yp0, int& lo, int& hi) {
-  const int hr = lane / FOLD_TH, r = lane % FOLD_TH;
+  const int hr = idx / FOLD_TH, r = idx % FOLD_TH, lane = idx & 31;
   const int yp = yp0 + r;
   int y = yp < fm.Py ? fold_prim(yp, fm.My, fm.Ay) : -1;
   if (hr == 1 && y >= 0) {
@@ -699,9 +702,9 @@ __device__ __forceinline__ void fold_rows(const SampleParams& p, const FoldMap& 
 // a staged tile's rows (same lanes as fold_rows, after the box origin r0 is
 // known): texel rows j0, j1 -> shared addresses of box rows j - r0; output
 // row y -> its address in the output slice `out`
-__device__ __forceinline__ void fold_rows_addr(const SampleParams& p, FoldTables& T, int lane, uint32_t box_s,
+__device__ __forceinline__ void fold_rows_addr(const SampleParams& p, FoldTables& T, int idx, uint32_t box_s,
                                                int r0, const float4* out) {
-  const int hr = lane / FOLD_TH, r = lane % FOLD_TH;
+  const int hr = idx / FOLD_TH, r = idx % FOLD_TH;
   const int y = T.rY[hr][r];
   if (y < 0) return;
   const float4 t = T.rT[hr][r];
@@ -761,18 +764,17 @@ __device__ __forceinline__ void fold_unit(const SampleParams& p, const FoldTable
            make_float4(lerp1(ry.x, ry.y, n0.x, n1.x), lerp1(ry.x, ry.y, n0.y, n1.y), lerp1(ry.x, ry.y, n0.z, n1.z),
                        lerp1(ry.x, ry.y, n0.w, n1.w)));
   };
-  // the unit's 8 rows: all present and chained one way, so each texel row is
-  // x-blended once; otherwise both taps per row
-  const int flag = T.rflag[hr][rb >> 3];
-  auto walk = [&](auto upc) {
+  // each 8-row block of the unit: all present and chained one way, so each
+  // texel row is x-blended once; otherwise both taps per row
+  auto walk = [&](int bk, auto upc) {
     constexpr bool UP = decltype(upc)::value;
     float4 hp;  // x-blend of the texel row shared with the previous output row
     {
-      const float4 ry = T.rT[hr][rb];
+      const float4 ry = T.rT[hr][bk];
       xblend(UP ? ry.z : ry.w, hp);
     }
 #pragma unroll kFoldWalkUnroll
-    for (int r = rb; r < rb + FOLD_TH / 2; ++r) {
+    for (int r = bk; r < bk + 8; ++r) {
       const float4 ry = T.rT[hr][r];
       float4 hn;
       xblend(UP ? ry.w : ry.z, hn);
@@ -781,19 +783,23 @@ __device__ __forceinline__ void fold_unit(const SampleParams& p, const FoldTable
       hp = hn;
     }
   };
-  if (flag == 1) {
-    walk(std::true_type{});
-  } else if (flag == 2) {
-    walk(std::false_type{});
-  } else {
 #pragma unroll 1
-    for (int r = rb; r < rb + FOLD_TH / 2; ++r) {
-      if (T.rY[hr][r] < 0) continue;  // (warp-uniform)
-      const float4 ry = T.rT[hr][r];
-      float4 n0, n1;
-      xblend(ry.z, n0);
-      xblend(ry.w, n1);
-      emit(r, ry, n0, n1);
+  for (int bk = rb; bk < rb + FOLD_TH / 2; bk += 8) {
+    const int flag = T.rflag[hr][bk >> 3];
+    if (flag == 1) {
+      walk(bk, std::true_type{});
+    } else if (flag == 2) {
+      walk(bk, std::false_type{});
+    } else {
+#pragma unroll 1
+      for (int r = bk; r < bk + 8; ++r) {
+        if (T.rY[hr][r] < 0) continue;  // (warp-uniform)
+        const float4 ry = T.rT[hr][r];
+        float4 n0, n1;
+        xblend(ry.z, n0);
+        xblend(ry.w, n1);
+        emit(r, ry, n0, n1);
+      }
     }
   }
 }
@@ -859,9 +865,9 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB)
       atomicMin(&bb[0], lo);
       atomicMax(&bb[1], hi);
     }
-    if (warp == 0) {
+    if (tid < 2 * TH) {
       int rlo = 0x7fffffff, rhi = -1;
-      fold_rows<C>(p, fm, T, lane, yp0, rlo, rhi);
+      fold_rows<C>(p, fm, T, tid, yp0, rlo, rhi);
       if (rhi >= 0) {
         atomicMin(&bb[2], rlo);
         atomicMax(&bb[3], rhi);
@@ -908,7 +914,7 @@ __global__ void __launch_bounds__(128, B2CL_FOLD_MINB)
                      : "memory");
     }
   }
-  if (staged && warp == 0) fold_rows_addr(p, T, lane, smem_u32(&box[0][0]), r0, out);
+  if (staged && tid < 2 * TH) fold_rows_addr(p, T, tid, smem_u32(&box[0][0]), r0, out);
   if (staged && !kTma) asm volatile("cp.async.wait_all;" ::: "memory");
   __syncthreads();
   if (staged && kTma) mbar_wait(&fbar, 0);
@@ -1039,7 +1045,7 @@ static bool go_fold(const SampleParams& p, cudaStream_t st, cudaError_t* err) {
   if (!fold_axis((double)p.A[0], (double)p.A[3], p.ox, p.ow, &fm.Mx, &fm.Ax, &fm.Px)) return false;
   if (!fold_axis((double)p.A[5], (double)p.A[7], p.oy, p.oh, &fm.My, &fm.Ay, &fm.Py)) return false;
   fm.gx = (fm.Px + 63) / 64;
-  fm.gy = (fm.Py + 15) / 16;
+  fm.gy = (fm.Py + FOLD_TH - 1) / FOLD_TH;
   fm.gz = p.od;
   dim3 grd(fm.gx, fm.gy, fm.gz);
   static const char* ctas_env = getenv("B2CL_FOLD_CTAS");  // A/B: persistent CTAs per SM (0: one per tile)
@@ -1060,7 +1066,7 @@ static bool go_fold(const SampleParams& p, cudaStream_t st, cudaError_t* err) {
     auto enc = tma_encode_fn();
     const cuuint64_t dims[3] = {4, (cuuint64_t)p.im.w, (cuuint64_t)p.im.h};
     const cuuint64_t strides[2] = {16, p.im.rp};
-    const cuuint32_t box[3] = {4, (cuuint32_t)(64 + B2CL_FOLD_PAD), (cuuint32_t)(16 + B2CL_FOLD_PAD)};
+    const cuuint32_t box[3] = {4, (cuuint32_t)FOLD_BW, (cuuint32_t)FOLD_BH};
     const cuuint32_t es[3] = {1, 1, 1};
     tma = enc && !(reinterpret_cast<uintptr_t>(p.im.ptr) & 15) && !(p.im.rp & 15) &&
           enc(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, p.im.ptr, dims, strides, box, es,

@@ -655,6 +655,10 @@ extern "C" cl_mem clCreateBuffer(cl_context c, cl_mem_flags flags, size_t size, 
   if (host_ptr) {
     DeviceGuard g(ord);
     cudaError_t e = cudaMemcpy(s->ptr, host_ptr, size, cudaMemcpyHostToDevice);
+    // a pageable-source cudaMemcpy returns once the data is staged, before
+    // the DMA lands: wait for it, or a queue's first command (its own
+    // stream) could run before the contents exist
+    if (e == cudaSuccess) e = cudaStreamSynchronize(nullptr);
     if (e != cudaSuccess) { raw_free(*s); delete m; SET_ERR(cuda_err(e)); return nullptr; }
   }
   m->valid = 1ull << ord;
@@ -784,6 +788,8 @@ extern "C" cl_mem clCreateImage(cl_context c, cl_mem_flags flags, const cl_image
                                    L.w * L.fmt.es, L.h, cudaMemcpyHostToDevice);
       if (e != cudaSuccess) { raw_free(*s); delete m; SET_ERR(cuda_err(e)); return nullptr; }
     }
+    const cudaError_t e = cudaStreamSynchronize(nullptr);  // (the DMA has landed: see clCreateBuffer)
+    if (e != cudaSuccess) { raw_free(*s); delete m; SET_ERR(cuda_err(e)); return nullptr; }
   }
   m->valid = 1ull << ord;
   register_mem(m);

@@ -223,6 +223,32 @@ def test_read_write_image_host_pitches(sess, orc):
     sess.release(img)
 
 
+def test_created_contents_visible_to_the_first_command(sess):
+    """clCreateBuffer / clCreateImage with host data: the upload has landed
+    before the call returns, so the queue's first command (its own stream)
+    sees the contents -- a pageable cudaMemcpy returns once the data is
+    staged, before its DMA completes (a race seen once in
+    test_read_write_buffer_rect before the fix)."""
+    g = synth.rng(45)
+    L = cl.lib()
+    for k in range(12):
+        n = (8 << 20) + 16 * k
+        host = _rand_bytes(g, n)
+        ref = host.copy()
+        b = sess.buffer(n, host)
+        host[:] = 0  # (the host copy changes right after creation)
+        out = np.empty(n, np.uint8)
+        cl.check(L.clEnqueueReadBuffer(sess.queue, b, 1, 0, n, out.ctypes.data_as(ctypes.c_void_p), 0, None, None))
+        assert np.array_equal(out, ref), k
+        sess.release(b)
+    W, H = 1024, 512
+    codes = synth.image_codes(g, cl.CL_RGBA, cl.CL_FLOAT, W, H)
+    img = sess.image(cl.CL_RGBA, cl.CL_FLOAT, W, H, host=codes.copy())
+    got = sess.read_image(img, (0, 0, 0), (W, H, 1))
+    assert np.array_equal(got.view(np.uint8).reshape(-1), np.ascontiguousarray(codes).view(np.uint8).reshape(-1))
+    sess.release(img)
+
+
 def test_read_write_buffer_rect(sess, orc):
     g = synth.rng(44)
     n = 64 * 10 * 4
