@@ -36,15 +36,15 @@ def test_release_is_deferred_and_stream_ordered(sess):
     pat = np.array([0x3C], np.uint8)
     cl.check(L.clEnqueueFillBuffer(sess.queue, src, pat.ctypes.data, 1, 1 << 20, n - (1 << 20), 0, None, None))
     sess.finish()
-    # queue several long copies, then release the source while they run
-    for _ in range(8):
+    # queue several long copies (~7 ms), then release the source while they run
+    for _ in range(24):
         cl.check(L.clEnqueueCopyBuffer(sess.queue, src, dst, 0, 0, n, 0, None, None))
     t0 = time.perf_counter()
     cl.check(L.clReleaseMemObject(src))
     dt = time.perf_counter() - t0
     pending = L.clFinish(sess.queue)   # (reaps the deferred free)
     assert pending == 0
-    assert dt < 1e-3, f"release blocked the host for {dt * 1e3:.2f} ms"
+    assert dt < 2e-3, f"release blocked the host for {dt * 1e3:.2f} ms"
     got = sess.read(dst, 1 << 20)
     assert np.array_equal(got, head)
     assert np.all(sess.read(dst, 4096, offset=n - 4096) == 0x3C)
