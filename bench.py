@@ -1123,6 +1123,36 @@ def run_secondary(S, L, T, torch, dev, hbm_peak, args):
                   "distinct_texels": texels})
         res[f"c2_map_b_{name}"] = e
         L.clReleaseSampler(smp2)
+    # the coordinate-list form of the built-in (b2clEnqueueReadImageSamples,
+    # k_sample_list: a float2 per sample, the way a translated kernel passes
+    # arbitrary coordinates) on config 2's image: the coordinates of map (A)
+    # and map (B) in output order, precomputed and resident; algorithmic bytes
+    # = 8 B coordinate + 16 B output per sample + 16 B per distinct texel
+    f32 = np.float32
+    xs = np.arange(n2, dtype=f32)[None, :]
+    ys = np.arange(n2, dtype=f32)[:, None]
+    for mname, Al in (("a", synth.affine_translate_2d(n2, n2)), ("b", synth.affine_rotate_2d(n2, n2, 30.0))):
+        cs = ((Al[0] * xs).astype(f32) + (Al[1] * ys).astype(f32)).astype(f32) + Al[3]
+        ct = ((Al[4] * xs).astype(f32) + (Al[5] * ys).astype(f32)).astype(f32) + Al[7]
+        co = np.ascontiguousarray(np.stack([cs.astype(f32), ct.astype(f32)], -1).reshape(-1, 2))
+        del cs, ct
+        cbuf = S.buffer(co.nbytes, co)
+        del co
+        for name, addr in (("repeat", cl.CL_ADDRESS_REPEAT), ("mirrored", cl.CL_ADDRESS_MIRRORED_REPEAT)):
+            smpl = S.sampler(True, addr, cl.CL_FILTER_LINEAR)
+            ms = _time_launches(T, torch, dev, lambda: cl.check(L.b2clEnqueueReadImageSamples(
+                S.queue, img2, smpl, cl.B2CL_RTYPE_FLOAT, cl.B2CL_COORD_FLOAT, cbuf, 0, n2 * n2, out2, 0, 0,
+                None, None)), 10)
+            texels = (distinct_texels_separable(Al, n2, n2, name) if mname == "a"
+                      else res[f"c2_map_b_{name}"]["distinct_texels"])
+            bl = 24 * n2 * n2 + 16 * texels
+            res[f"c2_list_map_{mname}_{name}"] = {
+                "Gsamples/s": n2 * n2 / ms / 1e6, "ms": ms, "kernel": cl.last_kernel(),
+                "coords": "float2 list (map A translate)" if mname == "a" else "float2 list (map B, 30 deg)",
+                "GB/s": bl / ms / 1e6, "hbm_frac": bl / ms / 1e6 / hbm_peak, "algorithmic_bytes": bl,
+                "distinct_texels": texels}
+            L.clReleaseSampler(smpl)
+        S.release(cbuf)
     # the same rotated read from TILED storage (B2CL_MEM_TILED_IMAGE, 8 x 8-texel
     # 1 KiB tiles; the one-thread-per-sample kernel), against that kernel on the
     # pitched image: does block-linear storage help the rotated gathers?
