@@ -440,3 +440,30 @@ def test_config3_kernels_degenerate_maps(sess, orc, case):
         exp = orc.read_grid(oimg, True, cl.CL_ADDRESS_CLAMP_TO_EDGE, cl.CL_FILTER_LINEAR, orc.RT_F, A, out, 1)
         assert_parity(got, exp, True, f"{case} rotated={rotated}")
     sess.release(img)
+
+
+@pytest.mark.parametrize("n", [1, 2, 255, 256, 257, 511, 512, 513, 1000, 131073])
+def test_list_lengths(sess, orc, n):
+    """k_sample_list takes two samples per thread, strided by the grid: every
+    list length (one block, a partial second sample, an odd tail) maps each
+    coordinate to its own output slot and nothing past the end is written."""
+    W, H = 67, 45
+    img, oimg, _ = make_images(sess, orc, RGBA, F32, W, H, 1, 2, seed=n % 97)
+    g = synth.rng(500 + n)
+    co = g.uniform(-0.3, 1.3, size=(n, 2)).astype(np.float32)
+    for addr in (cl.CL_ADDRESS_REPEAT, cl.CL_ADDRESS_CLAMP_TO_EDGE):
+        smp = sess.sampler(1, addr, cl.CL_FILTER_LINEAR)
+        L = cl.lib()
+        cbuf = sess.buffer(co.nbytes, co)
+        guard = 64
+        obuf = sess.buffer(16 * (n + guard), np.full(16 * (n + guard), 0xA5, np.uint8))
+        cl.check(L.b2clEnqueueReadImageSamples(sess.queue, img, smp, cl.B2CL_RTYPE_FLOAT, cl.B2CL_COORD_FLOAT,
+                                               cbuf, 0, n, obuf, 0, 0, None, None))
+        raw = sess.read(obuf, 16 * (n + guard), np.uint8)
+        assert np.all(raw[16 * n:] == 0xA5), "a store past the list's end"
+        got = raw[:16 * n].view(np.float32).reshape(n, 4)
+        exp = orc.read_samples(oimg, 1, addr, cl.CL_FILTER_LINEAR, orc.RT_F, co)
+        assert_parity(got, exp, True, f"list n={n} addr {hex(addr)}")
+        sess.release(cbuf, obuf)
+        L.clReleaseSampler(smp)
+    sess.release(img)
