@@ -377,7 +377,9 @@ cl_int CL_API_CALL clFinish(cl_command_queue command_queue);
 
 /* [CL1.2 §5.2.1]  Device allocation of `size` bytes (rounded up internally
  * to 256 B; CL_MEM_SIZE reports `size`).  CL_MEM_COPY_HOST_PTR uploads
- * host_ptr (synchronously).  CL_MEM_USE_HOST_PTR -> CL_INVALID_VALUE
+ * host_ptr synchronously: the bytes are in device memory when the call
+ * returns (visible to any queue's next command; host_ptr may be reused).
+ * CL_MEM_USE_HOST_PTR -> CL_INVALID_VALUE
  * (reading A33); CL_MEM_ALLOC_HOST_PTR is accepted and ignored. */
 cl_mem CL_API_CALL clCreateBuffer(cl_context context, cl_mem_flags flags, size_t size,
                                   void* host_ptr, cl_int* errcode_ret);
@@ -403,7 +405,8 @@ cl_mem CL_API_CALL clCreateBuffer(cl_context context, cl_mem_flags flags, size_t
  * row_pitch*height (reported by clGetImageInfo).  With
  * CL_MEM_COPY_HOST_PTR the contents are uploaded from host_ptr honouring
  * desc->image_row_pitch / image_slice_pitch (0 = tight), as the paper's
- * clCreateImage wrapper does with cudaMemcpy. */
+ * clCreateImage wrapper does with cudaMemcpy, complete when the call
+ * returns (as clCreateBuffer). */
 cl_mem CL_API_CALL clCreateImage(cl_context context, cl_mem_flags flags,
                                  const cl_image_format* image_format,
                                  const cl_image_desc* image_desc, void* host_ptr,
