@@ -111,3 +111,59 @@ def test_trace_log_names_command_and_kernel():
                        capture_output=True, text=True, timeout=300)
     assert r.returncode == 0, r.stderr[-2000:]
     assert "[b2cl FILL_BUFFER" in r.stderr and "kernel=k_rect<FILL>" in r.stderr, r.stderr[-2000:]
+
+
+def test_threads_share_the_runtime(sess):
+    """Eight host threads (ctypes drops the GIL in every library call), each
+    with its own queue, create / copy / fill / read back / release buffers and
+    images concurrently -- objects released while their commands are still
+    queued (deferred frees) -- and retain / release one shared buffer: every
+    result exact, the shared object alive and intact, no error."""
+    import threading
+    L = cl.lib()
+    base = np.arange(1 << 20, dtype=np.uint32).view(np.uint8)
+    shared = sess.buffer(base.nbytes, base)
+    errors = []
+
+    def worker(tid):
+        try:
+            q = sess.queue_for(0)
+            g = np.random.default_rng(100 + tid)
+            for it in range(30):
+                n = int(g.integers(1, 1 << 16)) * 16
+                host = g.integers(0, 256, n, dtype=np.uint8)
+                a = sess.buffer(n, host)
+                b = sess.buffer(n)
+                cl.check(L.clEnqueueCopyBuffer(q, a, b, 0, 0, n, 0, None, None))
+                pat = np.array([tid, it, 7, 9], np.uint8)
+                cl.check(L.clEnqueueFillBuffer(q, a, pat.ctypes.data, 4, 0, n, 0, None, None))
+                cl.check(L.clReleaseMemObject(a))  # (its fill may still be queued)
+                cl.check(L.clRetainMemObject(shared))
+                out = np.empty(n, np.uint8)
+                cl.check(L.clEnqueueReadBuffer(q, b, 1, 0, n, out.ctypes.data_as(ctypes.c_void_p), 0, None, None))
+                cl.check(L.clReleaseMemObject(shared))
+                assert np.array_equal(out, host), (tid, it)
+                cl.check(L.clReleaseMemObject(b))
+                if it % 5 == 0:
+                    W, H = int(g.integers(1, 200)), int(g.integers(1, 100))
+                    codes = g.integers(0, 256, (H, W, 4), dtype=np.uint8)
+                    img = sess.image(cl.CL_RGBA, cl.CL_UNSIGNED_INT8, W, H, host=codes)
+                    got = np.empty(W * H * 4, np.uint8)
+                    cl.check(L.clEnqueueReadImage(q, img, 1, cl.sz3((0, 0, 0)), cl.sz3((W, H, 1)), 0, 0,
+                                                  got.ctypes.data_as(ctypes.c_void_p), 0, None, None))
+                    assert np.array_equal(got, codes.reshape(-1)), (tid, it, "image")
+                    cl.check(L.clReleaseMemObject(img))
+            assert L.clFinish(q) == 0
+            cl.check(L.clReleaseCommandQueue(q))
+        except Exception as exc:  # reported by the main thread
+            errors.append(f"thread {tid}: {exc!r}")
+
+    threads = [threading.Thread(target=worker, args=(t,)) for t in range(8)]
+    for t in threads:
+        t.start()
+    for t in threads:
+        t.join(timeout=300)
+    assert not any(t.is_alive() for t in threads), "a thread hung"
+    assert not errors, errors
+    assert np.array_equal(sess.read(shared, base.nbytes), base)
+    sess.release(shared)
