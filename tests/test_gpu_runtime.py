@@ -167,3 +167,17 @@ def test_threads_share_the_runtime(sess):
     assert not errors, errors
     assert np.array_equal(sess.read(shared, base.nbytes), base)
     sess.release(shared)
+
+
+def test_released_memory_is_reclaimed(sess):
+    """800 buffers of 256 MiB (200 GiB in total, more than the device holds),
+    each filled and released at once while its fill is still queued: the
+    deferred frees are reaped as allocations proceed, so nothing runs out."""
+    L = cl.lib()
+    n = 256 << 20
+    pat = np.array([1, 2, 3, 4], np.uint8)
+    for it in range(800):
+        b = sess.buffer(n)
+        cl.check(L.clEnqueueFillBuffer(sess.queue, b, pat.ctypes.data, 4, 0, n, 0, None, None))
+        cl.check(L.clReleaseMemObject(b))
+    sess.finish()
