@@ -521,13 +521,16 @@ def run_gpu(args):
     # device, as an OpenCL program would, and joins them with events: the
     # second queue starts after a marker of the first (the previous step is
     # complete) and the first queue's barrier waits for the second read.
+    # The REPEAT read is enqueued first (tools/time_c2_queues.py: 135.3 us per
+    # step against 137.4 us with the MIRRORED read first; across bench
+    # processes the step still varies 135-138.5 us either way).
     q_two = S.queue_for(gpu)
 
     def step():
         mk, e1 = ctypes.c_void_p(), ctypes.c_void_p()
         cl.check(L.clEnqueueMarkerWithWaitList(S.queue, 0, None, ctypes.byref(mk)))
-        launch(1, queue=q_two, nwait=1, wait=(ctypes.c_void_p * 1)(mk), ev=ctypes.byref(e1))
         launch(0)
+        launch(1, queue=q_two, nwait=1, wait=(ctypes.c_void_p * 1)(mk), ev=ctypes.byref(e1))
         cl.check(L.clEnqueueBarrierWithWaitList(S.queue, 1, (ctypes.c_void_p * 1)(e1), None))
         L.clReleaseEvent(mk)
         L.clReleaseEvent(e1)
