@@ -75,9 +75,26 @@ def peaks():
 
 
 # ------------------------------------------------------------------ clocks
+_CLOCK_POLLER = r"""
+import sys, time
+import pynvml
+idx, path = int(sys.argv[1]), sys.argv[2]
+pynvml.nvmlInit()
+h = pynvml.nvmlDeviceGetHandleByIndex(idx)
+mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+with open(path, "w", buffering=1) as f:
+    f.write(f"max,{mx},0\n")
+    while True:
+        f.write(f"{time.time():.6f},{pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)},"
+                f"{pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)}\n")
+        time.sleep(0.002)
+"""
+
+
 class Clocks:
-    """SM clock + throttle reasons sampled DURING the timed region: an NVML
-    polling thread (5 ms) when pynvml finds the driver library, else
+    """SM clock + throttle reasons sampled DURING the timed region: NVML polled
+    every 2 ms by a separate process (no GIL shared with the enqueue loop; only
+    the samples stamped between start() and stop() count), else
     `nvidia-smi -lms 100` in the background."""
 
     REASONS = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
@@ -86,49 +103,67 @@ class Clocks:
     def __init__(self, index: int):
         self.index = index
         self.samples, self.reasons, self.max_mhz = [], set(), None
-        self.thread = self.proc = None
-        self._stop = False
+        self.poller = self.proc = None
+        self.t0 = self.t1 = 0.0
 
     def start(self):
+        self.file = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.file.close()
         try:
-            import threading
-
-            import pynvml
-            pynvml.nvmlInit()
-            h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
-            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
-
-            def poll():
-                while not self._stop:
-                    self.samples.append(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM))
-                    r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
-                    for n, bit in self.REASONS.items():
-                        if r & bit:
-                            self.reasons.add(n)
-                    time.sleep(0.005)
-            self.thread = threading.Thread(target=poll, daemon=True)
-            self.thread.start()
-            time.sleep(0.01)
-            return
+            import pynvml  # noqa: F401  (the poller needs it)
+            self.poller = subprocess.Popen([sys.executable, "-c", _CLOCK_POLLER, str(self.index), self.file.name],
+                                           stdout=subprocess.DEVNULL, stderr=subprocess.DEVNULL)
+            deadline = time.time() + 20
+            while time.time() < deadline and self.poller.poll() is None:
+                if len(open(self.file.name).read().splitlines()) >= 2:
+                    break
+                time.sleep(0.01)
+            if self.poller.poll() is not None or len(open(self.file.name).read().splitlines()) < 2:
+                self.poller.kill()
+                self.poller = None
         except Exception:
-            self.thread = None
-        try:
-            self.file = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
-            self.proc = subprocess.Popen(
-                ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,"
-                 "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
-                 "--format=csv,noheader,nounits", "-lms", "100"],
-                stdout=self.file, stderr=subprocess.DEVNULL)
-        except (OSError, FileNotFoundError):
-            self.proc = None
+            self.poller = None
+        if self.poller is None:
+            try:
+                self.proc = subprocess.Popen(
+                    ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,"
+                     "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                     "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+                     "--format=csv,noheader,nounits", "-lms", "100"],
+                    stdout=open(self.file.name, "w"), stderr=subprocess.DEVNULL)
+            except (OSError, FileNotFoundError):
+                self.proc = None
+        self.t0 = time.time()
 
     def stop(self):
-        if self.thread is not None:
-            self._stop = True
-            self.thread.join(timeout=2)
-            sm = self.samples
-            src = "nvml 5 ms"
+        self.t1 = time.time()
+        if self.poller is not None:
+            time.sleep(0.005)
+            self.poller.terminate()
+            try:
+                self.poller.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.poller.kill()
+            rows = [ln.split(",") for ln in open(self.file.name).read().splitlines() if ln.strip()]
+            os.unlink(self.file.name)
+            timed, sm = [], []
+            for r in rows:
+                if r[0] == "max":
+                    self.max_mhz = float(r[1])
+                    continue
+                try:
+                    timed.append((float(r[0]), float(r[1]), int(r[2])))
+                except (ValueError, IndexError):
+                    continue
+            inside = [t for t in timed if self.t0 <= t[0] <= self.t1]
+            if not inside and timed:  # (a region shorter than the poll period: the nearest sample)
+                inside = [min(timed, key=lambda t: abs(t[0] - 0.5 * (self.t0 + self.t1)))]
+            for _, mhz, bits in inside:
+                sm.append(mhz)
+                for n, bit in self.REASONS.items():
+                    if bits & bit:
+                        self.reasons.add(n)
+            src = "nvml 2 ms (separate process)"
         elif self.proc is not None:
             time.sleep(0.15)
             self.proc.terminate()
@@ -136,7 +171,6 @@ class Clocks:
                 self.proc.wait(timeout=5)
             except subprocess.TimeoutExpired:
                 self.proc.kill()
-            self.file.flush()
             rows = [ln.split(",") for ln in open(self.file.name).read().splitlines() if ln.strip()]
             os.unlink(self.file.name)
             sm = []
